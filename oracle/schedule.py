@@ -1,0 +1,174 @@
+"""Oracle for the preemption scheduler: invariant checker + discrete-event model.
+
+Invariants (each from the paper, checked on any trace — the oracle's own simulated
+trace or the GPU runtime's recorded one):
+
+  I1  "no two GPU executors are scheduled on a single GPU simultaneously"
+      (section 3.4): on a device, compute intervals of different
+      models are disjoint.
+  I2  per-job order: "executors from consecutive runs of the same session follow
+      sequential order" (section 3.2); with "no work is lost"
+       every (iter, k) of a job runs exactly once, in order, and a
+      job's subgraphs never overlap each other.
+  I3  preemption latency is bounded by the outstanding work of the preemptee: "Only
+      waiting for the outstanding nodes of a preempted job to complete is on the
+      critical path" (section 5.2.3).  Checked as
+      start(infer) - max(arrival, end of the previous inference on that device)
+      <= max train-subgraph duration on that device + slack.
+  I4  cut rule (reading Q13): a request arriving while S_k runs is served at the
+      boundary after S_k.
+
+Event dicts: {"dev", "job", "kind": "train"|"infer", "iter", "k", "t0", "t1",
+"arrival" (infer only)}; times in any consistent unit.
+
+Pins (tests/test_oracle_schedule.py): hand-built violating traces for I1..I4 are
+rejected; the discrete-event model's traces satisfy them; closed-form latencies of
+the model for single arrivals.
+"""
+from __future__ import annotations
+
+import heapq
+from typing import Dict, List, Sequence
+
+
+class InvariantError(AssertionError):
+    pass
+
+
+def check_no_corun(events: Sequence[dict]) -> None:
+    """I1: per device, intervals of different jobs never overlap."""
+    by_dev: Dict[int, List[dict]] = {}
+    for e in events:
+        by_dev.setdefault(e["dev"], []).append(e)
+    for d, evs in by_dev.items():
+        evs = sorted(evs, key=lambda e: (e["t0"], e["t1"]))
+        for a, b in zip(evs, evs[1:]):
+            if a["job"] != b["job"] and b["t0"] < a["t1"]:
+                raise InvariantError(f"dev {d}: job {a['job']} [{a['t0']},{a['t1']}) overlaps "
+                                     f"job {b['job']} [{b['t0']},{b['t1']})")
+
+
+def check_job_order(events: Sequence[dict], n_sub: Dict[int, int],
+                    start: Dict[int, tuple] | None = None) -> None:
+    """I2: each training job's (iter, k) sequence is the contiguous enumeration."""
+    by_job: Dict[int, List[dict]] = {}
+    for e in events:
+        if e["kind"] == "train":
+            by_job.setdefault(e["job"], []).append(e)
+    for j, evs in by_job.items():
+        evs = sorted(evs, key=lambda e: e["t0"])
+        n = n_sub[j]
+        it, k = (start or {}).get(j, (evs[0]["iter"], evs[0]["k"]))
+        prev_t1 = None
+        for e in evs:
+            if (e["iter"], e["k"]) != (it, k):
+                raise InvariantError(f"job {j}: expected ({it},{k}) got ({e['iter']},{e['k']})")
+            if prev_t1 is not None and e["t0"] < prev_t1:
+                raise InvariantError(f"job {j}: subgraph ({it},{k}) overlaps its predecessor")
+            prev_t1 = e["t1"]
+            k += 1
+            if k == n:
+                it, k = it + 1, 0
+
+
+def check_preempt_latency(events: Sequence[dict], slack: float) -> None:
+    """I3: inference start - ready time <= longest training subgraph on that device + slack."""
+    by_dev: Dict[int, List[dict]] = {}
+    for e in events:
+        by_dev.setdefault(e["dev"], []).append(e)
+    for d, evs in by_dev.items():
+        longest = max([e["t1"] - e["t0"] for e in evs if e["kind"] == "train"], default=0.0)
+        prev_end = float("-inf")
+        for e in sorted([e for e in evs if e["kind"] == "infer"], key=lambda e: e["t0"]):
+            ready = max(e["arrival"], prev_end)
+            if e["t0"] - ready > longest + slack:
+                raise InvariantError(f"dev {d}: inference waited {e['t0'] - ready} > "
+                                     f"{longest} + {slack}")
+            prev_end = e["t1"]
+
+
+def check_cut_rule(events: Sequence[dict]) -> None:
+    """I4: the first training subgraph that starts on a device after an arrival but
+    before the inference ran must not exist (the job stops at the next boundary)."""
+    by_dev: Dict[int, List[dict]] = {}
+    for e in events:
+        by_dev.setdefault(e["dev"], []).append(e)
+    for d, evs in by_dev.items():
+        trains = [e for e in evs if e["kind"] == "train"]
+        for r in (e for e in evs if e["kind"] == "infer"):
+            for t in trains:
+                if r["arrival"] <= t["t0"] < r["t0"]:
+                    raise InvariantError(f"dev {d}: subgraph ({t['iter']},{t['k']}) started at "
+                                         f"{t['t0']} after arrival {r['arrival']} before the "
+                                         f"inference at {r['t0']}")
+
+
+def check_all(events: Sequence[dict], n_sub: Dict[int, int], slack: float = 0.0) -> None:
+    check_no_corun(events)
+    check_job_order(events, n_sub)
+    check_preempt_latency(events, slack)
+    check_cut_rule(events)
+
+
+def simulate(durations: Sequence[float], iters: int, arrivals: Sequence[float],
+             infer_dur: float, tier: str = "host", swap_out: float = 0.0,
+             swap_in: float = 0.0, gate: float = 0.0) -> List[dict]:
+    """Discrete-event model of one training job (job 0) + an inference stream (job 1).
+
+    Policy (readings Q4-Q7, Q13):
+      * training runs S_0..S_{n-1} per iteration back to back on device 0, ``gate``
+        between subgraphs;
+      * a request arriving while S_k runs is served once S_k finishes; requests are
+        FIFO by arrival and all queued ones run before the job resumes;
+      * host tier: state goes out (``swap_out``, concurrent with inference) and comes
+        back (``swap_in``) after the queue drained; the job resumes on device 0;
+      * peer tier: the job migrates (``swap_out``) and resumes on device 1, where it
+        stays (Q7); later requests on device 0 find no training job to preempt.
+    """
+    n = len(durations)
+    ev: List[dict] = []
+    t = 0.0
+    dev = 0
+    q = list(arrivals)
+    heapq.heapify(q)
+    it, k = 0, 0
+    free0 = 0.0  # device-0 time after the last inference
+
+    def serve_pending(now):
+        nonlocal free0
+        end = max(now, free0)
+        while q and q[0] <= end:
+            a = heapq.heappop(q)
+            s = max(end, a)
+            ev.append({"dev": 0, "job": 1, "kind": "infer", "iter": 0, "k": 0, "t0": s,
+                       "t1": s + infer_dur, "arrival": a})
+            end = s + infer_dur
+        free0 = end
+        return end
+
+    while it < iters:
+        if dev == 0 and q and q[0] <= t:
+            # preempt at this boundary
+            cut_t = t
+            drained = serve_pending(cut_t)
+            if tier == "host":
+                t = max(drained, cut_t + swap_out) + swap_in
+            else:
+                dev = 1
+                t = cut_t + swap_out
+            continue
+        s = t
+        e = s + durations[k]
+        ev.append({"dev": dev, "job": 0, "kind": "train", "iter": it, "k": k, "t0": s, "t1": e})
+        t = e + gate
+        k += 1
+        if k == n:
+            it, k = it + 1, 0
+    # serve requests that arrive after training finished (or on a now-free device 0)
+    while q:
+        a = heapq.heappop(q)
+        s = max(a, free0)
+        ev.append({"dev": 0, "job": 1, "kind": "infer", "iter": 0, "k": 0, "t0": s,
+                   "t1": s + infer_dur, "arrival": a})
+        free0 = s + infer_dur
+    return ev

@@ -1,0 +1,123 @@
+"""Pins for oracle/runner.py (trajectory, inference) and oracle/schedule.py (invariants).
+
+runner: C1 trains (loss falls over 100 iterations — sanity, not parity); inference
+vs a brute-force fp64 forward written with Python loops; the preempter running at the
+cut does not perturb the trajectory.
+schedule: hand-built traces violating I1..I4 are rejected; the discrete-event
+model's traces satisfy all four; closed-form latencies of the model.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import runner as R, schedule as SC, graph as OG
+from sf_inputs import graphs as G, data as D
+
+
+def test_c1_loss_decreases():
+    g = G.mlp_train()
+    tr = R.run(g, 100, D.init_state(g), D.datasets(g), keep_stagings=False)
+    losses = [float(o["loss"][0, 0]) for o in tr.outputs]
+    assert abs(losses[0] - math.log(10)) < 0.5
+    assert np.mean(losses[-10:]) < losses[0] - 0.1
+
+
+def test_inference_brute_force():
+    gi = G.mlp_infer((7, 5, 3))
+    params = D.init_state(gi, seed=9)
+    rng = np.random.default_rng(1)
+    for i, t in enumerate(gi.tensors):
+        if t.rows == 1 and t.kind == 0:
+            params[i] = rng.standard_normal((1, t.cols)).astype(np.float32)
+    x = D.infer_inputs(gi, 1)[0]
+    got = R.run_inference(gi, params, x)
+    W1, b1, W2, b2 = (params[gi.tid(n)] for n in ("W1", "b1", "W2", "b2"))
+    h = [max(0.0, sum(float(x[0, k]) * float(W1[k, j]) for k in range(7)) + float(b1[0, j]))
+         for j in range(5)]
+    l = [sum(h[k] * float(W2[k, j]) for k in range(5)) + float(b2[0, j]) for j in range(3)]
+    m = max(l)
+    e = [math.exp(v - m) for v in l]
+    p = [v / sum(e) for v in e]
+    np.testing.assert_allclose(got[0], p, rtol=1e-6)
+
+
+def test_preempter_at_cut_does_not_perturb():
+    g = G.mlp_train((5, 7, 3), batch=4, pool=2)
+    gi = G.mlp_infer((5, 7, 3))
+    st, ds = D.init_state(g), D.datasets(g)
+    ref = R.run(g, 3, st, ds)
+    got = R.run(g, 3, st, ds, schedule=[(1, 2, R.HOST), (2, 3, 1)],
+                inference=(gi, D.init_state(gi), D.infer_inputs(gi, 1)[0]))
+    for i in ref.state:
+        assert ref.state[i].tobytes() == got.state[i].tobytes()
+
+
+def _ev(dev, job, kind, t0, t1, it=0, k=0, arrival=None):
+    e = {"dev": dev, "job": job, "kind": kind, "iter": it, "k": k, "t0": t0, "t1": t1}
+    if arrival is not None:
+        e["arrival"] = arrival
+    return e
+
+
+def test_checker_rejects_corun():
+    evs = [_ev(0, 0, "train", 0, 10), _ev(0, 1, "infer", 5, 7, arrival=4)]
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun(evs)
+    SC.check_no_corun([_ev(0, 0, "train", 0, 10), _ev(1, 1, "infer", 5, 7, arrival=4)])
+
+
+def test_checker_rejects_order_gap_and_duplicate():
+    ok = [_ev(0, 0, "train", i, i + 1, it=i // 3, k=i % 3) for i in range(7)]
+    SC.check_job_order(ok, {0: 3})
+    gap = ok[:3] + ok[4:]
+    with pytest.raises(SC.InvariantError):
+        SC.check_job_order(gap, {0: 3})
+    dup = ok[:4] + [dict(ok[3], t0=4.5, t1=4.9)] + ok[4:]
+    with pytest.raises(SC.InvariantError):
+        SC.check_job_order(dup, {0: 3})
+    overlap = [dict(e) for e in ok]
+    overlap[2]["t0"] = 1.5
+    with pytest.raises(SC.InvariantError):
+        SC.check_job_order(overlap, {0: 3})
+
+
+def test_checker_rejects_long_wait_and_cut_rule():
+    evs = [_ev(0, 0, "train", 0, 10), _ev(0, 0, "train", 10, 20, k=1),
+           _ev(0, 1, "infer", 20, 21, arrival=5)]
+    ok = [_ev(0, 0, "train", 0, 10), _ev(0, 1, "infer", 10, 11, arrival=5),
+          _ev(0, 0, "train", 11, 21, k=1)]
+    SC.check_preempt_latency(ok, 0)
+    SC.check_cut_rule(ok)
+    with pytest.raises(SC.InvariantError):
+        SC.check_preempt_latency(evs, 0)  # waited 15 > longest subgraph 10
+    evs2 = [_ev(0, 0, "train", 0, 4), _ev(0, 0, "train", 4, 8, k=1),
+            _ev(0, 0, "train", 8, 12, k=2), _ev(0, 1, "infer", 12, 13, arrival=1)]
+    with pytest.raises(SC.InvariantError):
+        SC.check_preempt_latency(evs2, 0)
+    with pytest.raises(SC.InvariantError):
+        SC.check_cut_rule(evs)  # subgraph k=1 started at 10 after arrival 5
+
+
+def test_model_satisfies_invariants_host_and_peer():
+    dur = [3.0, 1.0, 2.0, 0.5, 1.5]
+    arr = list(D.poisson_arrivals(40, 0.2, seed=3))
+    for tier in ("host", "peer"):
+        evs = SC.simulate(dur, 30, arr, 0.7, tier=tier, swap_out=0.4, swap_in=0.4, gate=0.01)
+        SC.check_all(evs, {0: len(dur)}, slack=0.02)
+        trains = [e for e in evs if e["kind"] == "train"]
+        assert len(trains) == 30 * len(dur)
+        assert len([e for e in evs if e["kind"] == "infer"]) == 40
+
+
+def test_model_closed_form_single_arrival():
+    dur = [4.0, 4.0, 4.0]
+    # arrival at 5 while S_1 runs [4, 8): served at 8 (cut k=2), done 9; host swap
+    evs = SC.simulate(dur, 2, [5.0], 1.0, tier="host", swap_out=0.5, swap_in=2.0)
+    inf = [e for e in evs if e["kind"] == "infer"][0]
+    assert (inf["t0"], inf["t1"]) == (8.0, 9.0)
+    nxt = [e for e in evs if e["kind"] == "train" and e["t0"] >= 8.0][0]
+    assert (nxt["iter"], nxt["k"], nxt["t0"]) == (0, 2, 11.0)  # max(9, 8.5) + 2
+    evs = SC.simulate(dur, 2, [5.0], 1.0, tier="peer", swap_out=0.5)
+    nxt = [e for e in evs if e["kind"] == "train" and e["t0"] >= 8.0][0]
+    assert (nxt["dev"], nxt["k"], nxt["t0"]) == (1, 2, 8.5)
