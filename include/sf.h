@@ -1,0 +1,336 @@
+/*
+ * sf.h — C ABI of the SwitchFlow-on-B200 subgraph-preemption runtime.
+ *
+ * Method: SwitchFlow, "Preemptive Multitasking for Deep Learning" (Wu et al.,
+ * Middleware '21), /root/reference/PAPER.md.  The ABI follows the paper's problem
+ * statement: jobs are static computation graphs (section 2) submitted
+ * with a priority (section 4); the session is partitioned into
+ * subgraphs run by executors (section 2.1) and one executor version is
+ * built per device (section 3.2); a high-priority job "is allowed to
+ * start immediately after submission" (section 3.4); the preemptee is
+ * suspended, its graph re-pointed at another device, its persistent state copied
+ * asynchronously, and it resumes with no work lost (section 3.3); no two
+ * models' GPU executors co-run on one GPU (section 3.4).
+ *
+ * B200 design: a preemption cuts the job at its next subgraph boundary and
+ * migrates the live set L_k (variables, optimizer slots, in-flight activations) — to a
+ * peer B200 over NVLink with a fused peer-store kernel, or to pinned host memory
+ * (pack kernel + PCIe) — and resumes the pre-built CUDA-graph version of S_k there.
+ *
+ * Conventions (all entry points):
+ *  - every call returns sf_status; SF_OK == 0, errors < 0; no exception crosses the ABI;
+ *    the message of the last error on the calling thread is in sf_last_error();
+ *  - "device pointer" = CUDA global memory of the stated device (or a peer mapping);
+ *    "host pointer" = ordinary host memory; "pinned" = page-locked (cudaHostAlloc /
+ *    torch pin_memory) host memory;
+ *  - memory passed in (arenas, staging, request buffers, op operands) is CALLER-OWNED
+ *    and must stay valid until the call that uses it completes (for sf_bind: until
+ *    sf_destroy); runtime-owned memory (descriptor lists, CUDA graphs, workspaces,
+ *    events, threads) is freed only by sf_destroy;
+ *  - tensors are 2-D row-major; fp32 (SF_F32) or int32 (SF_I32); arenas place every
+ *    tensor at a 256-byte aligned offset, identical on every device;
+ *  - all sf_* calls are thread-safe.  sf_op_* kernel entry points are asynchronous on
+ *    the given stream (cudaStream_t passed as void*, NULL = legacy default stream).
+ */
+#ifndef SF_H_
+#define SF_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SF_ABI_VERSION 1
+
+typedef int32_t sf_status;
+#define SF_OK 0
+#define SF_EINVAL (-1)       /* bad argument / malformed graph */
+#define SF_ENOMEM (-2)       /* device budget exceeded or allocation failed */
+#define SF_ESTATE (-3)       /* call not valid in the object's current state */
+#define SF_EBUSY (-4)        /* a migration of this job is already in flight */
+#define SF_ECUDA (-5)        /* CUDA error; text in sf_last_error() */
+#define SF_ETIMEOUT (-6)
+#define SF_EUNSUPPORTED (-7) /* op outside the fixed op set, or dtype/shape not supported */
+
+/* ---- graph IR (nodes = ops, edges = dataflow) -------------------- */
+enum sf_dtype { SF_F32 = 0, SF_I32 = 1 };
+
+/* Kinds: PARAM/SLOT/SCALAR_STATE are persistent across iterations;
+ * DATASET is read-only and replicated on every candidate device (never migrated);
+ * INPUT/LABEL are fed each iteration (FEED op or request copy); ACT/GRAD are
+ * intermediates; OUTPUT is fetched at iteration end (live until then). */
+enum sf_tensor_kind {
+  SF_PARAM = 0, SF_SLOT = 1, SF_SCALAR_STATE = 2, SF_DATASET = 3, SF_INPUT = 4,
+  SF_LABEL = 5, SF_ACT = 6, SF_GRAD = 7, SF_OUTPUT = 8
+};
+
+/* The fixed op set of BASELINE.json north_star.  Operand conventions:
+ *  GEMM         in[A,B] out[C]        C = op(A) op(B) (+C if SF_GEMM_ACC); op = transpose
+ *                                     if SF_GEMM_TA / SF_GEMM_TB; fp32-accurate (3xTF32)
+ *  BIAS_ACT     in[z,b1(,b2,b3)] out[h]  h = act(z + b1 + b2 + b3), act = ReLU if SF_ACT_RELU
+ *  BIAS_ACT_BWD in[dh,h] out[dz,db]   dz = dh * [h > 0]; db = column sum of dz
+ *  COLSUM       in[x] out[s]          s = column sum of x (s is [1, cols])
+ *  SOFTMAX_CE   in[logits,labels] out[loss,dlogits]  mean sparse CE; (softmax-onehot)/B
+ *  SOFTMAX      in[logits] out[probs]
+ *  SGD_MOM      in[g] out[w,a]        a = mu * a + g; w = w - lr * a    (f = lr, mu)
+ *  ADAM         in[g,step] out[w,m,v] TF Adam, t = step + 1 (f = lr, beta1, beta2, eps)
+ *  FEED         in[pool,step] out[x]  x = pool rows [(step mod P) * rows, +rows)
+ *  STEP_INC     out[step]             step += 1
+ * Reductions are deterministic (fixed order): repeated runs are bitwise identical. */
+enum sf_op_type {
+  SF_OP_GEMM = 1, SF_OP_BIAS_ACT = 2, SF_OP_BIAS_ACT_BWD = 3, SF_OP_COLSUM = 4,
+  SF_OP_SOFTMAX_CE = 5, SF_OP_SOFTMAX = 6, SF_OP_SGD_MOM = 7, SF_OP_ADAM = 8,
+  SF_OP_FEED = 9, SF_OP_STEP_INC = 10
+};
+#define SF_GEMM_TA 1
+#define SF_GEMM_TB 2
+#define SF_GEMM_ACC 4
+#define SF_ACT_RELU 1
+
+typedef struct sf_tensor_desc {
+  int32_t rows, cols; /* 2-D row-major */
+  int32_t dtype;      /* sf_dtype */
+  int32_t kind;       /* sf_tensor_kind */
+} sf_tensor_desc;
+
+typedef struct sf_op_desc {
+  int32_t type;    /* sf_op_type */
+  int32_t n_in;    /* number of valid entries in in[] */
+  int32_t in[6];   /* tensor ids (index into sf_graph_desc.tensors) */
+  int32_t n_out;
+  int32_t out[3];
+  int32_t flags;   /* SF_GEMM_* / SF_ACT_RELU */
+  int32_t phase;   /* layer-phase id: PER_LAYER_PHASE cuts where it changes */
+  float f[4];      /* op scalars (lr, mu / lr, beta1, beta2, eps) */
+} sf_op_desc;
+
+typedef struct sf_graph_desc {
+  const char* name;               /* copied; may be NULL */
+  uint32_t n_tensors;
+  const sf_tensor_desc* tensors;  /* host pointer, copied before return */
+  uint32_t n_ops;
+  const sf_op_desc* ops;          /* host pointer, topological order, copied */
+} sf_graph_desc;
+
+/* ---- runtime --------------------------------------------------------------------- */
+typedef struct sf_runtime sf_runtime; /* opaque, one per process */
+typedef uint32_t sf_graph_id;
+typedef uint32_t sf_job_id;
+typedef uint64_t sf_req_id;
+#define SF_TARGET_HOST (-1) /* migrate the live set to pinned host memory (host tier) */
+
+/* Host-tier transfer strategy. */
+#define SF_HOST_CE 0 /* pack into device staging, copy-engine D2H; H2D, unpack */
+#define SF_HOST_ZC 1 /* zero-copy: pack kernel stores straight into mapped pinned memory,
+                        unpack kernel reads it back over PCIe */
+
+typedef struct sf_config {
+  int32_t n_devices;             /* logical device slots */
+  const int32_t* cuda_ordinals;  /* host array [n_devices]: CUDA device of each slot */
+  int32_t exclusive_gpu;         /* 1 (default behaviour): no two models' subgraphs co-run
+                                    on a device; 0: free co-run baseline
+                                    (multi-threaded TF) */
+  int32_t auto_preempt;          /* 1: sf_submit_inference preempts the training job that
+                                    owns the device */
+  int32_t iteration_granularity; /* 1: preempt only at iteration boundaries (session time
+                                    slicing baseline); 0: subgraph */
+  int32_t host_mode;             /* SF_HOST_CE or SF_HOST_ZC */
+  int32_t poison_released;       /* 1: fill released source arenas with 0xFF (tests) */
+  int32_t trace_capacity;        /* events kept; 0 -> 1<<16 */
+  uint64_t device_budget_bytes;  /* per device; 0 = unlimited */
+} sf_config;
+
+/* Create a runtime: enables peer access between distinct CUDA devices of the slots,
+ * creates per-slot streams (training, high-priority inference, migration) and one
+ * dispatcher thread per slot.  *out owned by the caller, freed by sf_destroy. */
+sf_status sf_create(const sf_config* cfg, sf_runtime** out);
+/* Wait for all jobs and requests, join threads, free runtime-owned memory. */
+void sf_destroy(sf_runtime* rt);
+/* Thread-local text of the last error (valid until the next failing call). */
+const char* sf_last_error(void);
+int32_t sf_abi_version(void);
+
+/* Validate and copy a graph (shapes, dtypes, op arity, read-before-write).
+ * priority > 0 marks an inference (preempter) graph.  SF_EUNSUPPORTED for ops outside
+ * the fixed set; SF_EINVAL for malformed graphs. */
+sf_status sf_register_graph(sf_runtime* rt, const sf_graph_desc* g, int32_t priority,
+                            sf_graph_id* out);
+
+#define SF_PART_PER_LAYER_PHASE 0
+#define SF_PART_MAX_OPS 1
+typedef struct sf_partition_opts {
+  int32_t policy;  /* SF_PART_PER_LAYER_PHASE (maximal runs of equal phase) or
+                      SF_PART_MAX_OPS (split runs to <= max_ops ops; optimizer runs whole) */
+  int32_t max_ops;
+} sf_partition_opts;
+typedef struct sf_partition_info {
+  int32_t n_subgraphs;
+  uint64_t arena_bytes;      /* device bytes each bound device must provide */
+  uint64_t staging_bytes;    /* bytes of the largest staging buffer (max over cuts) */
+  uint64_t persistent_bytes; /* PARAM + SLOT + SCALAR_STATE */
+  uint64_t max_live_bytes;   /* max over cuts of sum(nbytes of L_k) */
+} sf_partition_info;
+
+/* Partition into subgraphs S_0..S_{n-1}, compute the live set L_k of every cut and the
+ * arena layout.  May be called once per graph. */
+sf_status sf_partition(sf_runtime* rt, sf_graph_id g, const sf_partition_opts* o,
+                       sf_partition_info* out);
+/* Op range [begin, end) of subgraph k. */
+sf_status sf_subgraph_range(sf_runtime* rt, sf_graph_id g, int32_t k, int32_t* op_begin,
+                            int32_t* op_end);
+/* L_k as ascending tensor ids (host array ids[cap]); *n = |L_k|, *bytes = sum nbytes. */
+sf_status sf_live_set(sf_runtime* rt, sf_graph_id g, int32_t k, uint32_t* ids, uint32_t cap,
+                      uint32_t* n, uint64_t* bytes);
+/* Byte offset of a tensor inside every arena of this graph. */
+sf_status sf_tensor_offset(sf_runtime* rt, sf_graph_id g, uint32_t tensor_id, uint64_t* off);
+/* Staging layout of cut k: total bytes and payload offset of the e-th live tensor. */
+sf_status sf_staging_layout(sf_runtime* rt, sf_graph_id g, int32_t k, uint64_t* total,
+                            uint64_t* payload_offsets, uint32_t cap);
+
+/* Bind memory of device slot `dev` to graph g and build its versions: one CUDA graph per
+ * subgraph (the per-device executor replica) plus the pack / unpack /
+ * peer-store descriptor lists of every cut.
+ *   arena        device pointer, >= arena_bytes, 256-B aligned (caller fills DATASET /
+ *                PARAM / SLOT / SCALAR_STATE contents at sf_tensor_offset() offsets)
+ *   staging      device pointer, >= staging_bytes, or NULL (then host tier uses ZC)
+ *   host_staging pinned host pointer, >= staging_bytes, or NULL (no host tier)
+ * Peer-store lists to a slot are built when both slots are bound.  Returns SF_ENOMEM when
+ * the persistent bytes of all graphs bound to the slot exceed device_budget_bytes. */
+sf_status sf_bind(sf_runtime* rt, sf_graph_id g, int32_t dev, void* arena, void* staging,
+                  void* host_staging);
+
+/* ---- training jobs, preemption --------------------------------------------------- */
+enum sf_job_state {
+  SF_JOB_RUNNING = 0, SF_JOB_STOPPING = 1, SF_JOB_MIGRATING = 2, SF_JOB_PREEMPTED = 3,
+  SF_JOB_DONE = 4, SF_JOB_FAILED = 5
+};
+typedef struct sf_job_info {
+  int32_t state;        /* sf_job_state */
+  int32_t dev;          /* current device slot (source while migrating) */
+  int64_t iter;         /* next (iter, k) to run */
+  int32_t k;
+  int32_t n_preemptions;
+  uint64_t migrated_bytes;      /* cumulative live bytes moved */
+  double last_pack_us;          /* CUDA-event durations of the last migration's kernels */
+  double last_xfer_us;
+  double last_unpack_us;
+  uint64_t last_stop_ns;        /* CLOCK_MONOTONIC: cut decided (in-flight S_k done) */
+  uint64_t last_resume_ns;      /* CLOCK_MONOTONIC: first resumed subgraph launched */
+} sf_job_info;
+
+typedef struct sf_cut_info {
+  int64_t iter;          /* the cut sits before S_k of this iteration */
+  int32_t k;
+  int32_t n_tensors;     /* |L_k| */
+  uint64_t live_bytes;   /* sum nbytes(L_k) */
+  uint64_t t_req_ns;     /* CLOCK_MONOTONIC when the preemption was requested */
+  uint64_t t_stop_ns;    /* when the job stopped at the boundary */
+  int32_t src_dev, dst_dev;
+} sf_cut_info;
+
+/* A preemption scheduled at a fixed cut: before S_k of iteration `iter`, migrate the live
+ * set to `target` (peer slot or SF_TARGET_HOST) and resume right away (peer: on the
+ * target; host: swap back into the same slot once its inference queue drained). */
+typedef struct sf_cut_request {
+  int64_t iter;
+  int32_t k;
+  int32_t target;
+} sf_cut_request;
+
+/* Start a training job of graph g on bound slot `dev` for `iters` iterations (job
+ * driver thread).  `auto_target` = where an auto-preemption migrates it (peer slot or
+ * SF_TARGET_HOST).  `sched` (host array, n_sched entries, ascending (iter, k), copied)
+ * lists deterministic preemptions, e.g. for "preempted N times == unpreempted" checks. */
+sf_status sf_start_training(sf_runtime* rt, sf_graph_id g, int32_t dev, int64_t iters,
+                            int32_t auto_target, const sf_cut_request* sched, int32_t n_sched,
+                            sf_job_id* out);
+/* Preempt: block until the job stops at its next subgraph boundary (kernels of the
+ * in-flight subgraph finish) and its migration to `target` (peer slot
+ * or SF_TARGET_HOST) is enqueued; does not wait for the migration.  The job then stays
+ * SF_JOB_PREEMPTED until sf_resume.  SF_ESTATE if not RUNNING; SF_EINVAL if target is the
+ * current slot or unbound; SF_EBUSY if a migration is in flight. */
+sf_status sf_preempt(sf_runtime* rt, sf_job_id job, int32_t target, sf_cut_info* out);
+/* Resume a preempted job on `dev` (peer tier: the migration target; host tier: any bound
+ * slot) — stream-ordered after the migration, no host sync on the copy.  SF_ESTATE if
+ * the job is not preempted. */
+sf_status sf_resume(sf_runtime* rt, sf_job_id job, int32_t dev);
+sf_status sf_job_query(sf_runtime* rt, sf_job_id job, sf_job_info* out);
+/* Wait until the job finished all iterations (SF_ETIMEOUT after timeout_ns; <0 = inf). */
+sf_status sf_wait_job(sf_runtime* rt, sf_job_id job, int64_t timeout_ns);
+/* Ask a running job to stop at its next iteration boundary and finish. */
+sf_status sf_stop_job(sf_runtime* rt, sf_job_id job);
+
+/* ---- inference (the preempter) --------------------------------------------------- */
+typedef struct sf_timing {
+  uint64_t arrival_ns;   /* scheduled arrival (CLOCK_MONOTONIC) */
+  uint64_t start_ns;     /* inference launched on the device */
+  uint64_t end_ns;       /* completion observed */
+  int32_t dev;
+  int32_t preempted_job; /* job cut by this request, or -1 */
+  int64_t cut_iter;
+  int32_t cut_k;
+} sf_timing;
+
+/* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).
+ * in: pointer (device or pinned host) to the INPUT tensor's bytes; out: pointer (device
+ * or pinned host) receiving the OUTPUT tensor's bytes; both caller-owned until sf_wait.
+ * arrival_ns = scheduled arrival time (CLOCK_MONOTONIC ns; 0 = now).  With
+ * auto_preempt the training job owning dev is preempted to its auto_target. */
+sf_status sf_submit_inference(sf_runtime* rt, sf_graph_id g, int32_t dev, const void* in,
+                              void* out, uint64_t arrival_ns, sf_req_id* req);
+/* Wait for a request; fills *timing. */
+sf_status sf_wait(sf_runtime* rt, sf_req_id req, int64_t timeout_ns, sf_timing* timing);
+
+/* ---- trace (schedule invariants; oracle/schedule.py checks it) ------------------- */
+enum sf_event_kind { SF_EV_TRAIN = 0, SF_EV_INFER = 1, SF_EV_MIGRATE = 2 };
+typedef struct sf_trace_event {
+  int32_t dev, job, kind, k;   /* job: training job id, or 1<<20 | request for inference */
+  int64_t iter;
+  uint64_t t0_ns, t1_ns;       /* host CLOCK_MONOTONIC: launch .. completion observed */
+  uint64_t arrival_ns;         /* inference only */
+} sf_trace_event;
+sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* n_out);
+uint64_t sf_now_ns(void); /* CLOCK_MONOTONIC */
+
+/* ---- kernel entry points (operate on plain device pointers; async on `stream`) ---- */
+/* Multi-tensor copy descriptor: copy nbytes (multiple of 4) from src to dst, and write
+ * zeros from nbytes up to span (span >= nbytes, multiple of 16); src/dst 16-B aligned.
+ * This single descriptor walk is the pack (arena -> staging, span = round_up(nbytes,256)),
+ * unpack (staging -> arena) and peer-store (arena -> peer arena over NVLink) kernel. */
+typedef struct sf_copy_desc {
+  const void* src;
+  void* dst;
+  uint64_t nbytes;
+  uint64_t span;
+} sf_copy_desc;
+/* descs: HOST array [n].  patch_iter >= 0: overwrite bytes [16, 24) of descriptor 0's
+ * destination with patch_iter (the staging header's iter field). */
+sf_status sf_op_mtcopy(const sf_copy_desc* descs, int32_t n, int64_t patch_iter, void* stream);
+/* C = op(A) op(B) (+C); lda/ldb/ldc = row strides (elements) of the stored matrices. */
+sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N,
+                     int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
+                     void* stream);
+sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
+                         float* h, int32_t rows, int32_t cols, int32_t relu, void* stream);
+sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* db,
+                             int32_t rows, int32_t cols, void* stream);
+sf_status sf_op_colsum(const float* x, float* s, int32_t rows, int32_t cols, void* stream);
+sf_status sf_op_softmax_ce(const float* logits, const int32_t* labels, float* loss,
+                           float* dlogits, int32_t rows, int32_t cols, void* stream);
+sf_status sf_op_softmax(const float* logits, float* probs, int32_t rows, int32_t cols,
+                        void* stream);
+sf_status sf_op_sgd_mom(float* w, float* a, const float* g, int64_t n, float lr, float mu,
+                        void* stream);
+sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t* step,
+                     int64_t n, float lr, float beta1, float beta2, float eps, void* stream);
+/* Fill n bytes at dst (device) with byte value (0xFF = poison). */
+sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream);
+/* Number of kernels this process launched through the library so far. */
+uint64_t sf_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SF_H_ */

@@ -1,0 +1,477 @@
+// GEMM for the training subgraphs: C = op(A) op(B) (+C), fp32-accurate on
+// the 5th-generation tensor cores via split-TF32 ("3xTF32"):
+//     x = hi + lo,  hi = x with the low 13 mantissa bits cleared (exactly tf32),
+//                   lo = tf32(x - hi) (x - hi is exact in fp32);
+//     A B ~= A_lo B_hi + A_hi B_lo + A_hi B_hi  (the dropped A_lo B_lo is ~2^-22 relative).
+// The paper's GEMMs are cuBLAS sgemm calls inside TF ops; there is no
+// fp32-input tcgen05 MMA, and plain TF32 (~1e-3 relative) would miss the 1e-4 parity bar
+// of BASELINE.json north_star, hence the split.
+//
+// Kernel (one 128 x BN output tile per CTA, optional deterministic split-K):
+//   warps 0-3 : producers for A (LDG from global with bounds -> split -> st.shared into
+//               the canonical K-major SWIZZLE_128B layout), then the epilogue
+//               (tcgen05.ld TMEM -> registers -> global)
+//   warps 4-7 : producers for B
+//   warp  8   : TMEM allocation + a single elected thread issuing tcgen05.mma.kind::tf32
+//               (M=128, N=BN, K=8), 3 MMAs per k-step, tcgen05.commit -> mbarriers.
+// The producers transpose on the fly, so every operand (N/T) lands in one K-major layout.
+// A STAGES-deep mbarrier ring (full / empty) overlaps loads with MMAs.
+//
+// Batch-1 inference GEMMs (M <= 8) are HBM-bound weight streaming and
+// go to a split-K GEMV kernel instead of padding M to 128.
+#include <algorithm>
+#include <atomic>
+
+#include "sf_device.cuh"
+#include "sf_kernels.h"
+
+namespace sfk {
+namespace {
+
+constexpr int BM = 128;
+constexpr int BK = 32;  // fp32 elements = 128 B = one SWIZZLE_128B row
+constexpr int kProducerWarps = 8;
+constexpr int kMmaWarp = 8;
+constexpr int kThreads = 9 * 32;
+
+template <int BN>
+struct Cfg {
+  static constexpr int STAGES = BN == 64 ? 4 : 3;
+  static constexpr int A_BYTES = BM * BK * 4;
+  static constexpr int B_BYTES = BN * BK * 4;
+  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = BN;
+  static constexpr uint32_t IDESC = (1u << 4)                       // D = f32
+                                    | (2u << 7) | (2u << 10)        // A, B = tf32
+                                    | (0u << 15) | (0u << 16)       // both K-major
+                                    | (uint32_t(BN >> 3) << 17)     // N
+                                    | (uint32_t(BM >> 4) << 24);    // M
+};
+
+struct Params {
+  const float* A; const float* B; float* C;
+  int M, N, K, lda, ldb, ldc;
+  int acc, vec_a, vec_b, vec_c;
+  int splits, kb_per_split;
+  float* ws; unsigned* counters;
+};
+
+// Canonical K-major SWIZZLE_128B UMMA smem descriptor (8-row groups 1024 B apart).
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
+  return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (static_cast<uint64_t>(1) << 16) |
+         (static_cast<uint64_t>(1024 >> 4) << 32) | (static_cast<uint64_t>(1) << 46) |
+         (static_cast<uint64_t>(2) << 61);
+}
+
+__device__ __forceinline__ void split_tf32(float x, float& hi, float& lo) {
+  hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+  lo = __uint_as_float(__float_as_uint(x - hi) & 0xFFFFE000u);
+}
+
+// Element (r, 4c..4c+3) of a K-major SW128 tile: row r at (r/8)*1024 + (r%8)*128, 16-B
+// chunk c stored at chunk position c ^ (r % 8).
+__device__ __forceinline__ void store_split(uint8_t* hi, uint8_t* lo, int r, int c, float4 v) {
+  const uint32_t off = (r >> 3) * 1024 + (r & 7) * 128 + ((c ^ (r & 7)) << 4);
+  float4 h, l;
+  split_tf32(v.x, h.x, l.x);
+  split_tf32(v.y, h.y, l.y);
+  split_tf32(v.z, h.z, l.z);
+  split_tf32(v.w, h.w, l.w);
+  *reinterpret_cast<float4*>(hi + off) = h;
+  *reinterpret_cast<float4*>(lo + off) = l;
+}
+
+// Operand stored contiguous along K: element (r, k) at src[(row0 + r) * ld + k].
+template <int ROWS>
+__device__ __forceinline__ void produce_kc(uint8_t* hi, uint8_t* lo, const float* __restrict__ src,
+                                           int ld, int nrows, int K, int row0, int k0, int t,
+                                           bool vec) {
+  constexpr int PER = ROWS * 8 / 128;
+  float4 v[PER];
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    const int idx = i * 128 + t, r = idx >> 3, c = idx & 7;
+    const int gr = row0 + r, gk = k0 + c * 4;
+    v[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (gr < nrows) {
+      const float* p = src + static_cast<size_t>(gr) * ld + gk;
+      if (vec && gk + 3 < K) {
+        v[i] = __ldg(reinterpret_cast<const float4*>(p));
+      } else {
+        if (gk < K) v[i].x = __ldg(p);
+        if (gk + 1 < K) v[i].y = __ldg(p + 1);
+        if (gk + 2 < K) v[i].z = __ldg(p + 2);
+        if (gk + 3 < K) v[i].w = __ldg(p + 3);
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    const int idx = i * 128 + t;
+    store_split(hi, lo, idx >> 3, idx & 7, v[i]);
+  }
+}
+
+// Operand stored contiguous along rows (M or N): element (r, k) at src[(k0 + k) * ld + row0 + r].
+// Lanes take consecutive rows (coalesced 128-B loads) and each gathers 4 k's per chunk.
+template <int ROWS>
+__device__ __forceinline__ void produce_mn(uint8_t* hi, uint8_t* lo, const float* __restrict__ src,
+                                           int ld, int nrows, int K, int row0, int k0, int t) {
+  constexpr int PER = ROWS * 8 / 128;
+  float4 v[PER];
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    const int idx = i * 128 + t, r = idx % ROWS, c = idx / ROWS;
+    const int gr = row0 + r;
+    float e[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int gk = k0 + 4 * c + j;
+      e[j] = (gr < nrows && gk < K) ? __ldg(src + static_cast<size_t>(gk) * ld + gr) : 0.f;
+    }
+    v[i] = make_float4(e[0], e[1], e[2], e[3]);
+  }
+#pragma unroll
+  for (int i = 0; i < PER; ++i) {
+    const int idx = i * 128 + t;
+    store_split(hi, lo, idx % ROWS, idx / ROWS, v[i]);
+  }
+}
+
+__device__ __forceinline__ void epi_barrier() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+template <int BN, bool A_KC, bool B_KC>
+__global__ void __launch_bounds__(kThreads, 1) gemm_tf32x3_kernel(Params p) {
+  using C = Cfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* done = empty + C::STAGES;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(done + 1);
+  int* last_flag = reinterpret_cast<int*>(tmem_slot + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM, z = blockIdx.z;
+  const int nkb_total = (p.K + BK - 1) / BK;
+  const int kb_begin = z * p.kb_per_split;
+  const int nkb = max(0, min(nkb_total, kb_begin + p.kb_per_split) - kb_begin);
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < C::STAGES; ++s) {
+      sfdev::mbar_init(&full[s], kProducerWarps);
+      sfdev::mbar_init(&empty[s], 1);
+    }
+    sfdev::mbar_init(done, 1);
+    sfdev::mbar_fence_init();
+  }
+  if (warp == kMmaWarp) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
+  sfdev::tc_fence_before();
+  __syncthreads();
+  sfdev::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp < kProducerWarps) {
+    const bool is_a = warp < 4;
+    const int t = threadIdx.x & 127;
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % C::STAGES, round = i / C::STAGES;
+      if (round > 0) sfdev::mbar_wait(&empty[s], (round - 1) & 1);
+      uint8_t* st = smem + s * C::STAGE_BYTES;
+      const int k0 = (kb_begin + i) * BK;
+      if (is_a) {
+        if constexpr (A_KC) produce_kc<BM>(st, st + C::A_BYTES, p.A, p.lda, p.M, p.K, m0, k0, t, p.vec_a);
+        else produce_mn<BM>(st, st + C::A_BYTES, p.A, p.lda, p.M, p.K, m0, k0, t);
+      } else {
+        uint8_t* bh = st + 2 * C::A_BYTES;
+        if constexpr (B_KC) produce_kc<BN>(bh, bh + C::B_BYTES, p.B, p.ldb, p.N, p.K, n0, k0, t, p.vec_b);
+        else produce_mn<BN>(bh, bh + C::B_BYTES, p.B, p.ldb, p.N, p.K, n0, k0, t);
+      }
+      sfdev::fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) sfdev::mbar_arrive(&full[s]);
+    }
+  } else {
+    // MMA issuer: one elected thread.
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % C::STAGES;
+      sfdev::mbar_wait(&full[s], (i / C::STAGES) & 1);
+      sfdev::tc_fence_after();
+      if (lane == 0) {
+        const uint32_t base = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
+        const uint32_t a_hi = base, a_lo = base + C::A_BYTES;
+        const uint32_t b_hi = base + 2 * C::A_BYTES, b_lo = b_hi + C::B_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < BK / 8; ++kk) {
+          const uint32_t off = kk * 32;
+          sfdev::mma_tf32(tmem, sw128_desc(a_lo + off), sw128_desc(b_hi + off), C::IDESC,
+                          (i | kk) != 0);
+          sfdev::mma_tf32(tmem, sw128_desc(a_hi + off), sw128_desc(b_lo + off), C::IDESC, 1u);
+          sfdev::mma_tf32(tmem, sw128_desc(a_hi + off), sw128_desc(b_hi + off), C::IDESC, 1u);
+        }
+        sfdev::mma_commit(&empty[s]);
+      }
+      __syncwarp();
+    }
+    if (lane == 0) sfdev::mma_commit(done);
+    __syncwarp();
+  }
+
+  if (warp < 4) {
+    sfdev::mbar_wait(done, 0);
+    sfdev::tc_fence_after();
+    const int row = m0 + warp * 32 + lane;
+    float* out_base;
+    int ld_out;
+    bool add_old, vec_out;
+    if (p.splits == 1) {
+      out_base = p.C; ld_out = p.ldc; add_old = p.acc != 0; vec_out = p.vec_c != 0;
+    } else {
+      out_base = p.ws + static_cast<size_t>(z) * p.M * p.N; ld_out = p.N; add_old = false;
+      vec_out = (p.N & 3) == 0;
+    }
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 32) {
+      uint32_t r[32];
+      sfdev::tmem_ld32(tmem + (static_cast<uint32_t>(warp * 32) << 16) + c0, r);
+      sfdev::tmem_ld_wait();
+      const int col = n0 + c0;
+      if (nkb == 0) {
+#pragma unroll
+        for (int j = 0; j < 32; ++j) r[j] = 0u;
+      }
+      if (row < p.M && col < p.N) {
+        float* o = out_base + static_cast<size_t>(row) * ld_out + col;
+        const int nvalid = min(32, p.N - col);
+        if (vec_out && nvalid == 32) {
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            float4 v = make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]),
+                                   __uint_as_float(r[4 * q + 2]), __uint_as_float(r[4 * q + 3]));
+            if (add_old) {
+              const float4 old = *reinterpret_cast<const float4*>(o + 4 * q);
+              v.x += old.x; v.y += old.y; v.z += old.z; v.w += old.w;
+            }
+            *reinterpret_cast<float4*>(o + 4 * q) = v;
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            if (j < nvalid) {
+              float v = __uint_as_float(r[j]);
+              if (add_old) v += o[j];
+              o[j] = v;
+            }
+          }
+        }
+      }
+    }
+    if (p.splits > 1) {
+      // Deterministic split-K: the last CTA of this tile sums the partials in order z=0..S-1.
+      __threadfence();
+      epi_barrier();
+      const unsigned tile = blockIdx.y * gridDim.x + blockIdx.x;
+      if (threadIdx.x == 0) {
+        const unsigned prev = atomicAdd(&p.counters[tile], 1u);
+        *last_flag = (prev == static_cast<unsigned>(p.splits - 1));
+      }
+      epi_barrier();
+      if (*last_flag) {
+        __threadfence();
+        const int rows = min(BM, p.M - m0), cols = min(BN, p.N - n0);
+        for (int e = threadIdx.x; e < rows * cols; e += 128) {
+          const int rr = m0 + e / cols, cc = n0 + e % cols;
+          float s = 0.f;
+          for (int zz = 0; zz < p.splits; ++zz)
+            s += __ldcg(p.ws + (static_cast<size_t>(zz) * p.M + rr) * p.N + cc);
+          float* o = p.C + static_cast<size_t>(rr) * p.ldc + cc;
+          if (p.acc) s += *o;
+          *o = s;
+        }
+        if (threadIdx.x == 0) p.counters[tile] = 0u;
+      }
+    }
+  }
+  sfdev::tc_fence_before();
+  __syncthreads();
+  sfdev::tc_fence_after();
+  if (warp == kMmaWarp) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
+}
+
+struct Plan {
+  int bn, splits, kb_per_split, tiles_n, tiles_m;
+};
+
+Plan plan_gemm(int M, int N, int K) {
+  Plan pl;
+  pl.bn = N <= 64 ? 64 : 128;
+  pl.tiles_n = (N + pl.bn - 1) / pl.bn;
+  pl.tiles_m = (M + BM - 1) / BM;
+  const int tiles = pl.tiles_n * pl.tiles_m;
+  const int nkb = std::max(1, (K + BK - 1) / BK);
+  int splits = 1;
+  if (tiles < 148) {
+    splits = (148 + tiles - 1) / tiles;
+    splits = std::min(splits, std::max(1, nkb / 4));
+    splits = std::min(splits, 64);
+  }
+  pl.kb_per_split = (nkb + splits - 1) / splits;
+  pl.splits = (nkb + pl.kb_per_split - 1) / pl.kb_per_split;
+  return pl;
+}
+
+template <int BN, bool AK, bool BKc>
+cudaError_t launch_t(const Params& p, dim3 grid, cudaStream_t st) {
+  auto kern = gemm_tf32x3_kernel<BN, AK, BKc>;
+  static std::atomic<uint64_t> configured{0};  // per instantiation, bit per device
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (!(configured.load() & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg<BN>::SMEM);
+    if (e != cudaSuccess) return e;
+    configured.fetch_or(bit);
+  }
+  kern<<<grid, kThreads, Cfg<BN>::SMEM, st>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// ---- batch-1 GEMV (M <= 8, op(A) = A, op(B) = B) --------------------------------------
+template <int MR>
+__global__ void __launch_bounds__(256)
+gemv_kernel(const float* __restrict__ A, const float* __restrict__ B, float* __restrict__ C,
+            int M, int N, int K, int lda, int ldb, int ldc, int acc, int kper, int splits,
+            float* ws, unsigned* counters) {
+  const int n = blockIdx.x * 256 + threadIdx.x;
+  const int z = blockIdx.y;
+  const int k0 = z * kper, k1 = min(K, k0 + kper);
+  float a[MR];
+#pragma unroll
+  for (int m = 0; m < MR; ++m) a[m] = 0.f;
+  if (n < N) {
+    int k = k0;
+    for (; k + 8 <= k1; k += 8) {
+      float b[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) b[u] = __ldg(B + static_cast<size_t>(k + u) * ldb + n);
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+#pragma unroll
+        for (int m = 0; m < MR; ++m)
+          if (m < M) a[m] = fmaf(__ldg(A + static_cast<size_t>(m) * lda + k + u), b[u], a[m]);
+    }
+    for (; k < k1; ++k) {
+      const float b = __ldg(B + static_cast<size_t>(k) * ldb + n);
+#pragma unroll
+      for (int m = 0; m < MR; ++m)
+        if (m < M) a[m] = fmaf(__ldg(A + static_cast<size_t>(m) * lda + k), b, a[m]);
+    }
+  }
+  if (splits == 1) {
+    if (n < N)
+#pragma unroll
+      for (int m = 0; m < MR; ++m)
+        if (m < M) {
+          float* o = C + static_cast<size_t>(m) * ldc + n;
+          *o = acc ? *o + a[m] : a[m];
+        }
+    return;
+  }
+  if (n < N)
+#pragma unroll
+    for (int m = 0; m < MR; ++m)
+      if (m < M) ws[(static_cast<size_t>(z) * M + m) * N + n] = a[m];
+  __threadfence();
+  __syncthreads();
+  __shared__ int last;
+  if (threadIdx.x == 0) last = atomicAdd(&counters[blockIdx.x], 1u) == static_cast<unsigned>(splits - 1);
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  if (n < N)
+    for (int m = 0; m < M; ++m) {
+      float s = 0.f;
+      for (int zz = 0; zz < splits; ++zz) s += __ldcg(ws + (static_cast<size_t>(zz) * M + m) * N + n);
+      float* o = C + static_cast<size_t>(m) * ldc + n;
+      *o = acc ? *o + s : s;
+    }
+  if (threadIdx.x == 0) counters[blockIdx.x] = 0u;
+}
+
+struct GemvPlan { int splits, kper, cols_blocks; };
+GemvPlan plan_gemv(int N, int K) {
+  GemvPlan g;
+  g.cols_blocks = (N + 255) / 256;
+  int splits = std::max(1, (2 * 148 + g.cols_blocks - 1) / g.cols_blocks);
+  splits = std::min(splits, std::max(1, (K + 63) / 64));
+  g.kper = ((K + splits - 1) / splits + 7) / 8 * 8;
+  g.splits = (K + g.kper - 1) / g.kper;
+  return g;
+}
+
+bool use_gemv(int M, bool ta, bool tb) { return M <= 8 && !ta && !tb; }
+
+}  // namespace
+
+uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb) {
+  if (use_gemv(M, ta, tb)) {
+    GemvPlan g = plan_gemv(N, K);
+    return g.splits > 1 ? static_cast<uint64_t>(g.splits) * M * N : 0;
+  }
+  Plan pl = plan_gemm(M, N, K);
+  return pl.splits > 1 ? static_cast<uint64_t>(pl.splits) * M * N : 0;
+}
+
+uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
+  if (use_gemv(M, ta, tb)) return static_cast<uint64_t>(plan_gemv(N, K).cols_blocks);
+  Plan pl = plan_gemm(M, N, K);
+  return static_cast<uint64_t>(pl.tiles_m) * pl.tiles_n;
+}
+
+cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
+  if (a.M <= 0 || a.N <= 0) return cudaSuccess;
+  if (use_gemv(a.M, a.ta, a.tb)) {
+    GemvPlan g = plan_gemv(a.N, a.K);
+    if (g.splits > 1 && (!a.ws || !a.counters)) return cudaErrorInvalidValue;
+    dim3 grid(g.cols_blocks, g.splits);
+#define SF_GEMV(MR)                                                                          \
+  gemv_kernel<MR><<<grid, 256, 0, st>>>(a.A, a.B, a.C, a.M, a.N, a.K, a.lda, a.ldb, a.ldc,   \
+                                        a.acc ? 1 : 0, g.kper, g.splits, a.ws, a.counters)
+    if (a.M == 1) SF_GEMV(1);
+    else if (a.M == 2) SF_GEMV(2);
+    else if (a.M <= 4) SF_GEMV(4);
+    else SF_GEMV(8);
+#undef SF_GEMV
+    count_launch();
+    return cudaGetLastError();
+  }
+  Plan pl = plan_gemm(a.M, a.N, a.K);
+  if (pl.splits > 1 && (!a.ws || !a.counters)) return cudaErrorInvalidValue;
+  Params p;
+  p.A = a.A; p.B = a.B; p.C = a.C;
+  p.M = a.M; p.N = a.N; p.K = a.K; p.lda = a.lda; p.ldb = a.ldb; p.ldc = a.ldc;
+  p.acc = a.acc ? 1 : 0;
+  const bool a_kc = !a.ta, b_kc = a.tb;
+  p.vec_a = a_kc && (a.lda % 4 == 0) && (reinterpret_cast<uintptr_t>(a.A) % 16 == 0);
+  p.vec_b = b_kc && (a.ldb % 4 == 0) && (reinterpret_cast<uintptr_t>(a.B) % 16 == 0);
+  p.vec_c = (a.ldc % 4 == 0) && (reinterpret_cast<uintptr_t>(a.C) % 16 == 0);
+  p.splits = pl.splits; p.kb_per_split = pl.kb_per_split;
+  p.ws = a.ws; p.counters = a.counters;
+  dim3 grid(pl.tiles_n, pl.tiles_m, pl.splits);
+  if (pl.bn == 64) {
+    if (a_kc && b_kc) return launch_t<64, true, true>(p, grid, st);
+    if (a_kc) return launch_t<64, true, false>(p, grid, st);
+    if (b_kc) return launch_t<64, false, true>(p, grid, st);
+    return launch_t<64, false, false>(p, grid, st);
+  }
+  if (a_kc && b_kc) return launch_t<128, true, true>(p, grid, st);
+  if (a_kc) return launch_t<128, true, false>(p, grid, st);
+  if (b_kc) return launch_t<128, false, true>(p, grid, st);
+  return launch_t<128, false, false>(p, grid, st);
+}
+
+}  // namespace sfk

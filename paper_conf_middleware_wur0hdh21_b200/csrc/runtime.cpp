@@ -1,0 +1,1649 @@
+// SwitchFlow-on-B200 runtime: graph registry, partitioner, live-set analysis, per-device
+// versions (CUDA graphs), preemption scheduler and migration engine behind include/sf.h.
+//
+// Paper mapping (PAPER.md = /root/reference/PAPER.md):
+//  * graph / session partition into subgraphs ........ PAPER.md:279-291, 323-325 (s.2, 2.1)
+//  * one executor version per device ................... PAPER.md:635-637, 665-667 (s.3.2)
+//  * session order preserved, executors interleave ..... PAPER.md:669-673 (s.3.2)
+//  * task suspension: dispatched kernels finish ........ PAPER.md:699-704 (s.3.3)
+//  * graph reconstruction onto GPU2 / CPU .............. PAPER.md:705-716 (s.3.3)
+//  * context saving + async state transfer ............. PAPER.md:734-761 (s.3.3)
+//  * resumption, no work lost .......................... PAPER.md:750-754 (s.3.3)
+//  * invariant 1: no co-running GPU executors .......... PAPER.md:794-806 (s.3.4)
+//  * preempter starts immediately after submission ..... PAPER.md:808-814 (s.3.4)
+//  * atomic-flag executor sync, 1-LOC priority ......... PAPER.md:904-909, 920-923 (s.4)
+// B200 choices are described in DESIGN.md: cut at subgraph boundaries with in-flight
+// activations (reading Q1), one multi-tensor pack / unpack / peer-store launch per cut,
+// stream-ordered resume of a pre-instantiated CUDA graph on the target.
+#include <cuda_runtime.h>
+#include <time.h>
+
+#include <algorithm>
+#include <atomic>
+#include <condition_variable>
+#include <cstring>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "sf.h"
+#include "sf_kernels.h"
+
+namespace {
+
+thread_local std::string g_err;
+
+sf_status fail(sf_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+#define SF_CK(call)                                                                  \
+  do {                                                                               \
+    cudaError_t e_ = (call);                                                         \
+    if (e_ != cudaSuccess)                                                           \
+      return fail(SF_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_));    \
+  } while (0)
+
+uint64_t now_ns() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return static_cast<uint64_t>(ts.tv_sec) * 1000000000ull + static_cast<uint64_t>(ts.tv_nsec);
+}
+
+constexpr uint64_t kAlign = 256;
+uint64_t round_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+bool persistent(int kind) { return kind == SF_PARAM || kind == SF_SLOT || kind == SF_SCALAR_STATE; }
+bool optimizer_op(int t) { return t == SF_OP_SGD_MOM || t == SF_OP_ADAM || t == SF_OP_STEP_INC; }
+
+struct Tensor {
+  int rows, cols, dtype, kind;
+  uint64_t nbytes, offset;
+};
+
+// Per-device copy list uploaded to device memory (DCopy[n + 1], last = sentinel).
+struct CopyList {
+  sfk::DCopy* d = nullptr;
+  int n = 0;
+  uint64_t total_chunks = 0;
+  uint64_t bytes = 0;  // live bytes moved
+};
+
+struct Binding {
+  int slot = -1;
+  uint8_t* arena = nullptr;
+  uint8_t* staging = nullptr;
+  uint8_t* host_staging = nullptr;      // pinned host (host pointer)
+  uint8_t* host_staging_dev = nullptr;  // its device mapping
+  std::vector<cudaGraphExec_t> versions;
+  float* ws = nullptr;
+  unsigned* counters = nullptr;
+  std::vector<CopyList> pack, unpack, pack_zc, unpack_zc;
+  std::map<int, std::vector<CopyList>> peer;  // target slot -> per cut
+  std::vector<std::pair<uint64_t, uint64_t>> poison_ranges;  // non-DATASET arena ranges
+  std::vector<void*> dev_allocs;
+};
+
+struct Graph {
+  std::string name;
+  int priority = 0;
+  std::vector<Tensor> T;
+  std::vector<sf_op_desc> ops;
+  bool partitioned = false;
+  std::vector<std::pair<int, int>> parts;
+  std::vector<std::vector<uint32_t>> live;
+  std::vector<uint64_t> live_bytes, staging_total, payload_start;
+  std::vector<std::vector<uint64_t>> payload_off;
+  std::vector<std::vector<uint8_t>> header;  // per cut: bytes [0, payload_start)
+  uint64_t arena_bytes = 0, staging_bytes = 0, persistent_bytes = 0, max_live = 0;
+  uint64_t ws_floats = 0, counter_slots = 0;
+  std::vector<std::unique_ptr<Binding>> bind;  // per slot
+  int input_tid = -1, output_tid = -1;
+};
+
+constexpr int kInferOwner = 1 << 20;
+
+struct Request {
+  sf_req_id id;
+  Graph* g;
+  int dev;
+  const void* in;
+  void* out;
+  uint64_t arrival, start = 0, end = 0;
+  bool done = false;
+  int preempted_job = -1;
+  int64_t cut_iter = -1;
+  int cut_k = -1;
+  std::string error;
+};
+
+struct Slot {
+  int id, cuda;
+  cudaStream_t s_train = nullptr, s_infer = nullptr, s_mig = nullptr;
+  cudaEvent_t ev_infer = nullptr;
+  int owner = -1;
+  std::deque<Request*> q;
+  std::thread dispatcher;
+  uint64_t persistent_bound = 0;
+};
+
+struct Job {
+  sf_job_id id;
+  Graph* g;
+  int dev;
+  int64_t iters;
+  int auto_target;
+  int64_t it = 0;
+  int k = 0;
+  int state = SF_JOB_RUNNING;
+  bool preempt_req = false, preempt_park = false;
+  std::vector<sf_cut_request> sched;
+  size_t sched_pos = 0;
+  int preempt_target = 0;
+  uint64_t t_req = 0;
+  bool cut_ready = false;
+  bool mig_enqueued = false;
+  bool holds_token = false;
+  sf_cut_info cut{};
+  bool resume_req = false;
+  int resume_dev = -1;
+  bool stop_req = false;
+  bool stamp_resume = false;
+  int n_preempt = 0;
+  uint64_t migrated = 0;
+  double pack_us = 0, xfer_us = 0, unpack_us = 0;
+  uint64_t last_stop = 0, last_resume = 0;
+  std::string error;
+  std::thread driver;
+  std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c;  // per slot
+};
+
+}  // namespace
+
+struct sf_runtime {
+  sf_config cfg{};
+  std::vector<std::unique_ptr<Slot>> slots;
+  std::vector<std::unique_ptr<Graph>> graphs;
+  std::vector<std::unique_ptr<Job>> jobs;
+  std::unordered_map<sf_req_id, std::unique_ptr<Request>> reqs;
+  sf_req_id next_req = 1;
+  std::mutex m;
+  std::condition_variable cv;
+  bool shutting_down = false;
+  std::vector<sf_trace_event> trace;
+  size_t trace_cap = 1 << 16;
+  size_t trace_dropped = 0;
+};
+
+namespace {
+
+void push_trace(sf_runtime* rt, const sf_trace_event& e) {  // rt->m held
+  if (rt->trace.size() < rt->trace_cap) rt->trace.push_back(e);
+  else ++rt->trace_dropped;
+}
+
+// ---------------------------------------------------------------------------------------
+// Graph validation (mirrors the oracle's rules, written independently from the paper).
+// ---------------------------------------------------------------------------------------
+sf_status validate(const Graph& g) {
+  const int n = static_cast<int>(g.T.size());
+  auto chk = [&](bool c, sf_status s, const std::string& msg) -> sf_status {
+    return c ? SF_OK : fail(s, msg);
+  };
+  for (size_t j = 0; j < g.ops.size(); ++j) {
+    const sf_op_desc& o = g.ops[j];
+    const std::string at = "op " + std::to_string(j) + ": ";
+    if (o.type < SF_OP_GEMM || o.type > SF_OP_STEP_INC)
+      return fail(SF_EUNSUPPORTED, at + "op type outside the fixed op set");
+    if (o.n_in < 0 || o.n_in > 6 || o.n_out < 0 || o.n_out > 3) return fail(SF_EINVAL, at + "arity");
+    for (int i = 0; i < o.n_in; ++i)
+      if (o.in[i] < 0 || o.in[i] >= n) return fail(SF_EINVAL, at + "input id out of range");
+    for (int i = 0; i < o.n_out; ++i) {
+      if (o.out[i] < 0 || o.out[i] >= n) return fail(SF_EINVAL, at + "output id out of range");
+      const Tensor& t = g.T[o.out[i]];
+      if (t.kind == SF_DATASET) return fail(SF_EINVAL, at + "writes a DATASET tensor");
+      if (persistent(t.kind) && !optimizer_op(o.type))
+        return fail(SF_EINVAL, at + "only optimizer ops write persistent state");
+    }
+    auto T = [&](int id) -> const Tensor& { return g.T[id]; };
+    sf_status s = SF_OK;
+    switch (o.type) {
+      case SF_OP_GEMM: {
+        if ((s = chk(o.n_in == 2 && o.n_out == 1, SF_EINVAL, at + "gemm arity"))) return s;
+        const Tensor &A = T(o.in[0]), &B = T(o.in[1]), &C = T(o.out[0]);
+        const int M = (o.flags & SF_GEMM_TA) ? A.cols : A.rows;
+        const int K = (o.flags & SF_GEMM_TA) ? A.rows : A.cols;
+        const int K2 = (o.flags & SF_GEMM_TB) ? B.cols : B.rows;
+        const int N = (o.flags & SF_GEMM_TB) ? B.rows : B.cols;
+        if ((s = chk(K == K2 && C.rows == M && C.cols == N && K > 0, SF_EINVAL, at + "gemm shapes"))) return s;
+        if ((s = chk(A.dtype == SF_F32 && B.dtype == SF_F32 && C.dtype == SF_F32, SF_EUNSUPPORTED,
+                     at + "gemm dtype")))
+          return s;
+        break;
+      }
+      case SF_OP_BIAS_ACT: {
+        if ((s = chk(o.n_in >= 2 && o.n_in <= 4 && o.n_out == 1, SF_EINVAL, at + "bias_act arity"))) return s;
+        const Tensor &z = T(o.in[0]), &h = T(o.out[0]);
+        if ((s = chk(z.rows == h.rows && z.cols == h.cols, SF_EINVAL, at + "bias_act shape"))) return s;
+        for (int i = 1; i < o.n_in; ++i)
+          if ((s = chk(T(o.in[i]).rows == 1 && T(o.in[i]).cols == z.cols, SF_EINVAL, at + "bias shape")))
+            return s;
+        break;
+      }
+      case SF_OP_BIAS_ACT_BWD: {
+        if ((s = chk(o.n_in == 2 && o.n_out == 2, SF_EINVAL, at + "bias_act_bwd arity"))) return s;
+        const Tensor &dh = T(o.in[0]), &h = T(o.in[1]), &dz = T(o.out[0]), &db = T(o.out[1]);
+        if ((s = chk(dh.rows == h.rows && dh.cols == h.cols && dz.rows == h.rows && dz.cols == h.cols &&
+                         db.rows == 1 && db.cols == h.cols,
+                     SF_EINVAL, at + "bias_act_bwd shapes")))
+          return s;
+        break;
+      }
+      case SF_OP_COLSUM: {
+        if ((s = chk(o.n_in == 1 && o.n_out == 1 && T(o.out[0]).rows == 1 &&
+                         T(o.out[0]).cols == T(o.in[0]).cols,
+                     SF_EINVAL, at + "colsum")))
+          return s;
+        break;
+      }
+      case SF_OP_SOFTMAX_CE: {
+        if ((s = chk(o.n_in == 2 && o.n_out == 2, SF_EINVAL, at + "softmax_ce arity"))) return s;
+        const Tensor &l = T(o.in[0]), &y = T(o.in[1]), &loss = T(o.out[0]), &d = T(o.out[1]);
+        if ((s = chk(y.dtype == SF_I32 && y.rows == l.rows && y.cols == 1 && loss.rows == 1 &&
+                         loss.cols == 1 && d.rows == l.rows && d.cols == l.cols,
+                     SF_EINVAL, at + "softmax_ce shapes")))
+          return s;
+        break;
+      }
+      case SF_OP_SOFTMAX: {
+        if ((s = chk(o.n_in == 1 && o.n_out == 1 && T(o.in[0]).rows == T(o.out[0]).rows &&
+                         T(o.in[0]).cols == T(o.out[0]).cols,
+                     SF_EINVAL, at + "softmax")))
+          return s;
+        break;
+      }
+      case SF_OP_SGD_MOM: {
+        if ((s = chk(o.n_in == 1 && o.n_out == 2, SF_EINVAL, at + "sgd arity"))) return s;
+        const Tensor &gr = T(o.in[0]), &w = T(o.out[0]), &a = T(o.out[1]);
+        if ((s = chk(gr.rows == w.rows && gr.cols == w.cols && a.rows == w.rows && a.cols == w.cols,
+                     SF_EINVAL, at + "sgd shapes")))
+          return s;
+        break;
+      }
+      case SF_OP_ADAM: {
+        if ((s = chk(o.n_in == 2 && o.n_out == 3, SF_EINVAL, at + "adam arity"))) return s;
+        const Tensor &gr = T(o.in[0]), &st = T(o.in[1]);
+        for (int i = 0; i < 3; ++i)
+          if ((s = chk(T(o.out[i]).rows == gr.rows && T(o.out[i]).cols == gr.cols, SF_EINVAL,
+                       at + "adam shapes")))
+            return s;
+        if ((s = chk(st.dtype == SF_I32 && st.rows * st.cols == 1, SF_EINVAL, at + "adam step"))) return s;
+        break;
+      }
+      case SF_OP_FEED: {
+        if ((s = chk(o.n_in == 2 && o.n_out == 1, SF_EINVAL, at + "feed arity"))) return s;
+        const Tensor &pool = T(o.in[0]), &st = T(o.in[1]), &x = T(o.out[0]);
+        if ((s = chk(pool.kind == SF_DATASET && pool.cols == x.cols && x.rows > 0 &&
+                         pool.rows % x.rows == 0 && pool.dtype == x.dtype && st.dtype == SF_I32,
+                     SF_EINVAL, at + "feed shapes")))
+          return s;
+        break;
+      }
+      case SF_OP_STEP_INC: {
+        if ((s = chk(o.n_out == 1 && T(o.out[0]).dtype == SF_I32, SF_EINVAL, at + "step_inc"))) return s;
+        break;
+      }
+    }
+  }
+  // read-before-write within an iteration
+  std::vector<char> written(n, 0), has_writer(n, 0);
+  for (const auto& o : g.ops)
+    for (int i = 0; i < o.n_out; ++i) has_writer[o.out[i]] = 1;
+  for (size_t j = 0; j < g.ops.size(); ++j) {
+    const sf_op_desc& o = g.ops[j];
+    std::vector<int> reads(o.in, o.in + o.n_in);
+    if (o.type == SF_OP_GEMM && (o.flags & SF_GEMM_ACC)) reads.push_back(o.out[0]);
+    if (optimizer_op(o.type)) reads.insert(reads.end(), o.out, o.out + o.n_out);
+    for (int t : reads) {
+      const int k = g.T[t].kind;
+      if (persistent(k) || k == SF_DATASET || written[t]) continue;
+      if ((k == SF_INPUT || k == SF_LABEL) && !has_writer[t]) continue;
+      return fail(SF_EINVAL, "op " + std::to_string(j) + ": reads tensor " + std::to_string(t) +
+                                 " before it is written");
+    }
+    for (int i = 0; i < o.n_out; ++i) written[o.out[i]] = 1;
+  }
+  return SF_OK;
+}
+
+std::vector<int> op_reads(const sf_op_desc& o) {
+  std::vector<int> r(o.in, o.in + o.n_in);
+  if (o.type == SF_OP_GEMM && (o.flags & SF_GEMM_ACC)) r.push_back(o.out[0]);
+  if (optimizer_op(o.type)) r.insert(r.end(), o.out, o.out + o.n_out);
+  return r;
+}
+
+// Live set at cut k: persistent state, plus every tensor written
+// before S_k that an op at/after S_k reads before overwriting it, plus OUTPUT tensors
+// already produced (fetched at iteration end).  Externally fed INPUT/LABEL count as
+// written at the start of S_0.
+std::vector<uint32_t> compute_live(const Graph& g, int k) {
+  const int start = g.parts[k].first;
+  const int nT = static_cast<int>(g.T.size()), nO = static_cast<int>(g.ops.size());
+  std::vector<char> written_before(nT, 0), has_writer(nT, 0);
+  for (int j = 0; j < nO; ++j)
+    for (int i = 0; i < g.ops[j].n_out; ++i) {
+      has_writer[g.ops[j].out[i]] = 1;
+      if (j < start) written_before[g.ops[j].out[i]] = 1;
+    }
+  // first access at/after start: +1 read first, -1 write first, 0 none
+  std::vector<int> first(nT, 0);
+  for (int j = start; j < nO; ++j) {
+    const sf_op_desc& o = g.ops[j];
+    for (int t : op_reads(o))
+      if (first[t] == 0) first[t] = 1;
+    for (int i = 0; i < o.n_out; ++i)
+      if (first[o.out[i]] == 0) first[o.out[i]] = -1;
+  }
+  std::vector<uint32_t> live;
+  for (int t = 0; t < nT; ++t) {
+    const Tensor& x = g.T[t];
+    if (persistent(x.kind)) { live.push_back(t); continue; }
+    if (x.kind == SF_DATASET) continue;
+    const bool fed_ext = (x.kind == SF_INPUT || x.kind == SF_LABEL) && !has_writer[t];
+    const bool wb = written_before[t] || (fed_ext && start > 0);
+    if (!wb) continue;
+    if (x.kind == SF_OUTPUT || first[t] == 1) live.push_back(t);
+  }
+  return live;
+}
+
+sf_status do_partition(Graph& g, const sf_partition_opts& o) {
+  g.parts.clear();
+  std::vector<std::pair<int, int>> runs;
+  int s = 0;
+  const int nO = static_cast<int>(g.ops.size());
+  for (int j = 1; j <= nO; ++j)
+    if (j == nO || g.ops[j].phase != g.ops[s].phase) {
+      runs.emplace_back(s, j);
+      s = j;
+    }
+  if (o.policy == SF_PART_PER_LAYER_PHASE) {
+    g.parts = runs;
+  } else if (o.policy == SF_PART_MAX_OPS && o.max_ops > 0) {
+    for (auto [a, b] : runs) {
+      bool opt = false;
+      for (int j = a; j < b; ++j) opt |= optimizer_op(g.ops[j].type);
+      if (opt) { g.parts.emplace_back(a, b); continue; }
+      for (int c = a; c < b; c += o.max_ops) g.parts.emplace_back(c, std::min(b, c + o.max_ops));
+    }
+  } else {
+    return fail(SF_EINVAL, "unknown partition policy");
+  }
+  // arena layout: every tensor at a 256-B aligned offset, ascending id
+  uint64_t off = 0;
+  g.persistent_bytes = 0;
+  for (auto& t : g.T) {
+    t.offset = off;
+    off += round_up(std::max<uint64_t>(t.nbytes, 1), kAlign);
+    if (persistent(t.kind)) g.persistent_bytes += t.nbytes;
+  }
+  g.arena_bytes = off;
+  const int n = static_cast<int>(g.parts.size());
+  g.live.assign(n, {});
+  g.live_bytes.assign(n, 0);
+  g.staging_total.assign(n, 0);
+  g.payload_start.assign(n, 0);
+  g.payload_off.assign(n, {});
+  g.header.assign(n, {});
+  g.staging_bytes = 0;
+  g.max_live = 0;
+  for (int k = 0; k < n; ++k) {
+    g.live[k] = compute_live(g, k);
+    const auto& L = g.live[k];
+    // staging format: 32-B header, 24-B entries, payloads at 256-B offsets
+    const uint64_t ps = round_up(32 + 24 * static_cast<uint64_t>(L.size()), kAlign);
+    uint64_t p = ps, bytes = 0;
+    std::vector<uint64_t> offs;
+    for (uint32_t t : L) {
+      offs.push_back(p);
+      p += round_up(g.T[t].nbytes, kAlign);
+      bytes += g.T[t].nbytes;
+    }
+    std::vector<uint8_t> h(ps, 0);
+    auto put32 = [&](size_t at, uint32_t v) { std::memcpy(&h[at], &v, 4); };
+    auto put64 = [&](size_t at, uint64_t v) { std::memcpy(&h[at], &v, 8); };
+    std::memcpy(&h[0], "SFST", 4);
+    put32(4, 1);
+    put32(8, static_cast<uint32_t>(L.size()));
+    put32(12, static_cast<uint32_t>(k));
+    put64(16, 0);  // iter, patched by the pack kernel
+    put64(24, p);
+    for (size_t e = 0; e < L.size(); ++e) {
+      put32(32 + 24 * e, L[e]);
+      put32(36 + 24 * e, static_cast<uint32_t>(g.T[L[e]].dtype));
+      put64(40 + 24 * e, offs[e]);
+      put64(48 + 24 * e, g.T[L[e]].nbytes);
+    }
+    g.header[k] = std::move(h);
+    g.payload_start[k] = ps;
+    g.payload_off[k] = std::move(offs);
+    g.staging_total[k] = p;
+    g.live_bytes[k] = bytes;
+    g.staging_bytes = std::max(g.staging_bytes, p);
+    g.max_live = std::max(g.max_live, bytes);
+  }
+  // workspace: max over ops (ops of one subgraph run sequentially on one stream)
+  g.ws_floats = 0;
+  g.counter_slots = 1;
+  for (const auto& op : g.ops) {
+    if (op.type == SF_OP_GEMM) {
+      const Tensor &A = g.T[op.in[0]], &B = g.T[op.in[1]];
+      const bool ta = op.flags & SF_GEMM_TA, tb = op.flags & SF_GEMM_TB;
+      const int M = ta ? A.cols : A.rows, K = ta ? A.rows : A.cols, N = tb ? B.rows : B.cols;
+      g.ws_floats = std::max(g.ws_floats, sfk::gemm_workspace_floats(M, N, K, ta, tb));
+      g.counter_slots = std::max(g.counter_slots, sfk::gemm_counter_slots(M, N, K, ta, tb));
+    } else if (op.type == SF_OP_BIAS_ACT_BWD || op.type == SF_OP_COLSUM) {
+      const Tensor& x = g.T[op.in[0]];
+      g.ws_floats = std::max(g.ws_floats, sfk::colsum_ws_floats(x.rows, x.cols));
+      g.counter_slots = std::max(g.counter_slots, sfk::colsum_counter_slots(x.rows, x.cols));
+    } else if (op.type == SF_OP_SOFTMAX_CE) {
+      g.ws_floats = std::max(g.ws_floats, sfk::softmax_ce_ws_floats(g.T[op.in[0]].rows));
+    }
+  }
+  g.partitioned = true;
+  return SF_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// Version build: launch the ops of subgraph k for one binding (captured into a CUDA graph).
+// ---------------------------------------------------------------------------------------
+struct Capture {
+  Graph& g;
+  Binding& b;
+  cudaStream_t st;
+  bool dry;                          // prepare pass: upload descriptor arrays, launch nothing
+  std::map<int, void*>* prepared;    // first op index of an optimizer group -> device array
+  uint8_t* ptr(int t) const { return b.arena + g.T[t].offset; }
+  float* f(int t) const { return reinterpret_cast<float*>(ptr(t)); }
+};
+
+sf_status upload(Binding& b, const void* host, size_t bytes, void** out) {
+  void* d = nullptr;
+  SF_CK(cudaMalloc(&d, std::max<size_t>(bytes, 16)));
+  SF_CK(cudaMemcpy(d, host, bytes, cudaMemcpyHostToDevice));
+  b.dev_allocs.push_back(d);
+  *out = d;
+  return SF_OK;
+}
+
+sf_status launch_subgraph_ops(Capture& c, int k) {
+  Graph& g = c.g;
+  const auto [a, e] = g.parts[k];
+  int j = a;
+  while (j < e) {
+    const sf_op_desc& o = g.ops[j];
+    cudaError_t err = cudaSuccess;
+    if (o.type == SF_OP_SGD_MOM) {
+      const int first = j;
+      std::vector<sfk::SgdDesc> ds;
+      uint64_t q = 0;
+      while (j < e && g.ops[j].type == SF_OP_SGD_MOM) {
+        const sf_op_desc& s = g.ops[j];
+        sfk::SgdDesc d{c.f(s.out[0]), c.f(s.out[1]), c.f(s.in[0]),
+                       static_cast<uint64_t>(g.T[s.out[0]].rows) * g.T[s.out[0]].cols, s.f[0], s.f[1], q};
+        q += (d.n + 3) / 4;
+        ds.push_back(d);
+        ++j;
+      }
+      sfk::SgdDesc sent{};
+      sent.begin = q;
+      ds.push_back(sent);
+      void* dd;
+      if (c.dry) {
+        if (sf_status s = upload(c.b, ds.data(), ds.size() * sizeof(sfk::SgdDesc), &dd)) return s;
+        (*c.prepared)[first] = dd;
+        continue;
+      }
+      dd = (*c.prepared)[first];
+      err = sfk::launch_sgd(static_cast<sfk::SgdDesc*>(dd), static_cast<int>(ds.size()) - 1, q, c.st);
+      if (err != cudaSuccess) return fail(SF_ECUDA, std::string("sgd: ") + cudaGetErrorString(err));
+      continue;
+    }
+    if (o.type == SF_OP_ADAM) {
+      const int first = j;
+      std::vector<sfk::AdamDesc> ds;
+      uint64_t q = 0;
+      const int step_t = o.in[1];
+      while (j < e && g.ops[j].type == SF_OP_ADAM && g.ops[j].in[1] == step_t) {
+        const sf_op_desc& s = g.ops[j];
+        sfk::AdamDesc d{c.f(s.out[0]), c.f(s.out[1]), c.f(s.out[2]), c.f(s.in[0]),
+                        static_cast<uint64_t>(g.T[s.out[0]].rows) * g.T[s.out[0]].cols,
+                        s.f[0], s.f[1], s.f[2], s.f[3], q};
+        q += (d.n + 3) / 4;
+        ds.push_back(d);
+        ++j;
+      }
+      sfk::AdamDesc sent{};
+      sent.begin = q;
+      ds.push_back(sent);
+      void* dd;
+      if (c.dry) {
+        if (sf_status s = upload(c.b, ds.data(), ds.size() * sizeof(sfk::AdamDesc), &dd)) return s;
+        (*c.prepared)[first] = dd;
+        continue;
+      }
+      dd = (*c.prepared)[first];
+      err = sfk::launch_adam(static_cast<sfk::AdamDesc*>(dd), static_cast<int>(ds.size()) - 1, q,
+                             reinterpret_cast<const int32_t*>(c.ptr(step_t)), c.st);
+      if (err != cudaSuccess) return fail(SF_ECUDA, std::string("adam: ") + cudaGetErrorString(err));
+      continue;
+    }
+    if (c.dry) {
+      ++j;
+      continue;
+    }
+    switch (o.type) {
+      case SF_OP_GEMM: {
+        const Tensor &A = g.T[o.in[0]], &B = g.T[o.in[1]], &C = g.T[o.out[0]];
+        sfk::GemmArgs ga;
+        ga.A = c.f(o.in[0]); ga.B = c.f(o.in[1]); ga.C = c.f(o.out[0]);
+        ga.ta = o.flags & SF_GEMM_TA; ga.tb = o.flags & SF_GEMM_TB; ga.acc = o.flags & SF_GEMM_ACC;
+        ga.M = C.rows; ga.N = C.cols; ga.K = ga.ta ? A.rows : A.cols;
+        ga.lda = A.cols; ga.ldb = B.cols; ga.ldc = C.cols;
+        ga.ws = c.b.ws; ga.counters = c.b.counters;
+        err = sfk::launch_gemm(ga, c.st);
+        break;
+      }
+      case SF_OP_BIAS_ACT: {
+        const Tensor& z = g.T[o.in[0]];
+        err = sfk::launch_bias_act(c.f(o.in[0]), c.f(o.in[1]), o.n_in > 2 ? c.f(o.in[2]) : nullptr,
+                                   o.n_in > 3 ? c.f(o.in[3]) : nullptr, c.f(o.out[0]), z.rows, z.cols,
+                                   o.flags & SF_ACT_RELU, c.st);
+        break;
+      }
+      case SF_OP_BIAS_ACT_BWD: {
+        const Tensor& x = g.T[o.in[0]];
+        err = sfk::launch_colsum(c.f(o.in[0]), c.f(o.in[1]), c.f(o.out[0]), c.f(o.out[1]), x.rows,
+                                 x.cols, c.b.ws, c.b.counters, c.st);
+        break;
+      }
+      case SF_OP_COLSUM: {
+        const Tensor& x = g.T[o.in[0]];
+        err = sfk::launch_colsum(c.f(o.in[0]), nullptr, nullptr, c.f(o.out[0]), x.rows, x.cols,
+                                 c.b.ws, c.b.counters, c.st);
+        break;
+      }
+      case SF_OP_SOFTMAX_CE: {
+        const Tensor& l = g.T[o.in[0]];
+        err = sfk::launch_softmax_ce(c.f(o.in[0]), reinterpret_cast<const int32_t*>(c.ptr(o.in[1])),
+                                     c.f(o.out[0]), c.f(o.out[1]), l.rows, l.cols, c.b.ws,
+                                     c.b.counters, c.st);
+        break;
+      }
+      case SF_OP_SOFTMAX: {
+        const Tensor& l = g.T[o.in[0]];
+        err = sfk::launch_softmax(c.f(o.in[0]), c.f(o.out[0]), l.rows, l.cols, c.st);
+        break;
+      }
+      case SF_OP_FEED: {
+        const Tensor &pool = g.T[o.in[0]], &x = g.T[o.out[0]];
+        err = sfk::launch_feed(c.ptr(o.in[0]), reinterpret_cast<const int32_t*>(c.ptr(o.in[1])),
+                               c.ptr(o.out[0]), x.nbytes, pool.rows / x.rows, c.st);
+        break;
+      }
+      case SF_OP_STEP_INC:
+        err = sfk::launch_step_inc(reinterpret_cast<int32_t*>(c.ptr(o.out[0])), c.st);
+        break;
+      default:
+        return fail(SF_EUNSUPPORTED, "op type");
+    }
+    if (err != cudaSuccess)
+      return fail(SF_ECUDA, "op " + std::to_string(j) + ": " + cudaGetErrorString(err));
+    ++j;
+  }
+  return SF_OK;
+}
+
+sf_status build_copy_list(Binding& b, const std::vector<sf_copy_desc>& descs, CopyList* out) {
+  std::vector<sfk::DCopy> d;
+  uint64_t chunks = 0, bytes = 0;
+  for (const auto& s : descs) {
+    sfk::DCopy x;
+    x.src = static_cast<const uint8_t*>(s.src);
+    x.dst = static_cast<uint8_t*>(s.dst);
+    x.nbytes = s.nbytes;
+    x.chunk_begin = chunks;
+    chunks += s.span / 16;
+    bytes += s.nbytes;
+    d.push_back(x);
+  }
+  sfk::DCopy sent{};
+  sent.chunk_begin = chunks;
+  d.push_back(sent);
+  void* dd;
+  if (sf_status s = upload(b, d.data(), d.size() * sizeof(sfk::DCopy), &dd)) return s;
+  out->d = static_cast<sfk::DCopy*>(dd);
+  out->n = static_cast<int>(descs.size());
+  out->total_chunks = chunks;
+  out->bytes = bytes;
+  return SF_OK;
+}
+
+sf_status build_peer_lists(sf_runtime* rt, Graph& g, Binding& src, Binding& dst) {
+  SF_CK(cudaSetDevice(rt->slots[src.slot]->cuda));
+  std::vector<CopyList> lists(g.parts.size());
+  for (size_t k = 0; k < g.parts.size(); ++k) {
+    std::vector<sf_copy_desc> ds;
+    for (uint32_t t : g.live[k]) {
+      const Tensor& x = g.T[t];
+      ds.push_back({src.arena + x.offset, dst.arena + x.offset, x.nbytes, round_up(x.nbytes, 16)});
+    }
+    if (sf_status s = build_copy_list(src, ds, &lists[k])) return s;
+  }
+  src.peer[dst.slot] = std::move(lists);
+  return SF_OK;
+}
+
+// ---------------------------------------------------------------------------------------
+// Scheduler
+// ---------------------------------------------------------------------------------------
+Slot& slot_of(sf_runtime* rt, int s) { return *rt->slots[s]; }
+
+sf_status ensure_events(sf_runtime* rt, Job& J) {
+  if (!J.ev_sub.empty()) return SF_OK;
+  const size_t n = rt->slots.size();
+  J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  for (size_t s = 0; s < n; ++s) {
+    SF_CK(cudaSetDevice(rt->slots[s]->cuda));
+    SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
+    SF_CK(cudaEventCreate(&J.ev_a[s]));
+    SF_CK(cudaEventCreate(&J.ev_b[s]));
+    SF_CK(cudaEventCreate(&J.ev_c[s]));
+  }
+  SF_CK(cudaSetDevice(cur));
+  return SF_OK;
+}
+
+cudaError_t spin_event(cudaEvent_t ev) {
+  for (;;) {
+    cudaError_t e = cudaEventQuery(ev);
+    if (e != cudaErrorNotReady) return e;
+  }
+}
+
+float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) return 0.f;
+  return ms * 1000.f;
+}
+
+bool slot_has_inference(sf_runtime* rt, int s) { return !slot_of(rt, s).q.empty(); }
+
+// Poison the non-DATASET tensors of a released arena (test mode): a missing live tensor
+// then reads as NaN / -1 after resume.
+cudaError_t poison(Binding& b, cudaStream_t st) {
+  for (auto [off, len] : b.poison_ranges) {
+    cudaError_t e = sfk::launch_fill(b.arena + off, len, 0xFF, st);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+// Preempt J at its current boundary (rt->m held on entry and on return).
+sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
+  Graph& g = *J.g;
+  const bool expl = J.preempt_park;  // explicit sf_preempt: park until sf_resume
+  const int target = J.preempt_target;
+  const int src = J.dev;
+  const int k = J.k;
+  J.preempt_req = false;
+  J.state = SF_JOB_MIGRATING;
+  J.last_stop = now_ns();
+  J.cut = sf_cut_info{};
+  J.cut.iter = J.it;
+  J.cut.k = k;
+  J.cut.n_tensors = static_cast<int32_t>(g.live[k].size());
+  J.cut.live_bytes = g.live_bytes[k];
+  J.cut.t_req_ns = J.t_req;
+  J.cut.t_stop_ns = J.last_stop;
+  J.cut.src_dev = src;
+  J.cut.dst_dev = target;
+  J.cut_ready = true;
+  J.mig_enqueued = false;
+  for (Request* r : slot_of(rt, src).q)
+    if (r->preempted_job < 0) {
+      r->preempted_job = static_cast<int>(J.id);
+      r->cut_iter = J.it;
+      r->cut_k = k;
+    }
+  rt->cv.notify_all();
+  Slot& S = slot_of(rt, src);
+  Binding& B = *g.bind[src];
+  lk.unlock();
+
+  auto cuda_fail = [&](cudaError_t e, const char* what) {
+    lk.lock();
+    J.error = std::string(what) + ": " + cudaGetErrorString(e);
+    J.state = SF_JOB_FAILED;
+    rt->cv.notify_all();
+    return fail(SF_ECUDA, J.error);
+  };
+  cudaError_t e;
+  if (target == SF_TARGET_HOST) {
+    // ---- host tier: pack (+ D2H), park, swap back in ------------------------------
+    if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+    const bool zc = rt->cfg.host_mode == SF_HOST_ZC || B.staging == nullptr;
+    cudaEventRecord(J.ev_a[src], S.s_mig);
+    if (zc) {
+      const CopyList& L = B.pack_zc[k];
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig);
+      cudaEventRecord(J.ev_b[src], S.s_mig);
+    } else {
+      const CopyList& L = B.pack[k];
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig);
+      cudaEventRecord(J.ev_b[src], S.s_mig);
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(B.host_staging, B.staging, g.staging_total[k], cudaMemcpyDeviceToHost, S.s_mig);
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "pack");
+    cudaEventRecord(J.ev_c[src], S.s_mig);
+    lk.lock();
+    J.mig_enqueued = true;
+    rt->cv.notify_all();
+    lk.unlock();
+    if ((e = spin_event(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
+    const float pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
+    const float d2h_us = elapsed_us(J.ev_b[src], J.ev_c[src]);
+    if (rt->cfg.poison_released) {
+      if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
+      if ((e = cudaStreamSynchronize(S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison sync");
+    }
+    lk.lock();
+    J.pack_us = pack_us;
+    J.xfer_us = d2h_us;
+    int dst = src;
+    if (expl) {
+      J.state = SF_JOB_PREEMPTED;
+      rt->cv.notify_all();
+      rt->cv.wait(lk, [&] { return J.resume_req || J.stop_req || rt->shutting_down; });
+      if (!J.resume_req) { J.state = SF_JOB_DONE; rt->cv.notify_all(); return SF_OK; }
+      dst = J.resume_dev;
+      J.resume_req = false;
+    } else {
+      // swap back in once the device's inference queue drained (reading Q4/Q13)
+      rt->cv.wait(lk, [&] {
+        return rt->shutting_down || (!slot_has_inference(rt, src) && S.owner != kInferOwner);
+      });
+    }
+    Slot& D = slot_of(rt, dst);
+    Binding& BD = *g.bind[dst];
+    lk.unlock();
+    if ((e = cudaSetDevice(D.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+    cudaEventRecord(J.ev_a[dst], D.s_train);
+    // the parked bytes live in the source binding's pinned staging; a ZC swap-in reads
+    // them in place when resuming on the same slot, otherwise H2D + unpack
+    if (zc && dst == src) {
+      const CopyList& L = BD.unpack_zc[k];
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train);
+      cudaEventRecord(J.ev_b[dst], D.s_train);
+    } else if (!BD.staging) {
+      e = cudaErrorInvalidValue;
+    } else {
+      e = cudaMemcpyAsync(BD.staging, B.host_staging, g.staging_total[k], cudaMemcpyHostToDevice,
+                          D.s_train);
+      cudaEventRecord(J.ev_b[dst], D.s_train);
+      if (e == cudaSuccess) {
+        const CopyList& L = BD.unpack[k];
+        e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train);
+      }
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "unpack");
+    cudaEventRecord(J.ev_c[dst], D.s_train);
+    lk.lock();
+    J.dev = dst;
+  } else {
+    // ---- peer tier: fused peer store into the target's arena over NVLink -----------
+    if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+    auto it = B.peer.find(target);
+    if (it == B.peer.end()) {
+      lk.lock();
+      J.state = SF_JOB_FAILED;
+      J.error = "no peer list to target slot";
+      rt->cv.notify_all();
+      return fail(SF_EINVAL, J.error);
+    }
+    const CopyList& L = it->second[k];
+    cudaEventRecord(J.ev_a[src], S.s_mig);
+    e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S.s_mig);
+    if (e != cudaSuccess) return cuda_fail(e, "peer store");
+    cudaEventRecord(J.ev_b[src], S.s_mig);
+    Slot& T = slot_of(rt, target);
+    // stream-ordered resume: the target's training stream waits on the source's copy
+    // (a cross-device event wait when the slots are different GPUs)
+    e = cudaStreamWaitEvent(T.s_train, J.ev_b[src], 0);
+    if (e != cudaSuccess) return cuda_fail(e, "stream wait");
+    if (rt->cfg.poison_released) {
+      if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
+    }
+    lk.lock();
+    J.mig_enqueued = true;
+    J.dev = target;
+    if (expl) {
+      J.state = SF_JOB_PREEMPTED;
+      rt->cv.notify_all();
+      rt->cv.wait(lk, [&] { return J.resume_req || J.stop_req || rt->shutting_down; });
+      if (!J.resume_req) { J.state = SF_JOB_DONE; rt->cv.notify_all(); return SF_OK; }
+      J.resume_req = false;
+    }
+  }
+  J.n_preempt++;
+  J.migrated += g.live_bytes[k];
+  J.state = SF_JOB_RUNNING;
+  J.stamp_resume = true;
+  rt->cv.notify_all();
+  return SF_OK;
+}
+
+void driver_main(sf_runtime* rt, Job* Jp) {
+  Job& J = *Jp;
+  Graph& g = *J.g;
+  const int n = static_cast<int>(g.parts.size());
+  std::unique_lock<std::mutex> lk(rt->m);
+  bool pending_peer_stats = false;
+  int stats_slot = -1;
+  auto release = [&] {
+    if (J.holds_token) {
+      Slot& S = slot_of(rt, J.dev);
+      if (S.owner == static_cast<int>(J.id)) S.owner = -1;
+      J.holds_token = false;
+      rt->cv.notify_all();
+    }
+  };
+  while (true) {
+    if (J.state == SF_JOB_FAILED) break;
+    if (J.it >= J.iters || (J.stop_req && J.k == 0) || rt->shutting_down) {
+      release();
+      J.state = SF_JOB_DONE;
+      rt->cv.notify_all();
+      break;
+    }
+    // boundary gate: preempt here if asked to (explicitly, or because a
+    // request is queued on this device and auto-preemption is on)
+    const bool at_cut_ok = !rt->cfg.iteration_granularity || J.k == 0;
+    if (!J.preempt_req && J.sched_pos < J.sched.size() && J.sched[J.sched_pos].iter == J.it &&
+        J.sched[J.sched_pos].k == J.k) {
+      J.preempt_req = J.sched[J.sched_pos].target != J.dev;  // a move to itself is a no-op
+      J.preempt_park = false;
+      J.preempt_target = J.sched[J.sched_pos].target;
+      J.t_req = now_ns();
+      ++J.sched_pos;
+    }
+    const bool has_inf = slot_has_inference(rt, J.dev);
+    const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu && has_inf &&
+                           J.auto_target != J.dev;
+    if (J.preempt_req || (auto_want && at_cut_ok)) {
+      release();
+      if (!J.preempt_req) {
+        J.preempt_park = false;
+        J.preempt_target = J.auto_target;
+        J.t_req = slot_of(rt, J.dev).q.front()->arrival;
+      }
+      const int src = J.dev;
+      const bool peer = J.preempt_target != SF_TARGET_HOST;
+      if (do_preempt(rt, J, lk) != SF_OK) break;
+      if (J.state == SF_JOB_DONE) break;
+      if (peer) { pending_peer_stats = true; stats_slot = src; }
+      continue;
+    }
+    Slot& S = slot_of(rt, J.dev);
+    if (rt->cfg.exclusive_gpu && !J.holds_token) {
+      // invariant 1: wait until no other model owns the device; with no
+      // preemption possible here, yield to queued inference at this boundary
+      const bool yield_to_inf = has_inf && !(auto_want && !at_cut_ok);
+      if (S.owner != -1 || yield_to_inf) {
+        rt->cv.wait(lk);
+        continue;
+      }
+      S.owner = static_cast<int>(J.id);
+      J.holds_token = true;
+    }
+    const int dev = J.dev, k = J.k;
+    const int64_t it = J.it;
+    cudaGraphExec_t ver = g.bind[dev]->versions[k];
+    const bool stamp = J.stamp_resume;
+    J.stamp_resume = false;
+    const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
+    lk.unlock();
+    cudaSetDevice(S.cuda);
+    cudaError_t e = cudaGraphLaunch(ver, S.s_train);
+    if (e == cudaSuccess) e = cudaEventRecord(J.ev_sub[dev], S.s_train);
+    if (e == cudaSuccess) e = spin_event(J.ev_sub[dev]);
+    const uint64_t t1 = now_ns();
+    float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
+    if (e == cudaSuccess && stamp) {
+      if (pending_peer_stats) {
+        peer_us = elapsed_us(J.ev_a[stats_slot], J.ev_b[stats_slot]);
+        pending_peer_stats = false;
+      } else {
+        h2d_us = elapsed_us(J.ev_a[dev], J.ev_b[dev]);
+        unpack_us = elapsed_us(J.ev_b[dev], J.ev_c[dev]);
+      }
+    }
+    lk.lock();
+    if (stamp) {
+      J.last_resume = t0;
+      if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += h2d_us; }
+      if (peer_us >= 0.f) { J.pack_us = 0.0; J.xfer_us = peer_us; J.unpack_us = 0.0; }
+    }
+    if (e != cudaSuccess) {
+      release();
+      J.error = std::string("subgraph launch: ") + cudaGetErrorString(e);
+      J.state = SF_JOB_FAILED;
+      rt->cv.notify_all();
+      break;
+    }
+    sf_trace_event ev{};
+    ev.dev = dev; ev.job = static_cast<int32_t>(J.id); ev.kind = SF_EV_TRAIN; ev.k = k; ev.iter = it;
+    ev.t0_ns = t0; ev.t1_ns = t1;
+    push_trace(rt, ev);
+    if (++J.k == n) { J.k = 0; ++J.it; }
+    // iteration-granularity (session time slicing baseline) keeps the device for the whole
+    // iteration; otherwise every subgraph boundary is a scheduling point
+    if (!rt->cfg.iteration_granularity || J.k == 0) release();
+    rt->cv.notify_all();
+  }
+}
+
+void dispatcher_main(sf_runtime* rt, Slot* S) {
+  cudaSetDevice(S->cuda);
+  std::unique_lock<std::mutex> lk(rt->m);
+  while (true) {
+    rt->cv.wait(lk, [&] {
+      return rt->shutting_down ||
+             (!S->q.empty() && (!rt->cfg.exclusive_gpu || S->owner == -1 || S->owner == kInferOwner));
+    });
+    if (S->q.empty() && rt->shutting_down) break;
+    if (S->q.empty()) continue;
+    if (rt->cfg.exclusive_gpu) S->owner = kInferOwner;
+    Request* r = S->q.front();
+    Graph& g = *r->g;
+    Binding* B = g.bind[S->id].get();
+    const uint64_t t0 = now_ns();
+    lk.unlock();
+    cudaError_t e = cudaSuccess;
+    const Tensor& tin = g.T[g.input_tid];
+    const Tensor& tout = g.T[g.output_tid];
+    e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
+    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k)
+      e = cudaGraphLaunch(B->versions[k], S->s_infer);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
+    if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
+    if (e == cudaSuccess) e = spin_event(S->ev_infer);
+    const uint64_t t1 = now_ns();
+    lk.lock();
+    r->start = t0;
+    r->end = t1;
+    if (e != cudaSuccess) r->error = cudaGetErrorString(e);
+    r->done = true;
+    S->q.pop_front();
+    sf_trace_event ev{};
+    ev.dev = S->id; ev.job = static_cast<int32_t>(kInferOwner | (r->id & 0xFFFFF)); ev.kind = SF_EV_INFER;
+    ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
+    push_trace(rt, ev);
+    if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
+    rt->cv.notify_all();
+  }
+}
+
+Graph* get_graph(sf_runtime* rt, sf_graph_id g) {
+  return g < rt->graphs.size() ? rt->graphs[g].get() : nullptr;
+}
+Job* get_job(sf_runtime* rt, sf_job_id j) { return j < rt->jobs.size() ? rt->jobs[j].get() : nullptr; }
+
+}  // namespace
+
+// =========================================================================================
+// C ABI
+// =========================================================================================
+extern "C" {
+
+const char* sf_last_error(void) { return g_err.c_str(); }
+int32_t sf_abi_version(void) { return SF_ABI_VERSION; }
+uint64_t sf_now_ns(void) { return now_ns(); }
+uint64_t sf_kernel_launches(void) { return sfk::launches(); }
+
+sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
+  if (!cfg || !out || cfg->n_devices <= 0 || !cfg->cuda_ordinals) return fail(SF_EINVAL, "bad config");
+  int ndev = 0;
+  SF_CK(cudaGetDeviceCount(&ndev));
+  auto rt = std::make_unique<sf_runtime>();
+  rt->cfg = *cfg;
+  rt->cfg.cuda_ordinals = nullptr;
+  if (cfg->trace_capacity > 0) rt->trace_cap = static_cast<size_t>(cfg->trace_capacity);
+  rt->trace.reserve(std::min<size_t>(rt->trace_cap, 1 << 16));
+  for (int s = 0; s < cfg->n_devices; ++s) {
+    const int c = cfg->cuda_ordinals[s];
+    if (c < 0 || c >= ndev) return fail(SF_EINVAL, "cuda ordinal out of range");
+    auto S = std::make_unique<Slot>();
+    S->id = s;
+    S->cuda = c;
+    SF_CK(cudaSetDevice(c));
+    int lo = 0, hi = 0;
+    SF_CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    SF_CK(cudaStreamCreateWithFlags(&S->s_train, cudaStreamNonBlocking));
+    SF_CK(cudaStreamCreateWithPriority(&S->s_infer, cudaStreamNonBlocking, hi));
+    SF_CK(cudaStreamCreateWithFlags(&S->s_mig, cudaStreamNonBlocking));
+    SF_CK(cudaEventCreateWithFlags(&S->ev_infer, cudaEventDisableTiming));
+    rt->slots.push_back(std::move(S));
+  }
+  // peer access between distinct physical devices (NVLink / NVSwitch)
+  for (auto& a : rt->slots)
+    for (auto& b : rt->slots)
+      if (a->cuda != b->cuda) {
+        int can = 0;
+        SF_CK(cudaDeviceCanAccessPeer(&can, a->cuda, b->cuda));
+        if (!can) return fail(SF_EUNSUPPORTED, "no peer access between devices");
+        SF_CK(cudaSetDevice(a->cuda));
+        cudaError_t e = cudaDeviceEnablePeerAccess(b->cuda, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+          return fail(SF_ECUDA, std::string("enable peer access: ") + cudaGetErrorString(e));
+        cudaGetLastError();
+      }
+  sf_runtime* p = rt.release();
+  for (auto& S : p->slots) S->dispatcher = std::thread(dispatcher_main, p, S.get());
+  *out = p;
+  return SF_OK;
+}
+
+void sf_destroy(sf_runtime* rt) {
+  if (!rt) return;
+  {
+    std::unique_lock<std::mutex> lk(rt->m);
+    rt->cv.wait(lk, [&] {
+      for (auto& S : rt->slots)
+        if (!S->q.empty()) return false;
+      for (auto& J : rt->jobs)
+        if (J->state == SF_JOB_RUNNING || J->state == SF_JOB_STOPPING || J->state == SF_JOB_MIGRATING)
+          return false;
+      return true;
+    });
+    rt->shutting_down = true;
+    rt->cv.notify_all();
+  }
+  for (auto& J : rt->jobs)
+    if (J->driver.joinable()) J->driver.join();
+  for (auto& S : rt->slots)
+    if (S->dispatcher.joinable()) S->dispatcher.join();
+  for (auto& S : rt->slots) {
+    cudaSetDevice(S->cuda);
+    cudaDeviceSynchronize();
+  }
+  for (auto& G : rt->graphs)
+    for (auto& B : G->bind) {
+      if (!B) continue;
+      cudaSetDevice(rt->slots[B->slot]->cuda);
+      for (auto v : B->versions) cudaGraphExecDestroy(v);
+      for (void* d : B->dev_allocs) cudaFree(d);
+      if (B->ws) cudaFree(B->ws);
+      if (B->counters) cudaFree(B->counters);
+    }
+  for (auto& J : rt->jobs)
+    for (size_t s = 0; s < J->ev_sub.size(); ++s) {
+      cudaSetDevice(rt->slots[s]->cuda);
+      cudaEventDestroy(J->ev_sub[s]);
+      cudaEventDestroy(J->ev_a[s]);
+      cudaEventDestroy(J->ev_b[s]);
+      cudaEventDestroy(J->ev_c[s]);
+    }
+  for (auto& S : rt->slots) {
+    cudaSetDevice(S->cuda);
+    cudaStreamDestroy(S->s_train);
+    cudaStreamDestroy(S->s_infer);
+    cudaStreamDestroy(S->s_mig);
+    cudaEventDestroy(S->ev_infer);
+  }
+  delete rt;
+}
+
+sf_status sf_register_graph(sf_runtime* rt, const sf_graph_desc* gd, int32_t priority,
+                            sf_graph_id* out) {
+  if (!rt || !gd || !out || (gd->n_tensors && !gd->tensors) || (gd->n_ops && !gd->ops))
+    return fail(SF_EINVAL, "null argument");
+  auto g = std::make_unique<Graph>();
+  g->name = gd->name ? gd->name : "";
+  g->priority = priority;
+  for (uint32_t i = 0; i < gd->n_tensors; ++i) {
+    const sf_tensor_desc& t = gd->tensors[i];
+    if (t.rows <= 0 || t.cols <= 0) return fail(SF_EINVAL, "tensor " + std::to_string(i) + ": shape");
+    if (t.dtype != SF_F32 && t.dtype != SF_I32) return fail(SF_EUNSUPPORTED, "tensor dtype");
+    if (t.kind < SF_PARAM || t.kind > SF_OUTPUT) return fail(SF_EINVAL, "tensor kind");
+    g->T.push_back({t.rows, t.cols, t.dtype, t.kind, static_cast<uint64_t>(t.rows) * t.cols * 4, 0});
+  }
+  g->ops.assign(gd->ops, gd->ops + gd->n_ops);
+  if (g->ops.empty()) return fail(SF_EINVAL, "graph has no ops");
+  if (sf_status s = validate(*g)) return s;
+  for (size_t i = 0; i < g->T.size(); ++i) {
+    if (g->T[i].kind == SF_INPUT && g->input_tid < 0) g->input_tid = static_cast<int>(i);
+    if (g->T[i].kind == SF_OUTPUT && g->output_tid < 0) g->output_tid = static_cast<int>(i);
+  }
+  std::lock_guard<std::mutex> lk(rt->m);
+  g->bind.resize(rt->slots.size());
+  rt->graphs.push_back(std::move(g));
+  *out = static_cast<sf_graph_id>(rt->graphs.size() - 1);
+  return SF_OK;
+}
+
+sf_status sf_partition(sf_runtime* rt, sf_graph_id gid, const sf_partition_opts* o,
+                       sf_partition_info* out) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g) return fail(SF_EINVAL, "bad graph id");
+  if (g->partitioned) return fail(SF_ESTATE, "graph already partitioned");
+  sf_partition_opts def{SF_PART_PER_LAYER_PHASE, 0};
+  if (sf_status s = do_partition(*g, o ? *o : def)) return s;
+  if (out) {
+    out->n_subgraphs = static_cast<int32_t>(g->parts.size());
+    out->arena_bytes = g->arena_bytes;
+    out->staging_bytes = g->staging_bytes;
+    out->persistent_bytes = g->persistent_bytes;
+    out->max_live_bytes = g->max_live;
+  }
+  return SF_OK;
+}
+
+sf_status sf_subgraph_range(sf_runtime* rt, sf_graph_id gid, int32_t k, int32_t* b, int32_t* e) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned || k < 0 || k >= static_cast<int>(g->parts.size()))
+    return fail(SF_EINVAL, "bad graph / cut");
+  if (b) *b = g->parts[k].first;
+  if (e) *e = g->parts[k].second;
+  return SF_OK;
+}
+
+sf_status sf_live_set(sf_runtime* rt, sf_graph_id gid, int32_t k, uint32_t* ids, uint32_t cap,
+                      uint32_t* n, uint64_t* bytes) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned || k < 0 || k >= static_cast<int>(g->parts.size()))
+    return fail(SF_EINVAL, "bad graph / cut");
+  const auto& L = g->live[k];
+  if (n) *n = static_cast<uint32_t>(L.size());
+  if (bytes) *bytes = g->live_bytes[k];
+  if (ids) std::copy(L.begin(), L.begin() + std::min<size_t>(cap, L.size()), ids);
+  return SF_OK;
+}
+
+sf_status sf_tensor_offset(sf_runtime* rt, sf_graph_id gid, uint32_t t, uint64_t* off) {
+  if (!rt || !off) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned || t >= g->T.size()) return fail(SF_EINVAL, "bad graph / tensor");
+  *off = g->T[t].offset;
+  return SF_OK;
+}
+
+sf_status sf_staging_layout(sf_runtime* rt, sf_graph_id gid, int32_t k, uint64_t* total,
+                            uint64_t* offs, uint32_t cap) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned || k < 0 || k >= static_cast<int>(g->parts.size()))
+    return fail(SF_EINVAL, "bad graph / cut");
+  if (total) *total = g->staging_total[k];
+  if (offs)
+    std::copy(g->payload_off[k].begin(),
+              g->payload_off[k].begin() + std::min<size_t>(cap, g->payload_off[k].size()), offs);
+  return SF_OK;
+}
+
+sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, void* staging,
+                  void* host_staging) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* gp = get_graph(rt, gid);
+  if (!gp || !gp->partitioned) return fail(SF_ESTATE, "graph not partitioned");
+  Graph& g = *gp;
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size())) return fail(SF_EINVAL, "bad slot");
+  if (g.bind[dev]) return fail(SF_ESTATE, "slot already bound");
+  if (!arena || reinterpret_cast<uintptr_t>(arena) % kAlign)
+    return fail(SF_EINVAL, "arena must be a 256-B aligned device pointer");
+  if (staging && reinterpret_cast<uintptr_t>(staging) % kAlign)
+    return fail(SF_EINVAL, "staging must be 256-B aligned");
+  Slot& S = *rt->slots[dev];
+  if (rt->cfg.device_budget_bytes &&
+      S.persistent_bound + g.persistent_bytes > rt->cfg.device_budget_bytes)
+    return fail(SF_ENOMEM, "persistent state of the graphs sharing this device exceeds its budget");
+  SF_CK(cudaSetDevice(S.cuda));
+  auto b = std::make_unique<Binding>();
+  b->slot = dev;
+  b->arena = static_cast<uint8_t*>(arena);
+  b->staging = static_cast<uint8_t*>(staging);
+  b->host_staging = static_cast<uint8_t*>(host_staging);
+  if (host_staging) {
+    void* dp = nullptr;
+    SF_CK(cudaHostGetDevicePointer(&dp, host_staging, 0));
+    b->host_staging_dev = static_cast<uint8_t*>(dp);
+  }
+  SF_CK(cudaMalloc(&b->ws, std::max<uint64_t>(g.ws_floats, 4) * sizeof(float)));
+  SF_CK(cudaMalloc(&b->counters, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));
+  SF_CK(cudaMemset(b->counters, 0, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));
+  // versions: one CUDA graph per subgraph
+  cudaStream_t cap;
+  SF_CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+  std::map<int, void*> prepared;
+  {
+    Capture prep{g, *b, cap, true, &prepared};
+    for (size_t k = 0; k < g.parts.size(); ++k)
+      if (sf_status s = launch_subgraph_ops(prep, static_cast<int>(k))) { cudaStreamDestroy(cap); return s; }
+  }
+  for (size_t k = 0; k < g.parts.size(); ++k) {
+    SF_CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
+    Capture c{g, *b, cap, false, &prepared};
+    sf_status s = launch_subgraph_ops(c, static_cast<int>(k));
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(cap, &graph);
+    if (s != SF_OK) { if (graph) cudaGraphDestroy(graph); cudaStreamDestroy(cap); return s; }
+    if (e != cudaSuccess) { cudaStreamDestroy(cap); return fail(SF_ECUDA, std::string("capture: ") + cudaGetErrorString(e)); }
+    cudaGraphExec_t exec = nullptr;
+    e = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) { cudaStreamDestroy(cap); return fail(SF_ECUDA, std::string("instantiate: ") + cudaGetErrorString(e)); }
+    b->versions.push_back(exec);
+  }
+  cudaStreamDestroy(cap);
+  // copy lists per cut
+  const size_t n = g.parts.size();
+  b->pack.resize(n); b->unpack.resize(n); b->pack_zc.resize(n); b->unpack_zc.resize(n);
+  for (size_t k = 0; k < n; ++k) {
+    void* hdr_dev;
+    if (sf_status s = upload(*b, g.header[k].data(), g.header[k].size(), &hdr_dev)) return s;
+    for (int mode = 0; mode < 2; ++mode) {
+      uint8_t* stg = mode == 0 ? b->staging : b->host_staging_dev;
+      if (!stg) continue;
+      std::vector<sf_copy_desc> pk, up;
+      pk.push_back({hdr_dev, stg, g.payload_start[k], g.payload_start[k]});
+      for (size_t e = 0; e < g.live[k].size(); ++e) {
+        const Tensor& t = g.T[g.live[k][e]];
+        pk.push_back({b->arena + t.offset, stg + g.payload_off[k][e], t.nbytes, round_up(t.nbytes, kAlign)});
+        up.push_back({stg + g.payload_off[k][e], b->arena + t.offset, t.nbytes, round_up(t.nbytes, 16)});
+      }
+      if (sf_status s = build_copy_list(*b, pk, mode == 0 ? &b->pack[k] : &b->pack_zc[k])) return s;
+      if (sf_status s = build_copy_list(*b, up, mode == 0 ? &b->unpack[k] : &b->unpack_zc[k])) return s;
+    }
+  }
+  // poison ranges: maximal runs of non-DATASET tensors
+  for (size_t t = 0; t < g.T.size();) {
+    if (g.T[t].kind == SF_DATASET) { ++t; continue; }
+    const uint64_t a = g.T[t].offset;
+    size_t u = t;
+    while (u < g.T.size() && g.T[u].kind != SF_DATASET) ++u;
+    const uint64_t end = (u < g.T.size()) ? g.T[u].offset : g.arena_bytes;
+    b->poison_ranges.emplace_back(a, end - a);
+    t = u;
+  }
+  S.persistent_bound += g.persistent_bytes;
+  g.bind[dev] = std::move(b);
+  // peer lists with every other bound slot, both directions
+  for (size_t o = 0; o < g.bind.size(); ++o) {
+    if (static_cast<int>(o) == dev || !g.bind[o]) continue;
+    if (sf_status s = build_peer_lists(rt, g, *g.bind[dev], *g.bind[o])) return s;
+    if (sf_status s = build_peer_lists(rt, g, *g.bind[o], *g.bind[dev])) return s;
+  }
+  SF_CK(cudaSetDevice(S.cuda));
+  SF_CK(cudaDeviceSynchronize());
+  return SF_OK;
+}
+
+sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters,
+                            int32_t auto_target, const sf_cut_request* sched, int32_t n_sched,
+                            sf_job_id* out) {
+  if (!rt || !out || n_sched < 0 || (n_sched > 0 && !sched)) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned) return fail(SF_ESTATE, "graph not partitioned");
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev])
+    return fail(SF_EINVAL, "slot not bound");
+  if (auto_target != SF_TARGET_HOST &&
+      (auto_target < 0 || auto_target >= static_cast<int>(rt->slots.size()) || !g->bind[auto_target]))
+    return fail(SF_EINVAL, "auto_target not bound");
+  if (auto_target == SF_TARGET_HOST && !g->bind[dev]->host_staging)
+    return fail(SF_EINVAL, "host tier needs host_staging");
+  auto J = std::make_unique<Job>();
+  J->id = static_cast<sf_job_id>(rt->jobs.size());
+  J->g = g;
+  J->dev = dev;
+  J->iters = iters;
+  J->auto_target = auto_target;
+  for (int i = 0; i < n_sched; ++i) {
+    const sf_cut_request& c = sched[i];
+    if (c.k < 0 || c.k >= static_cast<int>(g->parts.size()) || c.iter < 0)
+      return fail(SF_EINVAL, "scheduled cut out of range");
+    if (i > 0 && (c.iter < sched[i - 1].iter || (c.iter == sched[i - 1].iter && c.k <= sched[i - 1].k)))
+      return fail(SF_EINVAL, "scheduled cuts must be strictly ascending");
+    if (c.target != SF_TARGET_HOST &&
+        (c.target < 0 || c.target >= static_cast<int>(rt->slots.size()) || !g->bind[c.target]))
+      return fail(SF_EINVAL, "scheduled target not bound");
+    J->sched.push_back(c);
+  }
+  if (sf_status s = ensure_events(rt, *J)) return s;
+  Job* jp = J.get();
+  rt->jobs.push_back(std::move(J));
+  jp->driver = std::thread(driver_main, rt, jp);
+  *out = jp->id;
+  return SF_OK;
+}
+
+sf_status sf_preempt(sf_runtime* rt, sf_job_id jid, int32_t target, sf_cut_info* out) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::unique_lock<std::mutex> lk(rt->m);
+  Job* J = get_job(rt, jid);
+  if (!J) return fail(SF_EINVAL, "bad job id");
+  if (J->state == SF_JOB_MIGRATING) return fail(SF_EBUSY, "migration in flight");
+  if (J->state != SF_JOB_RUNNING || J->preempt_req) return fail(SF_ESTATE, "job not running");
+  if (target == J->dev) return fail(SF_EINVAL, "target is the current device");
+  if (target == SF_TARGET_HOST) {
+    if (!J->g->bind[J->dev]->host_staging) return fail(SF_EINVAL, "no host staging bound");
+  } else if (target < 0 || target >= static_cast<int>(rt->slots.size()) || !J->g->bind[target]) {
+    return fail(SF_EINVAL, "target slot not bound");
+  }
+  J->cut_ready = false;
+  J->preempt_req = true;
+  J->preempt_park = true;
+  J->preempt_target = target;
+  J->t_req = now_ns();
+  rt->cv.notify_all();
+  rt->cv.wait(lk, [&] { return J->cut_ready || J->state == SF_JOB_DONE || J->state == SF_JOB_FAILED; });
+  if (!J->cut_ready) return fail(SF_ESTATE, "job finished before reaching a boundary: " + J->error);
+  rt->cv.wait(lk, [&] { return J->mig_enqueued || J->state == SF_JOB_FAILED; });
+  if (J->state == SF_JOB_FAILED) return fail(SF_ECUDA, J->error);
+  if (out) *out = J->cut;
+  return SF_OK;
+}
+
+sf_status sf_resume(sf_runtime* rt, sf_job_id jid, int32_t dev) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Job* J = get_job(rt, jid);
+  if (!J) return fail(SF_EINVAL, "bad job id");
+  if (J->state != SF_JOB_PREEMPTED) return fail(SF_ESTATE, "job not preempted");
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !J->g->bind[dev])
+    return fail(SF_EINVAL, "slot not bound");
+  if (J->cut.dst_dev != SF_TARGET_HOST && dev != J->cut.dst_dev)
+    return fail(SF_EINVAL, "peer-migrated job resumes on its migration target");
+  J->resume_req = true;
+  J->resume_dev = dev;
+  J->state = SF_JOB_RUNNING;  // visible to the caller at once; the driver continues
+  rt->cv.notify_all();
+  return SF_OK;
+}
+
+sf_status sf_job_query(sf_runtime* rt, sf_job_id jid, sf_job_info* out) {
+  if (!rt || !out) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Job* J = get_job(rt, jid);
+  if (!J) return fail(SF_EINVAL, "bad job id");
+  out->state = J->state;
+  out->dev = J->dev;
+  out->iter = J->it;
+  out->k = J->k;
+  out->n_preemptions = J->n_preempt;
+  out->migrated_bytes = J->migrated;
+  out->last_pack_us = J->pack_us;
+  out->last_xfer_us = J->xfer_us;
+  out->last_unpack_us = J->unpack_us;
+  out->last_stop_ns = J->last_stop;
+  out->last_resume_ns = J->last_resume;
+  if (J->state == SF_JOB_FAILED) return fail(SF_ECUDA, J->error);
+  return SF_OK;
+}
+
+sf_status sf_wait_job(sf_runtime* rt, sf_job_id jid, int64_t timeout_ns) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::unique_lock<std::mutex> lk(rt->m);
+  Job* J = get_job(rt, jid);
+  if (!J) return fail(SF_EINVAL, "bad job id");
+  auto done = [&] { return J->state == SF_JOB_DONE || J->state == SF_JOB_FAILED; };
+  if (timeout_ns < 0) rt->cv.wait(lk, done);
+  else if (!rt->cv.wait_for(lk, std::chrono::nanoseconds(timeout_ns), done))
+    return fail(SF_ETIMEOUT, "job still running");
+  if (J->state == SF_JOB_FAILED) return fail(SF_ECUDA, J->error);
+  return SF_OK;
+}
+
+sf_status sf_stop_job(sf_runtime* rt, sf_job_id jid) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Job* J = get_job(rt, jid);
+  if (!J) return fail(SF_EINVAL, "bad job id");
+  J->stop_req = true;
+  rt->cv.notify_all();
+  return SF_OK;
+}
+
+sf_status sf_submit_inference(sf_runtime* rt, sf_graph_id gid, int32_t dev, const void* in,
+                              void* out, uint64_t arrival_ns, sf_req_id* req) {
+  if (!rt || !in || !out || !req) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || !g->partitioned) return fail(SF_ESTATE, "graph not partitioned");
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev])
+    return fail(SF_EINVAL, "slot not bound");
+  if (g->input_tid < 0 || g->output_tid < 0) return fail(SF_EINVAL, "graph has no INPUT/OUTPUT");
+  auto r = std::make_unique<Request>();
+  r->id = rt->next_req++;
+  r->g = g;
+  r->dev = dev;
+  r->in = in;
+  r->out = out;
+  r->arrival = arrival_ns ? arrival_ns : now_ns();
+  Request* rp = r.get();
+  rt->reqs.emplace(r->id, std::move(r));
+  rt->slots[dev]->q.push_back(rp);
+  *req = rp->id;
+  rt->cv.notify_all();
+  return SF_OK;
+}
+
+sf_status sf_wait(sf_runtime* rt, sf_req_id id, int64_t timeout_ns, sf_timing* t) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::unique_lock<std::mutex> lk(rt->m);
+  auto it = rt->reqs.find(id);
+  if (it == rt->reqs.end()) return fail(SF_EINVAL, "unknown request");
+  Request* r = it->second.get();
+  auto done = [&] { return r->done; };
+  if (timeout_ns < 0) rt->cv.wait(lk, done);
+  else if (!rt->cv.wait_for(lk, std::chrono::nanoseconds(timeout_ns), done))
+    return fail(SF_ETIMEOUT, "request pending");
+  if (t) {
+    t->arrival_ns = r->arrival;
+    t->start_ns = r->start;
+    t->end_ns = r->end;
+    t->dev = r->dev;
+    t->preempted_job = r->preempted_job;
+    t->cut_iter = r->cut_iter;
+    t->cut_k = r->cut_k;
+  }
+  std::string err = r->error;
+  rt->reqs.erase(it);
+  if (!err.empty()) return fail(SF_ECUDA, err);
+  return SF_OK;
+}
+
+sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* n_out) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  const size_t n = std::min(cap, rt->trace.size());
+  if (buf) std::copy(rt->trace.begin(), rt->trace.begin() + n, buf);
+  if (n_out) *n_out = buf ? n : rt->trace.size();
+  return SF_OK;
+}
+
+// ---- direct kernel entry points --------------------------------------------------------
+static cudaStream_t as_stream(void* s) { return static_cast<cudaStream_t>(s); }
+
+sf_status sf_op_mtcopy(const sf_copy_desc* descs, int32_t n, int64_t patch_iter, void* stream) {
+  if (n < 0 || (n > 0 && !descs)) return fail(SF_EINVAL, "descs");
+  if (n == 0) return SF_OK;
+  std::vector<sfk::DCopy> d;
+  uint64_t chunks = 0;
+  for (int i = 0; i < n; ++i) {
+    const sf_copy_desc& s = descs[i];
+    if (s.span < s.nbytes || s.span % 16 || s.nbytes % 4 ||
+        reinterpret_cast<uintptr_t>(s.src) % 16 || reinterpret_cast<uintptr_t>(s.dst) % 16)
+      return fail(SF_EINVAL, "descriptor " + std::to_string(i) + ": alignment / span");
+    d.push_back({static_cast<const uint8_t*>(s.src), static_cast<uint8_t*>(s.dst), s.nbytes, chunks});
+    chunks += s.span / 16;
+  }
+  sfk::DCopy sent{};
+  sent.chunk_begin = chunks;
+  d.push_back(sent);
+  cudaStream_t st = as_stream(stream);
+  void* dd = nullptr;
+  SF_CK(cudaMallocAsync(&dd, d.size() * sizeof(sfk::DCopy), st));
+  SF_CK(cudaMemcpyAsync(dd, d.data(), d.size() * sizeof(sfk::DCopy), cudaMemcpyHostToDevice, st));
+  SF_CK(sfk::launch_mtcopy(static_cast<sfk::DCopy*>(dd), n, chunks, patch_iter, st));
+  SF_CK(cudaFreeAsync(dd, st));
+  SF_CK(cudaStreamSynchronize(st));  // the host descriptor array is released on return
+  return SF_OK;
+}
+
+sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
+                     int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
+  if (!A || !B || !C || M <= 0 || N <= 0 || K <= 0) return fail(SF_EINVAL, "gemm args");
+  sfk::GemmArgs ga{A, B, C, M, N, K, lda, ldb, ldc, (flags & SF_GEMM_TA) != 0,
+                   (flags & SF_GEMM_TB) != 0, (flags & SF_GEMM_ACC) != 0, nullptr, nullptr};
+  cudaStream_t st = as_stream(stream);
+  const uint64_t wsf = sfk::gemm_workspace_floats(M, N, K, ga.ta, ga.tb);
+  const uint64_t cs = sfk::gemm_counter_slots(M, N, K, ga.ta, ga.tb);
+  void* ws = nullptr;
+  void* cnt = nullptr;
+  if (wsf) {
+    SF_CK(cudaMallocAsync(&ws, wsf * 4, st));
+    SF_CK(cudaMallocAsync(&cnt, cs * 4, st));
+    SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
+    ga.ws = static_cast<float*>(ws);
+    ga.counters = static_cast<unsigned*>(cnt);
+  }
+  SF_CK(sfk::launch_gemm(ga, st));
+  if (ws) {
+    SF_CK(cudaFreeAsync(ws, st));
+    SF_CK(cudaFreeAsync(cnt, st));
+  }
+  return SF_OK;
+}
+
+sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
+                         float* h, int32_t rows, int32_t cols, int32_t relu, void* stream) {
+  if (!z || !b1 || !h) return fail(SF_EINVAL, "bias_act args");
+  SF_CK(sfk::launch_bias_act(z, b1, b2, b3, h, rows, cols, relu != 0, as_stream(stream)));
+  return SF_OK;
+}
+
+static sf_status colsum_common(const float* x, const float* mask, float* dz, float* s, int rows,
+                               int cols, cudaStream_t st) {
+  const uint64_t wsf = sfk::colsum_ws_floats(rows, cols);
+  const uint64_t cs = sfk::colsum_counter_slots(rows, cols);
+  void* ws = nullptr;
+  void* cnt = nullptr;
+  if (wsf) {
+    SF_CK(cudaMallocAsync(&ws, wsf * 4, st));
+    SF_CK(cudaMallocAsync(&cnt, cs * 4, st));
+    SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
+  }
+  SF_CK(sfk::launch_colsum(x, mask, dz, s, rows, cols, static_cast<float*>(ws),
+                           static_cast<unsigned*>(cnt), st));
+  if (ws) {
+    SF_CK(cudaFreeAsync(ws, st));
+    SF_CK(cudaFreeAsync(cnt, st));
+  }
+  return SF_OK;
+}
+
+sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* db, int32_t rows,
+                             int32_t cols, void* stream) {
+  if (!dh || !h || !dz || !db) return fail(SF_EINVAL, "bias_act_bwd args");
+  return colsum_common(dh, h, dz, db, rows, cols, as_stream(stream));
+}
+
+sf_status sf_op_colsum(const float* x, float* s, int32_t rows, int32_t cols, void* stream) {
+  if (!x || !s) return fail(SF_EINVAL, "colsum args");
+  return colsum_common(x, nullptr, nullptr, s, rows, cols, as_stream(stream));
+}
+
+sf_status sf_op_softmax_ce(const float* logits, const int32_t* labels, float* loss, float* dlogits,
+                           int32_t rows, int32_t cols, void* stream) {
+  if (!logits || !labels || !loss || !dlogits || rows <= 0 || cols <= 0)
+    return fail(SF_EINVAL, "softmax_ce args");
+  cudaStream_t st = as_stream(stream);
+  void *ws = nullptr, *cnt = nullptr;
+  SF_CK(cudaMallocAsync(&ws, sfk::softmax_ce_ws_floats(rows) * 4, st));
+  SF_CK(cudaMallocAsync(&cnt, 16, st));
+  SF_CK(cudaMemsetAsync(cnt, 0, 16, st));
+  SF_CK(sfk::launch_softmax_ce(logits, labels, loss, dlogits, rows, cols, static_cast<float*>(ws),
+                               static_cast<unsigned*>(cnt), st));
+  SF_CK(cudaFreeAsync(ws, st));
+  SF_CK(cudaFreeAsync(cnt, st));
+  return SF_OK;
+}
+
+sf_status sf_op_softmax(const float* logits, float* probs, int32_t rows, int32_t cols, void* stream) {
+  if (!logits || !probs) return fail(SF_EINVAL, "softmax args");
+  SF_CK(sfk::launch_softmax(logits, probs, rows, cols, as_stream(stream)));
+  return SF_OK;
+}
+
+static bool al16(const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; }
+
+sf_status sf_op_sgd_mom(float* w, float* a, const float* g, int64_t n, float lr, float mu,
+                        void* stream) {
+  if (!w || !a || !g || n < 0 || !al16(w) || !al16(a) || !al16(g))
+    return fail(SF_EINVAL, "sgd args (16-B aligned pointers)");
+  cudaStream_t st = as_stream(stream);
+  sfk::SgdDesc d[2] = {{w, a, g, static_cast<uint64_t>(n), lr, mu, 0}, {}};
+  d[1].begin = (static_cast<uint64_t>(n) + 3) / 4;
+  void* dd = nullptr;
+  SF_CK(cudaMallocAsync(&dd, sizeof(d), st));
+  SF_CK(cudaMemcpyAsync(dd, d, sizeof(d), cudaMemcpyHostToDevice, st));
+  SF_CK(sfk::launch_sgd(static_cast<sfk::SgdDesc*>(dd), 1, d[1].begin, st));
+  SF_CK(cudaFreeAsync(dd, st));
+  SF_CK(cudaStreamSynchronize(st));
+  return SF_OK;
+}
+
+sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t* step, int64_t n,
+                     float lr, float beta1, float beta2, float eps, void* stream) {
+  if (!w || !m || !v || !g || !step || n < 0 || !al16(w) || !al16(m) || !al16(v) || !al16(g))
+    return fail(SF_EINVAL, "adam args (16-B aligned pointers)");
+  cudaStream_t st = as_stream(stream);
+  sfk::AdamDesc d[2] = {{w, m, v, g, static_cast<uint64_t>(n), lr, beta1, beta2, eps, 0}, {}};
+  d[1].begin = (static_cast<uint64_t>(n) + 3) / 4;
+  void* dd = nullptr;
+  SF_CK(cudaMallocAsync(&dd, sizeof(d), st));
+  SF_CK(cudaMemcpyAsync(dd, d, sizeof(d), cudaMemcpyHostToDevice, st));
+  SF_CK(sfk::launch_adam(static_cast<sfk::AdamDesc*>(dd), 1, d[1].begin, step, st));
+  SF_CK(cudaFreeAsync(dd, st));
+  SF_CK(cudaStreamSynchronize(st));
+  return SF_OK;
+}
+
+sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream) {
+  if (!dst) return fail(SF_EINVAL, "fill args");
+  SF_CK(sfk::launch_fill(dst, n, static_cast<uint8_t>(value), as_stream(stream)));
+  return SF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,69 @@
+// Host-side launchers of the sm_100a kernels (internal to libswitchflow_b200.so).
+// Every launcher is asynchronous on `st` and returns the cudaError_t of the launch.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace sfk {
+
+// Device-side copy descriptor of the multi-tensor walk: chunk_begin = prefix sum of
+// span/16 over preceding descriptors; the array has n + 1 entries (sentinel holds the
+// total chunk count).
+struct DCopy {
+  const uint8_t* src;
+  uint8_t* dst;
+  uint64_t nbytes;       // valid bytes copied (multiple of 4)
+  uint64_t chunk_begin;  // first 16-B chunk of this descriptor in the flat chunk space
+};
+
+// Multi-tensor copy / pack / unpack / peer-store over a device descriptor array.
+// patch_iter >= 0 overwrites bytes [16,24) of descriptor 0's destination (staging iter).
+cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
+                          int64_t patch_iter, cudaStream_t st);
+cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st);
+
+// GEMM C[M,N] = op(A) op(B) (+C).  a_kcontig: A stored [M][K] (not transposed);
+// b_kcontig: B stored [N][K] (i.e. TB).  ws / counters: split-K workspace (may be null
+// when gemm_workspace_floats() == 0).  Deterministic (fixed split, fixed order).
+struct GemmArgs {
+  const float* A; const float* B; float* C;
+  int M, N, K, lda, ldb, ldc;
+  bool ta, tb, acc;
+  float* ws; unsigned* counters;
+};
+uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
+uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);
+cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
+
+// Elementwise / reduction ops (deterministic).  ws / counters sized by *_ws().
+uint64_t colsum_ws_floats(int rows, int cols);
+uint64_t colsum_counter_slots(int rows, int cols);
+cudaError_t launch_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
+                            float* h, int rows, int cols, bool relu, cudaStream_t st);
+cudaError_t launch_colsum(const float* x, const float* h_mask, float* dz, float* s, int rows,
+                          int cols, float* ws, unsigned* counters, cudaStream_t st);
+uint64_t softmax_ce_ws_floats(int rows);
+cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float* loss,
+                              float* dlogits, int rows, int cols, float* ws, unsigned* counter,
+                              cudaStream_t st);
+cudaError_t launch_softmax(const float* logits, float* probs, int rows, int cols,
+                           cudaStream_t st);
+
+struct SgdDesc { float* w; float* a; const float* g; uint64_t n; float lr, mu; uint64_t begin; };
+struct AdamDesc {
+  float* w; float* m; float* v; const float* g; uint64_t n; float lr, b1, b2, eps;
+  uint64_t begin;
+};
+// Multi-tensor optimizer updates over device descriptor arrays (n + 1 entries, sentinel).
+cudaError_t launch_sgd(const SgdDesc* d, int n, uint64_t total, cudaStream_t st);
+cudaError_t launch_adam(const AdamDesc* d, int n, uint64_t total, const int32_t* step,
+                        cudaStream_t st);
+cudaError_t launch_feed(const void* pool, const int32_t* step, void* x, uint64_t x_bytes,
+                        int64_t pool_period, cudaStream_t st);
+cudaError_t launch_step_inc(int32_t* step, cudaStream_t st);
+
+// Library-wide kernel launch counter (evidence of the native path).
+void count_launch(uint64_t n = 1);
+uint64_t launches();
+
+}  // namespace sfk
