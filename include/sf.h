@@ -139,6 +139,9 @@ typedef struct sf_config {
   int32_t host_mode;             /* SF_HOST_CE or SF_HOST_ZC */
   int32_t poison_released;       /* 1: fill released source arenas with 0xFF (tests) */
   int32_t trace_capacity;        /* events kept; 0 -> 1<<16 */
+  int32_t defer_migration;       /* 1: start the migration copy only after the device's
+                                    queued inference drained (the paper defers the transfer
+                                    past the preemption); 0: concurrent */
   uint64_t device_budget_bytes;  /* per device; 0 = unlimited */
 } sf_config;
 

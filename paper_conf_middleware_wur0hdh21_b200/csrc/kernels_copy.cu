@@ -122,6 +122,29 @@ cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+__global__ void copy_kernel(const uint8_t* __restrict__ src, uint8_t* __restrict__ dst,
+                            uint64_t nb) {
+  const uint64_t full = nb >> 4;
+  for (uint64_t j = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; j < (nb + 15) / 16;
+       j += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    if (j < full) {
+      sfdev::st16(dst + j * 16, sfdev::ld_stream16(src + j * 16));
+    } else {
+      for (uint64_t b = j * 16; b < nb; b += 4)
+        *reinterpret_cast<uint32_t*>(dst + b) = *reinterpret_cast<const uint32_t*>(src + b);
+    }
+  }
+}
+
+cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st) {
+  if (nbytes == 0) return cudaSuccess;
+  const uint64_t blocks = std::min<uint64_t>((nbytes / 16 + 255) / 256 + 1, 148ull * 4);
+  copy_kernel<<<static_cast<unsigned>(blocks), 256, 0, st>>>(static_cast<const uint8_t*>(src),
+                                                             static_cast<uint8_t*>(dst), nbytes);
+  count_launch();
+  return cudaGetLastError();
+}
+
 // FEED: x = pool[(step mod P) * x_bytes ...] (data cursor read on device, reading Q3).
 __global__ void feed_kernel(const uint8_t* __restrict__ pool, const int32_t* __restrict__ step,
                             uint8_t* __restrict__ x, uint64_t x_bytes, int64_t period) {

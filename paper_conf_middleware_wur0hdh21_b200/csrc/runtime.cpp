@@ -82,6 +82,7 @@ struct Binding {
   uint8_t* host_staging = nullptr;      // pinned host (host pointer)
   uint8_t* host_staging_dev = nullptr;  // its device mapping
   std::vector<cudaGraphExec_t> versions;
+  std::vector<uint64_t> version_kernels;  // kernel nodes per version (launch accounting)
   float* ws = nullptr;
   unsigned* counters = nullptr;
   std::vector<CopyList> pack, unpack, pack_zc, unpack_zc;
@@ -728,6 +729,12 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
   rt->cv.notify_all();
   Slot& S = slot_of(rt, src);
   Binding& B = *g.bind[src];
+  if (rt->cfg.defer_migration) {
+    // the preempter runs first with the whole device; the copy starts once it drained
+    rt->cv.wait(lk, [&] {
+      return rt->shutting_down || (!slot_has_inference(rt, src) && S.owner != kInferOwner);
+    });
+  }
   lk.unlock();
 
   auto cuda_fail = [&](cudaError_t e, const char* what) {
@@ -919,6 +926,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     const int dev = J.dev, k = J.k;
     const int64_t it = J.it;
     cudaGraphExec_t ver = g.bind[dev]->versions[k];
+    sfk::count_launch(g.bind[dev]->version_kernels[k]);
     const bool stamp = J.stamp_resume;
     J.stamp_resume = false;
     const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
@@ -982,11 +990,24 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     cudaError_t e = cudaSuccess;
     const Tensor& tin = g.T[g.input_tid];
     const Tensor& tout = g.T[g.output_tid];
-    e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
-    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k)
+    // Request I/O with the SM copy kernel on the high-priority stream: device or pinned
+    // (UVA-mapped) host buffers alike, never queued behind a copy-engine migration.
+    const bool aligned = reinterpret_cast<uintptr_t>(r->in) % 16 == 0 &&
+                         reinterpret_cast<uintptr_t>(r->out) % 16 == 0 && tin.nbytes % 4 == 0 &&
+                         tout.nbytes % 4 == 0;
+    if (aligned) {
+      e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
+    } else {
+      e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
+    }
+    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
       e = cudaGraphLaunch(B->versions[k], S->s_infer);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
+      sfk::count_launch(B->version_kernels[k]);
+    }
+    if (e == cudaSuccess) {
+      if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
+      else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
+    }
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
     if (e == cudaSuccess) e = spin_event(S->ev_infer);
     const uint64_t t1 = now_ns();
@@ -1253,7 +1274,10 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
   for (size_t k = 0; k < g.parts.size(); ++k) {
     SF_CK(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
     Capture c{g, *b, cap, false, &prepared};
+    const uint64_t l0 = sfk::launches();
     sf_status s = launch_subgraph_ops(c, static_cast<int>(k));
+    const uint64_t nk = sfk::launches() - l0;
+    sfk::count_launch(uint64_t(0) - nk);  // captured, not launched: counted at each replay
     cudaGraph_t graph = nullptr;
     cudaError_t e = cudaStreamEndCapture(cap, &graph);
     if (s != SF_OK) { if (graph) cudaGraphDestroy(graph); cudaStreamDestroy(cap); return s; }
@@ -1263,6 +1287,7 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
     cudaGraphDestroy(graph);
     if (e != cudaSuccess) { cudaStreamDestroy(cap); return fail(SF_ECUDA, std::string("instantiate: ") + cudaGetErrorString(e)); }
     b->versions.push_back(exec);
+    b->version_kernels.push_back(nk);
   }
   cudaStreamDestroy(cap);
   // copy lists per cut

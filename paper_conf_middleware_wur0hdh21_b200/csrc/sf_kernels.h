@@ -21,6 +21,8 @@ struct DCopy {
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
                           int64_t patch_iter, cudaStream_t st);
 cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st);
+// Single-buffer copy with pointer arguments (request I/O; 16-B aligned, nbytes % 4 == 0).
+cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st);
 
 // GEMM C[M,N] = op(A) op(B) (+C).  a_kcontig: A stored [M][K] (not transposed);
 // b_kcontig: B stored [N][K] (i.e. TB).  ws / counters: split-K workspace (may be null
