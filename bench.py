@@ -131,7 +131,7 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
                  iteration_granularity=iteration_granularity,
                  defer_migration=args.defer if defer is None else defer)
     gh = rt.register(g)
-    info = gh.partition()
+    info = gh.partition(update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
     arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
     gh.load(0, arrays)
@@ -321,6 +321,8 @@ def main():
     ap.add_argument("--spatial-div", type=int, default=1)
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--update-chunks", type=int, default=8,
+                    help="split the SGD update subgraph into byte-balanced chunks (Q2)")
     ap.add_argument("--defer", type=int, default=1,
                     help="1: migrate after the preempter drained (default); 0: concurrently")
     args = ap.parse_args()
@@ -398,6 +400,7 @@ def main():
         "config": {"workload": WORKLOAD, "batch": args.batch, "spatial_div": args.spatial_div,
                    "tensors_live_cut0": 535, "inference_model": "MLP 2048-4096-4096-1000 (29.3M params)",
                    "tier": "host (pinned, copy engine)", "parallelism": f"replicas x{args.world}",
+                   "update_chunks": args.update_chunks,
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets > 126 MB L2 (no flush needed)"},

@@ -164,9 +164,14 @@ sf_status sf_register_graph(sf_runtime* rt, const sf_graph_desc* g, int32_t prio
 #define SF_PART_PER_LAYER_PHASE 0
 #define SF_PART_MAX_OPS 1
 typedef struct sf_partition_opts {
-  int32_t policy;  /* SF_PART_PER_LAYER_PHASE (maximal runs of equal phase) or
-                      SF_PART_MAX_OPS (split runs to <= max_ops ops; optimizer runs whole) */
+  int32_t policy;        /* SF_PART_PER_LAYER_PHASE (maximal runs of equal phase) or
+                            SF_PART_MAX_OPS (split runs to <= max_ops ops; optimizer runs whole) */
   int32_t max_ops;
+  int32_t update_chunks; /* > 1: split each optimizer run into this many byte-balanced
+                            subgraphs: op j (weight = nbytes of its variable, 0 for STEP_INC,
+                            C_j = weight of the run's earlier ops, W = run total) goes to chunk
+                            min(U-1, floor(U*C_j/W)); bounds the longest subgraph, i.e. the
+                            preemption latency */
 } sf_partition_opts;
 typedef struct sf_partition_info {
   int32_t n_subgraphs;

@@ -6,8 +6,9 @@
   subgraph).  Granularity within a device is not specified by the paper; reading Q2:
   PER_LAYER_PHASE = maximal runs of ops with equal phase id; MAX_OPS = n splits each
   run into chunks of at most n ops, except that a run containing optimizer ops
-  (SGD_MOM / ADAM / STEP_INC) is never split (no partial weight update is visible at
-  a cut).
+  (SGD_MOM / ADAM / STEP_INC) is kept whole unless ``update_chunks`` > 1, which splits it
+  into byte-balanced chunks (``_split_update``); resuming inside it continues with the
+  remaining updates, so nothing is applied twice or lost.
 * Live set — PAPER.md:734-744 (section 3.3 "Context saving": persistent variables are
   tracked and saved; intermediate data is discarded at iteration end) extended by
   north_star to in-flight activations crossing the cut (reading Q1/Q3):
@@ -129,7 +130,32 @@ def validate(g: Graph) -> None:
         written.update(op_writes(op))
 
 
-def partition(g: Graph, policy: str = "phase", max_ops: int = 0) -> List[Tuple[int, int]]:
+def _split_update(g: Graph, a: int, b: int, chunks: int) -> List[Tuple[int, int]]:
+    """Split an optimizer run into byte-balanced chunks (reading Q2, update_chunks > 1).
+
+    Op j gets weight w_j = nbytes of its updated variable (0 for STEP_INC); with
+    C_j = sum of weights of the run's ops before j and W the run total, op j belongs to
+    chunk min(U - 1, floor(U * C_j / W)); maximal equal-chunk runs are the subgraphs.
+    """
+    w = [g.tensors[g.ops[j].outs[0]].nbytes if g.ops[j].type in (SGD_MOM, ADAM) else 0
+         for j in range(a, b)]
+    W = sum(w)
+    if chunks <= 1 or W == 0:
+        return [(a, b)]
+    out, c, start, prev = [], 0, a, None
+    for i, j in enumerate(range(a, b)):
+        ch = min(chunks - 1, (chunks * c) // W)
+        if prev is not None and ch != prev:
+            out.append((start, j))
+            start = j
+        prev = ch
+        c += w[i]
+    out.append((start, b))
+    return out
+
+
+def partition(g: Graph, policy: str = "phase", max_ops: int = 0,
+              update_chunks: int = 1) -> List[Tuple[int, int]]:
     """Contiguous op ranges [start, end) for S_0..S_{n-1} (reading Q2)."""
     runs = []
     s = 0
@@ -137,6 +163,14 @@ def partition(g: Graph, policy: str = "phase", max_ops: int = 0) -> List[Tuple[i
         if j == len(g.ops) or g.ops[j].phase != g.ops[s].phase:
             runs.append((s, j))
             s = j
+    if update_chunks > 1:
+        split = []
+        for (a, b) in runs:
+            if any(g.ops[j].type in OPTIMIZER_OPS for j in range(a, b)):
+                split.extend(_split_update(g, a, b, update_chunks))
+            else:
+                split.append((a, b))
+        runs = split
     if policy == "phase":
         return runs
     if policy != "max_ops" or max_ops <= 0:
@@ -144,7 +178,7 @@ def partition(g: Graph, policy: str = "phase", max_ops: int = 0) -> List[Tuple[i
     out = []
     for (a, b) in runs:
         if any(g.ops[j].type in OPTIMIZER_OPS for j in range(a, b)):
-            out.append((a, b))
+            out.append((a, b))  # optimizer runs are split only by update_chunks
             continue
         for c in range(a, b, max_ops):
             out.append((c, min(b, c + max_ops)))

@@ -54,7 +54,7 @@ class sf_config(C.Structure):
 
 
 class sf_partition_opts(C.Structure):
-    _fields_ = [("policy", C.c_int32), ("max_ops", C.c_int32)]
+    _fields_ = [("policy", C.c_int32), ("max_ops", C.c_int32), ("update_chunks", C.c_int32)]
 
 
 class sf_partition_info(C.Structure):

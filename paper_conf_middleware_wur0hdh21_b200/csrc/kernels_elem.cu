@@ -119,6 +119,198 @@ colsum_kernel(const float* __restrict__ x, const float* __restrict__ mask, float
   if (threadIdx.x == 0) counters[blockIdx.x] = 0u;
 }
 
+// Vectorized column sum (cols % 4 == 0, 16-B aligned): block = 16 column quads x 16 row
+// lanes, 4 rows in flight per thread; split partials [rsplit][cols] are combined by the last
+// CTA of the column tile in index order (rows lanes in parallel, then a fixed tree).
+struct Colsum4Plan { int col_tiles, rsplit, rper; };
+Colsum4Plan plan_colsum4(int rows, int cols) {
+  Colsum4Plan p;
+  p.col_tiles = (cols / 4 + 15) / 16;
+  int rs = std::max(1, (2 * 148 + p.col_tiles - 1) / p.col_tiles);
+  rs = std::min(rs, std::max(1, (rows + 127) / 128));
+  p.rper = (rows + rs - 1) / rs;
+  p.rsplit = (rows + p.rper - 1) / p.rper;
+  return p;
+}
+
+__global__ void __launch_bounds__(256)
+colsum4_kernel(const float* __restrict__ x, const float* __restrict__ mask, float* __restrict__ dz,
+               float* __restrict__ s, int rows, int cols, int rper, int rsplit, float* ws,
+               unsigned* counters) {
+  const int cq = threadIdx.x & 15, rl = threadIdx.x >> 4;
+  const int quad = blockIdx.x * 16 + cq;
+  const int nq = cols / 4;
+  const int z = blockIdx.y;
+  const int r0 = z * rper, r1 = min(rows, r0 + rper);
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (quad < nq) {
+    const float4* x4 = reinterpret_cast<const float4*>(x);
+    const float4* m4 = reinterpret_cast<const float4*>(mask);
+    float4* d4 = reinterpret_cast<float4*>(dz);
+    int r = r0 + rl;
+    for (; r + 48 < r1; r += 64) {
+      float4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) v[u] = __ldcs(x4 + static_cast<size_t>(r + 16 * u) * nq + quad);
+      if (mask) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const size_t i = static_cast<size_t>(r + 16 * u) * nq + quad;
+          const float4 mk = __ldcs(m4 + i);
+          v[u].x = mk.x > 0.f ? v[u].x : 0.f; v[u].y = mk.y > 0.f ? v[u].y : 0.f;
+          v[u].z = mk.z > 0.f ? v[u].z : 0.f; v[u].w = mk.w > 0.f ? v[u].w : 0.f;
+          d4[i] = v[u];
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        acc.x += v[u].x; acc.y += v[u].y; acc.z += v[u].z; acc.w += v[u].w;
+      }
+    }
+    for (; r < r1; r += 16) {
+      const size_t i = static_cast<size_t>(r) * nq + quad;
+      float4 v = __ldcs(x4 + i);
+      if (mask) {
+        const float4 mk = __ldcs(m4 + i);
+        v.x = mk.x > 0.f ? v.x : 0.f; v.y = mk.y > 0.f ? v.y : 0.f;
+        v.z = mk.z > 0.f ? v.z : 0.f; v.w = mk.w > 0.f ? v.w : 0.f;
+        d4[i] = v;
+      }
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+  }
+  __shared__ float4 red[16][16];
+  __shared__ int last;
+  red[rl][cq] = acc;
+  __syncthreads();
+  float4 part = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (rl == 0) {
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      part.x += red[j][cq].x; part.y += red[j][cq].y; part.z += red[j][cq].z; part.w += red[j][cq].w;
+    }
+  }
+  if (rsplit == 1) {
+    if (rl == 0 && quad < nq) reinterpret_cast<float4*>(s)[quad] = part;
+    return;
+  }
+  if (rl == 0 && quad < nq) reinterpret_cast<float4*>(ws)[static_cast<size_t>(z) * nq + quad] = part;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicAdd(&counters[blockIdx.x], 1u) == static_cast<unsigned>(rsplit - 1);
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  // 16 row lanes each sum a strided subset of the splits, then a fixed-order combine
+  float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (quad < nq)
+    for (int zz = rl; zz < rsplit; zz += 16) {
+      const float4 v = __ldcg(reinterpret_cast<const float4*>(ws) + static_cast<size_t>(zz) * nq + quad);
+      t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+    }
+  __syncthreads();
+  red[rl][cq] = t;
+  __syncthreads();
+  if (rl == 0 && quad < nq) {
+    float4 u = red[0][cq];
+#pragma unroll
+    for (int j = 1; j < 16; ++j) {
+      u.x += red[j][cq].x; u.y += red[j][cq].y; u.z += red[j][cq].z; u.w += red[j][cq].w;
+    }
+    reinterpret_cast<float4*>(s)[quad] = u;
+  }
+  if (threadIdx.x == 0) counters[blockIdx.x] = 0u;
+}
+
+// Softmax-CE for narrow rows (cols % 4 == 0, cols <= 8 L): L lanes per row, each lane keeps
+// up to two float4 of the row in registers (one read pass); shuffles within the L-lane group.
+template <int L>
+__global__ void __launch_bounds__(256)
+softmax_ce_narrow_kernel(const float* __restrict__ l, const int32_t* __restrict__ y,
+                         float* __restrict__ loss, float* __restrict__ dl, int rows, int cols,
+                         float* row_loss, unsigned* counter) {
+  const int lane = threadIdx.x & 31;
+  const int sub = lane % L;                       // lane within the row group
+  const int groups_per_block = 256 / L;
+  const int g0 = blockIdx.x * groups_per_block + threadIdx.x / L;
+  const int stride = gridDim.x * groups_per_block;
+  const int warp_first = blockIdx.x * groups_per_block + (threadIdx.x >> 5) * (32 / L);
+  const int nq = cols / 4;
+  const float inv_b = 1.0f / static_cast<float>(rows);
+  // warp-uniform trip count: every lane joins every shuffle; rows past the end are masked
+  for (int base = warp_first, row = g0; base < rows; base += stride, row += stride) {
+    const bool active = row < rows;
+    if (!active) {
+      float m = -INFINITY, s = 0.f;
+#pragma unroll
+      for (int o = L / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+#pragma unroll
+      for (int o = L / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      continue;
+    }
+    const float4* lr = reinterpret_cast<const float4*>(l + static_cast<size_t>(row) * cols);
+    float4* dr = reinterpret_cast<float4*>(dl + static_cast<size_t>(row) * cols);
+    float4 v[2];
+    bool have[2];
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int q = sub + u * L;
+      have[u] = q < nq;
+      v[u] = have[u] ? __ldcs(lr + q) : make_float4(-INFINITY, -INFINITY, -INFINITY, -INFINITY);
+    }
+    float m = fmaxf(fmaxf(fmaxf(v[0].x, v[0].y), fmaxf(v[0].z, v[0].w)),
+                    fmaxf(fmaxf(v[1].x, v[1].y), fmaxf(v[1].z, v[1].w)));
+#pragma unroll
+    for (int o = L / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float4 e[2];
+    float s = 0.f;
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      if (have[u]) {
+        e[u] = make_float4(expf(v[u].x - m), expf(v[u].y - m), expf(v[u].z - m), expf(v[u].w - m));
+        s += ((e[u].x + e[u].y) + e[u].z) + e[u].w;
+      }
+    }
+#pragma unroll
+    for (int o = L / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const int lab = y[row];
+    const bool ok = lab >= 0 && lab < cols;
+    const float nan = __int_as_float(0x7fffffff);
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      if (!have[u]) continue;
+      const int c0 = 4 * (sub + u * L);
+      float4 d;
+      d.x = ok ? (e[u].x / s - (c0 == lab ? 1.f : 0.f)) * inv_b : nan;
+      d.y = ok ? (e[u].y / s - (c0 + 1 == lab ? 1.f : 0.f)) * inv_b : nan;
+      d.z = ok ? (e[u].z / s - (c0 + 2 == lab ? 1.f : 0.f)) * inv_b : nan;
+      d.w = ok ? (e[u].w / s - (c0 + 3 == lab ? 1.f : 0.f)) * inv_b : nan;
+      dr[sub + u * L] = d;
+    }
+    if (sub == 0) row_loss[row] = ok ? (m + logf(s)) - l[static_cast<size_t>(row) * cols + lab] : nan;
+  }
+  __shared__ int last;
+  __shared__ float red[256];
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicAdd(counter, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  float t = 0.f;
+  for (int r = threadIdx.x; r < rows; r += 256) t += __ldcg(row_loss + r);
+  red[threadIdx.x] = t;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *loss = red[0] / static_cast<float>(rows);
+    *counter = 0u;
+  }
+}
+
 // ---- softmax cross-entropy: one warp per row ------------------------------------------
 __global__ void __launch_bounds__(256)
 softmax_ce_kernel(const float* __restrict__ l, const int32_t* __restrict__ y, float* __restrict__ loss,
@@ -179,6 +371,33 @@ softmax_kernel(const float* __restrict__ l, float* __restrict__ p, int rows, int
     s = warp_sum(s);
     for (int c = lane; c < cols; c += 32) p[static_cast<size_t>(row) * cols + c] = expf(lr[c] - m) / s;
   }
+}
+
+// Block-per-row softmax for few, wide rows (batch-1 inference head): 256 threads share a row;
+// max / sum reduced through shared memory in a fixed tree order.
+__global__ void __launch_bounds__(256)
+softmax_block_kernel(const float* __restrict__ l, float* __restrict__ p, int cols) {
+  const float* lr = l + static_cast<size_t>(blockIdx.x) * cols;
+  float* pr = p + static_cast<size_t>(blockIdx.x) * cols;
+  __shared__ float red[8];
+  float m = -INFINITY;
+  for (int c = threadIdx.x; c < cols; c += 256) m = fmaxf(m, lr[c]);
+  m = warp_max(m);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  m = red[0];
+#pragma unroll
+  for (int j = 1; j < 8; ++j) m = fmaxf(m, red[j]);
+  __syncthreads();
+  float s = 0.f;
+  for (int c = threadIdx.x; c < cols; c += 256) s += expf(lr[c] - m);
+  s = warp_sum(s);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  s = 0.f;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) s += red[j];
+  for (int c = threadIdx.x; c < cols; c += 256) pr[c] = expf(lr[c] - m) / s;
 }
 
 // ---- multi-tensor optimizer updates ---------------------------------------------------
@@ -302,13 +521,26 @@ cudaError_t launch_bias_act(const float* z, const float* b1, const float* b2, co
 
 uint64_t colsum_ws_floats(int rows, int cols) {
   ColsumPlan p = plan_colsum(rows, cols);
-  return p.rsplit > 1 ? static_cast<uint64_t>(p.rsplit) * cols : 0;
+  Colsum4Plan q = plan_colsum4(rows, cols);
+  return std::max<uint64_t>(p.rsplit > 1 ? static_cast<uint64_t>(p.rsplit) * cols : 0,
+                            q.rsplit > 1 ? static_cast<uint64_t>(q.rsplit) * cols : 0);
 }
-uint64_t colsum_counter_slots(int rows, int cols) { return plan_colsum(rows, cols).col_tiles; }
+uint64_t colsum_counter_slots(int rows, int cols) {
+  return std::max(plan_colsum(rows, cols).col_tiles, plan_colsum4(rows, cols).col_tiles);
+}
 
 cudaError_t launch_colsum(const float* x, const float* mask, float* dz, float* s, int rows,
                           int cols, float* ws, unsigned* counters, cudaStream_t st) {
   if (cols <= 0) return cudaSuccess;
+  auto al = [](const void* p) { return p == nullptr || reinterpret_cast<uintptr_t>(p) % 16 == 0; };
+  if (cols % 4 == 0 && rows > 0 && al(x) && al(mask) && al(dz) && al(s) && al(ws)) {
+    Colsum4Plan q = plan_colsum4(rows, cols);
+    if (q.rsplit > 1 && (!ws || !counters)) return cudaErrorInvalidValue;
+    dim3 grid(q.col_tiles, q.rsplit);
+    colsum4_kernel<<<grid, 256, 0, st>>>(x, mask, dz, s, rows, cols, q.rper, q.rsplit, ws, counters);
+    count_launch();
+    return cudaGetLastError();
+  }
   ColsumPlan p = plan_colsum(rows, std::max(cols, 1));
   if (rows <= 0) {
     p.rsplit = 1;
@@ -328,6 +560,18 @@ cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float*
                               cudaStream_t st) {
   if (rows <= 0) return cudaSuccess;
   if (!ws || !counter) return cudaErrorInvalidValue;
+  auto al = [](const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; };
+  if (cols % 4 == 0 && cols <= 256 && al(logits) && al(dlogits)) {
+    const int L = cols <= 16 ? 2 : cols <= 32 ? 4 : cols <= 64 ? 8 : cols <= 128 ? 16 : 32;
+    const int per_block = 256 / L;
+    const unsigned blocks = grid_for(static_cast<uint64_t>(rows), per_block * 4, 148 * 8);
+#define SF_SCE(LL) softmax_ce_narrow_kernel<LL><<<blocks, 256, 0, st>>>(logits, labels, loss, dlogits, rows, cols, ws, counter)
+    if (L == 2) SF_SCE(2); else if (L == 4) SF_SCE(4); else if (L == 8) SF_SCE(8);
+    else if (L == 16) SF_SCE(16); else SF_SCE(32);
+#undef SF_SCE
+    count_launch();
+    return cudaGetLastError();
+  }
   const unsigned blocks = grid_for(static_cast<uint64_t>(rows), 8, 148 * 8);
   softmax_ce_kernel<<<blocks, 256, 0, st>>>(logits, labels, loss, dlogits, rows, cols, ws, counter);
   count_launch();
@@ -336,6 +580,11 @@ cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float*
 
 cudaError_t launch_softmax(const float* logits, float* probs, int rows, int cols, cudaStream_t st) {
   if (rows <= 0) return cudaSuccess;
+  if (rows <= 64 && cols >= 256) {
+    softmax_block_kernel<<<rows, 256, 0, st>>>(logits, probs, cols);
+    count_launch();
+    return cudaGetLastError();
+  }
   const unsigned blocks = grid_for(static_cast<uint64_t>(rows), 8, 148 * 8);
   softmax_kernel<<<blocks, 256, 0, st>>>(logits, probs, rows, cols);
   count_launch();

@@ -21,6 +21,8 @@
 // go to a split-K GEMV kernel instead of padding M to 128.
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
+#include <string>
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
@@ -313,8 +315,9 @@ Plan plan_gemm(int M, int N, int K) {
   const int nkb = std::max(1, (K + BK - 1) / BK);
   int splits = 1;
   if (tiles < 148) {
-    splits = (148 + tiles - 1) / tiles;
-    splits = std::min(splits, std::max(1, nkb / 4));
+    // fill the 148 SMs in ONE wave: floor, never a small second wave
+    splits = std::max(1, 148 / tiles);
+    splits = std::min(splits, std::max(1, nkb / 2));
     splits = std::min(splits, 64);
   }
   pl.kb_per_split = (nkb + splits - 1) / splits;
@@ -402,6 +405,107 @@ gemv_kernel(const float* __restrict__ A, const float* __restrict__ B, float* __r
   if (threadIdx.x == 0) counters[blockIdx.x] = 0u;
 }
 
+// Bandwidth-oriented GEMV (N % 4 == 0): each thread owns 4 adjacent columns (16-B loads of
+// W rows), 8 W rows in flight per thread, K split over enough CTAs to fill every SM several
+// times; partials [S][M][N] are summed in index order by a second, fully parallel kernel.
+template <int MR>
+__global__ void __launch_bounds__(256)
+gemv4_kernel(const float* __restrict__ A, const float* __restrict__ B, float* __restrict__ ws,
+             int M, int N, int K, int lda, int ldb, int kper) {
+  const int q = blockIdx.x * 256 + threadIdx.x;  // column quad
+  const int z = blockIdx.y;
+  const int k0 = z * kper, k1 = min(K, k0 + kper);
+  __shared__ float xs[MR][64];
+  for (int i = threadIdx.x; i < MR * kper; i += 256) {
+    const int m = i / kper, kk = i % kper;
+    xs[m][kk] = (m < M && k0 + kk < k1) ? A[static_cast<size_t>(m) * lda + k0 + kk] : 0.f;
+  }
+  __syncthreads();
+  if (4 * q >= N) return;
+  float4 acc[MR];
+#pragma unroll
+  for (int m = 0; m < MR; ++m) acc[m] = make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* col = B + 4 * q;
+  int k = k0;
+  for (; k + 8 <= k1; k += 8) {
+    float4 w[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      w[u] = __ldcs(reinterpret_cast<const float4*>(col + static_cast<size_t>(k + u) * ldb));
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+#pragma unroll
+      for (int m = 0; m < MR; ++m) {
+        const float xv = xs[m][k - k0 + u];
+        acc[m].x = fmaf(xv, w[u].x, acc[m].x); acc[m].y = fmaf(xv, w[u].y, acc[m].y);
+        acc[m].z = fmaf(xv, w[u].z, acc[m].z); acc[m].w = fmaf(xv, w[u].w, acc[m].w);
+      }
+  }
+  for (; k < k1; ++k) {
+    const float4 w = __ldcs(reinterpret_cast<const float4*>(col + static_cast<size_t>(k) * ldb));
+#pragma unroll
+    for (int m = 0; m < MR; ++m) {
+      const float xv = xs[m][k - k0];
+      acc[m].x = fmaf(xv, w.x, acc[m].x); acc[m].y = fmaf(xv, w.y, acc[m].y);
+      acc[m].z = fmaf(xv, w.z, acc[m].z); acc[m].w = fmaf(xv, w.w, acc[m].w);
+    }
+  }
+#pragma unroll
+  for (int m = 0; m < MR; ++m)
+    if (m < M) *reinterpret_cast<float4*>(ws + (static_cast<size_t>(z) * M + m) * N + 4 * q) = acc[m];
+}
+
+// Split reduction of the GEMV partials, parallel over columns AND splits: block = 32 output
+// elements x 8 split lanes; lane zl sums z = zl, zl+8, ... (two accumulators), then the 8
+// lane partials are combined in index order.  Optional fused bias + ReLU epilogue.
+__global__ void __launch_bounds__(256)
+gemv_reduce_kernel(const float* __restrict__ ws, float* __restrict__ C, int M, int N, int S, int ldc,
+                   int acc, const float* __restrict__ b1, const float* __restrict__ b2,
+                   const float* __restrict__ b3, int relu) {
+  const int lane = threadIdx.x & 31, zl = threadIdx.x >> 5;
+  const int total = M * N;
+  const int e = blockIdx.x * 32 + lane;
+  float s0 = 0.f, s1 = 0.f;
+  if (e < total) {
+    int z = zl;
+    for (; z + 8 < S; z += 16) {
+      s0 += __ldcs(ws + static_cast<size_t>(z) * total + e);
+      s1 += __ldcs(ws + static_cast<size_t>(z + 8) * total + e);
+    }
+    if (z < S) s0 += __ldcs(ws + static_cast<size_t>(z) * total + e);
+  }
+  __shared__ float red[8][33];
+  red[zl][lane] = s0 + s1;
+  __syncthreads();
+  if (zl != 0 || e >= total) return;
+  float t = 0.f;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) t += red[j][lane];
+  const int m = e / N, n = e % N;
+  float* o = C + static_cast<size_t>(m) * ldc + n;
+  if (acc) t = *o + t;
+  if (b1) t += b1[n];
+  if (b2) t += b2[n];
+  if (b3) t += b3[n];
+  if (relu) t = fmaxf(t, 0.f);
+  *o = t;
+}
+
+struct Gemv4Plan { int splits, kper, col_blocks; };
+Gemv4Plan plan_gemv4(int N, int K) {
+  Gemv4Plan g;
+  g.col_blocks = (N / 4 + 255) / 256;
+  // ~4 CTAs per SM in one pass, at least 16 weight rows per CTA
+  int splits = std::max(1, (148 * 4 + g.col_blocks - 1) / g.col_blocks);
+  g.kper = std::min(64, std::max(16, ((K + splits - 1) / splits + 7) / 8 * 8));
+  g.splits = (K + g.kper - 1) / g.kper;
+  return g;
+}
+
+bool gemv4_ok(const float* A, const float* B, float* C, int N, int ldb) {
+  return N % 4 == 0 && ldb % 4 == 0 && reinterpret_cast<uintptr_t>(B) % 16 == 0;
+}
+
 struct GemvPlan { int splits, kper, cols_blocks; };
 GemvPlan plan_gemv(int N, int K) {
   GemvPlan g;
@@ -417,7 +521,15 @@ bool use_gemv(int M, bool ta, bool tb) { return M <= 8 && !ta && !tb; }
 
 }  // namespace
 
+bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb) {
+  return use_gemv(M, ta, tb) && N % 4 == 0 && ldb % 4 == 0;
+}
+
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb) {
+  if (use_gemv(M, ta, tb) && N % 4 == 0) {
+    Gemv4Plan g = plan_gemv4(N, K);
+    return static_cast<uint64_t>(g.splits) * M * N;
+  }
   if (use_gemv(M, ta, tb)) {
     GemvPlan g = plan_gemv(N, K);
     return g.splits > 1 ? static_cast<uint64_t>(g.splits) * M * N : 0;
@@ -434,6 +546,27 @@ uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0) return cudaSuccess;
+  if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb) && a.ws))
+    return cudaErrorInvalidValue;  // fused epilogue only exists on the GEMV path
+  if (use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb) && a.ws) {
+    Gemv4Plan g = plan_gemv4(a.N, a.K);
+    dim3 grid(g.col_blocks, g.splits);
+#define SF_GEMV4(MR) gemv4_kernel<MR><<<grid, 256, 0, st>>>(a.A, a.B, a.ws, a.M, a.N, a.K, a.lda, a.ldb, g.kper)
+    if (a.M == 1) SF_GEMV4(1);
+    else if (a.M == 2) SF_GEMV4(2);
+    else if (a.M <= 4) SF_GEMV4(4);
+    else SF_GEMV4(8);
+#undef SF_GEMV4
+    count_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    const int total = a.M * a.N;
+    gemv_reduce_kernel<<<(total + 31) / 32, 256, 0, st>>>(a.ws, a.C, a.M, a.N, g.splits, a.ldc,
+                                                          a.acc ? 1 : 0, a.bias[0], a.bias[1],
+                                                          a.bias[2], a.relu ? 1 : 0);
+    count_launch();
+    return cudaGetLastError();
+  }
   if (use_gemv(a.M, a.ta, a.tb)) {
     GemvPlan g = plan_gemv(a.N, a.K);
     if (g.splits > 1 && (!a.ws || !a.counters)) return cudaErrorInvalidValue;
@@ -451,6 +584,15 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   }
   Plan pl = plan_gemm(a.M, a.N, a.K);
   if (pl.splits > 1 && (!a.ws || !a.counters)) return cudaErrorInvalidValue;
+  // SF_GEMM_PATH=legacy forces the LDG-producer kernel; SF_GEMM_RAWHI=1 feeds raw fp32 as
+  // the hi operand (relies on the tensor core ignoring the low 13 mantissa bits).
+  static const char* path = std::getenv("SF_GEMM_PATH");
+  // default: raw (the tcgen05 tf32 datapath truncates the low 13 bits — bit-identical to the
+  // explicitly masked hi on B200, scripts/rawhi_check.py); SF_GEMM_RAWHI=0 masks explicitly.
+  static const bool raw_hi = !(std::getenv("SF_GEMM_RAWHI") && std::getenv("SF_GEMM_RAWHI")[0] == '0');
+  const bool legacy = path && std::string(path) == "legacy";
+  if (!legacy && gemm_tma_eligible(a, pl.splits))
+    return launch_gemm_tma(a, pl.bn, pl.splits, pl.kb_per_split, pl.tiles_n, pl.tiles_m, raw_hi, st);
   Params p;
   p.A = a.A; p.B = a.B; p.C = a.C;
   p.M = a.M; p.N = a.N; p.K = a.K; p.lda = a.lda; p.ldb = a.ldb; p.ldc = a.ldc;

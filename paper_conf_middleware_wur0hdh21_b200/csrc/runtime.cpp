@@ -88,6 +88,9 @@ struct Binding {
   std::vector<CopyList> pack, unpack, pack_zc, unpack_zc;
   std::map<int, std::vector<CopyList>> peer;  // target slot -> per cut
   std::vector<std::pair<uint64_t, uint64_t>> poison_ranges;  // non-DATASET arena ranges
+  // padded-pitch copies of DATASET GEMM operands whose row pitch is not 16-B aligned (the
+  // TMA tensor-map requirement); refreshed from the arena at sf_start_training
+  std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
   std::vector<void*> dev_allocs;
 };
 
@@ -375,6 +378,29 @@ sf_status do_partition(Graph& g, const sf_partition_opts& o) {
       runs.emplace_back(s, j);
       s = j;
     }
+  if (o.update_chunks > 1) {
+    std::vector<std::pair<int, int>> split;
+    for (auto [a, b] : runs) {
+      bool opt = false;
+      for (int j = a; j < b; ++j) opt |= optimizer_op(g.ops[j].type);
+      uint64_t W = 0;
+      for (int j = a; j < b; ++j)
+        if (g.ops[j].type == SF_OP_SGD_MOM || g.ops[j].type == SF_OP_ADAM) W += g.T[g.ops[j].out[0]].nbytes;
+      if (!opt || W == 0) { split.emplace_back(a, b); continue; }
+      const uint64_t U = static_cast<uint64_t>(o.update_chunks);
+      uint64_t c = 0;
+      int start = a;
+      int64_t prev = -1;
+      for (int j = a; j < b; ++j) {
+        const int64_t ch = static_cast<int64_t>(std::min<uint64_t>(U - 1, (U * c) / W));
+        if (prev >= 0 && ch != prev) { split.emplace_back(start, j); start = j; }
+        prev = ch;
+        if (g.ops[j].type == SF_OP_SGD_MOM || g.ops[j].type == SF_OP_ADAM) c += g.T[g.ops[j].out[0]].nbytes;
+      }
+      split.emplace_back(start, b);
+    }
+    runs = std::move(split);
+  }
   if (o.policy == SF_PART_PER_LAYER_PHASE) {
     g.parts = runs;
   } else if (o.policy == SF_PART_MAX_OPS && o.max_ops > 0) {
@@ -559,6 +585,29 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         ga.M = C.rows; ga.N = C.cols; ga.K = ga.ta ? A.rows : A.cols;
         ga.lda = A.cols; ga.ldb = B.cols; ga.ldc = C.cols;
         ga.ws = c.b.ws; ga.counters = c.b.counters;
+        auto sa = c.b.shadow.find(o.in[0]);
+        if (sa != c.b.shadow.end()) { ga.A = sa->second.first; ga.lda = sa->second.second; }
+        auto sb = c.b.shadow.find(o.in[1]);
+        if (sb != c.b.shadow.end()) { ga.B = sb->second.first; ga.ldb = sb->second.second; }
+        // Fuse a following BIAS_ACT into the GEMV epilogue when the GEMM output has no other
+        // reader (same arithmetic order as the unfused pair, so results are bit-identical).
+        if (j + 1 < e && !ga.acc && g.ops[j + 1].type == SF_OP_BIAS_ACT && g.ops[j + 1].in[0] == o.out[0] &&
+            C.kind != SF_OUTPUT && sfk::gemm_can_fuse_bias(ga.M, ga.N, ga.K, ga.ta, ga.tb, ga.ldb)) {
+          int readers = 0;
+          for (const auto& q : g.ops)
+            for (int t : op_reads(q)) readers += (t == o.out[0]);
+          if (readers == 1) {
+            const sf_op_desc& ba = g.ops[j + 1];
+            ga.C = c.f(ba.out[0]);
+            for (int i = 1; i < ba.n_in; ++i) ga.bias[i - 1] = c.f(ba.in[i]);
+            ga.relu = ba.flags & SF_ACT_RELU;
+            ga.ldc = g.T[ba.out[0]].cols;
+            err = sfk::launch_gemm(ga, c.st);
+            if (err != cudaSuccess) return fail(SF_ECUDA, "op " + std::to_string(j) + ": " + cudaGetErrorString(err));
+            j += 2;
+            continue;
+          }
+        }
         err = sfk::launch_gemm(ga, c.st);
         break;
       }
@@ -1171,7 +1220,7 @@ sf_status sf_partition(sf_runtime* rt, sf_graph_id gid, const sf_partition_opts*
   Graph* g = get_graph(rt, gid);
   if (!g) return fail(SF_EINVAL, "bad graph id");
   if (g->partitioned) return fail(SF_ESTATE, "graph already partitioned");
-  sf_partition_opts def{SF_PART_PER_LAYER_PHASE, 0};
+  sf_partition_opts def{SF_PART_PER_LAYER_PHASE, 0, 1};
   if (sf_status s = do_partition(*g, o ? *o : def)) return s;
   if (out) {
     out->n_subgraphs = static_cast<int32_t>(g->parts.size());
@@ -1258,6 +1307,19 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
     void* dp = nullptr;
     SF_CK(cudaHostGetDevicePointer(&dp, host_staging, 0));
     b->host_staging_dev = static_cast<uint8_t*>(dp);
+  }
+  for (const auto& op : g.ops) {
+    if (op.type != SF_OP_GEMM) continue;
+    for (int t : {op.in[0], op.in[1]}) {
+      const Tensor& x = g.T[t];
+      if (x.kind != SF_DATASET || x.cols % 4 == 0 || b->shadow.count(t)) continue;
+      const int pitch = (x.cols + 3) / 4 * 4;
+      float* d = nullptr;
+      SF_CK(cudaMalloc(&d, static_cast<size_t>(x.rows) * pitch * sizeof(float)));
+      SF_CK(cudaMemset(d, 0, static_cast<size_t>(x.rows) * pitch * sizeof(float)));
+      b->shadow[t] = {d, pitch};
+      b->dev_allocs.push_back(d);
+    }
   }
   SF_CK(cudaMalloc(&b->ws, std::max<uint64_t>(g.ws_floats, 4) * sizeof(float)));
   SF_CK(cudaMalloc(&b->counters, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));
@@ -1353,6 +1415,17 @@ sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_
   J->dev = dev;
   J->iters = iters;
   J->auto_target = auto_target;
+  // DATASET contents are final once training starts: refresh padded-pitch copies
+  for (auto& Bp : g->bind) {
+    if (!Bp) continue;
+    for (auto& [t, sh] : Bp->shadow) {
+      const Tensor& x = g->T[t];
+      SF_CK(cudaSetDevice(rt->slots[Bp->slot]->cuda));
+      SF_CK(cudaMemcpy2D(sh.first, static_cast<size_t>(sh.second) * 4, Bp->arena + x.offset,
+                         static_cast<size_t>(x.cols) * 4, static_cast<size_t>(x.cols) * 4, x.rows,
+                         cudaMemcpyDeviceToDevice));
+    }
+  }
   for (int i = 0; i < n_sched; ++i) {
     const sf_cut_request& c = sched[i];
     if (c.k < 0 || c.k >= static_cast<int>(g->parts.size()) || c.iter < 0)

@@ -32,10 +32,19 @@ struct GemmArgs {
   int M, N, K, lda, ldb, ldc;
   bool ta, tb, acc;
   float* ws; unsigned* counters;
+  // optional fused epilogue (batch-1 GEMV path only): C = act(AB + b1 + b2 + b3)
+  const float* bias[3] = {nullptr, nullptr, nullptr};
+  bool relu = false;
 };
+// True when launch_gemm can fuse a following BIAS_ACT into this GEMM's epilogue.
+bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb);
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
+// TMA-fed variant (kernels_gemm_tma.cu): needs 16-B aligned pointers and row pitches.
+bool gemm_tma_eligible(const GemmArgs& a, int splits);
+cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_split, int tiles_n,
+                            int tiles_m, bool raw_hi, cudaStream_t st);
 
 // Elementwise / reduction ops (deterministic).  ws / counters sized by *_ws().
 uint64_t colsum_ws_floats(int rows, int cols);

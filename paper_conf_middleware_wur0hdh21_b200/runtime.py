@@ -51,9 +51,10 @@ class GraphHandle:
         self.mem: Dict[int, dict] = {}
 
     # ---- partition / analysis ---------------------------------------------------------
-    def partition(self, policy: str = "phase", max_ops: int = 0) -> A.sf_partition_info:
+    def partition(self, policy: str = "phase", max_ops: int = 0,
+                  update_chunks: int = 1) -> A.sf_partition_info:
         o = A.sf_partition_opts(A.SF_PART_PER_LAYER_PHASE if policy == "phase" else A.SF_PART_MAX_OPS,
-                                max_ops)
+                                max_ops, update_chunks)
         info = A.sf_partition_info()
         check(lib().sf_partition(self.rt.h, self.gid, C.byref(o), C.byref(info)), "sf_partition")
         self.info = info

@@ -131,7 +131,8 @@ def test_bias_act(ops, rows, cols, nb, relu):
     assert rel(h.cpu().numpy(), O.bias_act(z, bs, relu)) <= TOL
 
 
-@pytest.mark.parametrize("rows,cols", [(64, 256), (25088, 64), (3, 1000), (513, 33), (1, 5)])
+@pytest.mark.parametrize("rows,cols", [(64, 256), (25088, 64), (3, 1000), (513, 33), (1, 5),
+                                       (100352, 64), (17, 4), (4097, 2048), (7, 12)])
 def test_bias_act_bwd_and_colsum(ops, rows, cols):
     rng = np.random.default_rng(rows * cols)
     dh = rng.standard_normal((rows, cols)).astype(np.float32)
@@ -150,7 +151,8 @@ def test_bias_act_bwd_and_colsum(ops, rows, cols):
     assert torch.equal(s, s2)
 
 
-@pytest.mark.parametrize("rows,cols", [(64, 10), (1, 1000), (3136, 256), (512, 30522), (7, 3)])
+@pytest.mark.parametrize("rows,cols", [(64, 10), (1, 1000), (3136, 256), (512, 30522), (7, 3),
+                                       (20000, 64), (33, 16), (5, 128), (9, 4), (100, 8)])
 def test_softmax_ce_and_softmax(ops, rows, cols):
     rng = np.random.default_rng(rows + cols)
     l = (rng.standard_normal((rows, cols)) * 3).astype(np.float32)

@@ -128,6 +128,31 @@ def test_random_schedule_ping_pong_resnet_prefix(P):
             assert rel(got[i], ref.state[i]) <= TOL, g.tensors[i].name
 
 
+def test_update_chunk_cuts_bit_identical(P):
+    g = G.resnet50_forest(batch=1, spatial_div=4, max_layers=10)
+    RT, A = P
+
+    def go(schedule):
+        rt = RT.Runtime([0, 0], poison=True)
+        gh = rt.register(g)
+        gh.partition(update_chunks=4)
+        st, ds = D.init_state(g), D.datasets(g)
+        for s_ in (0, 1):
+            gh.bind(s_, host_staging=True)
+            gh.load(s_, ds)
+        gh.load(0, st)
+        job = rt.start_training(gh, 0, 2, HOST, schedule=schedule)
+        rt.wait_job(job, 120)
+        dev = rt.job_info(job)["dev"]
+        out = {i: gh.read(dev, i) for i in st}
+        n = gh.n_subgraphs
+        rt.close()
+        return out, n
+    base, n = go(())
+    got, _ = go([(0, n - 3, 1), (0, n - 2, HOST), (1, n - 1, 0)])
+    assert_bitwise(base, got)
+
+
 def test_cut0_staging_bytes_equal_oracle_pack(P):
     g = G.mlp_train()
     st, ds = D.init_state(g), D.datasets(g)
@@ -255,14 +280,15 @@ def test_error_paths(P):
     rt.close()
 
 
-def test_live_sets_match_oracle(P):
+@pytest.mark.parametrize("U", [1, 3, 8])
+def test_live_sets_match_oracle(P, U):
     RT, A = P
     rt = RT.Runtime([0])
     for g in (G.mlp_train(), G.resnet50_forest(batch=1, spatial_div=8),
               G.bert_chain(layers=2, hidden=8, inter=16, vocab=11, tokens=6, positions=6)):
         gh = rt.register(g)
-        gh.partition()
-        parts = OG.partition(g)
+        gh.partition(update_chunks=U)
+        parts = OG.partition(g, update_chunks=U)
         assert gh.n_subgraphs == len(parts)
         for k in range(len(parts)):
             assert gh.subgraph_range(k) == parts[k]

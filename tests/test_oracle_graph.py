@@ -17,7 +17,7 @@ import pytest
 from oracle import graph as OG, runner as R
 from sf_inputs import graphs as G, data as D
 from sf_inputs.ir import (OP_NAMES, PERSISTENT_KINDS, Graph, F32, I32, PARAM, ACT, INPUT,
-                          DATASET, GEMM, BIAS_ACT, SCALAR_STATE, SGD_MOM, SLOT, GRAD)
+                          DATASET, GEMM, BIAS_ACT, SCALAR_STATE, SGD_MOM, SLOT, GRAD, STEP_INC)
 
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 
@@ -154,6 +154,40 @@ def test_max_ops_partition_keeps_update_whole():
     assert parts[-1] == (12, 17)
     assert parts[0][0] == 0 and parts[-1][1] == len(g.ops)
     assert all(p[1] == q[0] for p, q in zip(parts, parts[1:]))
+
+
+@pytest.mark.parametrize("U", [2, 3, 8])
+def test_update_chunks_rule(U):
+    g = G.resnet50_forest(batch=1, spatial_div=8)
+    whole = OG.partition(g)
+    parts = OG.partition(g, update_chunks=U)
+    a, b = whole[-1]
+    upd = [p for p in parts if p[0] >= a]
+    assert parts[:len(whole) - 1] == whole[:-1]
+    assert upd[0][0] == a and upd[-1][1] == b and len(upd) == U
+    assert all(p[1] == q[0] for p, q in zip(upd, upd[1:]))
+    w = lambda j: g.tensors[g.ops[j].outs[0]].nbytes if g.ops[j].type != STEP_INC else 0
+    W = sum(w(j) for j in range(a, b))
+    biggest = max(w(j) for j in range(a, b))
+    for (x, y) in upd:
+        assert sum(w(j) for j in range(x, y)) <= W / U + biggest
+
+
+@pytest.mark.parametrize("mk,U", [(lambda: G.mlp_train((5, 7, 3), batch=4, pool=2), 3),
+                                  (lambda: G.resnet50_forest(batch=1, spatial_div=8, max_layers=6), 4)])
+def test_cut_inside_update_is_bitwise(mk, U):
+    """Cutting between optimizer ops resumes with the remaining updates only."""
+    g = mk()
+    parts = OG.partition(g, update_chunks=U)
+    st, ds = D.init_state(g), D.datasets(g)
+    ref = R.run(g, 2, st, ds, parts=parts, keep_stagings=False)
+    n_upd = sum(1 for p in parts if any(g.ops[j].type in (SGD_MOM, STEP_INC) for j in range(*p)))
+    for k in range(len(parts) - n_upd + 1, len(parts)):
+        got = R.run(g, 2, st, ds, parts=parts, schedule=[(1, k, 1)], keep_stagings=False)
+        for i in ref.state:
+            assert _bitwise_equal(ref.state[i], got.state[i]), (k, g.tensors[i].name)
+        L = OG.live_set(g, parts, k)
+        assert any(g.tensors[i].kind == GRAD for i in L)  # not-yet-applied gradients
 
 
 def test_validate_rejects_bad_graphs():
