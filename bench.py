@@ -308,7 +308,7 @@ def reference_main(args):
             "cpu_baseline": {"value": p99, "unit": UNIT, "cores": cores(), "kind": "oracle",
                              "sample": o["sample"]},
             "e2e": {"value": p99, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line))
+    print(json.dumps(line), flush=True)
 
 
 def main():
@@ -431,7 +431,7 @@ def main():
                                 "kind": "oracle", "sample": o["sample"],
                                 "preempt_to_resume_ms": float(np.mean(o["p2r"])),
                                 "elapsed_s": o["elapsed_s"]}
-    print(json.dumps(line))
+    print(json.dumps(line), flush=True)
 
 
 if __name__ == "__main__":

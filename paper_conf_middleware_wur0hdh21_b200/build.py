@@ -50,7 +50,7 @@ def build(verbose: bool = False) -> str:
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
     if verbose:
-        print(LIB)
+        print(LIB, file=sys.stderr)
     return LIB
 
 

@@ -13,9 +13,14 @@
 // flight before the stores.  Roofline: HBM, 2 bytes of traffic per migrated byte.
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
+
+#ifndef SF_COPY_UNROLL
+#define SF_COPY_UNROLL 8
+#endif
 
 namespace sfk {
 
@@ -24,7 +29,7 @@ void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxe
 uint64_t launches() { return g_launches.load(std::memory_order_relaxed); }
 
 constexpr int kCopyThreads = 256;
-constexpr int kCopyUnroll = 4;
+constexpr int kCopyUnroll = SF_COPY_UNROLL;
 
 __device__ __forceinline__ uint4 load_chunk(const uint8_t* src, uint64_t j, uint64_t full,
                                             uint64_t nb) {
@@ -42,9 +47,14 @@ __device__ __forceinline__ uint4 load_chunk(const uint8_t* src, uint64_t j, uint
 
 __global__ void __launch_bounds__(kCopyThreads)
 mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t total, uint64_t per_block,
-              int64_t patch_iter) {
+              int64_t patch_iter, unsigned long long* tstamp) {
+  // optional device-side duration: [0] = earliest CTA start, [1] = latest CTA end (ns)
+  if (tstamp && threadIdx.x == 0) atomicMin(&tstamp[0], sfdev::globaltimer());
   const uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * per_block;
-  if (c0 >= total) return;
+  if (c0 >= total) {
+    if (tstamp && threadIdx.x == 0) atomicMax(&tstamp[1], sfdev::globaltimer());
+    return;
+  }
   const uint64_t c1 = min(c0 + per_block, total);
   __shared__ int s_first;
   if (threadIdx.x == 0) {
@@ -81,25 +91,34 @@ mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t total, uint64_t per_b
             v[u].x = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter));
             v[u].y = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter) >> 32);
           }
-          sfdev::st16(dst + j * 16, v[u]);
+          sfdev::st16_cs(dst + j * 16, v[u]);
         }
       }
+    }
+  }
+  if (tstamp) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicMax(&tstamp[1], sfdev::globaltimer());
     }
   }
 }
 
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
-                          int64_t patch_iter, cudaStream_t st) {
+                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp) {
   if (n <= 0 || total_chunks == 0) return cudaSuccess;
   // Grid: a multiple of the 148 SMs, enough bytes per CTA to amortise the search.
-  const uint64_t min_chunks = 2048;  // 32 KiB per CTA minimum
+  static const int bps = std::getenv("SF_COPY_BPS") ? std::atoi(std::getenv("SF_COPY_BPS")) : 8;
+  static const uint64_t min_chunks =
+      std::getenv("SF_COPY_MINCHUNKS") ? std::atoll(std::getenv("SF_COPY_MINCHUNKS")) : 2048;
   uint64_t blocks = (total_chunks + min_chunks - 1) / min_chunks;
-  blocks = std::min<uint64_t>(blocks, 148ull * 8);
+  blocks = std::min<uint64_t>(blocks, 148ull * bps);
   blocks = std::max<uint64_t>(blocks, 1);
   const uint64_t per_block = (total_chunks + blocks - 1) / blocks;
   blocks = (total_chunks + per_block - 1) / per_block;
   mtcopy_kernel<<<static_cast<unsigned>(blocks), kCopyThreads, 0, st>>>(d_descs, n, total_chunks,
-                                                                        per_block, patch_iter);
+                                                                        per_block, patch_iter, tstamp);
   count_launch();
   return cudaGetLastError();
 }

@@ -131,6 +131,7 @@ struct Slot {
   int id, cuda;
   cudaStream_t s_train = nullptr, s_infer = nullptr, s_mig = nullptr;
   cudaEvent_t ev_infer = nullptr;
+  unsigned long long* tstamp = nullptr;  // device {start, end} x 2 (pack/peer, unpack)
   int owner = -1;
   std::deque<Request*> q;
   std::thread dispatcher;
@@ -738,6 +739,17 @@ float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
 
 bool slot_has_inference(sf_runtime* rt, int s) { return !slot_of(rt, s).q.empty(); }
 
+// Device-side kernel duration stamps (globaltimer): reset {start, end} = {~0, 0}.
+cudaError_t tstamp_reset(unsigned long long* t, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(t, 0xFF, sizeof(unsigned long long), st);
+  return e == cudaSuccess ? cudaMemsetAsync(t + 1, 0, sizeof(unsigned long long), st) : e;
+}
+double tstamp_us(const unsigned long long* t) {  // after the stream completed
+  unsigned long long h[2] = {0, 0};
+  if (cudaMemcpy(h, t, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess || h[1] < h[0]) return -1.0;
+  return (h[1] - h[0]) * 1e-3;
+}
+
 // Poison the non-DATASET tensors of a released arena (test mode): a missing live tensor
 // then reads as NaN / -1 after resume.
 cudaError_t poison(Binding& b, cudaStream_t st) {
@@ -798,14 +810,15 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     // ---- host tier: pack (+ D2H), park, swap back in ------------------------------
     if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
     const bool zc = rt->cfg.host_mode == SF_HOST_ZC || B.staging == nullptr;
+    tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
     if (zc) {
       const CopyList& L = B.pack_zc[k];
-      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig);
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig, S.tstamp);
       cudaEventRecord(J.ev_b[src], S.s_mig);
     } else {
       const CopyList& L = B.pack[k];
-      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig);
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig, S.tstamp);
       cudaEventRecord(J.ev_b[src], S.s_mig);
       if (e == cudaSuccess)
         e = cudaMemcpyAsync(B.host_staging, B.staging, g.staging_total[k], cudaMemcpyDeviceToHost, S.s_mig);
@@ -817,7 +830,8 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     rt->cv.notify_all();
     lk.unlock();
     if ((e = spin_event(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
-    const float pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
+    float pack_us = static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
+    if (pack_us < 0.f) pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
     const float d2h_us = elapsed_us(J.ev_b[src], J.ev_c[src]);
     if (rt->cfg.poison_released) {
       if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
@@ -847,9 +861,10 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     cudaEventRecord(J.ev_a[dst], D.s_train);
     // the parked bytes live in the source binding's pinned staging; a ZC swap-in reads
     // them in place when resuming on the same slot, otherwise H2D + unpack
+    tstamp_reset(D.tstamp + 2, D.s_train);
     if (zc && dst == src) {
       const CopyList& L = BD.unpack_zc[k];
-      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train);
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
       cudaEventRecord(J.ev_b[dst], D.s_train);
     } else if (!BD.staging) {
       e = cudaErrorInvalidValue;
@@ -859,7 +874,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       cudaEventRecord(J.ev_b[dst], D.s_train);
       if (e == cudaSuccess) {
         const CopyList& L = BD.unpack[k];
-        e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train);
+        e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
       }
     }
     if (e != cudaSuccess) return cuda_fail(e, "unpack");
@@ -878,8 +893,9 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       return fail(SF_EINVAL, J.error);
     }
     const CopyList& L = it->second[k];
+    tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
-    e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S.s_mig);
+    e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S.s_mig, S.tstamp);
     if (e != cudaSuccess) return cuda_fail(e, "peer store");
     cudaEventRecord(J.ev_b[src], S.s_mig);
     Slot& T = slot_of(rt, target);
@@ -988,11 +1004,13 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
     if (e == cudaSuccess && stamp) {
       if (pending_peer_stats) {
-        peer_us = elapsed_us(J.ev_a[stats_slot], J.ev_b[stats_slot]);
+        peer_us = static_cast<float>(tstamp_us(slot_of(rt, stats_slot).tstamp));
+        if (peer_us < 0.f) peer_us = elapsed_us(J.ev_a[stats_slot], J.ev_b[stats_slot]);
         pending_peer_stats = false;
       } else {
         h2d_us = elapsed_us(J.ev_a[dev], J.ev_b[dev]);
-        unpack_us = elapsed_us(J.ev_b[dev], J.ev_c[dev]);
+        unpack_us = static_cast<float>(tstamp_us(S.tstamp + 2));
+        if (unpack_us < 0.f) unpack_us = elapsed_us(J.ev_b[dev], J.ev_c[dev]);
       }
     }
     lk.lock();
@@ -1114,6 +1132,7 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
     SF_CK(cudaStreamCreateWithPriority(&S->s_infer, cudaStreamNonBlocking, hi));
     SF_CK(cudaStreamCreateWithFlags(&S->s_mig, cudaStreamNonBlocking));
     SF_CK(cudaEventCreateWithFlags(&S->ev_infer, cudaEventDisableTiming));
+    SF_CK(cudaMalloc(&S->tstamp, 4 * sizeof(unsigned long long)));
     rt->slots.push_back(std::move(S));
   }
   // peer access between distinct physical devices (NVLink / NVSwitch)
@@ -1181,6 +1200,7 @@ void sf_destroy(sf_runtime* rt) {
     cudaStreamDestroy(S->s_infer);
     cudaStreamDestroy(S->s_mig);
     cudaEventDestroy(S->ev_infer);
+    cudaFree(S->tstamp);
   }
   delete rt;
 }

@@ -18,8 +18,10 @@ struct DCopy {
 
 // Multi-tensor copy / pack / unpack / peer-store over a device descriptor array.
 // patch_iter >= 0 overwrites bytes [16,24) of descriptor 0's destination (staging iter).
+// tstamp (optional, device): {earliest CTA start, latest CTA end} in %globaltimer ns; the
+// caller initialises it to {~0, 0}.
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
-                          int64_t patch_iter, cudaStream_t st);
+                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp = nullptr);
 cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st);
 // Single-buffer copy with pointer arguments (request I/O; 16-B aligned, nbytes % 4 == 0).
 cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st);
