@@ -233,6 +233,68 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
     return S
 
 
+def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, gloo):
+    """N>1: ranks (2i, 2i+1) ping-pong one training job; each request preempts it into the
+    partner's arena (peer-store kernel over NVLink, CUDA IPC mapping); pairs are independent."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_wur0hdh21_b200.pairs import PairLink, RuntimeOps, run_pair_steps
+    from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches
+    from sf_inputs import data as D
+
+    g, gi = build_workload(args.batch, args.spatial_div)
+    rt = Runtime([local_dev, -1], exclusive=True, auto_preempt=True, defer_migration=bool(args.defer))
+    gh = rt.register(g)
+    info = gh.partition(update_chunks=args.update_chunks)
+    gh.bind(0, staging=False, host_staging=False)
+    arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
+    link = PairLink(gloo)
+    gh.load(0, arrays if link.starts_holding else {i: a for i, a in arrays.items()
+                                                   if g.tensors[i].kind == 3})
+    ghi = rt.register(gi, priority=1)
+    ghi.partition()
+    ghi.bind(0, staging=False)
+    ghi.load(0, arrays_i)
+    rt.import_arena(gh, 1, link.exchange_bytes(rt.export_arena(gh, 0)))
+    xs = D.infer_inputs(gi, 64)
+    dev = torch.device("cuda", local_dev)
+    if host_io:
+        x_t, out_t = torch.from_numpy(xs).pin_memory(), torch.zeros(64, 1, 1000).pin_memory()
+    else:
+        x_t, out_t = torch.from_numpy(xs).to(dev), torch.zeros(64, 1, 1000, device=dev)
+    ops = RuntimeOps(rt, gh, ghi, 0, 1, [x.data_ptr() for x in x_t], [o.data_ptr() for o in out_t],
+                     sub_ms=0.06, rng=np.random.default_rng(4321 + args.rank))
+    if link.starts_holding:
+        ops.start()
+    Sw = run_pair_steps(link, ops, 0, warmup)
+    dist.barrier(group=gloo)
+    torch.cuda.synchronize(dev)
+    sampler = ClockSampler(local_dev).__enter__() if not host_io else None
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    launches0 = kernel_launches()
+    S = run_pair_steps(link, ops, steps, 0, holding=Sw["holding_at_end"])
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev1.record()
+    torch.cuda.synchronize(dev)
+    dist.barrier(group=gloo)
+    if sampler:
+        sampler.__exit__()
+    S["region_ms"] = ev0.elapsed_time(ev1)
+    S["launches"] = kernel_launches() - launches0
+    S["clocks"] = sampler.summary() if sampler else None
+    S["n_subgraphs"] = gh.n_subgraphs
+    S["sub_ms"] = 0.06
+    S["xfer_us"] = [c["xfer_us"] for c in S["out"]]
+    S["bytes"] = [c["bytes"] for c in S["out"]]
+    if S["holding_at_end"] and ops.job is not None:
+        rt.stop_job(ops.job)
+        rt.wait_job(ops.job, 120)
+    dist.barrier(group=gloo)
+    rt.close()
+    return S
+
+
 # ------------------------------------------------------------------------------------------
 def oracle_sample(args, steps: int):
     """CPU oracle on a bounded sample: each distinct sampled subgraph timed once."""
@@ -311,6 +373,59 @@ def reference_main(args):
     print(json.dumps(line), flush=True)
 
 
+def pair_main(args, local):
+    """N>1 bench: independent GPU pairs, peer tier over NVLink."""
+    import torch.distributed as dist
+    gloo = dist.new_group(backend="gloo")
+    main_s = run_pair_arm(args, local, args.steps, args.warmup, host_io=False, gloo=gloo)
+    e2e_s = run_pair_arm(args, local, max(20, args.steps // 2), 4, host_io=True, gloo=gloo)
+    allv = [None] * args.world
+    dist.all_gather_object(allv, {"main": main_s, "e2e": e2e_s}, group=gloo)
+    dist.barrier(group=gloo)
+    if args.rank != 0:
+        dist.destroy_process_group()
+        return
+    lat = sum((a["main"]["lat"] for a in allv), [])
+    pre = sum((a["main"]["pre"] for a in allv), [])
+    p2r = sum((a["main"]["p2r"] for a in allv), [])
+    xfer = np.asarray(sum((a["main"]["xfer_us"] for a in allv), []), np.float64)
+    byts = np.asarray(sum((a["main"]["bytes"] for a in allv), []), np.float64)
+    # each adopted job migrates exactly once, so its counter is that migration's live bytes
+    live = float(np.median(byts)) if len(byts) else float("nan")
+    ok = xfer > 0
+    link_gbs = float(live / (np.median(xfer[ok]) * 1e-6) / 1e9) if ok.any() else None
+    E = sum((a["e2e"]["lat"] for a in allv), [])
+    region_ms = max(a["main"]["region_ms"] for a in allv)
+    nvl_peak = 770.0  # B200_PROFILING.md: measured peer copy per direction (900 nominal)
+    line = {
+        "metric": METRIC, "value": pct(lat, 99), "unit": UNIT, "n_gpus": args.world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
+        "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded: glorot weights, U[0,1) features, uniform labels)",
+        "config": {"workload": f"C4@{args.world}GPU: {args.world // 2} independent GPU pairs, each one "
+                               "ResNet-50-shaped training job ping-ponged by batch-1 requests "
+                               "(peer-tier migration, CUDA IPC + NVLink peer store)",
+                   "batch": args.batch, "update_chunks": args.update_chunks,
+                   "parallelism": f"{args.world // 2} pairs", "tier": "peer (NVLink)"},
+        "p50_ms": pct(lat, 50), "p95_ms": pct(lat, 95), "p99_ms": pct(lat, 99),
+        "preempt_latency_p50_ms": pct(pre, 50), "preempt_latency_p99_ms": pct(pre, 99),
+        "preempt_to_resume_p50_ms": pct(p2r, 50), "preempt_to_resume_p99_ms": pct(p2r, 99),
+        "migration": {"live_bytes_median": live, "peer_store_us_median": float(np.median(xfer[ok])) if ok.any() else None,
+                      "peer_gbs": link_gbs},
+        "roofline": {"kernel": "mtcopy_kernel (peer store: local arena -> partner arena over NVLink)",
+                     "bound": "nvlink", "achieved": link_gbs, "peak": nvl_peak, "unit": "GB/s",
+                     "frac": (link_gbs / nvl_peak) if link_gbs else None, "traffic": None,
+                     "peak_source": "B200_PROFILING.md measured peer copy (770 GB/s/dir)",
+                     "algorithmic_bytes": "live bytes per migration (one direction)"},
+        "e2e": {"value": pct(E, 99), "unit": UNIT, "h2d_bytes_per_step": 2048 * 4,
+                "d2h_bytes_per_step": 1000 * 4, "p50_ms": pct(E, 50)},
+        "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),
+        "clocks": allv[0]["main"]["clocks"],
+    }
+    print(json.dumps(line), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -329,6 +444,8 @@ def main():
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("SF_BENCH_SAME_GPU") == "1":
+        local = 0  # functional check of the N>1 path on a 1-GPU box (not a scaling number)
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
         return reference_main(args)
@@ -340,11 +457,16 @@ def main():
     if args.world > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if os.environ.get("SF_BENCH_SAME_GPU") == "1":
+            dist.init_process_group("gloo")  # NCCL refuses two ranks on one device
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         dist.barrier()
         __graft_entry__.build()
     torch.cuda.set_device(local)
 
+    if args.world > 1:
+        return pair_main(args, local)
     main_s = run_arm(args, local, args.steps, args.warmup, host_io=False)
     e2e_steps = max(20, args.steps // 2)
     e2e_s = run_arm(args, local, e2e_steps, 3, host_io=True, measure=False)

@@ -128,7 +128,9 @@ typedef uint64_t sf_req_id;
 
 typedef struct sf_config {
   int32_t n_devices;             /* logical device slots */
-  const int32_t* cuda_ordinals;  /* host array [n_devices]: CUDA device of each slot */
+  const int32_t* cuda_ordinals;  /* host array [n_devices]: CUDA device of each slot, or -1
+                                    for a REMOTE slot: another process's device whose arena
+                                    is mapped with sf_import_arena (process-per-GPU peers) */
   int32_t exclusive_gpu;         /* 1 (default behaviour): no two models' subgraphs co-run
                                     on a device; 0: free co-run baseline
                                     (multi-threaded TF) */
@@ -212,7 +214,8 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id g, int32_t dev, void* arena, void*
 /* ---- training jobs, preemption --------------------------------------------------- */
 enum sf_job_state {
   SF_JOB_RUNNING = 0, SF_JOB_STOPPING = 1, SF_JOB_MIGRATING = 2, SF_JOB_PREEMPTED = 3,
-  SF_JOB_DONE = 4, SF_JOB_FAILED = 5
+  SF_JOB_DONE = 4, SF_JOB_FAILED = 5,
+  SF_JOB_MIGRATED_OUT = 6 /* state copied into a REMOTE slot; the partner adopts the job */
 };
 typedef struct sf_job_info {
   int32_t state;        /* sf_job_state */
@@ -269,6 +272,31 @@ sf_status sf_job_query(sf_runtime* rt, sf_job_id job, sf_job_info* out);
 sf_status sf_wait_job(sf_runtime* rt, sf_job_id job, int64_t timeout_ns);
 /* Ask a running job to stop at its next iteration boundary and finish. */
 sf_status sf_stop_job(sf_runtime* rt, sf_job_id job);
+
+/* ---- process-per-GPU peers (CUDA IPC) ------------------------------------------------
+ * The paper migrates a job between devices of one machine; with
+ * one process per GPU the target arena lives in another process.  Each process exports its
+ * arena once; the partner maps it into a REMOTE slot; a preemption to that slot runs the
+ * peer-store kernel straight into the partner's HBM over NVLink, waits for the copy, and
+ * leaves the job SF_JOB_MIGRATED_OUT with its cut in sf_cut_info; the partner process then
+ * calls sf_adopt_job with that cut (handoff message carried by the caller, e.g.
+ * torch.distributed). */
+typedef struct sf_ipc_arena {
+  uint8_t handle[64];     /* cudaIpcMemHandle_t of the allocation holding the arena */
+  uint64_t offset;        /* arena offset inside that allocation */
+  uint64_t arena_bytes;
+  int32_t cuda_ordinal;   /* device of the exporting process (informational) */
+  int32_t pad;
+} sf_ipc_arena;
+/* Export the arena of graph g bound on local slot dev. */
+sf_status sf_export_arena(sf_runtime* rt, sf_graph_id g, int32_t dev, sf_ipc_arena* out);
+/* Map a partner's exported arena as REMOTE slot `slot` of graph g (opened on the device of
+ * the first local slot g is bound to) and build peer-store lists from every local binding. */
+sf_status sf_import_arena(sf_runtime* rt, sf_graph_id g, int32_t slot, const sf_ipc_arena* a);
+/* Start a job whose live state at cut (iter, k) is already in dev's arena (copied there by a
+ * partner's peer store); runs until `iters` iterations are complete. */
+sf_status sf_adopt_job(sf_runtime* rt, sf_graph_id g, int32_t dev, int64_t iters, int64_t iter,
+                       int32_t k, int32_t auto_target, sf_job_id* out);
 
 /* ---- inference (the preempter) --------------------------------------------------- */
 typedef struct sf_timing {

@@ -24,7 +24,8 @@ SF_HOST_CE = 0
 SF_HOST_ZC = 1
 SF_PART_PER_LAYER_PHASE = 0
 SF_PART_MAX_OPS = 1
-JOB_STATES = {0: "running", 1: "stopping", 2: "migrating", 3: "preempted", 4: "done", 5: "failed"}
+JOB_STATES = {0: "running", 1: "stopping", 2: "migrating", 3: "preempted", 4: "done", 5: "failed",
+              6: "migrated_out"}
 EV_TRAIN, EV_INFER, EV_MIGRATE = 0, 1, 2
 INFER_JOB_FLAG = 1 << 20
 
@@ -93,6 +94,11 @@ class sf_cut_request(C.Structure):
     _fields_ = [("iter", C.c_int64), ("k", C.c_int32), ("target", C.c_int32)]
 
 
+class sf_ipc_arena(C.Structure):
+    _fields_ = [("handle", C.c_uint8 * 64), ("offset", C.c_uint64), ("arena_bytes", C.c_uint64),
+                ("cuda_ordinal", C.c_int32), ("pad", C.c_int32)]
+
+
 class sf_copy_desc(C.Structure):
     _fields_ = [("src", C.c_void_p), ("dst", C.c_void_p), ("nbytes", C.c_uint64),
                 ("span", C.c_uint64)]
@@ -119,6 +125,10 @@ PROTOTYPES = {
     "sf_start_training": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int64, C.c_int32,
                                 _P(sf_cut_request), C.c_int32, _P(C.c_uint32)]),
     "sf_preempt": (_st, [_vp, C.c_uint32, C.c_int32, _P(sf_cut_info)]),
+    "sf_export_arena": (_st, [_vp, C.c_uint32, C.c_int32, _P(sf_ipc_arena)]),
+    "sf_import_arena": (_st, [_vp, C.c_uint32, C.c_int32, _P(sf_ipc_arena)]),
+    "sf_adopt_job": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int64, C.c_int64, C.c_int32, C.c_int32,
+                           _P(C.c_uint32)]),
     "sf_resume": (_st, [_vp, C.c_uint32, C.c_int32]),
     "sf_job_query": (_st, [_vp, C.c_uint32, _P(sf_job_info)]),
     "sf_wait_job": (_st, [_vp, C.c_uint32, C.c_int64]),

@@ -15,6 +15,7 @@
 // B200 choices are described in DESIGN.md: cut at subgraph boundaries with in-flight
 // activations (reading Q1), one multi-tensor pack / unpack / peer-store launch per cut,
 // stream-ordered resume of a pre-instantiated CUDA graph on the target.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <time.h>
 
@@ -77,6 +78,9 @@ struct CopyList {
 
 struct Binding {
   int slot = -1;
+  bool remote = false;       // partner arena mapped over CUDA IPC (no versions, no staging)
+  void* ipc_base = nullptr;  // cudaIpcOpenMemHandle mapping (closed at sf_destroy)
+  int ipc_device = -1;
   uint8_t* arena = nullptr;
   uint8_t* staging = nullptr;
   uint8_t* host_staging = nullptr;      // pinned host (host pointer)
@@ -129,6 +133,7 @@ struct Request {
 
 struct Slot {
   int id, cuda;
+  bool remote = false;  // another process's device (arena mapped over CUDA IPC)
   cudaStream_t s_train = nullptr, s_infer = nullptr, s_mig = nullptr;
   cudaEvent_t ev_infer = nullptr;
   unsigned long long* tstamp = nullptr;  // device {start, end} x 2 (pack/peer, unpack)
@@ -160,6 +165,7 @@ struct Job {
   int resume_dev = -1;
   bool stop_req = false;
   bool stamp_resume = false;
+  bool adopted_pending = false;  // first launch of an adopted job: stamp time, no copy stats
   int n_preempt = 0;
   uint64_t migrated = 0;
   double pack_us = 0, xfer_us = 0, unpack_us = 0;
@@ -714,6 +720,7 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   int cur = 0;
   cudaGetDevice(&cur);
   for (size_t s = 0; s < n; ++s) {
+    if (rt->slots[s]->remote) continue;
     SF_CK(cudaSetDevice(rt->slots[s]->cuda));
     SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
@@ -733,7 +740,10 @@ cudaError_t spin_event(cudaEvent_t ev) {
 
 float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
   float ms = 0.f;
-  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) return 0.f;
+  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+    cudaGetLastError();  // statistics only: never leave a stale error for the next launch
+    return -1.f;
+  }
   return ms * 1000.f;
 }
 
@@ -746,7 +756,11 @@ cudaError_t tstamp_reset(unsigned long long* t, cudaStream_t st) {
 }
 double tstamp_us(const unsigned long long* t) {  // after the stream completed
   unsigned long long h[2] = {0, 0};
-  if (cudaMemcpy(h, t, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess || h[1] < h[0]) return -1.0;
+  if (cudaMemcpy(h, t, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess) {
+    cudaGetLastError();
+    return -1.0;
+  }
+  if (h[1] < h[0]) return -1.0;
   return (h[1] - h[0]) * 1e-3;
 }
 
@@ -899,6 +913,26 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     if (e != cudaSuccess) return cuda_fail(e, "peer store");
     cudaEventRecord(J.ev_b[src], S.s_mig);
     Slot& T = slot_of(rt, target);
+    if (T.remote) {
+      // process-per-GPU handoff: the copy must be complete before the partner adopts the job
+      if ((e = spin_event(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
+      const float us = static_cast<float>(tstamp_us(S.tstamp));
+      if (rt->cfg.poison_released) {
+        if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
+        if ((e = cudaStreamSynchronize(S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison sync");
+      }
+      lk.lock();
+      J.mig_enqueued = true;
+      J.dev = target;
+      J.n_preempt++;
+      J.migrated += g.live_bytes[k];
+      J.pack_us = 0.0;
+      J.unpack_us = 0.0;
+      J.xfer_us = us >= 0.f ? us : elapsed_us(J.ev_a[src], J.ev_b[src]);
+      J.state = SF_JOB_MIGRATED_OUT;
+      rt->cv.notify_all();
+      return SF_OK;
+    }
     // stream-ordered resume: the target's training stream waits on the source's copy
     // (a cross-device event wait when the slots are different GPUs)
     e = cudaStreamWaitEvent(T.s_train, J.ev_b[src], 0);
@@ -972,7 +1006,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       const int src = J.dev;
       const bool peer = J.preempt_target != SF_TARGET_HOST;
       if (do_preempt(rt, J, lk) != SF_OK) break;
-      if (J.state == SF_JOB_DONE) break;
+      if (J.state == SF_JOB_DONE || J.state == SF_JOB_MIGRATED_OUT) break;
       if (peer) { pending_peer_stats = true; stats_slot = src; }
       continue;
     }
@@ -1002,7 +1036,9 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     if (e == cudaSuccess) e = spin_event(J.ev_sub[dev]);
     const uint64_t t1 = now_ns();
     float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
-    if (e == cudaSuccess && stamp) {
+    if (e == cudaSuccess && stamp && J.adopted_pending) {
+      J.adopted_pending = false;  // the copy was timed by the exporting process
+    } else if (e == cudaSuccess && stamp) {
       if (pending_peer_stats) {
         peer_us = static_cast<float>(tstamp_us(slot_of(rt, stats_slot).tstamp));
         if (peer_us < 0.f) peer_us = elapsed_us(J.ev_a[stats_slot], J.ev_b[stats_slot]);
@@ -1016,7 +1052,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     lk.lock();
     if (stamp) {
       J.last_resume = t0;
-      if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += h2d_us; }
+      if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += std::max(h2d_us, 0.f); }
       if (peer_us >= 0.f) { J.pack_us = 0.0; J.xfer_us = peer_us; J.unpack_us = 0.0; }
     }
     if (e != cudaSuccess) {
@@ -1121,6 +1157,14 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
   rt->trace.reserve(std::min<size_t>(rt->trace_cap, 1 << 16));
   for (int s = 0; s < cfg->n_devices; ++s) {
     const int c = cfg->cuda_ordinals[s];
+    if (c == -1) {
+      auto S = std::make_unique<Slot>();
+      S->id = s;
+      S->cuda = -1;
+      S->remote = true;
+      rt->slots.push_back(std::move(S));
+      continue;
+    }
     if (c < 0 || c >= ndev) return fail(SF_EINVAL, "cuda ordinal out of range");
     auto S = std::make_unique<Slot>();
     S->id = s;
@@ -1138,7 +1182,7 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
   // peer access between distinct physical devices (NVLink / NVSwitch)
   for (auto& a : rt->slots)
     for (auto& b : rt->slots)
-      if (a->cuda != b->cuda) {
+      if (!a->remote && !b->remote && a->cuda != b->cuda) {
         int can = 0;
         SF_CK(cudaDeviceCanAccessPeer(&can, a->cuda, b->cuda));
         if (!can) return fail(SF_EUNSUPPORTED, "no peer access between devices");
@@ -1149,7 +1193,8 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
         cudaGetLastError();
       }
   sf_runtime* p = rt.release();
-  for (auto& S : p->slots) S->dispatcher = std::thread(dispatcher_main, p, S.get());
+  for (auto& S : p->slots)
+    if (!S->remote) S->dispatcher = std::thread(dispatcher_main, p, S.get());
   *out = p;
   return SF_OK;
 }
@@ -1174,12 +1219,20 @@ void sf_destroy(sf_runtime* rt) {
   for (auto& S : rt->slots)
     if (S->dispatcher.joinable()) S->dispatcher.join();
   for (auto& S : rt->slots) {
+    if (S->remote) continue;
     cudaSetDevice(S->cuda);
     cudaDeviceSynchronize();
   }
   for (auto& G : rt->graphs)
     for (auto& B : G->bind) {
       if (!B) continue;
+      if (B->remote) {
+        if (B->ipc_base) {
+          cudaSetDevice(B->ipc_device);
+          cudaIpcCloseMemHandle(B->ipc_base);
+        }
+        continue;
+      }
       cudaSetDevice(rt->slots[B->slot]->cuda);
       for (auto v : B->versions) cudaGraphExecDestroy(v);
       for (void* d : B->dev_allocs) cudaFree(d);
@@ -1188,6 +1241,7 @@ void sf_destroy(sf_runtime* rt) {
     }
   for (auto& J : rt->jobs)
     for (size_t s = 0; s < J->ev_sub.size(); ++s) {
+      if (rt->slots[s]->remote) continue;
       cudaSetDevice(rt->slots[s]->cuda);
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_a[s]);
@@ -1195,6 +1249,7 @@ void sf_destroy(sf_runtime* rt) {
       cudaEventDestroy(J->ev_c[s]);
     }
   for (auto& S : rt->slots) {
+    if (S->remote) continue;
     cudaSetDevice(S->cuda);
     cudaStreamDestroy(S->s_train);
     cudaStreamDestroy(S->s_infer);
@@ -1309,6 +1364,7 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
   Graph& g = *gp;
   if (dev < 0 || dev >= static_cast<int>(rt->slots.size())) return fail(SF_EINVAL, "bad slot");
   if (g.bind[dev]) return fail(SF_ESTATE, "slot already bound");
+  if (rt->slots[dev]->remote) return fail(SF_EINVAL, "remote slots are mapped with sf_import_arena");
   if (!arena || reinterpret_cast<uintptr_t>(arena) % kAlign)
     return fail(SF_EINVAL, "arena must be a 256-B aligned device pointer");
   if (staging && reinterpret_cast<uintptr_t>(staging) % kAlign)
@@ -1408,6 +1464,7 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
   for (size_t o = 0; o < g.bind.size(); ++o) {
     if (static_cast<int>(o) == dev || !g.bind[o]) continue;
     if (sf_status s = build_peer_lists(rt, g, *g.bind[dev], *g.bind[o])) return s;
+    if (g.bind[o]->remote) continue;  // a remote arena is only ever a destination here
     if (sf_status s = build_peer_lists(rt, g, *g.bind[o], *g.bind[dev])) return s;
   }
   SF_CK(cudaSetDevice(S.cuda));
@@ -1415,15 +1472,16 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
   return SF_OK;
 }
 
-sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters,
-                            int32_t auto_target, const sf_cut_request* sched, int32_t n_sched,
-                            sf_job_id* out) {
+static sf_status start_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters,
+                           int32_t auto_target, const sf_cut_request* sched, int32_t n_sched,
+                           int64_t it0, int32_t k0, sf_job_id* out) {
   if (!rt || !out || n_sched < 0 || (n_sched > 0 && !sched)) return fail(SF_EINVAL, "null argument");
   std::lock_guard<std::mutex> lk(rt->m);
   Graph* g = get_graph(rt, gid);
   if (!g || !g->partitioned) return fail(SF_ESTATE, "graph not partitioned");
-  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev])
-    return fail(SF_EINVAL, "slot not bound");
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || rt->slots[dev]->remote)
+    return fail(SF_EINVAL, "slot not bound locally");
+  if (k0 < 0 || k0 >= static_cast<int>(g->parts.size()) || it0 < 0) return fail(SF_EINVAL, "bad cut");
   if (auto_target != SF_TARGET_HOST &&
       (auto_target < 0 || auto_target >= static_cast<int>(rt->slots.size()) || !g->bind[auto_target]))
     return fail(SF_EINVAL, "auto_target not bound");
@@ -1435,9 +1493,13 @@ sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_
   J->dev = dev;
   J->iters = iters;
   J->auto_target = auto_target;
+  J->it = it0;
+  J->k = k0;
+  J->stamp_resume = it0 > 0 || k0 > 0;  // an adopted job: its first launch is the resume
+  J->adopted_pending = J->stamp_resume;
   // DATASET contents are final once training starts: refresh padded-pitch copies
   for (auto& Bp : g->bind) {
-    if (!Bp) continue;
+    if (!Bp || Bp->remote) continue;
     for (auto& [t, sh] : Bp->shadow) {
       const Tensor& x = g->T[t];
       SF_CK(cudaSetDevice(rt->slots[Bp->slot]->cuda));
@@ -1462,6 +1524,84 @@ sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_
   rt->jobs.push_back(std::move(J));
   jp->driver = std::thread(driver_main, rt, jp);
   *out = jp->id;
+  return SF_OK;
+}
+
+sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters,
+                            int32_t auto_target, const sf_cut_request* sched, int32_t n_sched,
+                            sf_job_id* out) {
+  return start_job(rt, gid, dev, iters, auto_target, sched, n_sched, 0, 0, out);
+}
+
+sf_status sf_adopt_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters, int64_t iter,
+                       int32_t k, int32_t auto_target, sf_job_id* out) {
+  return start_job(rt, gid, dev, iters, auto_target, nullptr, 0, iter, k, out);
+}
+
+sf_status sf_export_arena(sf_runtime* rt, sf_graph_id gid, int32_t dev, sf_ipc_arena* out) {
+  if (!rt || !out) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || g->bind[dev]->remote)
+    return fail(SF_EINVAL, "slot not bound locally");
+  Binding& B = *g->bind[dev];
+  SF_CK(cudaSetDevice(rt->slots[dev]->cuda));
+  // driver entry point resolved at run time (no link-time libcuda dependency)
+  using GetRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+  static GetRange get_range = nullptr;
+  if (!get_range) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return fail(SF_ECUDA, "cuMemGetAddressRange entry point unavailable");
+    get_range = reinterpret_cast<GetRange>(fn);
+  }
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (get_range(&base, &size, reinterpret_cast<CUdeviceptr>(B.arena)) != CUDA_SUCCESS)
+    return fail(SF_ECUDA, "cuMemGetAddressRange failed for the arena");
+  cudaIpcMemHandle_t h;
+  SF_CK(cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base)));
+  std::memset(out, 0, sizeof(*out));
+  std::memcpy(out->handle, &h, sizeof(h));
+  out->offset = reinterpret_cast<uint64_t>(B.arena) - static_cast<uint64_t>(base);
+  out->arena_bytes = g->arena_bytes;
+  out->cuda_ordinal = rt->slots[dev]->cuda;
+  return SF_OK;
+}
+
+sf_status sf_import_arena(sf_runtime* rt, sf_graph_id gid, int32_t slot, const sf_ipc_arena* a) {
+  if (!rt || !a) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* gp = get_graph(rt, gid);
+  if (!gp || !gp->partitioned) return fail(SF_ESTATE, "graph not partitioned");
+  Graph& g = *gp;
+  if (slot < 0 || slot >= static_cast<int>(rt->slots.size()) || !rt->slots[slot]->remote)
+    return fail(SF_EINVAL, "not a remote slot");
+  if (g.bind[slot]) return fail(SF_ESTATE, "remote slot already mapped");
+  if (a->arena_bytes != g.arena_bytes) return fail(SF_EINVAL, "arena layout mismatch");
+  int local = -1;
+  for (size_t o = 0; o < g.bind.size(); ++o)
+    if (g.bind[o] && !g.bind[o]->remote) { local = static_cast<int>(o); break; }
+  if (local < 0) return fail(SF_ESTATE, "bind a local slot before importing a remote arena");
+  const int cuda = rt->slots[local]->cuda;
+  SF_CK(cudaSetDevice(cuda));
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, a->handle, sizeof(h));
+  void* p = nullptr;
+  SF_CK(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+  auto b = std::make_unique<Binding>();
+  b->slot = slot;
+  b->remote = true;
+  b->ipc_base = p;
+  b->ipc_device = cuda;
+  b->arena = static_cast<uint8_t*>(p) + a->offset;
+  g.bind[slot] = std::move(b);
+  for (size_t o = 0; o < g.bind.size(); ++o) {
+    if (static_cast<int>(o) == slot || !g.bind[o] || g.bind[o]->remote) continue;
+    if (sf_status s = build_peer_lists(rt, g, *g.bind[o], *g.bind[slot])) return s;
+  }
   return SF_OK;
 }
 
@@ -1534,7 +1674,9 @@ sf_status sf_wait_job(sf_runtime* rt, sf_job_id jid, int64_t timeout_ns) {
   std::unique_lock<std::mutex> lk(rt->m);
   Job* J = get_job(rt, jid);
   if (!J) return fail(SF_EINVAL, "bad job id");
-  auto done = [&] { return J->state == SF_JOB_DONE || J->state == SF_JOB_FAILED; };
+  auto done = [&] {
+    return J->state == SF_JOB_DONE || J->state == SF_JOB_FAILED || J->state == SF_JOB_MIGRATED_OUT;
+  };
   if (timeout_ns < 0) rt->cv.wait(lk, done);
   else if (!rt->cv.wait_for(lk, std::chrono::nanoseconds(timeout_ns), done))
     return fail(SF_ETIMEOUT, "job still running");
@@ -1558,8 +1700,8 @@ sf_status sf_submit_inference(sf_runtime* rt, sf_graph_id gid, int32_t dev, cons
   std::lock_guard<std::mutex> lk(rt->m);
   Graph* g = get_graph(rt, gid);
   if (!g || !g->partitioned) return fail(SF_ESTATE, "graph not partitioned");
-  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev])
-    return fail(SF_EINVAL, "slot not bound");
+  if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || rt->slots[dev]->remote)
+    return fail(SF_EINVAL, "slot not bound locally");
   if (g->input_tid < 0 || g->output_tid < 0) return fail(SF_EINVAL, "graph has no INPUT/OUTPUT");
   auto r = std::make_unique<Request>();
   r->id = rt->next_req++;

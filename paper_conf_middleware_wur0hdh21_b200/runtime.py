@@ -172,6 +172,23 @@ class Runtime:
                                       C.byref(j)), "sf_start_training")
         return j.value
 
+    def adopt_job(self, gh: GraphHandle, slot: int, iters: int, it: int, k: int,
+                  auto_target: int) -> int:
+        """Continue a job whose cut-(it, k) state a partner peer-stored into this slot."""
+        j = C.c_uint32()
+        check(lib().sf_adopt_job(self.h, gh.gid, slot, iters, it, k, auto_target, C.byref(j)),
+              "sf_adopt_job")
+        return j.value
+
+    def export_arena(self, gh: GraphHandle, slot: int) -> bytes:
+        a = A.sf_ipc_arena()
+        check(lib().sf_export_arena(self.h, gh.gid, slot, C.byref(a)), "sf_export_arena")
+        return bytes(C.string_at(C.addressof(a), C.sizeof(a)))
+
+    def import_arena(self, gh: GraphHandle, slot: int, blob: bytes) -> None:
+        a = A.sf_ipc_arena.from_buffer_copy(blob)
+        check(lib().sf_import_arena(self.h, gh.gid, slot, C.byref(a)), "sf_import_arena")
+
     def preempt(self, job: int, target: int) -> dict:
         c = A.sf_cut_info()
         check(lib().sf_preempt(self.h, job, target, C.byref(c)), "sf_preempt")
