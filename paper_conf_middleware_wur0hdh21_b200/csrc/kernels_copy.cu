@@ -164,6 +164,30 @@ cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_
   return cudaGetLastError();
 }
 
+// 2-D pitched copy (rows x width bytes, width % 4 == 0, 4-B aligned pitches): pads or unpads
+// a GEMM operand whose row pitch is not a multiple of 16 B (TMA tensor-map requirement).
+__global__ void copy2d_kernel(const uint8_t* __restrict__ src, uint64_t spitch, uint8_t* __restrict__ dst,
+                              uint64_t dpitch, uint64_t rows, uint64_t width) {
+  const uint64_t words = width / 4;
+  const uint64_t total = rows * words;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < total;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    const uint64_t r = i / words, w = i % words;
+    reinterpret_cast<uint32_t*>(dst + r * dpitch)[w] = reinterpret_cast<const uint32_t*>(src + r * spitch)[w];
+  }
+}
+
+cudaError_t launch_copy2d(const void* src, uint64_t spitch, void* dst, uint64_t dpitch, uint64_t rows,
+                          uint64_t width, cudaStream_t st) {
+  if (rows == 0 || width == 0) return cudaSuccess;
+  const uint64_t total = rows * (width / 4);
+  const uint64_t blocks = std::min<uint64_t>((total + 255) / 256, 148ull * 8);
+  copy2d_kernel<<<static_cast<unsigned>(blocks), 256, 0, st>>>(static_cast<const uint8_t*>(src), spitch,
+                                                               static_cast<uint8_t*>(dst), dpitch, rows, width);
+  count_launch();
+  return cudaGetLastError();
+}
+
 // FEED: x = pool[(step mod P) * x_bytes ...] (data cursor read on device, reading Q3).
 __global__ void feed_kernel(const uint8_t* __restrict__ pool, const int32_t* __restrict__ step,
                             uint8_t* __restrict__ x, uint64_t x_bytes, int64_t period) {

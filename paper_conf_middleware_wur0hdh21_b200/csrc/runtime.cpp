@@ -20,6 +20,7 @@
 #include <time.h>
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <condition_variable>
 #include <cstring>
@@ -95,6 +96,10 @@ struct Binding {
   // padded-pitch copies of DATASET GEMM operands whose row pitch is not 16-B aligned (the
   // TMA tensor-map requirement); refreshed from the arena at sf_start_training
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
+  // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
+  // refreshed inside the version graph (copy2d before / after the GEMM)
+  struct PadBuf { float* p = nullptr; int pitch = 0; };
+  std::map<int, std::array<PadBuf, 3>> gemm_pad;  // op index -> {A, B, C}
   std::vector<void*> dev_allocs;
 };
 
@@ -596,6 +601,32 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         if (sa != c.b.shadow.end()) { ga.A = sa->second.first; ga.lda = sa->second.second; }
         auto sb = c.b.shadow.find(o.in[1]);
         if (sb != c.b.shadow.end()) { ga.B = sb->second.first; ga.ldb = sb->second.second; }
+        auto pd = c.b.gemm_pad.find(j);
+        if (pd != c.b.gemm_pad.end()) {
+          const auto& pads = pd->second;
+          const Tensor* xs[3] = {&A, &B, &C};
+          const int ids[3] = {o.in[0], o.in[1], o.out[0]};
+          for (int q = 0; q < 3; ++q) {
+            if (!pads[q].p) continue;
+            const Tensor& x = *xs[q];
+            const bool load = q < 2 || ga.acc;  // C is read only when accumulating
+            if (load) {
+              err = sfk::launch_copy2d(c.ptr(ids[q]), static_cast<uint64_t>(x.cols) * 4, pads[q].p,
+                                       static_cast<uint64_t>(pads[q].pitch) * 4, x.rows,
+                                       static_cast<uint64_t>(x.cols) * 4, c.st);
+              if (err != cudaSuccess) return fail(SF_ECUDA, std::string("pad: ") + cudaGetErrorString(err));
+            }
+          }
+          if (pads[0].p) { ga.A = pads[0].p; ga.lda = pads[0].pitch; }
+          if (pads[1].p) { ga.B = pads[1].p; ga.ldb = pads[1].pitch; }
+          if (pads[2].p) { ga.C = pads[2].p; ga.ldc = pads[2].pitch; }
+          err = sfk::launch_gemm(ga, c.st);
+          if (err == cudaSuccess && pads[2].p)
+            err = sfk::launch_copy2d(pads[2].p, static_cast<uint64_t>(pads[2].pitch) * 4, c.ptr(o.out[0]),
+                                     static_cast<uint64_t>(C.cols) * 4, C.rows,
+                                     static_cast<uint64_t>(C.cols) * 4, c.st);
+          break;
+        }
         // Fuse a following BIAS_ACT into the GEMV epilogue when the GEMM output has no other
         // reader (same arithmetic order as the unfused pair, so results are bit-identical).
         if (j + 1 < e && !ga.acc && g.ops[j + 1].type == SF_OP_BIAS_ACT && g.ops[j + 1].in[0] == o.out[0] &&
@@ -1396,6 +1427,29 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
       b->shadow[t] = {d, pitch};
       b->dev_allocs.push_back(d);
     }
+  }
+  for (size_t j = 0; j < g.ops.size(); ++j) {
+    const sf_op_desc& op = g.ops[j];
+    if (op.type != SF_OP_GEMM) continue;
+    const Tensor &A = g.T[op.in[0]], &B = g.T[op.in[1]], &C = g.T[op.out[0]];
+    const bool ta = op.flags & SF_GEMM_TA, tb = op.flags & SF_GEMM_TB;
+    if (C.rows <= 8 && !ta && !tb) continue;  // GEMV path has no pitch requirement
+    std::array<Binding::PadBuf, 3> pads{};
+    bool any = false;
+    const Tensor* ops3[3] = {&A, &B, &C};
+    const int ids[3] = {op.in[0], op.in[1], op.out[0]};
+    for (int q = 0; q < 3; ++q) {
+      const Tensor& x = *ops3[q];
+      if (x.cols % 4 == 0 || (q < 2 && b->shadow.count(ids[q]))) continue;
+      const int pitch = (x.cols + 3) / 4 * 4;
+      float* d = nullptr;
+      SF_CK(cudaMalloc(&d, static_cast<size_t>(x.rows) * pitch * sizeof(float)));
+      SF_CK(cudaMemset(d, 0, static_cast<size_t>(x.rows) * pitch * sizeof(float)));
+      b->dev_allocs.push_back(d);
+      pads[q] = {d, pitch};
+      any = true;
+    }
+    if (any) b->gemm_pad[static_cast<int>(j)] = pads;
   }
   SF_CK(cudaMalloc(&b->ws, std::max<uint64_t>(g.ws_floats, 4) * sizeof(float)));
   SF_CK(cudaMalloc(&b->counters, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));

@@ -23,6 +23,8 @@ struct DCopy {
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
                           int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp = nullptr);
 cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st);
+cudaError_t launch_copy2d(const void* src, uint64_t spitch, void* dst, uint64_t dpitch, uint64_t rows,
+                          uint64_t width, cudaStream_t st);
 // Single-buffer copy with pointer arguments (request I/O; 16-B aligned, nbytes % 4 == 0).
 cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st);
 
