@@ -228,7 +228,9 @@ typedef struct sf_job_info {
   double last_xfer_us;
   double last_unpack_us;
   uint64_t last_stop_ns;        /* CLOCK_MONOTONIC: cut decided (in-flight S_k done) */
-  uint64_t last_resume_ns;      /* CLOCK_MONOTONIC: first resumed subgraph launched */
+  uint64_t last_resume_ns;      /* CLOCK_MONOTONIC: first resumed subgraph began on the device
+                                   (host-observed completion of a marker recorded right before it,
+                                   i.e. after the stream-ordered copy / unpack finished) */
 } sf_job_info;
 
 typedef struct sf_cut_info {

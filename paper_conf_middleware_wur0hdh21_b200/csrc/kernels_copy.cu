@@ -45,55 +45,87 @@ __device__ __forceinline__ uint4 load_chunk(const uint8_t* src, uint64_t j, uint
   return v;
 }
 
+// One CTA owns the contiguous chunk range [c0, c1) of the flat 16-B chunk space.  Its
+// descriptors are staged in shared memory in batches of kBatch (no dependent global
+// descriptor loads on the copy path), then all threads walk the range flat — thread t takes
+// chunks c0 + t, c0 + t + 256, ... — each advancing a private monotonic cursor over the
+// staged descriptors.  Every thread stays busy whatever the tensor sizes (4-B scalars, 4-KB
+// slots, multi-GB tensors alike); kCopyUnroll loads are in flight per thread.
+constexpr int kBatch = 256;
+struct SDesc {
+  const uint8_t* src;
+  uint8_t* dst;
+  uint64_t nbytes;
+  uint64_t begin;
+};
+
 __global__ void __launch_bounds__(kCopyThreads)
 mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t total, uint64_t per_block,
               int64_t patch_iter, unsigned long long* tstamp) {
   // optional device-side duration: [0] = earliest CTA start, [1] = latest CTA end (ns)
   if (tstamp && threadIdx.x == 0) atomicMin(&tstamp[0], sfdev::globaltimer());
   const uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * per_block;
-  if (c0 >= total) {
-    if (tstamp && threadIdx.x == 0) atomicMax(&tstamp[1], sfdev::globaltimer());
-    return;
-  }
   const uint64_t c1 = min(c0 + per_block, total);
-  __shared__ int s_first;
-  if (threadIdx.x == 0) {
-    int lo = 0, hi = n - 1;
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (d[mid].chunk_begin <= c0) lo = mid; else hi = mid - 1;
+  __shared__ SDesc sd[kBatch + 1];
+  __shared__ int s_first, s_last;
+  if (c0 < total) {
+    if (threadIdx.x == 0) {
+      int lo = 0, hi = n - 1;  // last descriptor with begin <= c0
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (d[mid].chunk_begin <= c0) lo = mid; else hi = mid - 1;
+      }
+      s_first = lo;
+    } else if (threadIdx.x == 32) {
+      int lo = 0, hi = n - 1;  // last descriptor with begin <= c1 - 1
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (d[mid].chunk_begin <= c1 - 1) lo = mid; else hi = mid - 1;
+      }
+      s_last = lo;
     }
-    s_first = lo;
   }
   __syncthreads();
-  for (int i = s_first; i < n; ++i) {
-    const uint64_t b = d[i].chunk_begin, e = d[i + 1].chunk_begin;
-    if (b >= c1) break;
-    if (e <= c0 || e == b) continue;
-    const uint64_t lo = (c0 > b ? c0 : b) - b;
-    const uint64_t hi = (c1 < e ? c1 : e) - b;
-    const uint8_t* src = d[i].src;
-    uint8_t* dst = d[i].dst;
-    const uint64_t nb = d[i].nbytes;
-    const uint64_t full = nb >> 4;
-    for (uint64_t j0 = lo + threadIdx.x; j0 < hi; j0 += kCopyThreads * kCopyUnroll) {
-      uint4 v[kCopyUnroll];
-#pragma unroll
-      for (int u = 0; u < kCopyUnroll; ++u) {
-        const uint64_t j = j0 + static_cast<uint64_t>(u) * kCopyThreads;
-        v[u] = (j < hi) ? load_chunk(src, j, full, nb) : make_uint4(0u, 0u, 0u, 0u);
+  if (c0 < total) {
+    const int first = s_first, last = s_last;
+    for (int b0 = first; b0 <= last; b0 += kBatch) {
+      const int bn = min(kBatch, last - b0 + 1);
+      for (int t = threadIdx.x; t <= bn; t += kCopyThreads) {
+        const DCopy& x = d[b0 + t];  // t == bn: the next descriptor (or the sentinel)
+        sd[t] = {x.src, x.dst, x.nbytes, x.chunk_begin};
       }
+      __syncthreads();
+      const uint64_t lo = max(c0, sd[0].begin), hi = min(c1, sd[bn].begin);
+      int cur = 0;
+      for (uint64_t base = lo + threadIdx.x; base < hi; base += kCopyThreads * kCopyUnroll) {
+        uint4 v[kCopyUnroll];
+        uint8_t* dst[kCopyUnroll];
+        int di[kCopyUnroll];
 #pragma unroll
-      for (int u = 0; u < kCopyUnroll; ++u) {
-        const uint64_t j = j0 + static_cast<uint64_t>(u) * kCopyThreads;
-        if (j < hi) {
-          if (patch_iter >= 0 && i == 0 && j == 1) {
+        for (int u = 0; u < kCopyUnroll; ++u) {
+          const uint64_t c = base + static_cast<uint64_t>(u) * kCopyThreads;
+          dst[u] = nullptr;
+          di[u] = -1;
+          v[u] = make_uint4(0u, 0u, 0u, 0u);
+          if (c < hi) {
+            while (sd[cur + 1].begin <= c) ++cur;
+            const uint64_t j = c - sd[cur].begin;
+            v[u] = load_chunk(sd[cur].src, j, sd[cur].nbytes >> 4, sd[cur].nbytes);
+            dst[u] = sd[cur].dst + j * 16;
+            di[u] = (b0 + cur == 0 && j == 1) ? 1 : 0;
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < kCopyUnroll; ++u) {
+          if (!dst[u]) continue;
+          if (patch_iter >= 0 && di[u] == 1) {
             v[u].x = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter));
             v[u].y = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter) >> 32);
           }
-          sfdev::st16_cs(dst + j * 16, v[u]);
+          sfdev::st16_cs(dst[u], v[u]);
         }
       }
+      __syncthreads();
     }
   }
   if (tstamp) {

@@ -177,7 +177,7 @@ struct Job {
   uint64_t last_stop = 0, last_resume = 0;
   std::string error;
   std::thread driver;
-  std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c;  // per slot
+  std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
 };
 
 }  // namespace
@@ -748,12 +748,14 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   if (!J.ev_sub.empty()) return SF_OK;
   const size_t n = rt->slots.size();
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
+  J.ev_r.assign(n, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
   for (size_t s = 0; s < n; ++s) {
     if (rt->slots[s]->remote) continue;
     SF_CK(cudaSetDevice(rt->slots[s]->cuda));
     SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
+    SF_CK(cudaEventCreateWithFlags(&J.ev_r[s], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
     SF_CK(cudaEventCreate(&J.ev_b[s]));
     SF_CK(cudaEventCreate(&J.ev_c[s]));
@@ -1062,10 +1064,21 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
     lk.unlock();
     cudaSetDevice(S.cuda);
-    cudaError_t e = cudaGraphLaunch(ver, S.s_train);
+    // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
+    // wait on the peer store) has executed when this event completes on the device
+    cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
+    if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
     if (e == cudaSuccess) e = cudaEventRecord(J.ev_sub[dev], S.s_train);
-    if (e == cudaSuccess) e = spin_event(J.ev_sub[dev]);
+    uint64_t t_res = 0;
+    while (e == cudaSuccess) {
+      if (stamp && !t_res && cudaEventQuery(J.ev_r[dev]) == cudaSuccess) t_res = now_ns();
+      const cudaError_t q = cudaEventQuery(J.ev_sub[dev]);
+      if (q == cudaErrorNotReady) continue;
+      e = q;
+      break;
+    }
     const uint64_t t1 = now_ns();
+    if (stamp && !t_res) t_res = t1;
     float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
     if (e == cudaSuccess && stamp && J.adopted_pending) {
       J.adopted_pending = false;  // the copy was timed by the exporting process
@@ -1082,7 +1095,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     lk.lock();
     if (stamp) {
-      J.last_resume = t0;
+      J.last_resume = t_res;  // host-observed device resume (CLOCK_MONOTONIC)
       if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += std::max(h2d_us, 0.f); }
       if (peer_us >= 0.f) { J.pack_us = 0.0; J.xfer_us = peer_us; J.unpack_us = 0.0; }
     }
@@ -1275,6 +1288,7 @@ void sf_destroy(sf_runtime* rt) {
       if (rt->slots[s]->remote) continue;
       cudaSetDevice(rt->slots[s]->cuda);
       cudaEventDestroy(J->ev_sub[s]);
+      cudaEventDestroy(J->ev_r[s]);
       cudaEventDestroy(J->ev_a[s]);
       cudaEventDestroy(J->ev_b[s]);
       cudaEventDestroy(J->ev_c[s]);
