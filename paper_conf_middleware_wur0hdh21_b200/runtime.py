@@ -93,6 +93,8 @@ class GraphHandle:
     # ---- memory -------------------------------------------------------------------------
     def bind(self, slot: int, staging: bool = True, host_staging: bool = False) -> None:
         """Allocate this slot's arena (+ device / pinned host staging) with torch and bind."""
+        if self.rt.ordinals[slot] < 0:  # REMOTE slot: the C call reports the error
+            check(lib().sf_bind(self.rt.h, self.gid, slot, None, None, None), "sf_bind")
         dev = torch.device("cuda", self.rt.ordinals[slot])
         arena = torch.empty(self.info.arena_bytes, dtype=torch.uint8, device=dev)
         stg = torch.empty(self.info.staging_bytes, dtype=torch.uint8, device=dev) if staging else None

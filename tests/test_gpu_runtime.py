@@ -11,6 +11,8 @@ North_star bars:
 Two logical slots on one physical B200 exercise the peer-store path (same kernel; a
 different-GPU slot only changes the destination aperture to NVLink).
 """
+import ctypes
+
 import numpy as np
 import pytest
 import torch
@@ -379,3 +381,78 @@ def test_c3_full_size_mid_cut_peer_bitwise_and_sampled_oracle(P):
             elif op.type == BIAS_ACT:
                 h = O.bias_act(z, [T[b] for b in op.ins[1:]], True)
         assert rel(logits[r:r + 1], z) <= TOL, r
+
+
+@pytest.mark.parametrize("host_mode,defer", [(1, 0), (1, 1), (0, 1)])
+def test_host_modes_and_deferred_migration_bitwise(P, host_mode, defer):
+    """Zero-copy host tier (pack straight into mapped pinned memory) and deferred migration
+    give the same trajectory, bit for bit, as the unpreempted run."""
+    g = G.mlp_train((784, 256, 10))
+    base, _, _, _, _ = run_gpu(P, g, 30, slots=1)
+    sched = [(5, k, HOST) for k in range(5)] + [(20, 2, HOST)]
+    got, _, info, _, hs = run_gpu(P, g, 30, schedule=sched, slots=1, poison=True,
+                                  host_mode=host_mode, defer_migration=bool(defer))
+    assert info["n_preemptions"] == 6
+    assert_bitwise(base, got)
+
+
+def _run_with_requests(P, g, gi, n_req, **kw):
+    RT, A = P
+    rt, gh, st, ds = setup(P, g, slots=1, **kw)
+    ghi = rt.register(gi, priority=1)
+    ghi.partition()
+    ghi.bind(0, staging=False)
+    ghi.load(0, D.init_state(gi, seed=D.SEED_INFER))
+    job = rt.start_training(gh, 0, 100000, HOST)
+    x = torch.from_numpy(D.infer_inputs(gi, 1)[0]).cuda()
+    out = torch.zeros(1, 10, device="cuda")
+    import time
+    tms = []
+    for _ in range(n_req):
+        time.sleep(0.002)
+        tms.append(rt.wait(rt.submit(ghi, 0, x.data_ptr(), out.data_ptr()), 30))
+    rt.stop_job(job)
+    rt.wait_job(job, 60)
+    info = rt.job_info(job)
+    trace = rt.trace()
+    n = gh.n_subgraphs
+    rt.close()
+    return info, tms, trace, n
+
+
+def test_iteration_granularity_cuts_only_at_iteration_boundaries(P):
+    """Session time slicing baseline: requests wait for the iteration."""
+    info, tms, trace, n = _run_with_requests(P, G.mlp_train(), G.mlp_infer(), 10,
+                                             iteration_granularity=True)
+    assert info["n_preemptions"] >= 5
+    assert all(t["cut_k"] in (-1, 0) for t in tms)
+    evs = [dict(e, job=(1 if e["kind"] == "infer" else 0)) for e in trace]
+    SC.check_no_corun(evs)
+    SC.check_job_order([e for e in evs if e["kind"] == "train"], {0: n}, start={0: (0, 0)})
+
+
+def test_free_corun_baseline_never_preempts(P):
+    """exclusive_gpu=0 (multi-threaded TF analogue)."""
+    info, tms, trace, n = _run_with_requests(P, G.mlp_train(), G.mlp_infer(), 10, exclusive=False)
+    assert info["n_preemptions"] == 0
+    assert all(t["preempted_job"] == -1 for t in tms)
+
+
+def test_remote_slot_errors(P):
+    RT, A = P
+    g = G.mlp_train()
+    rt = RT.Runtime([0, -1])
+    gh = rt.register(g)
+    gh.partition()
+    with pytest.raises(A.SFError) as e:
+        gh.bind(1)  # remote slots are mapped, not bound
+    assert e.value.status == A.SF_EINVAL
+    with pytest.raises(A.SFError) as e:
+        rt.import_arena(gh, 1, bytes(96))  # no local binding yet
+    assert e.value.status in (A.SF_ESTATE, A.SF_EINVAL)
+    gh.bind(0)
+    blob = rt.export_arena(gh, 0)
+    assert len(blob) == ctypes.sizeof(A.sf_ipc_arena) == 88
+    with pytest.raises(A.SFError):
+        rt.import_arena(gh, 0, blob)  # slot 0 is local
+    rt.close()
