@@ -128,10 +128,11 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
 
     g, gi = build_workload(args.batch, args.spatial_div)
     rt = Runtime([local_dev], exclusive=exclusive, auto_preempt=True,
-                 iteration_granularity=iteration_granularity,
+                 iteration_granularity=iteration_granularity, max_inflight=args.max_inflight,
                  defer_migration=args.defer if defer is None else defer)
     gh = rt.register(g)
-    info = gh.partition(update_chunks=args.update_chunks)
+    info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
+                        update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
     arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
     gh.load(0, arrays)
@@ -223,7 +224,13 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
     S["launches"] = launches
     S["clocks"] = sampler.summary() if sampler else None
     S["sub_ms"] = sub_ms
-    S["iter_ms"] = iters_ms
+    tr = [e for e in rt.trace() if e["kind"] == "train"]
+    per_it = {}
+    for e in tr:
+        a, b_ = per_it.get(e["iter"], (e["t0"], e["t1"]))
+        per_it[e["iter"]] = (min(a, e["t0"]), max(b_, e["t1"]))
+    spans = sorted((b_ - a) * 1e-6 for a, b_ in per_it.values())
+    S["iter_ms"] = spans[len(spans) // 2] if spans else iters_ms
     S["n_subgraphs"] = gh.n_subgraphs
     S["info"] = {"arena_bytes": info.arena_bytes, "persistent_bytes": info.persistent_bytes,
                  "max_live_bytes": info.max_live_bytes, "staging_bytes": info.staging_bytes}
@@ -243,9 +250,11 @@ def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, g
     from sf_inputs import data as D
 
     g, gi = build_workload(args.batch, args.spatial_div)
-    rt = Runtime([local_dev, -1], exclusive=True, auto_preempt=True, defer_migration=bool(args.defer))
+    rt = Runtime([local_dev, -1], exclusive=True, auto_preempt=True, defer_migration=bool(args.defer),
+                 max_inflight=args.max_inflight)
     gh = rt.register(g)
-    info = gh.partition(update_chunks=args.update_chunks)
+    info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
+                        update_chunks=args.update_chunks)
     gh.bind(0, staging=False, host_staging=False)
     arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
     link = PairLink(gloo)
@@ -436,6 +445,10 @@ def main():
     ap.add_argument("--spatial-div", type=int, default=1)
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--max-ops", type=int, default=1,
+                    help="MAX_OPS partition: at most this many ops per subgraph (0 = per layer)")
+    ap.add_argument("--max-inflight", type=int, default=2,
+                    help="subgraphs queued on the GPU ahead of the host (1 = strict boundaries)")
     ap.add_argument("--update-chunks", type=int, default=8,
                     help="split the SGD update subgraph into byte-balanced chunks (Q2)")
     ap.add_argument("--defer", type=int, default=1,
@@ -523,6 +536,8 @@ def main():
                    "tensors_live_cut0": 535, "inference_model": "MLP 2048-4096-4096-1000 (29.3M params)",
                    "tier": "host (pinned, copy engine)", "parallelism": f"replicas x{args.world}",
                    "update_chunks": args.update_chunks,
+                   "partition": f"MAX_OPS={args.max_ops}" if args.max_ops else "PER_LAYER_PHASE",
+                   "max_inflight": args.max_inflight,
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets > 126 MB L2 (no flush needed)"},
@@ -536,6 +551,7 @@ def main():
                       "host_link_gbs": migr_gbs,
                       "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},
         "training_subgraph_ms_mean": m0["sub_ms"], "n_subgraphs": m0["n_subgraphs"],
+        "training_iteration_ms_median": m0["iter_ms"],
         "baselines": base,
         "roofline": {"kernel": "mtcopy_kernel (pack: arena -> staging)", "bound": "hbm",
                      "achieved": pack_achieved, "peak": hbm, "unit": "GB/s",

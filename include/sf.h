@@ -141,6 +141,9 @@ typedef struct sf_config {
   int32_t host_mode;             /* SF_HOST_CE or SF_HOST_ZC */
   int32_t poison_released;       /* 1: fill released source arenas with 0xFF (tests) */
   int32_t trace_capacity;        /* events kept; 0 -> 1<<16 */
+  int32_t max_inflight;          /* subgraphs queued on the device ahead of the host (1..4;
+                                    0 -> 1): >1 removes the host gap between subgraphs; a
+                                    preemption then waits for at most this many subgraphs */
   int32_t defer_migration;       /* 1: start the migration copy only after the device's
                                     queued inference drained (the paper defers the transfer
                                     past the preemption); 0: concurrent */
@@ -327,7 +330,8 @@ typedef struct sf_trace_event {
   int32_t dev, job, kind, k;   /* job: training job id, or 1<<20 | request for inference */
   int64_t iter;
   uint64_t t0_ns, t1_ns;       /* host CLOCK_MONOTONIC: launch .. completion observed */
-  uint64_t arrival_ns;         /* inference only */
+  uint64_t arrival_ns;         /* inference: scheduled arrival; train: host dispatch time
+                                  (<= t0 when queued behind an in-flight predecessor) */
 } sf_trace_event;
 sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* n_out);
 uint64_t sf_now_ns(void); /* CLOCK_MONOTONIC */

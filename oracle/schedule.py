@@ -16,7 +16,10 @@ trace or the GPU runtime's recorded one):
       start(infer) - max(arrival, end of the previous inference on that device)
       <= max train-subgraph duration on that device + slack.
   I4  cut rule (reading Q13): a request arriving while S_k runs is served at the
-      boundary after S_k.
+      boundary after S_k — more precisely, no training subgraph is DISPATCHED after the
+      arrival and before the inference starts (subgraphs already dispatched to the GPU are
+      allowed to finish); events may carry "launch" (dispatch time),
+      else t0 is the dispatch time.
 
 Event dicts: {"dev", "job", "kind": "train"|"infer", "iter", "k", "t0", "t1",
 "arrival" (infer only)}; times in any consistent unit.
@@ -97,7 +100,7 @@ def check_cut_rule(events: Sequence[dict]) -> None:
         trains = [e for e in evs if e["kind"] == "train"]
         for r in (e for e in evs if e["kind"] == "infer"):
             for t in trains:
-                if r["arrival"] <= t["t0"] < r["t0"]:
+                if r["arrival"] <= t.get("launch", t["t0"]) < r["t0"]:
                     raise InvariantError(f"dev {d}: subgraph ({t['iter']},{t['k']}) started at "
                                          f"{t['t0']} after arrival {r['arrival']} before the "
                                          f"inference at {r['t0']}")

@@ -51,7 +51,8 @@ class sf_config(C.Structure):
                 ("exclusive_gpu", C.c_int32), ("auto_preempt", C.c_int32),
                 ("iteration_granularity", C.c_int32), ("host_mode", C.c_int32),
                 ("poison_released", C.c_int32), ("trace_capacity", C.c_int32),
-                ("defer_migration", C.c_int32), ("device_budget_bytes", C.c_uint64)]
+                ("max_inflight", C.c_int32), ("defer_migration", C.c_int32),
+                ("device_budget_bytes", C.c_uint64)]
 
 
 class sf_partition_opts(C.Structure):

@@ -121,6 +121,7 @@ struct Graph {
 };
 
 constexpr int kInferOwner = 1 << 20;
+constexpr int kMaxInflight = 4;
 
 struct Request {
   sf_req_id id;
@@ -178,6 +179,7 @@ struct Job {
   std::string error;
   std::thread driver;
   std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
+  std::vector<cudaEvent_t> ev_ring;  // [slot * kMaxInflight + i]: in-flight subgraph ends
 };
 
 }  // namespace
@@ -749,6 +751,7 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   const size_t n = rt->slots.size();
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
   J.ev_r.assign(n, nullptr);
+  J.ev_ring.assign(n * kMaxInflight, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
   for (size_t s = 0; s < n; ++s) {
@@ -756,6 +759,8 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
     SF_CK(cudaSetDevice(rt->slots[s]->cuda));
     SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
     SF_CK(cudaEventCreateWithFlags(&J.ev_r[s], cudaEventDisableTiming));
+    for (int i = 0; i < kMaxInflight; ++i)
+      SF_CK(cudaEventCreateWithFlags(&J.ev_ring[s * kMaxInflight + i], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
     SF_CK(cudaEventCreate(&J.ev_b[s]));
     SF_CK(cudaEventCreate(&J.ev_c[s]));
@@ -992,10 +997,25 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
   return SF_OK;
 }
 
+// Job driver.  J.it / J.k is the LAUNCH cursor (the next subgraph not yet launched); up to
+// max_inflight subgraphs are queued on the device back to back (no host gap between them).
+// When a preemption is requested or a request is queued on the device, launching stops,
+// the in-flight subgraphs finish (dispatched kernels are allowed to
+// finish), and the cut is taken at the cursor.
 void driver_main(sf_runtime* rt, Job* Jp) {
   Job& J = *Jp;
   Graph& g = *J.g;
   const int n = static_cast<int>(g.parts.size());
+  const int W = std::max(1, std::min(rt->cfg.max_inflight, kMaxInflight));
+  struct Inflight {
+    int64_t it;
+    int k, dev, ev;
+    uint64_t t0;
+    bool stamp;
+  };
+  std::deque<Inflight> q;
+  int ev_next = 0;
+  uint64_t last_t1 = 0;
   std::unique_lock<std::mutex> lk(rt->m);
   bool pending_peer_stats = false;
   int stats_slot = -1;
@@ -1009,111 +1029,160 @@ void driver_main(sf_runtime* rt, Job* Jp) {
   };
   while (true) {
     if (J.state == SF_JOB_FAILED) break;
-    if (J.it >= J.iters || (J.stop_req && J.k == 0) || rt->shutting_down) {
-      release();
-      J.state = SF_JOB_DONE;
-      rt->cv.notify_all();
-      break;
-    }
-    // boundary gate: preempt here if asked to (explicitly, or because a
-    // request is queued on this device and auto-preemption is on)
-    const bool at_cut_ok = !rt->cfg.iteration_granularity || J.k == 0;
-    if (!J.preempt_req && J.sched_pos < J.sched.size() && J.sched[J.sched_pos].iter == J.it &&
-        J.sched[J.sched_pos].k == J.k) {
-      J.preempt_req = J.sched[J.sched_pos].target != J.dev;  // a move to itself is a no-op
-      J.preempt_park = false;
-      J.preempt_target = J.sched[J.sched_pos].target;
-      J.t_req = now_ns();
-      ++J.sched_pos;
-    }
-    const bool has_inf = slot_has_inference(rt, J.dev);
-    const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu && has_inf &&
-                           J.auto_target != J.dev;
-    if (J.preempt_req || (auto_want && at_cut_ok)) {
-      release();
-      if (!J.preempt_req) {
-        J.preempt_park = false;
-        J.preempt_target = J.auto_target;
-        J.t_req = slot_of(rt, J.dev).q.front()->arrival;
+    bool launch = false;
+    const bool finished = J.it >= J.iters || (J.stop_req && J.k == 0) || rt->shutting_down;
+    if (finished) {
+      if (q.empty()) {
+        release();
+        J.state = SF_JOB_DONE;
+        rt->cv.notify_all();
+        break;
       }
-      const int src = J.dev;
-      const bool peer = J.preempt_target != SF_TARGET_HOST;
-      if (do_preempt(rt, J, lk) != SF_OK) break;
-      if (J.state == SF_JOB_DONE || J.state == SF_JOB_MIGRATED_OUT) break;
-      if (peer) { pending_peer_stats = true; stats_slot = src; }
+    } else {
+      // boundary gate at the launch cursor
+      const bool at_cut_ok = !rt->cfg.iteration_granularity || J.k == 0;
+      if (!J.preempt_req && J.sched_pos < J.sched.size() && J.sched[J.sched_pos].iter == J.it &&
+          J.sched[J.sched_pos].k == J.k) {
+        J.preempt_req = J.sched[J.sched_pos].target != J.dev;  // a move to itself is a no-op
+        J.preempt_park = false;
+        J.preempt_target = J.sched[J.sched_pos].target;
+        J.t_req = now_ns();
+        ++J.sched_pos;
+      }
+      const bool has_inf = slot_has_inference(rt, J.dev);
+      const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu && has_inf &&
+                             J.auto_target != J.dev;
+      const bool want_cut = J.preempt_req || (auto_want && at_cut_ok);
+      // without a migration, yield the device to queued inference at this boundary (unless the
+      // session-slicing baseline keeps it for the rest of the iteration)
+      const bool yield_to_inf = rt->cfg.exclusive_gpu && has_inf && !(auto_want && !at_cut_ok);
+      if (want_cut) {
+        if (q.empty()) {
+          release();
+          if (!J.preempt_req) {
+            J.preempt_park = false;
+            J.preempt_target = J.auto_target;
+            J.t_req = slot_of(rt, J.dev).q.front()->arrival;
+          }
+          const int src = J.dev;
+          const bool peer = J.preempt_target != SF_TARGET_HOST;
+          if (do_preempt(rt, J, lk) != SF_OK) break;
+          if (J.state == SF_JOB_DONE || J.state == SF_JOB_MIGRATED_OUT) break;
+          if (peer) { pending_peer_stats = true; stats_slot = src; }
+          continue;
+        }
+      } else if (yield_to_inf) {
+        if (q.empty()) {
+          release();
+          rt->cv.wait(lk);
+          continue;
+        }
+      } else {
+        Slot& S = slot_of(rt, J.dev);
+        if (rt->cfg.exclusive_gpu && !J.holds_token) {
+          // invariant 1: no other model's subgraph on this device
+          if (S.owner != -1) {
+            if (q.empty()) {
+              rt->cv.wait(lk);
+              continue;
+            }
+          } else {
+            S.owner = static_cast<int>(J.id);
+            J.holds_token = true;
+          }
+        }
+        launch = (!rt->cfg.exclusive_gpu || J.holds_token) && static_cast<int>(q.size()) < W;
+      }
+    }
+    if (launch) {
+      Slot& S = slot_of(rt, J.dev);
+      const int dev = J.dev, k = J.k;
+      const int64_t it = J.it;
+      cudaGraphExec_t ver = g.bind[dev]->versions[k];
+      sfk::count_launch(g.bind[dev]->version_kernels[k]);
+      const bool stamp = J.stamp_resume;
+      J.stamp_resume = false;
+      const int ev = ev_next;
+      ev_next = (ev_next + 1) % W;
+      const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
+      lk.unlock();
+      cudaSetDevice(S.cuda);
+      // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
+      // wait on the peer store) has executed when this event completes on the device
+      cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
+      if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
+      if (e == cudaSuccess) e = cudaEventRecord(J.ev_ring[dev * kMaxInflight + ev], S.s_train);
+      lk.lock();
+      if (e != cudaSuccess) {
+        release();
+        J.error = std::string("subgraph launch: ") + cudaGetErrorString(e);
+        J.state = SF_JOB_FAILED;
+        rt->cv.notify_all();
+        break;
+      }
+      q.push_back({it, k, dev, ev, t0, stamp});
+      if (++J.k == n) { J.k = 0; ++J.it; }
       continue;
     }
-    Slot& S = slot_of(rt, J.dev);
-    if (rt->cfg.exclusive_gpu && !J.holds_token) {
-      // invariant 1: wait until no other model owns the device; with no
-      // preemption possible here, yield to queued inference at this boundary
-      const bool yield_to_inf = has_inf && !(auto_want && !at_cut_ok);
-      if (S.owner != -1 || yield_to_inf) {
-        rt->cv.wait(lk);
-        continue;
-      }
-      S.owner = static_cast<int>(J.id);
-      J.holds_token = true;
+    if (q.empty()) {  // nothing launched and nothing in flight: wait for a state change
+      rt->cv.wait(lk);
+      continue;
     }
-    const int dev = J.dev, k = J.k;
-    const int64_t it = J.it;
-    cudaGraphExec_t ver = g.bind[dev]->versions[k];
-    sfk::count_launch(g.bind[dev]->version_kernels[k]);
-    const bool stamp = J.stamp_resume;
-    J.stamp_resume = false;
-    const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
+    // retire the oldest in-flight subgraph
+    const Inflight f = q.front();
+    Slot& S = slot_of(rt, f.dev);
     lk.unlock();
     cudaSetDevice(S.cuda);
-    // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
-    // wait on the peer store) has executed when this event completes on the device
-    cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
-    if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
-    if (e == cudaSuccess) e = cudaEventRecord(J.ev_sub[dev], S.s_train);
     uint64_t t_res = 0;
-    while (e == cudaSuccess) {
-      if (stamp && !t_res && cudaEventQuery(J.ev_r[dev]) == cudaSuccess) t_res = now_ns();
-      const cudaError_t q = cudaEventQuery(J.ev_sub[dev]);
-      if (q == cudaErrorNotReady) continue;
-      e = q;
+    cudaError_t e = cudaSuccess;
+    for (;;) {
+      if (f.stamp && !t_res && cudaEventQuery(J.ev_r[f.dev]) == cudaSuccess) t_res = now_ns();
+      const cudaError_t qq = cudaEventQuery(J.ev_ring[f.dev * kMaxInflight + f.ev]);
+      if (qq == cudaErrorNotReady) continue;
+      e = qq;
       break;
     }
     const uint64_t t1 = now_ns();
-    if (stamp && !t_res) t_res = t1;
+    if (f.stamp && !t_res) t_res = t1;
     float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
-    if (e == cudaSuccess && stamp && J.adopted_pending) {
+    if (e == cudaSuccess && f.stamp && J.adopted_pending) {
       J.adopted_pending = false;  // the copy was timed by the exporting process
-    } else if (e == cudaSuccess && stamp) {
+    } else if (e == cudaSuccess && f.stamp) {
       if (pending_peer_stats) {
         peer_us = static_cast<float>(tstamp_us(slot_of(rt, stats_slot).tstamp));
         if (peer_us < 0.f) peer_us = elapsed_us(J.ev_a[stats_slot], J.ev_b[stats_slot]);
         pending_peer_stats = false;
       } else {
-        h2d_us = elapsed_us(J.ev_a[dev], J.ev_b[dev]);
+        h2d_us = elapsed_us(J.ev_a[f.dev], J.ev_b[f.dev]);
         unpack_us = static_cast<float>(tstamp_us(S.tstamp + 2));
-        if (unpack_us < 0.f) unpack_us = elapsed_us(J.ev_b[dev], J.ev_c[dev]);
+        if (unpack_us < 0.f) unpack_us = elapsed_us(J.ev_b[f.dev], J.ev_c[f.dev]);
       }
     }
     lk.lock();
-    if (stamp) {
+    q.pop_front();
+    if (f.stamp) {
       J.last_resume = t_res;  // host-observed device resume (CLOCK_MONOTONIC)
       if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += std::max(h2d_us, 0.f); }
       if (peer_us >= 0.f) { J.pack_us = 0.0; J.xfer_us = peer_us; J.unpack_us = 0.0; }
     }
     if (e != cudaSuccess) {
       release();
-      J.error = std::string("subgraph launch: ") + cudaGetErrorString(e);
+      J.error = std::string("subgraph: ") + cudaGetErrorString(e);
       J.state = SF_JOB_FAILED;
       rt->cv.notify_all();
       break;
     }
-    sf_trace_event ev{};
-    ev.dev = dev; ev.job = static_cast<int32_t>(J.id); ev.kind = SF_EV_TRAIN; ev.k = k; ev.iter = it;
-    ev.t0_ns = t0; ev.t1_ns = t1;
-    push_trace(rt, ev);
-    if (++J.k == n) { J.k = 0; ++J.it; }
+    sf_trace_event tev{};
+    tev.dev = f.dev; tev.job = static_cast<int32_t>(J.id); tev.kind = SF_EV_TRAIN; tev.k = f.k;
+    tev.iter = f.it;
+    tev.t0_ns = std::max(f.t0, last_t1);  // queued behind its predecessor on the stream
+    tev.t1_ns = t1;
+    tev.arrival_ns = f.t0;  // train events: host dispatch (launch) time
+    last_t1 = t1;
+    push_trace(rt, tev);
     // iteration-granularity (session time slicing baseline) keeps the device for the whole
-    // iteration; otherwise every subgraph boundary is a scheduling point
-    if (!rt->cfg.iteration_granularity || J.k == 0) release();
+    // iteration; otherwise an empty window is a scheduling point
+    if (q.empty() && (!rt->cfg.iteration_granularity || J.k == 0)) release();
     rt->cv.notify_all();
   }
 }
@@ -1289,6 +1358,7 @@ void sf_destroy(sf_runtime* rt) {
       cudaSetDevice(rt->slots[s]->cuda);
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_r[s]);
+      for (int i = 0; i < kMaxInflight; ++i) cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
       cudaEventDestroy(J->ev_a[s]);
       cudaEventDestroy(J->ev_b[s]);
       cudaEventDestroy(J->ev_c[s]);

@@ -102,14 +102,15 @@ def test_c2_prefix_long_trajectory_vs_oracle(P):
         assert rel(v, ref.outputs[-1][name]) <= TOL, name
 
 
-def test_c1_preempted_at_every_cut_is_bit_identical(P):
+@pytest.mark.parametrize("W", [1, 2, 4])
+def test_c1_preempted_at_every_cut_is_bit_identical(P, W):
     g = G.mlp_train()
-    base, bo, _, _, _ = run_gpu(P, g, 60)
+    base, bo, _, _, _ = run_gpu(P, g, 60, max_inflight=W)
     n = len(OG.partition(g))
     sched = [(50, k, HOST) for k in range(n)] + [(52, k, 1 - (k % 2)) for k in range(1, n)]
     sched += [(55, 2, 1), (56, 4, 0), (57, 1, HOST), (58, 3, 1)]
     sched = sorted(sched)
-    got, go, info, trace, _ = run_gpu(P, g, 60, schedule=sched, poison=True)
+    got, go, info, trace, _ = run_gpu(P, g, 60, schedule=sched, poison=True, max_inflight=W)
     assert info["n_preemptions"] >= 10
     assert_bitwise(base, got)
     assert bo["loss"].tobytes() == go["loss"].tobytes()
@@ -212,11 +213,12 @@ def test_explicit_preempt_resume_peer_and_host(P):
     assert_bitwise(base, got)
 
 
-def test_inference_vs_oracle_and_auto_preemption_invariants(P):
+@pytest.mark.parametrize("W", [1, 2])
+def test_inference_vs_oracle_and_auto_preemption_invariants(P, W):
     RT, A = P
     g = G.mlp_train()
     gi = G.mlp_infer()
-    rt, gh, st, ds = setup(P, g, slots=1)
+    rt, gh, st, ds = setup(P, g, slots=1, max_inflight=W)
     ghi = rt.register(gi, priority=1)
     ghi.partition()
     ghi.bind(0, staging=False)

@@ -99,6 +99,18 @@ def test_checker_rejects_long_wait_and_cut_rule():
         SC.check_cut_rule(evs)  # subgraph k=1 started at 10 after arrival 5
 
 
+def test_cut_rule_uses_dispatch_time():
+    # S_1 dispatched (launch 9) before the arrival (10) but queued behind S_0 (t0 = 12):
+    # allowed; a subgraph dispatched after the arrival is not
+    ok = [_ev(0, 0, "train", 0, 12), dict(_ev(0, 0, "train", 12, 20, k=1), launch=9),
+          _ev(0, 1, "infer", 20, 21, arrival=10)]
+    SC.check_cut_rule(ok)
+    bad = [_ev(0, 0, "train", 0, 12), dict(_ev(0, 0, "train", 12, 20, k=1), launch=11),
+           _ev(0, 1, "infer", 20, 21, arrival=10)]
+    with pytest.raises(SC.InvariantError):
+        SC.check_cut_rule(bad)
+
+
 def test_model_satisfies_invariants_host_and_peer():
     dur = [3.0, 1.0, 2.0, 0.5, 1.5]
     arr = list(D.poisson_arrivals(40, 0.2, seed=3))
