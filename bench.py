@@ -129,7 +129,9 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
     g, gi = build_workload(args.batch, args.spatial_div)
     rt = Runtime([local_dev], exclusive=exclusive, auto_preempt=True,
                  iteration_granularity=iteration_granularity, max_inflight=args.max_inflight,
-                 defer_migration=args.defer if defer is None else defer)
+                 defer_migration=args.defer if defer is None else defer,
+                 dispatch_spin_us=args.dispatch_spin_us,
+                 inflight_budget_us=args.inflight_budget_us)
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
                         update_chunks=args.update_chunks)
@@ -251,6 +253,7 @@ def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, g
 
     g, gi = build_workload(args.batch, args.spatial_div)
     rt = Runtime([local_dev, -1], exclusive=True, auto_preempt=True, defer_migration=bool(args.defer),
+                 dispatch_spin_us=args.dispatch_spin_us, inflight_budget_us=args.inflight_budget_us,
                  max_inflight=args.max_inflight)
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
@@ -451,6 +454,10 @@ def main():
                     help="subgraphs queued on the GPU ahead of the host (1 = strict boundaries)")
     ap.add_argument("--update-chunks", type=int, default=8,
                     help="split the SGD update subgraph into byte-balanced chunks (Q2)")
+    ap.add_argument("--dispatch-spin-us", type=int, default=-1,
+                    help="idle dispatcher busy-polls its queue (-1: always; one core per GPU)")
+    ap.add_argument("--inflight-budget-us", type=int, default=50,
+                    help="queue a subgraph behind in-flight ones only within this est. device time")
     ap.add_argument("--defer", type=int, default=1,
                     help="1: migrate after the preempter drained (default); 0: concurrently")
     args = ap.parse_args()
@@ -538,6 +545,8 @@ def main():
                    "update_chunks": args.update_chunks,
                    "partition": f"MAX_OPS={args.max_ops}" if args.max_ops else "PER_LAYER_PHASE",
                    "max_inflight": args.max_inflight,
+                   "dispatch_spin_us": args.dispatch_spin_us,
+                   "inflight_budget_us": args.inflight_budget_us,
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets > 126 MB L2 (no flush needed)"},

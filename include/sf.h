@@ -148,6 +148,14 @@ typedef struct sf_config {
                                     queued inference drained (the paper defers the transfer
                                     past the preemption); 0: concurrent */
   uint64_t device_budget_bytes;  /* per device; 0 = unlimited */
+  int32_t dispatch_spin_us;      /* an idle dispatcher busy-polls its request queue for this
+                                    long before blocking on the runtime's condition variable
+                                    (a futex wake-up adds tens of us to every request);
+                                    0 = block at once, -1 = poll forever (one core per slot) */
+  int32_t inflight_budget_us;    /* > 0: queue a subgraph behind in-flight ones only while
+                                    their estimated device time (EMA of observed subgraph
+                                    durations) stays within this budget, bounding what a
+                                    preemption drains; 0 = window limit only */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,
@@ -312,6 +320,8 @@ typedef struct sf_timing {
   int32_t preempted_job; /* job cut by this request, or -1 */
   int64_t cut_iter;
   int32_t cut_k;
+  float device_us;       /* device time of the request's kernel chain (input copy .. output
+                            copy), CUDA events on the inference stream */
 } sf_timing;
 
 /* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).
@@ -354,6 +364,15 @@ sf_status sf_op_mtcopy(const sf_copy_desc* descs, int32_t n, int64_t patch_iter,
 sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N,
                      int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
                      void* stream);
+/* C = act(op(A) op(B) (+C) + b1 (+ b2) (+ b3)), act = ReLU if relu else identity; the GEMM
+ * of a forward layer with its BIAS_ACT epilogue (PAPER.md:1213-1220 workload; SURVEY.md 8(a)
+ * K5).  b1 is required (SF_EINVAL otherwise); biases are 1 x N rows.  Batch <= 8 fuses the
+ * epilogue into the GEMV's cluster reduction; otherwise it runs as a second elementwise
+ * kernel in place (requires ldc == N). */
+sf_status sf_op_gemm_bias_act(const float* A, const float* B, float* C, int32_t M, int32_t N,
+                              int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
+                              const float* b1, const float* b2, const float* b3, int32_t relu,
+                              void* stream);
 sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
                          float* h, int32_t rows, int32_t cols, int32_t relu, void* stream);
 sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* db,

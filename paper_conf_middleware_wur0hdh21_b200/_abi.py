@@ -52,7 +52,8 @@ class sf_config(C.Structure):
                 ("iteration_granularity", C.c_int32), ("host_mode", C.c_int32),
                 ("poison_released", C.c_int32), ("trace_capacity", C.c_int32),
                 ("max_inflight", C.c_int32), ("defer_migration", C.c_int32),
-                ("device_budget_bytes", C.c_uint64)]
+                ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
+                ("inflight_budget_us", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):
@@ -82,7 +83,7 @@ class sf_cut_info(C.Structure):
 class sf_timing(C.Structure):
     _fields_ = [("arrival_ns", C.c_uint64), ("start_ns", C.c_uint64), ("end_ns", C.c_uint64),
                 ("dev", C.c_int32), ("preempted_job", C.c_int32), ("cut_iter", C.c_int64),
-                ("cut_k", C.c_int32)]
+                ("cut_k", C.c_int32), ("device_us", C.c_float)]
 
 
 class sf_trace_event(C.Structure):
@@ -142,6 +143,8 @@ PROTOTYPES = {
     "sf_op_mtcopy": (_st, [_P(sf_copy_desc), C.c_int32, C.c_int64, _vp]),
     "sf_op_gemm": (_st, [_vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                          C.c_int32, C.c_int32, _vp]),
+    "sf_op_gemm_bias_act": (_st, [_vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
+                                  C.c_int32, C.c_int32, C.c_int32, _vp, _vp, _vp, C.c_int32, _vp]),
     "sf_op_bias_act": (_st, [_vp, _vp, _vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, _vp]),
     "sf_op_bias_act_bwd": (_st, [_vp, _vp, _vp, _vp, C.c_int32, C.c_int32, _vp]),
     "sf_op_colsum": (_st, [_vp, _vp, C.c_int32, C.c_int32, _vp]),

@@ -17,6 +17,7 @@
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
+#include "sf_launch.cuh"
 
 #ifndef SF_COPY_UNROLL
 #define SF_COPY_UNROLL 8
@@ -27,6 +28,12 @@ namespace sfk {
 static std::atomic<uint64_t> g_launches{0};
 void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 uint64_t launches() { return g_launches.load(std::memory_order_relaxed); }
+
+namespace {
+thread_local bool t_pdl = false;
+}
+void set_pdl(bool on) { t_pdl = on; }
+bool pdl_enabled() { return t_pdl; }
 
 constexpr int kCopyThreads = 256;
 constexpr int kCopyUnroll = SF_COPY_UNROLL;
@@ -175,6 +182,8 @@ cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st) {
 
 __global__ void copy_kernel(const uint8_t* __restrict__ src, uint8_t* __restrict__ dst,
                             uint64_t nb) {
+  sfdev::griddep_wait();
+  sfdev::griddep_launch();
   const uint64_t full = nb >> 4;
   for (uint64_t j = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; j < (nb + 15) / 16;
        j += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
@@ -190,16 +199,16 @@ __global__ void copy_kernel(const uint8_t* __restrict__ src, uint8_t* __restrict
 cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st) {
   if (nbytes == 0) return cudaSuccess;
   const uint64_t blocks = std::min<uint64_t>((nbytes / 16 + 255) / 256 + 1, 148ull * 4);
-  copy_kernel<<<static_cast<unsigned>(blocks), 256, 0, st>>>(static_cast<const uint8_t*>(src),
-                                                             static_cast<uint8_t*>(dst), nbytes);
   count_launch();
-  return cudaGetLastError();
+  return launch_k(copy_kernel, dim3(static_cast<unsigned>(blocks)), dim3(256), 0, st,
+                  static_cast<const uint8_t*>(src), static_cast<uint8_t*>(dst), nbytes);
 }
 
 // 2-D pitched copy (rows x width bytes, width % 4 == 0, 4-B aligned pitches): pads or unpads
 // a GEMM operand whose row pitch is not a multiple of 16 B (TMA tensor-map requirement).
 __global__ void copy2d_kernel(const uint8_t* __restrict__ src, uint64_t spitch, uint8_t* __restrict__ dst,
                               uint64_t dpitch, uint64_t rows, uint64_t width) {
+  sfdev::griddep_wait();
   const uint64_t words = width / 4;
   const uint64_t total = rows * words;
   for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < total;
@@ -214,10 +223,9 @@ cudaError_t launch_copy2d(const void* src, uint64_t spitch, void* dst, uint64_t 
   if (rows == 0 || width == 0) return cudaSuccess;
   const uint64_t total = rows * (width / 4);
   const uint64_t blocks = std::min<uint64_t>((total + 255) / 256, 148ull * 8);
-  copy2d_kernel<<<static_cast<unsigned>(blocks), 256, 0, st>>>(static_cast<const uint8_t*>(src), spitch,
-                                                               static_cast<uint8_t*>(dst), dpitch, rows, width);
   count_launch();
-  return cudaGetLastError();
+  return launch_k(copy2d_kernel, dim3(static_cast<unsigned>(blocks)), dim3(256), 0, st,
+                  static_cast<const uint8_t*>(src), spitch, static_cast<uint8_t*>(dst), dpitch, rows, width);
 }
 
 // FEED: x = pool[(step mod P) * x_bytes ...] (data cursor read on device, reading Q3).

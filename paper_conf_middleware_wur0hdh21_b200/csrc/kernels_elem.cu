@@ -11,6 +11,7 @@
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
+#include "sf_launch.cuh"
 
 namespace sfk {
 namespace {
@@ -30,6 +31,8 @@ __device__ __forceinline__ float warp_max(float v) {
 __global__ void bias_act_kernel(const float* __restrict__ z, const float* __restrict__ b1,
                                 const float* __restrict__ b2, const float* __restrict__ b3,
                                 float* __restrict__ h, int rows, int cols, int relu, int vec) {
+  sfdev::griddep_wait();
+  sfdev::griddep_launch();
   const uint64_t total = static_cast<uint64_t>(rows) * cols;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
   if (vec) {
@@ -222,13 +225,49 @@ colsum4_kernel(const float* __restrict__ x, const float* __restrict__ mask, floa
   if (threadIdx.x == 0) counters[blockIdx.x] = 0u;
 }
 
+// Deterministic loss reduction shared by the softmax-CE kernels: every CTA reduces its
+// threads' partial sums in a fixed tree into ws[blockIdx.x]; the last CTA to arrive sums the
+// gridDim.x partials (strided per thread, then the same tree) and resets the counter.
+__device__ __forceinline__ float block_sum_tree(float v, float* red) {
+  red[threadIdx.x] = v;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
+    __syncthreads();
+  }
+  const float r = red[0];
+  __syncthreads();
+  return r;
+}
+
+__device__ __forceinline__ void loss_reduce(float part, float* ws, unsigned* counter, float* loss,
+                                            int rows) {
+  __shared__ float red[256];
+  __shared__ int last;
+  const float b = block_sum_tree(part, red);
+  if (threadIdx.x == 0) ws[blockIdx.x] = b;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicAdd(counter, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  float t = 0.f;
+  for (int i = threadIdx.x; i < static_cast<int>(gridDim.x); i += 256) t += __ldcg(ws + i);
+  const float tot = block_sum_tree(t, red);
+  if (threadIdx.x == 0) {
+    *loss = tot / static_cast<float>(rows);
+    *counter = 0u;
+  }
+}
+
 // Softmax-CE for narrow rows (cols % 4 == 0, cols <= 8 L): L lanes per row, each lane keeps
 // up to two float4 of the row in registers (one read pass); shuffles within the L-lane group.
 template <int L>
 __global__ void __launch_bounds__(256)
 softmax_ce_narrow_kernel(const float* __restrict__ l, const int32_t* __restrict__ y,
                          float* __restrict__ loss, float* __restrict__ dl, int rows, int cols,
-                         float* row_loss, unsigned* counter) {
+                         float* ws, unsigned* counter) {
   const int lane = threadIdx.x & 31;
   const int sub = lane % L;                       // lane within the row group
   const int groups_per_block = 256 / L;
@@ -237,6 +276,7 @@ softmax_ce_narrow_kernel(const float* __restrict__ l, const int32_t* __restrict_
   const int warp_first = blockIdx.x * groups_per_block + (threadIdx.x >> 5) * (32 / L);
   const int nq = cols / 4;
   const float inv_b = 1.0f / static_cast<float>(rows);
+  float part = 0.f;  // this thread's rows' losses, in row order
   // warp-uniform trip count: every lane joins every shuffle; rows past the end are masked
   for (int base = warp_first, row = g0; base < rows; base += stride, row += stride) {
     const bool active = row < rows;
@@ -287,37 +327,19 @@ softmax_ce_narrow_kernel(const float* __restrict__ l, const int32_t* __restrict_
       d.w = ok ? (e[u].w / s - (c0 + 3 == lab ? 1.f : 0.f)) * inv_b : nan;
       dr[sub + u * L] = d;
     }
-    if (sub == 0) row_loss[row] = ok ? (m + logf(s)) - l[static_cast<size_t>(row) * cols + lab] : nan;
+    if (sub == 0) part += ok ? (m + logf(s)) - l[static_cast<size_t>(row) * cols + lab] : nan;
   }
-  __shared__ int last;
-  __shared__ float red[256];
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) last = atomicAdd(counter, 1u) == gridDim.x - 1;
-  __syncthreads();
-  if (!last) return;
-  __threadfence();
-  float t = 0.f;
-  for (int r = threadIdx.x; r < rows; r += 256) t += __ldcg(row_loss + r);
-  red[threadIdx.x] = t;
-  __syncthreads();
-  for (int o = 128; o > 0; o >>= 1) {
-    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    *loss = red[0] / static_cast<float>(rows);
-    *counter = 0u;
-  }
+  loss_reduce(part, ws, counter, loss, rows);
 }
 
 // ---- softmax cross-entropy: one warp per row ------------------------------------------
 __global__ void __launch_bounds__(256)
 softmax_ce_kernel(const float* __restrict__ l, const int32_t* __restrict__ y, float* __restrict__ loss,
-                  float* __restrict__ dl, int rows, int cols, float* row_loss, unsigned* counter) {
+                  float* __restrict__ dl, int rows, int cols, float* ws, unsigned* counter) {
   const int lane = threadIdx.x & 31;
   const int warps_total = gridDim.x * 8;
   const float inv_b = 1.0f / static_cast<float>(rows);
+  float part = 0.f;
   for (int row = blockIdx.x * 8 + (threadIdx.x >> 5); row < rows; row += warps_total) {
     const float* lr = l + static_cast<size_t>(row) * cols;
     float* dr = dl + static_cast<size_t>(row) * cols;
@@ -333,33 +355,15 @@ softmax_ce_kernel(const float* __restrict__ l, const int32_t* __restrict__ y, fl
       const float p = expf(lr[c] - m) / s;
       dr[c] = ok ? (p - (c == lab ? 1.f : 0.f)) * inv_b : __int_as_float(0x7fffffff);
     }
-    if (lane == 0) row_loss[row] = ok ? (m + logf(s)) - lr[lab] : __int_as_float(0x7fffffff);
+    if (lane == 0) part += ok ? (m + logf(s)) - lr[lab] : __int_as_float(0x7fffffff);
   }
-  // The last CTA reduces the per-row losses in a fixed order.
-  __shared__ int last;
-  __shared__ float red[256];
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) last = atomicAdd(counter, 1u) == gridDim.x - 1;
-  __syncthreads();
-  if (!last) return;
-  __threadfence();
-  float t = 0.f;
-  for (int r = threadIdx.x; r < rows; r += 256) t += __ldcg(row_loss + r);
-  red[threadIdx.x] = t;
-  __syncthreads();
-  for (int o = 128; o > 0; o >>= 1) {
-    if (threadIdx.x < o) red[threadIdx.x] += red[threadIdx.x + o];
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    *loss = red[0] / static_cast<float>(rows);
-    *counter = 0u;
-  }
+  loss_reduce(part, ws, counter, loss, rows);
 }
 
 __global__ void __launch_bounds__(256)
 softmax_kernel(const float* __restrict__ l, float* __restrict__ p, int rows, int cols) {
+  sfdev::griddep_wait();
+  sfdev::griddep_launch();
   const int lane = threadIdx.x & 31;
   for (int row = blockIdx.x * 8 + (threadIdx.x >> 5); row < rows; row += gridDim.x * 8) {
     const float* lr = l + static_cast<size_t>(row) * cols;
@@ -377,6 +381,8 @@ softmax_kernel(const float* __restrict__ l, float* __restrict__ p, int rows, int
 // max / sum reduced through shared memory in a fixed tree order.
 __global__ void __launch_bounds__(256)
 softmax_block_kernel(const float* __restrict__ l, float* __restrict__ p, int cols) {
+  sfdev::griddep_wait();
+  sfdev::griddep_launch();
   const float* lr = l + static_cast<size_t>(blockIdx.x) * cols;
   float* pr = p + static_cast<size_t>(blockIdx.x) * cols;
   __shared__ float red[8];
@@ -514,9 +520,9 @@ cudaError_t launch_bias_act(const float* z, const float* b1, const float* b2, co
   auto al = [](const void* p) { return p == nullptr || reinterpret_cast<uintptr_t>(p) % 16 == 0; };
   const int vec = (cols % 4 == 0) && al(z) && al(b1) && al(b2) && al(b3) && al(h);
   const unsigned blocks = grid_for(vec ? total / 4 : total, 256 * 4, 148 * 8);
-  bias_act_kernel<<<blocks, 256, 0, st>>>(z, b1, b2, b3, h, rows, cols, relu ? 1 : 0, vec);
   count_launch();
-  return cudaGetLastError();
+  return launch_k(bias_act_kernel, dim3(blocks), dim3(256), 0, st, z, b1, b2, b3, h, rows, cols,
+                  relu ? 1 : 0, vec);
 }
 
 uint64_t colsum_ws_floats(int rows, int cols) {
@@ -553,7 +559,7 @@ cudaError_t launch_colsum(const float* x, const float* mask, float* dz, float* s
   return cudaGetLastError();
 }
 
-uint64_t softmax_ce_ws_floats(int rows) { return static_cast<uint64_t>(rows); }
+uint64_t softmax_ce_ws_floats(int rows) { return 148 * 8; }  // one partial per CTA (grid cap)
 
 cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float* loss,
                               float* dlogits, int rows, int cols, float* ws, unsigned* counter,
@@ -581,14 +587,12 @@ cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float*
 cudaError_t launch_softmax(const float* logits, float* probs, int rows, int cols, cudaStream_t st) {
   if (rows <= 0) return cudaSuccess;
   if (rows <= 64 && cols >= 256) {
-    softmax_block_kernel<<<rows, 256, 0, st>>>(logits, probs, cols);
     count_launch();
-    return cudaGetLastError();
+    return launch_k(softmax_block_kernel, dim3(rows), dim3(256), 0, st, logits, probs, cols);
   }
   const unsigned blocks = grid_for(static_cast<uint64_t>(rows), 8, 148 * 8);
-  softmax_kernel<<<blocks, 256, 0, st>>>(logits, probs, rows, cols);
   count_launch();
-  return cudaGetLastError();
+  return launch_k(softmax_kernel, dim3(blocks), dim3(256), 0, st, logits, probs, rows, cols);
 }
 
 cudaError_t launch_sgd(const SgdDesc* d, int n, uint64_t total, cudaStream_t st) {

@@ -19,6 +19,8 @@
 //
 // Batch-1 inference GEMMs (M <= 8) are HBM-bound weight streaming and
 // go to a split-K GEMV kernel instead of padding M to 128.
+#include <cooperative_groups.h>
+
 #include <algorithm>
 #include <atomic>
 #include <cstdlib>
@@ -26,6 +28,7 @@
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
+#include "sf_launch.cuh"
 
 namespace sfk {
 namespace {
@@ -491,6 +494,128 @@ gemv_reduce_kernel(const float* __restrict__ ws, float* __restrict__ C, int M, i
   *o = t;
 }
 
+// Cluster GEMV (N % 4 == 0): a cluster of kClusterK CTAs splits K; inside a CTA the 256
+// threads form RL = 256 / QW row lanes x QW column quads (lane = 4 adjacent columns, a row
+// segment of 16*QW contiguous bytes), row lane r taking rows k0 + r, k0 + r + RL, ...  x is
+// read through L1 (a warp-uniform broadcast), so weight streaming starts at the first
+// instruction.  The CTA reduces its row lanes in smem (fixed order), then the cluster leader
+// sums the kClusterK CTA partials through distributed shared memory in rank order and applies
+// bias + ReLU.  One launch per layer, deterministic, no global workspace.
+constexpr int kClusterK = 8;
+
+template <int MR, int QW>
+__global__ void __cluster_dims__(kClusterK, 1, 1) __launch_bounds__(256)
+gemv_cluster_kernel(const float* __restrict__ A, const float* __restrict__ B, float* __restrict__ C,
+                    int M, int N, int K, int lda, int ldb, int ldc, int kper, int acc,
+                    const float* __restrict__ b1, const float* __restrict__ b2,
+                    const float* __restrict__ b3, int relu) {
+  namespace cg = cooperative_groups;
+  constexpr int RL = 256 / QW;
+  sfdev::griddep_wait();
+  sfdev::griddep_launch();
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = static_cast<int>(cluster.block_rank());
+  const int cb = blockIdx.x / kClusterK;
+  const int qi = threadIdx.x % QW, rl = threadIdx.x / QW;
+  const int q = cb * QW + qi;
+  const int nq = N / 4;
+  const int k0 = rank * kper, k1 = min(K, k0 + kper);
+  __shared__ float4 red[RL][QW];
+  __shared__ float4 part[MR][QW];
+  float4 accv[MR];
+#pragma unroll
+  for (int m = 0; m < MR; ++m) accv[m] = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (q < nq) {
+    const float* col = B + 4 * q;
+    int k = k0 + rl;
+    for (; k + 7 * RL < k1; k += 8 * RL) {
+      float4 wv[8];
+      float xv[MR][8];
+      // all 8 weight rows in flight before any use: one asm block per 4 loads, so ptxas
+      // cannot interleave them with the FMAs that consume earlier rows
+      const size_t rs = static_cast<size_t>(RL) * ldb;
+      const float* p0 = col + static_cast<size_t>(k) * ldb;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const float* p = p0 + 4 * h * rs;
+        asm volatile(
+            "ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%16];\n\t"
+            "ld.global.nc.L1::no_allocate.v4.f32 {%4,%5,%6,%7}, [%17];\n\t"
+            "ld.global.nc.L1::no_allocate.v4.f32 {%8,%9,%10,%11}, [%18];\n\t"
+            "ld.global.nc.L1::no_allocate.v4.f32 {%12,%13,%14,%15}, [%19];"
+            : "=f"(wv[4 * h].x), "=f"(wv[4 * h].y), "=f"(wv[4 * h].z), "=f"(wv[4 * h].w),
+              "=f"(wv[4 * h + 1].x), "=f"(wv[4 * h + 1].y), "=f"(wv[4 * h + 1].z), "=f"(wv[4 * h + 1].w),
+              "=f"(wv[4 * h + 2].x), "=f"(wv[4 * h + 2].y), "=f"(wv[4 * h + 2].z), "=f"(wv[4 * h + 2].w),
+              "=f"(wv[4 * h + 3].x), "=f"(wv[4 * h + 3].y), "=f"(wv[4 * h + 3].z), "=f"(wv[4 * h + 3].w)
+            : "l"(p), "l"(p + rs), "l"(p + 2 * rs), "l"(p + 3 * rs));
+      }
+#pragma unroll
+      for (int m = 0; m < MR; ++m)
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+          xv[m][u] = m < M ? __ldg(A + static_cast<size_t>(m) * lda + k + RL * u) : 0.f;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+#pragma unroll
+        for (int m = 0; m < MR; ++m) {
+          const float xv_ = xv[m][u];
+          accv[m].x = fmaf(xv_, wv[u].x, accv[m].x); accv[m].y = fmaf(xv_, wv[u].y, accv[m].y);
+          accv[m].z = fmaf(xv_, wv[u].z, accv[m].z); accv[m].w = fmaf(xv_, wv[u].w, accv[m].w);
+        }
+    }
+    for (; k < k1; k += RL) {
+      const float4 wv = __ldcs(reinterpret_cast<const float4*>(col + static_cast<size_t>(k) * ldb));
+#pragma unroll
+      for (int m = 0; m < MR; ++m) {
+        const float xv = m < M ? __ldg(A + static_cast<size_t>(m) * lda + k) : 0.f;
+        accv[m].x = fmaf(xv, wv.x, accv[m].x); accv[m].y = fmaf(xv, wv.y, accv[m].y);
+        accv[m].z = fmaf(xv, wv.z, accv[m].z); accv[m].w = fmaf(xv, wv.w, accv[m].w);
+      }
+    }
+  }
+#pragma unroll
+  for (int m = 0; m < MR; ++m) {  // one row of x at a time keeps smem at 4 KB
+    red[rl][qi] = accv[m];
+    __syncthreads();
+    if (threadIdx.x < QW) {
+      float4 t = red[0][threadIdx.x];
+#pragma unroll 8
+      for (int j = 1; j < RL; ++j) {
+        const float4 v = red[j][threadIdx.x];
+        t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+      }
+      part[m][threadIdx.x] = t;
+    }
+    __syncthreads();
+  }
+  cluster.sync();  // every CTA's partial is visible cluster-wide
+  if (rank == 0 && threadIdx.x < MR * QW) {
+    const int m = threadIdx.x / QW, qq = cb * QW + threadIdx.x % QW;
+    if (m < M && qq < nq) {
+      float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int r = 0; r < kClusterK; ++r) {
+        const float4* remote = cluster.map_shared_rank(&part[0][0], r);
+        const float4 v = remote[threadIdx.x];
+        t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+      }
+      const int n = 4 * qq;
+      float* o = C + static_cast<size_t>(m) * ldc + n;
+      float r4[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float v = r4[j];
+        if (acc) v = o[j] + v;
+        if (b1) v += b1[n + j];
+        if (b2) v += b2[n + j];
+        if (b3) v += b3[n + j];
+        if (relu) v = fmaxf(v, 0.f);
+        o[j] = v;
+      }
+    }
+  }
+  cluster.sync();  // keep every CTA's smem alive until the leader has read it
+}
+
 struct Gemv4Plan { int splits, kper, col_blocks; };
 Gemv4Plan plan_gemv4(int N, int K) {
   Gemv4Plan g;
@@ -546,8 +671,43 @@ uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0) return cudaSuccess;
-  if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb) && a.ws))
+  if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)))
     return cudaErrorInvalidValue;  // fused epilogue only exists on the GEMV path
+  // M <= 8 paths: SF_GEMV = tma (default: TMA-streamed cluster GEMV) | cluster (register-
+  // streamed cluster GEMV) | split (split-K GEMV + separate reduce kernel)
+  static const char gemv_path = std::getenv("SF_GEMV") ? std::getenv("SF_GEMV")[0] : 't';
+  if (gemv_path == 't' && use_gemv(a.M, a.ta, a.tb) && gemv_tma_eligible(a)) return launch_gemv_tma(a, st);
+  if (gemv_path != 's' && use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)) {
+    // widest column block that still gives >= 2 CTAs per SM (the stream needs the MLP)
+    const int nq = a.N / 4;
+    int QW = 4;
+    for (int w : {32, 16, 8})
+      if ((nq + w - 1) / w * kClusterK >= 2 * 148) { QW = w; break; }
+    const int RL = 256 / QW;
+    int kper = (a.K + kClusterK - 1) / kClusterK;
+    kper = (kper + RL - 1) / RL * RL;
+    dim3 grid((nq + QW - 1) / QW * kClusterK);
+    cudaError_t e = cudaSuccess;
+#define SF_GEMVC2(MR, QWV)                                                                         \
+  e = launch_k(gemv_cluster_kernel<MR, QWV>, grid, dim3(256), 0, st, a.A, a.B, a.C, a.M, a.N, a.K, \
+               a.lda, a.ldb, a.ldc, kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2],      \
+               a.relu ? 1 : 0)
+#define SF_GEMVC(MR)                     \
+  do {                                   \
+    if (QW == 32) SF_GEMVC2(MR, 32);      \
+    else if (QW == 16) SF_GEMVC2(MR, 16); \
+    else if (QW == 8) SF_GEMVC2(MR, 8);   \
+    else SF_GEMVC2(MR, 4);                \
+  } while (0)
+    if (a.M == 1) SF_GEMVC(1);
+    else if (a.M == 2) SF_GEMVC(2);
+    else if (a.M <= 4) SF_GEMVC(4);
+    else SF_GEMVC(8);
+#undef SF_GEMVC
+#undef SF_GEMVC2
+    count_launch();
+    return e;
+  }
   if (use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb) && a.ws) {
     Gemv4Plan g = plan_gemv4(a.N, a.K);
     dim3 grid(g.col_blocks, g.splits);

@@ -15,6 +15,7 @@
 //                3-D workspace map and the last CTA of a tile sums them in order z=0..S-1.
 //
 // Same numerics as kernels_gemm.cu (parity-tested), different data movement.
+#include <cooperative_groups.h>
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -25,6 +26,7 @@
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
+#include "sf_launch.cuh"
 
 namespace sfk {
 namespace {
@@ -280,6 +282,228 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   if (warp == kMmaWarp) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
 }
 
+// ---- persistent variant -----------------------------------------------------------------
+// One CTA per SM loops over work units u = blockIdx.x + i * gridDim.x (tile_n fastest, then
+// tile_m, then split z).  TMEM holds two accumulators: the MMA warp fills unit i+1 while the
+// epilogue warps (10-13, one per TMEM lane quarter) drain unit i, so epilogue, prologue and
+// TMA latency overlap the tensor work.  Same per-tile arithmetic as gemm_tma_kernel.
+constexpr int kPThreads = 14 * 32;  // 0 TMA, 1-8 convert, 9 MMA, 10-13 epilogue
+
+template <int BN>
+struct PCfg {
+  static constexpr int STAGES = BN == 64 ? 4 : 3;
+  static constexpr int A_BYTES = BM * BK * 4;
+  static constexpr int B_BYTES = BN * BK * 4;
+  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int EPI_BYTES = 4 * 2 * 4096;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_BYTES + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = 2 * BN;
+};
+
+struct PParams {
+  int M, N, K, ldc;
+  int splits, kb_per_split, acc;
+  int tiles_n, tiles_m, units;
+  float* C;
+};
+
+template <int BN, bool A_MN, bool B_MN>
+__global__ void __launch_bounds__(kPThreads, 1)
+gemm_tma_persistent_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                           const __grid_constant__ CUtensorMap tmC, PParams p) {
+  using C = PCfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~static_cast<uintptr_t>(1023));
+  uint8_t* epi = smem + C::STAGES * C::STAGE_BYTES;
+  uint64_t* tma_full = reinterpret_cast<uint64_t*>(epi + C::EPI_BYTES);
+  uint64_t* conv_full = tma_full + C::STAGES;
+  uint64_t* empty = conv_full + C::STAGES;
+  uint64_t* acc_full = empty + C::STAGES;   // [2]
+  uint64_t* acc_empty = acc_full + 2;       // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nkb_total = (p.K + BK - 1) / BK;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < C::STAGES; ++s) {
+      sfdev::mbar_init(&tma_full[s], 1);
+      sfdev::mbar_init(&conv_full[s], kConvWarps);
+      sfdev::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      sfdev::mbar_init(&acc_full[a], 1);
+      sfdev::mbar_init(&acc_empty[a], 4);
+    }
+    sfdev::mbar_fence_init();
+    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
+  }
+  if (warp == kMmaWarp) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
+  sfdev::tc_fence_before();
+  __syncthreads();
+  sfdev::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  auto unit_coords = [&](int u, int& n0, int& m0, int& z, int& kb_begin, int& nkb) {
+    const int tn = u % p.tiles_n;
+    const int rest = u / p.tiles_n;
+    const int tm = rest % p.tiles_m;
+    z = rest / p.tiles_m;
+    n0 = tn * BN;
+    m0 = tm * BM;
+    kb_begin = z * p.kb_per_split;
+    nkb = max(0, min(nkb_total, kb_begin + p.kb_per_split) - kb_begin);
+  };
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int it = 0;  // global stage counter across units
+      for (int u = blockIdx.x; u < p.units; u += gridDim.x) {
+        int n0, m0, z, kb_begin, nkb;
+        unit_coords(u, n0, m0, z, kb_begin, nkb);
+        for (int i = 0; i < nkb; ++i, ++it) {
+          const int s = it % C::STAGES, round = it / C::STAGES;
+          if (round > 0) sfdev::mbar_wait(&empty[s], (round - 1) & 1);
+          const uint32_t st = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
+          const uint32_t bar = sfdev::smem_u32(&tma_full[s]);
+          expect_tx(&tma_full[s], C::A_BYTES + C::B_BYTES);
+          const int k0 = (kb_begin + i) * BK;
+          if constexpr (A_MN) {
+#pragma unroll
+            for (int b = 0; b < BM / 32; ++b) tma_load_2d(st + b * 4096, &tmA, bar, m0 + 32 * b, k0);
+          } else {
+            tma_load_2d(st, &tmA, bar, k0, m0);
+          }
+          const uint32_t sb = st + 2 * C::A_BYTES;
+          if constexpr (B_MN) {
+#pragma unroll
+            for (int b = 0; b < BN / 32; ++b) tma_load_2d(sb + b * 4096, &tmB, bar, n0 + 32 * b, k0);
+          } else {
+            tma_load_2d(sb, &tmB, bar, k0, n0);
+          }
+        }
+      }
+    }
+  } else if (warp <= kConvWarps) {
+    const int t = threadIdx.x - 32;
+    int it = 0;
+    for (int u = blockIdx.x; u < p.units; u += gridDim.x) {
+      int n0, m0, z, kb_begin, nkb;
+      unit_coords(u, n0, m0, z, kb_begin, nkb);
+      for (int i = 0; i < nkb; ++i, ++it) {
+        const int s = it % C::STAGES;
+        sfdev::mbar_wait(&tma_full[s], (it / C::STAGES) & 1);
+        uint8_t* st = smem + s * C::STAGE_BYTES;
+        split_tile<C::A_BYTES / 16 / 256, true>(reinterpret_cast<float4*>(st),
+                                                reinterpret_cast<float4*>(st + C::A_BYTES), t);
+        split_tile<C::B_BYTES / 16 / 256, true>(reinterpret_cast<float4*>(st + 2 * C::A_BYTES),
+                                                reinterpret_cast<float4*>(st + 2 * C::A_BYTES + C::B_BYTES), t);
+        sfdev::fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) sfdev::mbar_arrive(&conv_full[s]);
+      }
+    }
+  } else if (warp == kMmaWarp) {
+    constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((A_MN ? 1u : 0u) << 15) |
+                               ((B_MN ? 1u : 0u) << 16) | (uint32_t(BN >> 3) << 17) |
+                               (uint32_t(BM >> 4) << 24);
+    int it = 0, t_local = 0;
+    for (int u = blockIdx.x; u < p.units; u += gridDim.x, ++t_local) {
+      int n0, m0, z, kb_begin, nkb;
+      unit_coords(u, n0, m0, z, kb_begin, nkb);
+      const int a = t_local & 1;
+      sfdev::mbar_wait(&acc_empty[a], ((t_local >> 1) & 1) ^ 1);  // epilogue freed it
+      sfdev::tc_fence_after();
+      const uint32_t d = tmem + a * BN;
+      for (int i = 0; i < nkb; ++i, ++it) {
+        const int s = it % C::STAGES;
+        sfdev::mbar_wait(&conv_full[s], (it / C::STAGES) & 1);
+        sfdev::tc_fence_after();
+        if (lane == 0) {
+          const uint32_t base = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
+          const uint32_t a_hi = base, a_lo = base + C::A_BYTES;
+          const uint32_t b_hi = base + 2 * C::A_BYTES, b_lo = b_hi + C::B_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < BK / 8; ++kk) {
+            const uint32_t ao = A_MN ? kk * 1024 : kk * 32;
+            const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
+            auto da = [&](uint32_t x) { return A_MN ? desc_mn(x + ao) : desc_k(x + ao); };
+            auto db = [&](uint32_t x) { return B_MN ? desc_mn(x + bo) : desc_k(x + bo); };
+            sfdev::mma_tf32(d, da(a_lo), db(b_hi), idesc, (i | kk) != 0);
+            sfdev::mma_tf32(d, da(a_hi), db(b_lo), idesc, 1u);
+            sfdev::mma_tf32(d, da(a_hi), db(b_hi), idesc, 1u);
+          }
+          sfdev::mma_commit(&empty[s]);
+        }
+        __syncwarp();
+      }
+      if (lane == 0) sfdev::mma_commit(&acc_full[a]);
+      __syncwarp();
+    }
+  } else {
+    // epilogue warps 10-13: TMEM lane quarter (warp % 4)
+    const int q = warp & 3;
+    const int row0 = q * 32;
+    uint8_t* ebuf = epi + q * 2 * 4096;
+    int t_local = 0, nstore = 0;
+    for (int u = blockIdx.x; u < p.units; u += gridDim.x, ++t_local) {
+      int n0, m0, z, kb_begin, nkb;
+      unit_coords(u, n0, m0, z, kb_begin, nkb);
+      const int a = t_local & 1;
+      sfdev::mbar_wait(&acc_full[a], (t_local >> 1) & 1);
+      sfdev::tc_fence_after();
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN; c0 += 32, ++nstore) {
+        uint32_t r[32];
+        sfdev::tmem_ld32(tmem + a * BN + (static_cast<uint32_t>(row0) << 16) + c0, r);
+        sfdev::tmem_ld_wait();
+        if (c0 + 32 >= BN) {  // all of this accumulator read: hand it back to the MMA warp
+          sfdev::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) sfdev::mbar_arrive(&acc_empty[a]);
+        }
+        if (p.splits == 1 && p.acc) {
+          const int row = m0 + row0 + lane;
+          if (row < p.M)
+#pragma unroll
+            for (int j = 0; j < 32; ++j)
+              if (n0 + c0 + j < p.N)
+                r[j] = __float_as_uint(__uint_as_float(r[j]) + p.C[static_cast<size_t>(row) * p.ldc + n0 + c0 + j]);
+        }
+        uint8_t* buf = ebuf + (nstore & 1) * 4096;
+        if (nstore >= 2) {
+          if (lane == 0) bulk_wait_read1();
+          __syncwarp();
+        }
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) {
+          const uint32_t off = lane * 128 + ((ch ^ (lane & 7)) << 4);
+          *reinterpret_cast<uint4*>(buf + off) = make_uint4(r[4 * ch], r[4 * ch + 1], r[4 * ch + 2], r[4 * ch + 3]);
+        }
+        sfdev::fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          if (p.splits == 1) tma_store_2d(&tmC, sfdev::smem_u32(buf), n0 + c0, m0 + row0);
+          else tma_store_3d(&tmC, sfdev::smem_u32(buf), n0 + c0, m0 + row0, z);
+          bulk_commit();
+        }
+      }
+    }
+    if (lane == 0) {
+      bulk_wait_all();
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+    }
+    __syncwarp();
+  }
+  sfdev::tc_fence_before();
+  __syncthreads();
+  sfdev::tc_fence_after();
+  if (warp == kMmaWarp) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
+}
+
 // Deterministic split-K reduction: C[m][n] (+)= sum_{z} ws[z][m][n].  Block = 32 float4
 // output groups x 8 split lanes; lane zl sums z = zl, zl+8, ... (two accumulators), the 8
 // lane partials are then combined in index order — parallel over outputs AND splits.
@@ -322,6 +546,147 @@ splitk_reduce_kernel(const float* __restrict__ ws, float* __restrict__ C, int M,
     t.x = c.x + t.x; t.y = c.y + t.y; t.z = c.z + t.z; t.w = c.w + t.w;
   }
   *o = t;
+}
+
+
+// ---- TMA-streamed cluster GEMV (M <= 8, the inference path of SURVEY.md 8(a) C4) ----------
+// y[m][n] = sum_k x[m][k] W[k][n] (+ C if acc) (+ bias...) (ReLU): HBM-bound on W.  A cluster
+// of kGvCluster CTAs splits K; each CTA owns BC columns x kper rows of W.  Warp 8 (one thread)
+// streams W as {BC cols x 32 rows} TMA boxes through a 64 KB mbarrier ring, so every CTA has
+// 64 KB of loads in flight from its first cycle (the register-streamed kernels depended on
+// ptxas keeping loads ahead of their FMAs, which it does not).  Warps 0-7: thread = (row lane
+// rl, column quad qi), QW = BC/4 quads x RL = 256/QW row lanes; x is staged in smem while the
+// first boxes are in flight.  Reduction: row lanes in smem in fixed order, then the cluster
+// leader sums the kGvCluster partials over DSMEM in rank order (deterministic, one launch).
+constexpr int kGvCluster = 8;
+constexpr int kGvRows = 32;            // rows per TMA box
+constexpr int kGvRing = 64 * 1024;     // bytes of W in flight per CTA
+constexpr int kGvMaxKper = 1024;       // x slice staged in smem (K <= 8192)
+
+template <int MR, int BC>
+struct GvCfg {
+  static constexpr int QW = BC / 4, RL = 256 / QW, BOX = BC * kGvRows * 4, S = kGvRing / BOX;
+  static constexpr int RED = RL * QW * 16, PART = MR * QW * 16;
+  static size_t smem(int kper) { return kGvRing + RED + PART + 2 * S * 8 + size_t(MR) * kper * 4 + 128; }
+};
+
+template <int MR, int BC>
+__global__ void __cluster_dims__(kGvCluster, 1, 1) __launch_bounds__(288)
+gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict__ X,
+                float* __restrict__ Y, int M, int N, int K, int ldx, int ldy, int kper, int acc,
+                const float* __restrict__ b1, const float* __restrict__ b2,
+                const float* __restrict__ b3, int relu, int b_const) {
+  using Cfg = GvCfg<MR, BC>;
+  constexpr int QW = Cfg::QW, RL = Cfg::RL, S = Cfg::S;
+  extern __shared__ __align__(1024) unsigned char gv_smem[];
+  float4* ring = reinterpret_cast<float4*>(gv_smem);
+  float4* red = reinterpret_cast<float4*>(gv_smem + kGvRing);
+  float4* part = reinterpret_cast<float4*>(gv_smem + kGvRing + Cfg::RED);
+  uint64_t* full = reinterpret_cast<uint64_t*>(gv_smem + kGvRing + Cfg::RED + Cfg::PART);
+  uint64_t* empty = full + S;
+  float* xs = reinterpret_cast<float*>(empty + S);
+
+  namespace cg = cooperative_groups;
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = static_cast<int>(cluster.block_rank());
+  const int cb = blockIdx.x / kGvCluster;
+  const int c0 = cb * BC;
+  const int k0 = rank * kper, k1 = min(K, k0 + kper);
+  const int nbox = k1 > k0 ? (k1 - k0 + kGvRows - 1) / kGvRows : 0;
+  const int tid = threadIdx.x, warp = tid >> 5;
+
+  if (tid == 0) {
+    for (int i = 0; i < S; ++i) {
+      sfdev::mbar_init(&full[i], 1);
+      sfdev::mbar_init(&empty[i], 8);
+    }
+    sfdev::mbar_fence_init();
+  }
+  __syncthreads();
+
+  float4 accv[MR];
+#pragma unroll
+  for (int m = 0; m < MR; ++m) accv[m] = make_float4(0.f, 0.f, 0.f, 0.f);
+  const int qi = tid % QW, rl = tid / QW;
+
+  sfdev::griddep_launch();  // single wave: the next layer may start its own W stream now
+  if (warp == 8) {
+    if ((tid & 31) == 0) {
+      if (!b_const) sfdev::griddep_wait();  // W may be written by the predecessor
+      for (int i = 0; i < nbox; ++i) {
+        const int slot = i % S;
+        if (i >= S) sfdev::mbar_wait(&empty[slot], ((i / S) - 1) & 1);
+        expect_tx(&full[slot], Cfg::BOX);
+        tma_load_2d(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]), c0,
+                    k0 + i * kGvRows);
+      }
+    }
+    __syncwarp();
+  } else {
+    sfdev::griddep_wait();  // x is the predecessor's output
+    for (int i = tid; i < MR * kper; i += 256) {
+      const int m = i / kper, kk = i % kper;
+      xs[i] = (m < M && k0 + kk < k1) ? X[static_cast<size_t>(m) * ldx + k0 + kk] : 0.f;
+    }
+    asm volatile("bar.sync 1, 256;" ::: "memory");
+    for (int i = 0; i < nbox; ++i) {
+      const int slot = i % S;
+      sfdev::mbar_wait(&full[slot], (i / S) & 1);
+      const float4* tile = ring + slot * (Cfg::BOX / 16);
+#pragma unroll
+      for (int r = rl; r < kGvRows; r += RL) {
+        const float4 w = tile[r * QW + qi];
+        const int kk = i * kGvRows + r;
+#pragma unroll
+        for (int m = 0; m < MR; ++m) {
+          const float xv = xs[m * kper + kk];
+          accv[m].x = fmaf(xv, w.x, accv[m].x); accv[m].y = fmaf(xv, w.y, accv[m].y);
+          accv[m].z = fmaf(xv, w.z, accv[m].z); accv[m].w = fmaf(xv, w.w, accv[m].w);
+        }
+      }
+      __syncwarp();
+      if ((tid & 31) == 0) sfdev::mbar_arrive(&empty[slot]);
+    }
+  }
+#pragma unroll
+  for (int m = 0; m < MR; ++m) {
+    if (tid < 256) red[rl * QW + qi] = accv[m];
+    __syncthreads();
+    if (tid < QW) {
+      float4 t = red[tid];
+#pragma unroll 8
+      for (int j = 1; j < RL; ++j) {
+        const float4 v = red[j * QW + tid];
+        t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+      }
+      part[m * QW + tid] = t;
+    }
+    __syncthreads();
+  }
+  cluster.sync();
+  if (rank == 0 && tid < MR * QW) {
+    const int m = tid / QW, n = c0 + 4 * (tid % QW);
+    if (m < M && n < N) {
+      float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int r = 0; r < kGvCluster; ++r) {
+        const float4 v = cluster.map_shared_rank(part, r)[tid];
+        t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+      }
+      float* o = Y + static_cast<size_t>(m) * ldy + n;
+      const float r4[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float v = r4[j];
+        if (acc) v = o[j] + v;
+        if (b1) v += b1[n + j];
+        if (b2) v += b2[n + j];
+        if (b3) v += b3[n + j];
+        if (relu) v = fmaxf(v, 0.f);
+        o[j] = v;
+      }
+    }
+  }
+  cluster.sync();
 }
 
 // ---- host: tensor maps ------------------------------------------------------------------
@@ -382,6 +747,34 @@ cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUten
   return cudaGetLastError();
 }
 
+template <int BN, bool AM, bool BMn>
+cudaError_t launch_persistent_t(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
+                                const PParams& p, cudaStream_t st) {
+  auto kern = gemm_tma_persistent_kernel<BN, AM, BMn>;
+  static std::atomic<uint64_t> configured{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (!(configured.load() & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<BN>::SMEM);
+    if (e != cudaSuccess) return e;
+    configured.fetch_or(bit);
+  }
+  const int grid = std::min(p.units, 148);
+  kern<<<grid, kPThreads, PCfg<BN>::SMEM, st>>>(a, b, c, p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int BN>
+cudaError_t dispatch_persistent(bool a_mn, bool b_mn, const CUtensorMap& a, const CUtensorMap& b,
+                                const CUtensorMap& c, const PParams& p, cudaStream_t st) {
+  if (a_mn && b_mn) return launch_persistent_t<BN, true, true>(a, b, c, p, st);
+  if (a_mn) return launch_persistent_t<BN, true, false>(a, b, c, p, st);
+  if (b_mn) return launch_persistent_t<BN, false, true>(a, b, c, p, st);
+  return launch_persistent_t<BN, false, false>(a, b, c, p, st);
+}
+
 template <int BN, bool RAW>
 cudaError_t dispatch_major(bool a_mn, bool b_mn, const CUtensorMap& a, const CUtensorMap& b,
                            const CUtensorMap& c, const TParams& p, dim3 grid, cudaStream_t st) {
@@ -391,7 +784,59 @@ cudaError_t dispatch_major(bool a_mn, bool b_mn, const CUtensorMap& a, const CUt
   return launch_tma_t<BN, false, false, RAW>(a, b, c, p, grid, st);
 }
 
+
+template <int MR, int BC>
+cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cudaStream_t st) {
+  auto kern = gemv_tma_kernel<MR, BC>;
+  const size_t smem = GvCfg<MR, BC>::smem(kper);
+  static std::atomic<uint64_t> configured{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (!(configured.load() & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         GvCfg<MR, BC>::smem(kGvMaxKper));
+    if (e != cudaSuccess) return e;
+    configured.fetch_or(bit);
+  }
+  const int grid = (a.N + BC - 1) / BC * kGvCluster;
+  count_launch();
+  return launch_k(kern, dim3(grid), dim3(288), smem, st, w, a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc,
+                  kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
+                  a.b_const ? 1 : 0);
+}
+
+template <int BC>
+cudaError_t dispatch_gemv_mr(const CUtensorMap& w, const GemmArgs& a, int kper, cudaStream_t st) {
+  if (a.M == 1) return launch_gemv_t<1, BC>(w, a, kper, st);
+  if (a.M == 2) return launch_gemv_t<2, BC>(w, a, kper, st);
+  if (a.M <= 4) return launch_gemv_t<4, BC>(w, a, kper, st);
+  return launch_gemv_t<8, BC>(w, a, kper, st);
+}
+
 }  // namespace
+
+bool gemv_tma_eligible(const GemmArgs& a) {
+  auto al = [](const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; };
+  if (!encode_fn() || a.M < 1 || a.M > 8 || a.ta || a.tb) return false;
+  if (a.N % 4 || a.ldb % 4 || a.ldc % 4 || !al(a.B) || !al(a.C)) return false;
+  return (a.K + kGvCluster - 1) / kGvCluster <= kGvMaxKper;
+}
+
+cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st) {
+  // widest column block that still puts one CTA on every SM
+  int bc = 32;
+  for (int c : {128, 64})
+    if ((a.N + c - 1) / c * kGvCluster >= 148) { bc = c; break; }
+  int kper = (a.K + kGvCluster - 1) / kGvCluster;
+  kper = (kper + kGvRows - 1) / kGvRows * kGvRows;
+  CUtensorMap w;
+  if (!map2d(&w, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, bc, kGvRows, CU_TENSOR_MAP_SWIZZLE_NONE))
+    return cudaErrorInvalidValue;
+  if (bc == 128) return dispatch_gemv_mr<128>(w, a, kper, st);
+  if (bc == 64) return dispatch_gemv_mr<64>(w, a, kper, st);
+  return dispatch_gemv_mr<32>(w, a, kper, st);
+}
 
 bool gemm_tma_eligible(const GemmArgs& a, int splits) {
   auto al = [](const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; };
@@ -419,7 +864,15 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   TParams p{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, dbg, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;
-  if (bn == 64)
+  // persistent CTAs (double-buffered TMEM) measured equal to per-tile CTAs on the forest
+  // shapes (profiles/r01_ncu_summary.md); opt in with SF_GEMM_PERSISTENT=1
+  static const bool persistent = std::getenv("SF_GEMM_PERSISTENT") && std::getenv("SF_GEMM_PERSISTENT")[0] == '1';
+  if (persistent && raw_hi) {
+    PParams pp{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, tiles_n, tiles_m,
+               tiles_n * tiles_m * splits, a.C};
+    e = bn == 64 ? dispatch_persistent<64>(a_mn, b_mn, ma, mb, mc, pp, st)
+                 : dispatch_persistent<128>(a_mn, b_mn, ma, mb, mc, pp, st);
+  } else if (bn == 64)
     e = raw_hi ? dispatch_major<64, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<64, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
   else

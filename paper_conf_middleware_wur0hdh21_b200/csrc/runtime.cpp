@@ -37,6 +37,13 @@
 #include "sf_kernels.h"
 
 namespace {
+inline void cpu_relax() {
+#if defined(__x86_64__) || defined(__i386__)
+  __builtin_ia32_pause();
+#else
+  std::atomic_signal_fence(std::memory_order_seq_cst);
+#endif
+}
 
 thread_local std::string g_err;
 
@@ -96,6 +103,7 @@ struct Binding {
   // padded-pitch copies of DATASET GEMM operands whose row pitch is not 16-B aligned (the
   // TMA tensor-map requirement); refreshed from the arena at sf_start_training
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
+  std::map<int, void*> prepared;  // optimizer group first op -> uploaded descriptor array
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
   // refreshed inside the version graph (copy2d before / after the GEMM)
   struct PadBuf { float* p = nullptr; int pitch = 0; };
@@ -118,6 +126,7 @@ struct Graph {
   uint64_t ws_floats = 0, counter_slots = 0;
   std::vector<std::unique_ptr<Binding>> bind;  // per slot
   int input_tid = -1, output_tid = -1;
+  std::vector<char> op_written;  // tensor id -> some op of the graph writes it
 };
 
 constexpr int kInferOwner = 1 << 20;
@@ -134,6 +143,7 @@ struct Request {
   int preempted_job = -1;
   int64_t cut_iter = -1;
   int cut_k = -1;
+  float device_us = -1.f;
   std::string error;
 };
 
@@ -142,9 +152,11 @@ struct Slot {
   bool remote = false;  // another process's device (arena mapped over CUDA IPC)
   cudaStream_t s_train = nullptr, s_infer = nullptr, s_mig = nullptr;
   cudaEvent_t ev_infer = nullptr;
+  cudaEvent_t ev_i0 = nullptr;  // timing: request chain start (ev_infer marks its end)
   unsigned long long* tstamp = nullptr;  // device {start, end} x 2 (pack/peer, unpack)
-  int owner = -1;
+  std::atomic<int> owner{-1};  // device token (atomic: the spinning dispatcher polls it)
   std::deque<Request*> q;
+  std::atomic<int> qn{0};       // q.size(), readable without the runtime lock
   std::thread dispatcher;
   uint64_t persistent_bound = 0;
 };
@@ -194,6 +206,7 @@ struct sf_runtime {
   std::mutex m;
   std::condition_variable cv;
   bool shutting_down = false;
+  std::atomic<bool> stop_spin{false};
   std::vector<sf_trace_event> trace;
   size_t trace_cap = 1 << 16;
   size_t trace_dropped = 0;
@@ -599,6 +612,7 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         ga.M = C.rows; ga.N = C.cols; ga.K = ga.ta ? A.rows : A.cols;
         ga.lda = A.cols; ga.ldb = B.cols; ga.ldc = C.cols;
         ga.ws = c.b.ws; ga.counters = c.b.counters;
+        ga.b_const = !g.op_written[o.in[1]];
         auto sa = c.b.shadow.find(o.in[0]);
         if (sa != c.b.shadow.end()) { ga.A = sa->second.first; ga.lda = sa->second.second; }
         auto sb = c.b.shadow.find(o.in[1]);
@@ -620,7 +634,7 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
             }
           }
           if (pads[0].p) { ga.A = pads[0].p; ga.lda = pads[0].pitch; }
-          if (pads[1].p) { ga.B = pads[1].p; ga.ldb = pads[1].pitch; }
+          if (pads[1].p) { ga.B = pads[1].p; ga.ldb = pads[1].pitch; ga.b_const = false; }
           if (pads[2].p) { ga.C = pads[2].p; ga.ldc = pads[2].pitch; }
           err = sfk::launch_gemm(ga, c.st);
           if (err == cudaSuccess && pads[2].p)
@@ -1014,6 +1028,16 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     bool stamp;
   };
   std::deque<Inflight> q;
+  // device-time estimate per subgraph (EMA of host-observed busy intervals); with
+  // inflight_budget_us > 0 a subgraph is queued behind others only while the queued work
+  // stays within the budget, which bounds the drain a preemption waits for
+  std::vector<double> est_us(n, 0.0);
+  const double budget_us = rt->cfg.inflight_budget_us;
+  auto queued_us = [&] {
+    double t = 0.0;
+    for (const auto& f : q) t += est_us[f.k];
+    return t;
+  };
   int ev_next = 0;
   uint64_t last_t1 = 0;
   std::unique_lock<std::mutex> lk(rt->m);
@@ -1091,7 +1115,8 @@ void driver_main(sf_runtime* rt, Job* Jp) {
             J.holds_token = true;
           }
         }
-        launch = (!rt->cfg.exclusive_gpu || J.holds_token) && static_cast<int>(q.size()) < W;
+        launch = (!rt->cfg.exclusive_gpu || J.holds_token) && static_cast<int>(q.size()) < W &&
+                 (q.empty() || budget_us <= 0.0 || queued_us() + est_us[J.k] <= budget_us);
       }
     }
     if (launch) {
@@ -1177,6 +1202,10 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     tev.iter = f.it;
     tev.t0_ns = std::max(f.t0, last_t1);  // queued behind its predecessor on the stream
     tev.t1_ns = t1;
+    {
+      const double d = (t1 - tev.t0_ns) * 1e-3;
+      est_us[f.k] = est_us[f.k] > 0.0 ? 0.75 * est_us[f.k] + 0.25 * d : d;
+    }
     tev.arrival_ns = f.t0;  // train events: host dispatch (launch) time
     last_t1 = t1;
     push_trace(rt, tev);
@@ -1190,11 +1219,25 @@ void driver_main(sf_runtime* rt, Job* Jp) {
 void dispatcher_main(sf_runtime* rt, Slot* S) {
   cudaSetDevice(S->cuda);
   std::unique_lock<std::mutex> lk(rt->m);
+  const bool excl = rt->cfg.exclusive_gpu != 0;
+  const int64_t spin_us = rt->cfg.dispatch_spin_us;
+  auto free_for_inference = [&] {
+    const int o = S->owner.load(std::memory_order_acquire);
+    return !excl || o == -1 || o == kInferOwner;
+  };
+  auto ready = [&] { return rt->shutting_down || (!S->q.empty() && free_for_inference()); };
   while (true) {
-    rt->cv.wait(lk, [&] {
-      return rt->shutting_down ||
-             (!S->q.empty() && (!rt->cfg.exclusive_gpu || S->owner == -1 || S->owner == kInferOwner));
-    });
+    if (!ready() && spin_us != 0) {
+      // busy-poll (no futex wake-up on the request path) for dispatch_spin_us, -1 = forever
+      const uint64_t deadline = spin_us < 0 ? ~0ull : now_ns() + static_cast<uint64_t>(spin_us) * 1000;
+      lk.unlock();
+      while (!rt->stop_spin.load(std::memory_order_relaxed) && now_ns() < deadline) {
+        if (S->qn.load(std::memory_order_acquire) > 0 && free_for_inference()) break;
+        for (int i = 0; i < 32; ++i) cpu_relax();
+      }
+      lk.lock();
+    }
+    rt->cv.wait(lk, ready);
     if (S->q.empty() && rt->shutting_down) break;
     if (S->q.empty()) continue;
     if (rt->cfg.exclusive_gpu) S->owner = kInferOwner;
@@ -1211,28 +1254,53 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     const bool aligned = reinterpret_cast<uintptr_t>(r->in) % 16 == 0 &&
                          reinterpret_cast<uintptr_t>(r->out) % 16 == 0 && tin.nbytes % 4 == 0 &&
                          tout.nbytes % 4 == 0;
-    if (aligned) {
+    // Direct launches with programmatic dependent launch (default): each kernel of the chain
+    // is scheduled while its predecessor drains and GEMVs stream their (constant) weights
+    // before the previous layer finishes; SF_INFER_DIRECT=0 replays the captured versions.
+    static const bool direct = !(std::getenv("SF_INFER_DIRECT") && std::getenv("SF_INFER_DIRECT")[0] == '0');
+    static const bool use_pdl = !(std::getenv("SF_PDL") && std::getenv("SF_PDL")[0] == '0');
+    std::string op_err;
+    if (direct) sfk::set_pdl(use_pdl);
+    e = cudaEventRecord(S->ev_i0, S->s_infer);
+    if (e != cudaSuccess) {
+    } else if (aligned) {
       e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
     for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
-      e = cudaGraphLaunch(B->versions[k], S->s_infer);
-      sfk::count_launch(B->version_kernels[k]);
+      if (direct) {
+        Capture c{g, *B, S->s_infer, false, &B->prepared};
+        if (launch_subgraph_ops(c, static_cast<int>(k)) != SF_OK) {
+          op_err = g_err;
+          e = cudaErrorUnknown;
+        }
+      } else {
+        e = cudaGraphLaunch(B->versions[k], S->s_infer);
+        sfk::count_launch(B->version_kernels[k]);
+      }
     }
     if (e == cudaSuccess) {
       if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
       else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
     }
+    sfk::set_pdl(false);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
     if (e == cudaSuccess) e = spin_event(S->ev_infer);
     const uint64_t t1 = now_ns();
+    float dev_ms = -1.f;
+    if (e == cudaSuccess && cudaEventElapsedTime(&dev_ms, S->ev_i0, S->ev_infer) != cudaSuccess) {
+      dev_ms = -1.f;
+      cudaGetLastError();
+    }
     lk.lock();
     r->start = t0;
     r->end = t1;
-    if (e != cudaSuccess) r->error = cudaGetErrorString(e);
+    r->device_us = dev_ms >= 0.f ? dev_ms * 1e3f : -1.f;
+    if (e != cudaSuccess) r->error = op_err.empty() ? cudaGetErrorString(e) : op_err;
     r->done = true;
     S->q.pop_front();
+    S->qn.fetch_sub(1);
     sf_trace_event ev{};
     ev.dev = S->id; ev.job = static_cast<int32_t>(kInferOwner | (r->id & 0xFFFFF)); ev.kind = SF_EV_INFER;
     ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
@@ -1288,7 +1356,8 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
     SF_CK(cudaStreamCreateWithFlags(&S->s_train, cudaStreamNonBlocking));
     SF_CK(cudaStreamCreateWithPriority(&S->s_infer, cudaStreamNonBlocking, hi));
     SF_CK(cudaStreamCreateWithFlags(&S->s_mig, cudaStreamNonBlocking));
-    SF_CK(cudaEventCreateWithFlags(&S->ev_infer, cudaEventDisableTiming));
+    SF_CK(cudaEventCreate(&S->ev_infer));
+    SF_CK(cudaEventCreate(&S->ev_i0));
     SF_CK(cudaMalloc(&S->tstamp, 4 * sizeof(unsigned long long)));
     rt->slots.push_back(std::move(S));
   }
@@ -1325,6 +1394,7 @@ void sf_destroy(sf_runtime* rt) {
       return true;
     });
     rt->shutting_down = true;
+    rt->stop_spin = true;
     rt->cv.notify_all();
   }
   for (auto& J : rt->jobs)
@@ -1370,6 +1440,7 @@ void sf_destroy(sf_runtime* rt) {
     cudaStreamDestroy(S->s_infer);
     cudaStreamDestroy(S->s_mig);
     cudaEventDestroy(S->ev_infer);
+    cudaEventDestroy(S->ev_i0);
     cudaFree(S->tstamp);
   }
   delete rt;
@@ -1396,6 +1467,9 @@ sf_status sf_register_graph(sf_runtime* rt, const sf_graph_desc* gd, int32_t pri
     if (g->T[i].kind == SF_INPUT && g->input_tid < 0) g->input_tid = static_cast<int>(i);
     if (g->T[i].kind == SF_OUTPUT && g->output_tid < 0) g->output_tid = static_cast<int>(i);
   }
+  g->op_written.assign(g->T.size(), 0);
+  for (const auto& op : g->ops)
+    for (int q = 0; q < op.n_out; ++q) g->op_written[op.out[q]] = 1;
   std::lock_guard<std::mutex> lk(rt->m);
   g->bind.resize(rt->slots.size());
   rt->graphs.push_back(std::move(g));
@@ -1541,7 +1615,7 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
   // versions: one CUDA graph per subgraph
   cudaStream_t cap;
   SF_CK(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
-  std::map<int, void*> prepared;
+  std::map<int, void*>& prepared = b->prepared;
   {
     Capture prep{g, *b, cap, true, &prepared};
     for (size_t k = 0; k < g.parts.size(); ++k)
@@ -1851,6 +1925,7 @@ sf_status sf_submit_inference(sf_runtime* rt, sf_graph_id gid, int32_t dev, cons
   Request* rp = r.get();
   rt->reqs.emplace(r->id, std::move(r));
   rt->slots[dev]->q.push_back(rp);
+  rt->slots[dev]->qn.fetch_add(1);
   *req = rp->id;
   rt->cv.notify_all();
   return SF_OK;
@@ -1874,6 +1949,7 @@ sf_status sf_wait(sf_runtime* rt, sf_req_id id, int64_t timeout_ns, sf_timing* t
     t->preempted_job = r->preempted_job;
     t->cut_iter = r->cut_iter;
     t->cut_k = r->cut_k;
+    t->device_us = r->device_us;
   }
   std::string err = r->error;
   rt->reqs.erase(it);
@@ -1919,11 +1995,19 @@ sf_status sf_op_mtcopy(const sf_copy_desc* descs, int32_t n, int64_t patch_iter,
   return SF_OK;
 }
 
-sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
-                     int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
+static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
+                         int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, const float* b1,
+                         const float* b2, const float* b3, bool relu, void* stream) {
   if (!A || !B || !C || M <= 0 || N <= 0 || K <= 0) return fail(SF_EINVAL, "gemm args");
+  if (!b1 && (b2 || b3)) return fail(SF_EINVAL, "gemm bias args");
   sfk::GemmArgs ga{A, B, C, M, N, K, lda, ldb, ldc, (flags & SF_GEMM_TA) != 0,
                    (flags & SF_GEMM_TB) != 0, (flags & SF_GEMM_ACC) != 0, nullptr, nullptr};
+  const bool epi = b1 || relu;
+  const bool fuse = epi && sfk::gemm_can_fuse_bias(M, N, K, ga.ta, ga.tb, ldb);
+  if (fuse) {
+    ga.bias[0] = b1; ga.bias[1] = b2; ga.bias[2] = b3;
+    ga.relu = relu;
+  }
   cudaStream_t st = as_stream(stream);
   const uint64_t wsf = sfk::gemm_workspace_floats(M, N, K, ga.ta, ga.tb);
   const uint64_t cs = sfk::gemm_counter_slots(M, N, K, ga.ta, ga.tb);
@@ -1941,7 +2025,24 @@ sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_
     SF_CK(cudaFreeAsync(ws, st));
     SF_CK(cudaFreeAsync(cnt, st));
   }
+  if (epi && !fuse) {
+    if (ldc != N) return fail(SF_EINVAL, "unfused gemm epilogue needs ldc == N");
+    SF_CK(sfk::launch_bias_act(C, b1, b2, b3, C, M, N, relu, st));
+  }
   return SF_OK;
+}
+
+sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
+                     int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
+  return op_gemm(A, B, C, M, N, K, lda, ldb, ldc, flags, nullptr, nullptr, nullptr, false, stream);
+}
+
+sf_status sf_op_gemm_bias_act(const float* A, const float* B, float* C, int32_t M, int32_t N,
+                              int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
+                              const float* b1, const float* b2, const float* b3, int32_t relu,
+                              void* stream) {
+  if (!b1) return fail(SF_EINVAL, "gemm_bias_act needs b1");
+  return op_gemm(A, B, C, M, N, K, lda, ldb, ldc, flags, b1, b2, b3, relu != 0, stream);
 }
 
 sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,

@@ -108,4 +108,13 @@ __device__ __forceinline__ uint64_t globaltimer() {
   return t;
 }
 
+// ---- programmatic dependent launch (PDL) ----------------------------------------------
+// Kernels launched with the programmatic-serialization attribute may start while their
+// predecessor in the stream is still running: everything that reads the predecessor's output
+// must follow griddep_wait() (a no-op for normal launches), and every PDL-launched kernel calls
+// it before completing so the dependency stays transitive.  griddep_launch() lets this
+// kernel's own PDL successor be scheduled early.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch() { asm volatile("griddepcontrol.launch_dependents;"); }
+
 }  // namespace sfdev

@@ -39,14 +39,24 @@ struct GemmArgs {
   // optional fused epilogue (batch-1 GEMV path only): C = act(AB + b1 + b2 + b3)
   const float* bias[3] = {nullptr, nullptr, nullptr};
   bool relu = false;
+  // B is not written by any kernel that may still be running (inference weights): the GEMV
+  // may stream it before griddep_wait() under programmatic dependent launch
+  bool b_const = false;
 };
 // True when launch_gemm can fuse a following BIAS_ACT into this GEMM's epilogue.
+// Programmatic dependent launch for the launches this host thread makes (thread-local;
+// the inference dispatcher enables it around a request's kernel chain).
+void set_pdl(bool on);
+bool pdl_enabled();
 bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb);
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
 // TMA-fed variant (kernels_gemm_tma.cu): needs 16-B aligned pointers and row pitches.
 bool gemm_tma_eligible(const GemmArgs& a, int splits);
+// M <= 8 (inference): TMA-streamed cluster GEMV with fused reduction + bias/ReLU epilogue.
+bool gemv_tma_eligible(const GemmArgs& a);
+cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st);
 cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_split, int tiles_n,
                             int tiles_m, bool raw_hi, cudaStream_t st);
 

@@ -36,6 +36,18 @@ def gemm(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, flags: int = 0, st
                            flags, _s(stream)), "sf_op_gemm")
 
 
+def gemm_bias_act(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, biases: Sequence[torch.Tensor],
+                  relu: bool, flags: int = 0, stream=None) -> None:
+    """C = act(op(A) op(B) (+C if ACC) + sum(biases)) — forward layer with fused epilogue."""
+    bs = list(biases) + [None] * (3 - len(biases))
+    _need_cuda(A_, B, C_, *bs)
+    M, N = C_.shape
+    K = A_.shape[0] if flags & TA else A_.shape[1]
+    check(lib().sf_op_gemm_bias_act(_p(A_), _p(B), _p(C_), M, N, K, A_.shape[1], B.shape[1],
+                                    C_.shape[1], flags, _p(bs[0]), _p(bs[1]), _p(bs[2]), int(relu),
+                                    _s(stream)), "sf_op_gemm_bias_act")
+
+
 def bias_act(z, biases: Sequence[torch.Tensor], h, relu: bool, stream=None) -> None:
     bs = list(biases) + [None] * (3 - len(biases))
     _need_cuda(z, h, *bs)

@@ -80,6 +80,9 @@ GEMM_SHAPES = [
     (1, 4096, 2048, 0), (3, 17, 5, 0), (129, 65, 33, 0), (300, 200, 100, TA | TB),
     (128, 128, 32, ACC), (1000, 64, 576, 0), (576, 64, 3000, TA), (512, 1024, 1024, 0),
     (512, 300, 1024, TB), (7, 1000, 2048, 0), (1, 10, 256, ACC), (130, 8, 4, TA),
+    # GEMV paths (M <= 8): cluster kernel incl. empty K ranks, K tails, ACC; K/8 > 512 falls back
+    (8, 4096, 4096, 0), (4, 12, 13, 0), (1, 4, 1, 0), (5, 1024, 999, ACC), (2, 1000, 4100, 0),
+    (3, 516, 64, 0), (1, 2048, 20000, 0),
 ]
 
 
@@ -98,6 +101,69 @@ def test_gemm_vs_oracle(ops, M, N, K, flags):
     Ct2 = cu(C0)
     ops.gemm(cu(A), cu(B), Ct2, flags)
     assert torch.equal(Ct, Ct2)
+
+
+GEMM_EPI_SHAPES = [(1, 4096, 2048, 1, True), (1, 1000, 4096, 1, False), (8, 256, 784, 2, True),
+                   (5, 516, 333, 3, True), (64, 256, 784, 1, True), (130, 96, 40, 2, False)]
+
+
+@pytest.mark.parametrize("M,N,K,nb,relu", GEMM_EPI_SHAPES)
+def test_gemm_bias_act_vs_oracle(ops, M, N, K, nb, relu):
+    """Forward layer with its epilogue: fused into the GEMV reduction for M <= 8, a second
+    elementwise kernel otherwise; both equal the oracle's gemm -> bias_act."""
+    rng = np.random.default_rng(M + N + K + nb)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((K, N)).astype(np.float32)
+    bs = [rng.standard_normal((1, N)).astype(np.float32) for _ in range(nb)]
+    z = O.gemm(A, B, None, 0)
+    ref = O.bias_act(z, bs, relu)
+    C = torch.full((M, N), 7.0, device="cuda")
+    ops.gemm_bias_act(cu(A), cu(B), C, [cu(b) for b in bs], relu)
+    assert rel(C.cpu().numpy(), ref) <= TOL
+    C2 = torch.full((M, N), 7.0, device="cuda")
+    ops.gemm_bias_act(cu(A), cu(B), C2, [cu(b) for b in bs], relu)
+    assert torch.equal(C, C2)
+
+
+_GEMV_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, '.')
+from paper_conf_middleware_wur0hdh21_b200 import ops as K
+out = {}
+for (M, N, Kd, acc) in [(1, 4096, 2048, 0), (8, 1000, 4096, 1), (3, 12, 13, 0), (2, 516, 999, 1)]:
+    rng = np.random.default_rng(M * 100 + N + Kd)
+    A = rng.standard_normal((M, Kd)).astype(np.float32)
+    B = rng.standard_normal((Kd, N)).astype(np.float32)
+    C0 = rng.standard_normal((M, N)).astype(np.float32)
+    b = rng.standard_normal((1, N)).astype(np.float32)
+    C = torch.from_numpy(C0).cuda()
+    K.gemm_bias_act(torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda(), C,
+                    [torch.from_numpy(b).cuda()], True, 4 if acc else 0)
+    out[f"{M}_{N}_{Kd}"] = C.cpu().numpy()
+np.savez(sys.argv[1], **out)
+"""
+
+
+@pytest.mark.parametrize("path", ["tma", "cluster", "split"])
+def test_gemv_paths_agree_with_oracle(path, tmp_path):
+    """Every M <= 8 path (SF_GEMV=tma|cluster|split, read once per process) meets the bar."""
+    import os, subprocess, sys
+    f = tmp_path / "out.npz"
+    env = dict(os.environ, SF_GEMV=path)
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    subprocess.run([sys.executable, "-c", _GEMV_CHILD, str(f)], cwd=root, env=env, check=True,
+                   timeout=120)
+    got = np.load(f)
+    for key in got.files:
+        M, N, Kd = map(int, key.split("_"))
+        rng = np.random.default_rng(M * 100 + N + Kd)
+        A = rng.standard_normal((M, Kd)).astype(np.float32)
+        B = rng.standard_normal((Kd, N)).astype(np.float32)
+        C0 = rng.standard_normal((M, N)).astype(np.float32)
+        b = rng.standard_normal((1, N)).astype(np.float32)
+        acc = key in ("8_1000_4096", "2_516_999")
+        ref = O.bias_act(O.gemm(A, B, C0 if acc else None, ACC if acc else 0), [b], True)
+        assert rel(got[key], ref) <= TOL, (path, key)
 
 
 def test_gemm_plain_tf32_would_fail_the_bar(ops):
