@@ -373,6 +373,21 @@ sf_status sf_op_gemm_bias_act(const float* A, const float* B, float* C, int32_t 
                               int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
                               const float* b1, const float* b2, const float* b3, int32_t relu,
                               void* stream);
+/* Fused batch-M inference chain (M <= 8): h[l] = act_l(h[l-1] W[l] + b[l]) for l = 0..n-1
+ * with h[-1] = x, act_l = ReLU if relu[l] else identity, then probs = softmax(h[n-1]) row-wise
+ * when probs != NULL — the preempter's forward pass of SURVEY.md 8(a) a6
+ * in one persistent kernel.  widths: host [n+1] (K_0, N_0 = K_1, ..., N_{n-1}); W[l]:
+ * device K_l x N_l row-major (N_l % 4 == 0, 16-B aligned); b[l]: device 1 x N_l or NULL (b
+ * itself may be NULL); relu: host [n] or NULL; h[l]: device M x N_l, all written.  n <= 6,
+ * otherwise SF_EUNSUPPORTED. */
+/* Diagnostics: while dev_buf != NULL every fused-chain launch writes per-CTA phase
+ * timestamps (%globaltimer ns) to dev_buf, uint64 [n_SMs][64] = [cta][layer * 8 + event]
+ * (events: 0 layer start, 1 inputs ready, 2 x staged, 3 first W box, 4 units done,
+ * 5 partial published, 6 column block reduced, 7 chain done).  NULL turns it off. */
+sf_status sf_debug_chain_trace(void* dev_buf);
+sf_status sf_op_mlp_chain(const float* x, int32_t M, int32_t n_layers, const int32_t* widths,
+                          const float* const* W, const float* const* b, const int32_t* relu,
+                          float* const* h, float* probs, void* stream);
 sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
                          float* h, int32_t rows, int32_t cols, int32_t relu, void* stream);
 sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* db,

@@ -145,6 +145,9 @@ PROTOTYPES = {
                          C.c_int32, C.c_int32, _vp]),
     "sf_op_gemm_bias_act": (_st, [_vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                                   C.c_int32, C.c_int32, C.c_int32, _vp, _vp, _vp, C.c_int32, _vp]),
+    "sf_debug_chain_trace": (_st, [_vp]),
+    "sf_op_mlp_chain": (_st, [_vp, C.c_int32, C.c_int32, _P(C.c_int32), _P(_vp), _P(_vp),
+                              _P(C.c_int32), _P(_vp), _vp, _vp]),
     "sf_op_bias_act": (_st, [_vp, _vp, _vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, _vp]),
     "sf_op_bias_act_bwd": (_st, [_vp, _vp, _vp, _vp, C.c_int32, C.c_int32, _vp]),
     "sf_op_colsum": (_st, [_vp, _vp, C.c_int32, C.c_int32, _vp]),

@@ -104,6 +104,7 @@ struct Binding {
   // TMA tensor-map requirement); refreshed from the arena at sf_start_training
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
   std::map<int, void*> prepared;  // optimizer group first op -> uploaded descriptor array
+  std::map<int, std::pair<float*, unsigned*>> chain_bufs;  // chain first op -> (ws, counters)
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
   // refreshed inside the version graph (copy2d before / after the GEMM)
   struct PadBuf { float* p = nullptr; int pitch = 0; };
@@ -537,6 +538,64 @@ sf_status upload(Binding& b, const void* host, size_t bytes, void** out) {
   return SF_OK;
 }
 
+// Fused inference chain (kernels_chain.cu): GEMM(M <= 8, constant B) [-> BIAS_ACT] -> GEMM
+// [-> BIAS_ACT] ... [-> SOFTMAX] inside [j, e), each GEMM reading the previous layer's output.
+// Returns the number of ops covered (0 = no chain of >= 2 layers starts at j).
+int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
+  // opt-in (SF_CHAIN=1): parity-tested, but on the C4 model the per-layer GEMV kernels under
+  // programmatic dependent launch are faster (inference path)
+  static const bool enabled = std::getenv("SF_CHAIN") && std::getenv("SF_CHAIN")[0] == '1';
+  if (!enabled) return 0;
+  Graph& g = c.g;
+  sfk::ChainArgs a;
+  int i = j, prev_y = -1;
+  auto readers = [&](int t) {
+    int n = 0;
+    for (const auto& q : g.ops)
+      for (int r : op_reads(q)) n += (r == t);
+    return n;
+  };
+  while (i < e && a.n_layers < sfk::kChainMaxLayers) {
+    const sf_op_desc& o = g.ops[i];
+    if (o.type != SF_OP_GEMM || (o.flags & (SF_GEMM_TA | SF_GEMM_TB | SF_GEMM_ACC))) break;
+    const Tensor &A = g.T[o.in[0]], &B = g.T[o.in[1]], &C = g.T[o.out[0]];
+    if (C.rows > 8 || g.op_written[o.in[1]] || c.b.shadow.count(o.in[1]) || c.b.gemm_pad.count(i)) break;
+    if (a.n_layers > 0 && (o.in[0] != prev_y || C.rows != a.M)) break;
+    sfk::ChainLayerArgs& L = a.layer[a.n_layers];
+    L = sfk::ChainLayerArgs{};
+    L.W = c.f(o.in[1]); L.ldw = B.cols;
+    L.x = c.f(o.in[0]); L.ldx = A.cols;
+    L.K = A.cols; L.N = C.cols;
+    int y = o.out[0], used = 1;
+    if (i + 1 < e && g.ops[i + 1].type == SF_OP_BIAS_ACT && g.ops[i + 1].in[0] == o.out[0] &&
+        C.kind != SF_OUTPUT && readers(o.out[0]) == 1) {
+      const sf_op_desc& ba = g.ops[i + 1];
+      for (int q = 1; q < ba.n_in; ++q) L.b[q - 1] = c.f(ba.in[q]);
+      L.relu = ba.flags & SF_ACT_RELU;
+      y = ba.out[0];
+      used = 2;
+    }
+    L.y = c.f(y); L.ldy = g.T[y].cols;
+    a.M = C.rows;
+    ++a.n_layers;
+    prev_y = y;
+    i += used;
+  }
+  if (a.n_layers < 2) return 0;
+  if (i < e && g.ops[i].type == SF_OP_SOFTMAX && g.ops[i].in[0] == prev_y) {
+    const Tensor& P = g.T[g.ops[i].out[0]];
+    a.softmax = true;
+    a.sm_out = c.f(g.ops[i].out[0]);
+    a.sm_n = P.cols;
+    a.sm_ldi = g.T[prev_y].cols;
+    a.sm_ldo = P.cols;
+    ++i;
+  }
+  if (!sfk::chain_eligible(a)) return 0;
+  *out = a;
+  return i - j;
+}
+
 sf_status launch_subgraph_ops(Capture& c, int k) {
   Graph& g = c.g;
   const auto [a, e] = g.parts[k];
@@ -598,6 +657,34 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
                              reinterpret_cast<const int32_t*>(c.ptr(step_t)), c.st);
       if (err != cudaSuccess) return fail(SF_ECUDA, std::string("adam: ") + cudaGetErrorString(err));
       continue;
+    }
+    if (o.type == SF_OP_GEMM) {
+      sfk::ChainArgs ca;
+      const int n_ops = match_chain(c, j, e, &ca);
+      if (n_ops > 0) {
+        auto& buf = c.b.chain_bufs[j];
+        if (c.dry) {
+          if (!buf.first) {
+            void *w = nullptr, *cn = nullptr;
+            const uint64_t wf = sfk::chain_ws_floats(ca), cs = sfk::chain_counter_slots(ca);
+            if (cudaMalloc(&w, std::max<uint64_t>(wf, 4) * 4) != cudaSuccess || cudaMalloc(&cn, cs * 4) != cudaSuccess ||
+                cudaMemset(cn, 0, cs * 4) != cudaSuccess)
+              return fail(SF_ENOMEM, "chain workspace");
+            c.b.dev_allocs.push_back(w);
+            c.b.dev_allocs.push_back(cn);
+            buf = {static_cast<float*>(w), static_cast<unsigned*>(cn)};
+          }
+          j += n_ops;
+          continue;
+        }
+        ca.ws = buf.first;
+        ca.counters = buf.second;
+        if (!ca.counters) return fail(SF_ESTATE, "chain workspace not prepared");
+        err = sfk::launch_chain(ca, c.st);
+        if (err != cudaSuccess) return fail(SF_ECUDA, "op " + std::to_string(j) + " (chain): " + cudaGetErrorString(err));
+        j += n_ops;
+        continue;
+      }
     }
     if (c.dry) {
       ++j;
@@ -2035,6 +2122,51 @@ static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, in
 sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
                      int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
   return op_gemm(A, B, C, M, N, K, lda, ldb, ldc, flags, nullptr, nullptr, nullptr, false, stream);
+}
+
+sf_status sf_debug_chain_trace(void* dev_buf) {
+  sfk::set_chain_trace(dev_buf);
+  return SF_OK;
+}
+
+sf_status sf_op_mlp_chain(const float* x, int32_t M, int32_t n_layers, const int32_t* widths,
+                          const float* const* W, const float* const* b, const int32_t* relu,
+                          float* const* h, float* probs, void* stream) {
+  if (!x || !widths || !W || !h || n_layers < 1) return fail(SF_EINVAL, "mlp_chain args");
+  if (n_layers > sfk::kChainMaxLayers) return fail(SF_EUNSUPPORTED, "mlp_chain: too many layers");
+  sfk::ChainArgs a;
+  a.M = M;
+  a.n_layers = n_layers;
+  for (int l = 0; l < n_layers; ++l) {
+    sfk::ChainLayerArgs& L = a.layer[l];
+    L = sfk::ChainLayerArgs{};
+    L.K = widths[l];
+    L.N = widths[l + 1];
+    L.W = W[l]; L.ldw = L.N;
+    L.x = l == 0 ? x : h[l - 1]; L.ldx = L.K;
+    L.y = h[l]; L.ldy = L.N;
+    L.b[0] = b ? b[l] : nullptr;
+    L.relu = relu && relu[l];
+  }
+  if (probs) {
+    a.softmax = true;
+    a.sm_out = probs;
+    a.sm_n = widths[n_layers];
+    a.sm_ldi = a.sm_ldo = widths[n_layers];
+  }
+  if (!sfk::chain_eligible(a)) return fail(SF_EUNSUPPORTED, "mlp_chain: shape outside the fused kernel");
+  cudaStream_t st = as_stream(stream);
+  const uint64_t wf = sfk::chain_ws_floats(a), cs = sfk::chain_counter_slots(a);
+  void *ws = nullptr, *cnt = nullptr;
+  SF_CK(cudaMallocAsync(&ws, std::max<uint64_t>(wf, 4) * 4, st));
+  SF_CK(cudaMallocAsync(&cnt, cs * 4, st));
+  SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
+  a.ws = static_cast<float*>(ws);
+  a.counters = static_cast<unsigned*>(cnt);
+  SF_CK(sfk::launch_chain(a, st));
+  SF_CK(cudaFreeAsync(ws, st));
+  SF_CK(cudaFreeAsync(cnt, st));
+  return SF_OK;
 }
 
 sf_status sf_op_gemm_bias_act(const float* A, const float* B, float* C, int32_t M, int32_t N,

@@ -108,6 +108,18 @@ __device__ __forceinline__ uint64_t globaltimer() {
   return t;
 }
 
+// ---- TMA ---------------------------------------------------------------------------
+// 2-D tensor tile -> shared memory, completion counted in bytes on an mbarrier.
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, uint32_t bar, int x, int y) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      :: "r"(dst), "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar), "r"(x), "r"(y) : "memory");
+}
+__device__ __forceinline__ void expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;"
+               :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+
 // ---- programmatic dependent launch (PDL) ----------------------------------------------
 // Kernels launched with the programmatic-serialization attribute may start while their
 // predecessor in the stream is still running: everything that reads the predecessor's output

@@ -2,6 +2,7 @@
 // Every launcher is asynchronous on `st` and returns the cudaError_t of the launch.
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 namespace sfk {
@@ -56,6 +57,36 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
 bool gemm_tma_eligible(const GemmArgs& a, int splits);
 // M <= 8 (inference): TMA-streamed cluster GEMV with fused reduction + bias/ReLU epilogue.
 bool gemv_tma_eligible(const GemmArgs& a);
+bool make_map2d(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint64_t pitch_bytes,
+                uint32_t box_cols, uint32_t box_rows, bool swizzle128);
+
+// Fused batch-M (M <= 8) MLP chain: h_{l+1} = act(h_l W_l + b_l) for every layer (+ softmax)
+// in one persistent kernel (kernels_chain.cu).  layer[l].x must be layer[l-1].y.
+constexpr int kChainMaxLayers = 6;
+struct ChainLayerArgs {
+  const float* W; int ldw;
+  const float* x; int ldx;
+  float* y; int ldy;
+  const float* b[3];
+  int K, N;
+  bool relu;
+};
+struct ChainArgs {
+  int n_layers = 0, M = 0;
+  ChainLayerArgs layer[kChainMaxLayers];
+  bool softmax = false;
+  float* sm_out = nullptr;
+  int sm_n = 0, sm_ldi = 0, sm_ldo = 0;
+  float* ws = nullptr;
+  unsigned* counters = nullptr;  // zero before the first launch; the kernel re-zeroes them
+};
+bool chain_eligible(const ChainArgs& a);
+uint64_t chain_ws_floats(const ChainArgs& a);
+uint64_t chain_counter_slots(const ChainArgs& a);
+cudaError_t launch_chain(const ChainArgs& a, cudaStream_t st);
+// diagnostics: when set, every chain launch records per-CTA phase timestamps (u64 [SMs][64])
+void set_chain_trace(void* dev_buf);
+void* chain_trace_buffer();
 cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st);
 cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_split, int tiles_n,
                             int tiles_m, bool raw_hi, cudaStream_t st);

@@ -48,6 +48,21 @@ def gemm_bias_act(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, biases: S
                                     _s(stream)), "sf_op_gemm_bias_act")
 
 
+def mlp_chain(x: torch.Tensor, Ws: Sequence[torch.Tensor], bs: Sequence[Optional[torch.Tensor]],
+              relu: Sequence[bool], hs: Sequence[torch.Tensor], probs: Optional[torch.Tensor] = None,
+              stream=None) -> None:
+    """Fused batch-M MLP forward (+ softmax) in one persistent kernel (sf_op_mlp_chain)."""
+    n = len(Ws)
+    _need_cuda(x, *Ws, *[b for b in bs if b is not None], *hs, probs)
+    widths = (C.c_int32 * (n + 1))(*([x.shape[1]] + [W.shape[1] for W in Ws]))
+    Wp = (C.c_void_p * n)(*[W.data_ptr() for W in Ws])
+    bp = (C.c_void_p * n)(*[(b.data_ptr() if b is not None else None) for b in bs])
+    rl = (C.c_int32 * n)(*[int(r) for r in relu])
+    hp = (C.c_void_p * n)(*[h.data_ptr() for h in hs])
+    check(lib().sf_op_mlp_chain(_p(x), x.shape[0], n, widths, Wp, bp, rl, hp, _p(probs), _s(stream)),
+          "sf_op_mlp_chain")
+
+
 def bias_act(z, biases: Sequence[torch.Tensor], h, relu: bool, stream=None) -> None:
     bs = list(biases) + [None] * (3 - len(biases))
     _need_cuda(z, h, *bs)

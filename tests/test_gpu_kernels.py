@@ -166,6 +166,63 @@ def test_gemv_paths_agree_with_oracle(path, tmp_path):
         assert rel(got[key], ref) <= TOL, (path, key)
 
 
+CHAIN_CASES = [
+    ((2048, 4096, 4096, 1000), 1, True, True),   # C4 preempter model
+    ((784, 256, 12), 1, True, True),              # C1-like head (N % 4 == 0 for TMA)
+    ((100, 36, 516, 12), 2, True, False),         # ragged K / N, no softmax
+    ((256, 1024, 64, 1000), 8, False, True),      # M = 8, no biases
+    ((129, 260, 132, 8), 3, True, True),          # K tails inside a 128-row unit
+    ((2048, 4096, 1000), 8, True, True),          # M = 8 at full width
+    ((64, 64, 64, 64, 64, 64, 16), 5, True, True),  # 6 layers
+]
+
+
+@pytest.mark.parametrize("widths,M,biases,softmax", CHAIN_CASES)
+def test_mlp_chain_vs_oracle(ops, widths, M, biases, softmax):
+    """The fused chain equals the oracle's layer-by-layer gemm -> bias_act -> ... -> softmax;
+    every intermediate h is materialised and checked; two launches are bit-identical."""
+    rng = np.random.default_rng(sum(widths) + M)
+    n = len(widths) - 1
+    x = rng.standard_normal((M, widths[0])).astype(np.float32)
+    Ws = [(rng.standard_normal((widths[i], widths[i + 1])) / np.sqrt(widths[i])).astype(np.float32)
+          for i in range(n)]
+    bs = [rng.standard_normal((1, widths[i + 1])).astype(np.float32) if biases else None for i in range(n)]
+    relu = [i < n - 1 for i in range(n)]
+    refs, h = [], x
+    for i in range(n):
+        z = O.gemm(h, Ws[i], None, 0)
+        h = O.bias_act(z, [bs[i]] if biases else [], relu[i]) if (biases or relu[i]) else z
+        refs.append(h)
+    outs = []
+    for _ in range(2):
+        hs = [torch.full((M, widths[i + 1]), float("nan"), device="cuda") for i in range(n)]
+        probs = torch.full((M, widths[-1]), float("nan"), device="cuda") if softmax else None
+        ops.mlp_chain(cu(x), [cu(W) for W in Ws], [cu(b) if b is not None else None for b in bs],
+                      relu, hs, probs)
+        torch.cuda.synchronize()
+        outs.append((hs, probs))
+    hs, probs = outs[0]
+    for i in range(n):
+        assert rel(hs[i].cpu().numpy(), refs[i]) <= TOL, (i, rel(hs[i].cpu().numpy(), refs[i]))
+        assert torch.equal(hs[i], outs[1][0][i])
+    if softmax:
+        assert rel(probs.cpu().numpy(), O.softmax(refs[-1])) <= TOL
+        assert torch.equal(probs, outs[1][1])
+
+
+def test_mlp_chain_rejects_unsupported_shapes(ops):
+    """N % 4 != 0 (TMA row pitch) and more than 6 layers are refused, not silently wrong."""
+    from paper_conf_middleware_wur0hdh21_b200._abi import SFError
+    x = torch.zeros(1, 64, device="cuda")
+    with pytest.raises(SFError):
+        ops.mlp_chain(x, [torch.zeros(64, 10, device="cuda"), torch.zeros(10, 8, device="cuda")],
+                      [None, None], [True, False],
+                      [torch.zeros(1, 10, device="cuda"), torch.zeros(1, 8, device="cuda")])
+    Ws = [torch.zeros(64, 64, device="cuda") for _ in range(7)]
+    with pytest.raises(SFError):
+        ops.mlp_chain(x, Ws, [None] * 7, [True] * 7, [torch.zeros(1, 64, device="cuda") for _ in range(7)])
+
+
 def test_gemm_plain_tf32_would_fail_the_bar(ops):
     """Control: single-pass TF32 (torch allow_tf32) misses 1e-4 where 3xTF32 passes."""
     rng = np.random.default_rng(1)

@@ -458,3 +458,55 @@ def test_remote_slot_errors(P):
     with pytest.raises(A.SFError):
         rt.import_arena(gh, 0, blob)  # slot 0 is local
     rt.close()
+
+
+_INFER_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, '.')
+from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
+from sf_inputs import data as D, graphs as G
+g = G.mlp_train()
+gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths")
+rt = Runtime([0], dispatch_spin_us=int(sys.argv[2]))
+gh = rt.register(g); gh.partition(); gh.bind(0, staging=True, host_staging=True)
+gh.load(0, {**D.init_state(g), **D.datasets(g)})
+ghi = rt.register(gi, 1); ghi.partition(); ghi.bind(0, staging=False)
+ghi.load(0, D.init_state(gi, seed=D.SEED_INFER))
+xs = D.infer_inputs(gi, 6)
+job = rt.start_training(gh, 0, 100000, -1)
+xin = torch.from_numpy(xs).cuda()
+out = torch.zeros(6, 1, 128, device="cuda")
+host_out = torch.zeros(6, 1, 128).pin_memory()
+host_in = torch.from_numpy(xs).pin_memory()
+for r in range(6):
+    if r % 2:
+        req = rt.submit(ghi, 0, host_in[r].data_ptr(), host_out[r].data_ptr())
+        rt.wait(req, 60)
+        out[r] = host_out[r].cuda()
+    else:
+        req = rt.submit(ghi, 0, xin[r].data_ptr(), out[r].data_ptr())
+        rt.wait(req, 60)
+rt.stop_job(job); rt.wait_job(job, 60); rt.close()
+np.save(sys.argv[1], out.cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("env,spin", [({"SF_CHAIN": "1"}, -1), ({"SF_CHAIN": "1", "SF_PDL": "0"}, 0),
+                                      ({"SF_INFER_DIRECT": "0"}, 0), ({"SF_GEMV": "split"}, 2000),
+                                      ({"SF_GEMV": "cluster", "SF_INFER_DIRECT": "0"}, -1)],
+                         ids=["chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv"])
+def test_inference_paths_vs_oracle(env, spin, tmp_path):
+    """Every inference launch path (fused chain, PDL direct launches, captured graphs, the
+    GEMV variants; device and pinned-host request buffers; spinning and blocking dispatcher)
+    gives the oracle's forward pass while a training job is being preempted around it."""
+    import os, subprocess, sys
+    f = tmp_path / "out.npy"
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    subprocess.run([sys.executable, "-c", _INFER_CHILD, str(f), str(spin)], cwd=root,
+                   env=dict(os.environ, **env), check=True, timeout=240)
+    got = np.load(f)
+    gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths")
+    sti = D.init_state(gi, seed=D.SEED_INFER)
+    xs = D.infer_inputs(gi, 6)
+    for r in range(6):
+        assert rel(got[r], R.run_inference(gi, sti, xs[r])) <= TOL, (env, r)
