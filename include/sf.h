@@ -242,6 +242,9 @@ typedef struct sf_job_info {
   uint64_t last_resume_ns;      /* CLOCK_MONOTONIC: first resumed subgraph began on the device
                                    (host-observed completion of a marker recorded right before it,
                                    i.e. after the stream-ordered copy / unpack finished) */
+  int64_t n_reparks;            /* host-tier preemptions that found the parked copy of the
+                                   same cut still current (nothing ran since the swap-in) and
+                                   re-parked without pack / D2H */
 } sf_job_info;
 
 typedef struct sf_cut_info {

@@ -71,7 +71,7 @@ class sf_job_info(C.Structure):
                 ("n_preemptions", C.c_int32), ("migrated_bytes", C.c_uint64),
                 ("last_pack_us", C.c_double), ("last_xfer_us", C.c_double),
                 ("last_unpack_us", C.c_double), ("last_stop_ns", C.c_uint64),
-                ("last_resume_ns", C.c_uint64)]
+                ("last_resume_ns", C.c_uint64), ("n_reparks", C.c_int64)]
 
 
 class sf_cut_info(C.Structure):

@@ -185,6 +185,10 @@ struct Job {
   bool stop_req = false;
   bool stamp_resume = false;
   bool adopted_pending = false;  // first launch of an adopted job: stamp time, no copy stats
+  // host tier: the pinned staging of slot parked_slot holds L_k of cut (parked_iter, parked_k)
+  int parked_slot = -1, parked_k = -1;
+  int64_t parked_iter = -1;
+  int64_t n_repark = 0;
   int n_preempt = 0;
   uint64_t migrated = 0;
   double pack_us = 0, xfer_us = 0, unpack_us = 0;
@@ -959,13 +963,25 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     return fail(SF_ECUDA, J.error);
   };
   cudaError_t e;
+  // The migration stream reads the arena only after everything already enqueued on the
+  // training stream (a pending swap-in or stream-ordered peer arrival) has landed.
+  if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+  if ((e = cudaEventRecord(J.ev_sub[src], S.s_train)) != cudaSuccess ||
+      (e = cudaStreamWaitEvent(S.s_mig, J.ev_sub[src], 0)) != cudaSuccess)
+    return cuda_fail(e, "order migration after training stream");
+  // Re-preempted before running anything since its swap-in from this slot's pinned
+  // staging: that copy of L_k is still current, so park again without pack + D2H.
+  const bool repark = target == SF_TARGET_HOST && J.stamp_resume && J.parked_slot == src &&
+                      J.parked_iter == J.it && J.parked_k == k;
   if (target == SF_TARGET_HOST) {
     // ---- host tier: pack (+ D2H), park, swap back in ------------------------------
-    if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
     const bool zc = rt->cfg.host_mode == SF_HOST_ZC || B.staging == nullptr;
     tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
-    if (zc) {
+    if (repark) {
+      cudaEventRecord(J.ev_b[src], S.s_mig);
+      e = cudaSuccess;
+    } else if (zc) {
       const CopyList& L = B.pack_zc[k];
       e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig, S.tstamp);
       cudaEventRecord(J.ev_b[src], S.s_mig);
@@ -983,9 +999,9 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     rt->cv.notify_all();
     lk.unlock();
     if ((e = spin_event(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
-    float pack_us = static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
+    float pack_us = repark ? 0.f : static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
     if (pack_us < 0.f) pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
-    const float d2h_us = elapsed_us(J.ev_b[src], J.ev_c[src]);
+    const float d2h_us = repark ? 0.f : elapsed_us(J.ev_b[src], J.ev_c[src]);
     if (rt->cfg.poison_released) {
       if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
       if ((e = cudaStreamSynchronize(S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison sync");
@@ -993,6 +1009,10 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     lk.lock();
     J.pack_us = pack_us;
     J.xfer_us = d2h_us;
+    J.parked_slot = src;
+    J.parked_iter = J.it;
+    J.parked_k = k;
+    J.n_repark += repark ? 1 : 0;
     int dst = src;
     if (expl) {
       J.state = SF_JOB_PREEMPTED;
@@ -1036,7 +1056,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     J.dev = dst;
   } else {
     // ---- peer tier: fused peer store into the target's arena over NVLink -----------
-    if ((e = cudaSetDevice(S.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+    J.parked_slot = -1;
     auto it = B.peer.find(target);
     if (it == B.peer.end()) {
       lk.lock();
@@ -1964,6 +1984,7 @@ sf_status sf_job_query(sf_runtime* rt, sf_job_id jid, sf_job_info* out) {
   out->last_unpack_us = J->unpack_us;
   out->last_stop_ns = J->last_stop;
   out->last_resume_ns = J->last_resume;
+  out->n_reparks = J->n_repark;
   if (J->state == SF_JOB_FAILED) return fail(SF_ECUDA, J->error);
   return SF_OK;
 }
