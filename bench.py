@@ -8,12 +8,16 @@ requests that each preempt a running training job.
 Workload at N=1 ("C4@1GPU", the largest single-GPU config): a training
 job with the ResNet-50-shaped state (Keras variable list, 534 tensors, 204.9 MB params +
 momentum; per-layer softmax-regression compute at batch 8, reading Q16) runs
-on the GPU; one batch-1 request of a 2048-4096-4096-1000 MLP (29.3M params) arrives per
-step at a seeded random point inside a training subgraph; the job is stopped at the next
-subgraph boundary, its live set is packed and parked in pinned host memory (host tier),
-the request runs, the state is swapped back and the job resumes.  Inputs are resident in
-HBM for `value`; `e2e` repeats the measurement with the request's input / output in
-pinned host memory (H2D + D2H inside each step, through sf_submit_inference).
+on the GPU while an OPEN-LOOP Poisson stream of batch-1 requests of a 2048-4096-4096-1000
+MLP (29.3M params; rate --rate, default 100 req/s, arrival seed 7) arrives.  A request that
+finds the job on the GPU stops it at the next subgraph boundary; the job's live set is
+packed and parked in pinned host memory (host tier), the request runs, the state is
+swapped back and the job resumes.  `value` = p99 latency from the scheduled arrival to the
+completion observed on the host, inputs resident in HBM; `e2e` repeats it with the
+request's input / output in pinned host memory (H2D + D2H inside each request, through
+sf_submit_inference).  The closed-loop "chase" arm (every request preempts; the next one
+is issued after the resume) supplies the per-cycle migration numbers (pack GB/s,
+preempt-to-resume split).
 
 Under torchrun (N>1) every rank runs the same job + request stream on its own GPU
 (independent replicas, weak scaling) and rank 0 pools the samples.
@@ -39,8 +43,8 @@ sys.path.insert(0, ROOT)
 HOST = -1
 METRIC = "p99 inference latency + preempt-to-resume ms; migration GB/s vs NVLink/HBM peak"
 UNIT = "ms"
-WORKLOAD = "C4@1GPU: ResNet-50-shaped training state (534 tensors, 204.9 MB) + batch-1 " \
-           "inference preemption, host-tier migration"
+WORKLOAD = "C4@1GPU: ResNet-50-shaped training job (534 tensors, 204.9 MB) + open-loop Poisson " \
+           "batch-1 inference stream, repeated preemptions, host-tier migration"
 
 
 def pct(x, q):
@@ -240,6 +244,93 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
     rt.wait_job(job, 120)
     rt.close()
     return S
+
+
+def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
+                    iteration_granularity=False, measure=True, defer=None):
+    """C4 as specified: an OPEN-LOOP Poisson request stream (rate args.rate
+    req/s, arrival seed 7 + pair) against the running training job.  Each request is submitted
+    at its scheduled arrival time (passed to sf_submit_inference, so any host delay counts
+    against the latency); a request that finds the job on the GPU preempts it, one that
+    arrives while the job is parked / migrating runs at once.  Returns samples."""
+    import torch
+    from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
+    from sf_inputs import data as D
+
+    g, gi = build_workload(args.batch, args.spatial_div)
+    rt = Runtime([local_dev], exclusive=exclusive, auto_preempt=True,
+                 iteration_granularity=iteration_granularity, max_inflight=args.max_inflight,
+                 defer_migration=args.defer if defer is None else defer,
+                 dispatch_spin_us=args.dispatch_spin_us,
+                 inflight_budget_us=args.inflight_budget_us)
+    gh = rt.register(g)
+    gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
+    gh.bind(0, staging=True, host_staging=True)
+    arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
+    gh.load(0, arrays)
+    ghi = rt.register(gi, priority=1)
+    ghi.partition()
+    ghi.bind(0, staging=False)
+    ghi.load(0, arrays_i)
+    n_in = n_req + warmup
+    xs = D.infer_inputs(gi, min(n_in, 64))
+    dev = torch.device("cuda", local_dev)
+    if host_io:
+        x_t = torch.from_numpy(xs).pin_memory()
+        out_t = torch.zeros(len(xs), 1, 1000).pin_memory()
+    else:
+        x_t = torch.from_numpy(xs).to(dev)
+        out_t = torch.zeros(len(xs), 1, 1000, device=dev)
+    job = rt.start_training(gh, 0, 1 << 40, HOST)
+    time.sleep(0.3)
+    rng = np.random.default_rng(7 + args.rank // 2)
+    gaps_ns = (rng.exponential(1.0 / args.rate, n_in) * 1e9).astype(np.int64)
+    torch.cuda.synchronize(dev)
+    t0 = now_ns() + 2_000_000
+    arr = t0 + np.cumsum(gaps_ns)
+    reqs, p2r, last = [], [], None
+    sampler, ev0, launches0, t_region = None, None, None, None
+    for i in range(n_in):
+        if i == warmup:
+            sampler = ClockSampler(local_dev).__enter__() if measure else None
+            ev0 = torch.cuda.Event(enable_timing=True)
+            ev0.record()
+            t_region = time.perf_counter()
+            launches0 = kernel_launches()
+        while now_ns() < arr[i]:
+            ji = rt.job_info(job)  # preempt-to-resume of every completed cycle
+            key = (ji["last_stop_ns"], ji["last_resume_ns"])
+            if key != last and ji["last_resume_ns"] > ji["last_stop_ns"] > 0:
+                if i >= warmup:
+                    p2r.append((ji["last_resume_ns"] - ji["last_stop_ns"]) * 1e-6)
+                last = key
+        j = i % len(xs)
+        reqs.append(rt.submit(ghi, 0, x_t[j].data_ptr(), out_t[j].data_ptr(), arrival_ns=int(arr[i])))
+    tms = [rt.wait(r, 120) for r in reqs]
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev1.record()
+    torch.cuda.synchronize(dev)
+    wall = time.perf_counter() - t_region
+    launches = kernel_launches() - launches0
+    if sampler:
+        sampler.__exit__()
+    info_j = rt.job_info(job)
+    tr = [e for e in rt.trace() if e["kind"] == "train"]
+    rt.stop_job(job)
+    rt.wait_job(job, 120)
+    rt.close()
+    T = tms[warmup:]
+    lat = [(t["end_ns"] - t["arrival_ns"]) * 1e-6 for t in T]
+    pre = [(t["start_ns"] - t["arrival_ns"]) * 1e-6 for t in T if t["preempted_job"] == job]
+    dev_us = [t["device_us"] for t in T if t["device_us"] > 0]
+    per_it = {}
+    for e in tr:
+        a, b_ = per_it.get(e["iter"], (e["t0"], e["t1"]))
+        per_it[e["iter"]] = (min(a, e["t0"]), max(b_, e["t1"]))
+    return {"lat": lat, "pre": pre, "p2r": p2r, "frac_preempting": len(pre) / max(1, len(T)),
+            "device_us": dev_us, "region_ms": ev0.elapsed_time(ev1), "wall_s": wall,
+            "launches": launches, "clocks": sampler.summary() if sampler else None,
+            "reparks": info_j["n_reparks"], "iters_done": len(per_it)}
 
 
 def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, gloo):
@@ -458,6 +549,9 @@ def main():
                     help="idle dispatcher busy-polls its queue (-1: always; one core per GPU)")
     ap.add_argument("--inflight-budget-us", type=int, default=50,
                     help="queue a subgraph behind in-flight ones only within this est. device time")
+    ap.add_argument("--arrivals", default="poisson", choices=["poisson", "chase"],
+                    help="poisson: open-loop stream (C4); chase: one request per step, each preempts")
+    ap.add_argument("--rate", type=float, default=100.0, help="Poisson arrival rate, req/s")
     ap.add_argument("--defer", type=int, default=1,
                     help="1: migrate after the preempter drained (default); 0: concurrently")
     args = ap.parse_args()
@@ -487,23 +581,29 @@ def main():
 
     if args.world > 1:
         return pair_main(args, local)
-    main_s = run_arm(args, local, args.steps, args.warmup, host_io=False)
+    # headline: open-loop Poisson stream (C4 as specified); the closed-loop "chase" arm (every
+    # request preempts, the next one waits for the resume) gives the per-cycle migration numbers
+    arm = run_poisson_arm if args.arrivals == "poisson" else run_arm
+    main_s = arm(args, local, args.steps, args.warmup, host_io=False)
+    chase_s = run_arm(args, local, args.steps, args.warmup, host_io=False, measure=False) \
+        if args.arrivals == "poisson" else main_s
     e2e_steps = max(20, args.steps // 2)
-    e2e_s = run_arm(args, local, e2e_steps, 3, host_io=True, measure=False)
+    e2e_s = arm(args, local, e2e_steps, 3, host_io=True, measure=False)
     base = {}
     if not args.no_baselines:
-        nb = max(20, args.steps // 4)
-        co = run_arm(args, local, nb, 3, host_io=False, exclusive=False, measure=False)
-        itg = run_arm(args, local, nb, 3, host_io=False, iteration_granularity=True, measure=False)
-        alt = run_arm(args, local, nb, 3, host_io=False, measure=False, defer=not args.defer)
-        base = {"free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
+        nb = max(20, args.steps // 2)
+        co = arm(args, local, nb, 3, host_io=False, exclusive=False, measure=False)
+        itg = arm(args, local, nb, 3, host_io=False, iteration_granularity=True, measure=False)
+        alt = arm(args, local, nb, 3, host_io=False, measure=False, defer=not args.defer)
+        base = {"arrivals": args.arrivals,
+                "free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
                 ("concurrent" if args.defer else "deferred") + "_migration_p99_ms": pct(alt["lat"], 99),
-                ("concurrent" if args.defer else "deferred") + "_migration_p2r_p50_ms": pct(alt["p2r"], 50),
+                ("concurrent" if args.defer else "deferred") + "_migration_p50_ms": pct(alt["lat"], 50),
                 "iteration_slicing_p99_ms": pct(itg["lat"], 99),
                 "iteration_slicing_p50_ms": pct(itg["lat"], 50)}
 
     # pool samples across ranks (weak scaling replicas); max-over-ranks region time
-    samples = {"main": main_s, "e2e": e2e_s}
+    samples = {"main": main_s, "e2e": e2e_s, "chase": chase_s}
     if args.world > 1:
         import torch.distributed as dist
         allv = [None] * args.world
@@ -513,27 +613,28 @@ def main():
         allv = [samples]
     if args.rank != 0:
         return
-    M = {k: sum((a["main"][k] for a in allv), []) for k in ("lat", "pre", "p2r", "pack_us", "xfer_us",
-                                                          "unpack_us", "bytes")}
+    M = {k: sum((a["main"][k] for a in allv), []) for k in ("lat", "pre", "p2r")}
+    Cc = {k: sum((a["chase"][k] for a in allv), []) for k in ("lat", "pre", "p2r", "pack_us", "xfer_us",
+                                                            "unpack_us", "bytes")}
     E = sum((a["e2e"]["lat"] for a in allv), [])
     region_ms = max(a["main"]["region_ms"] for a in allv)
     peaks = load_peaks()
     hbm = peaks.get("hbm_gbs")
     peak_src = "measured (MEASURED_PEAKS.json)" if hbm else "fallback (B200_PROFILING.md)"
     hbm = hbm or 6650.0
-    pack_us = np.asarray(M["pack_us"], np.float64)
-    byts = np.asarray(M["bytes"], np.float64)
+    pack_us = np.asarray(Cc["pack_us"], np.float64)
+    byts = np.asarray(Cc["bytes"], np.float64)
     ok = pack_us > 0
     pack_achieved = float((2 * byts[ok]).mean() / (pack_us[ok].mean() * 1e-6) / 1e9) if ok.any() else None
-    xfer = np.asarray(M["xfer_us"], np.float64)
-    unpack = np.asarray(M["unpack_us"], np.float64)
+    xfer = np.asarray(Cc["xfer_us"], np.float64)
+    unpack = np.asarray(Cc["unpack_us"], np.float64)
     migr_gbs = float((2 * byts[ok]).mean() / (xfer[ok].mean() * 1e-6) / 1e9) if ok.any() else None
     traffic = None
     try:
         traffic = json.load(open(os.path.join(ROOT, "profiles", "pack_traffic.json")))["bytes_per_launch"]
     except Exception:
         pass
-    m0 = main_s
+    m0 = chase_s
     line = {
         "metric": METRIC, "value": pct(M["lat"], 99), "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
@@ -553,6 +654,15 @@ def main():
         "p50_ms": pct(M["lat"], 50), "p95_ms": pct(M["lat"], 95), "p99_ms": pct(M["lat"], 99),
         "preempt_latency_p50_ms": pct(M["pre"], 50), "preempt_latency_p99_ms": pct(M["pre"], 99),
         "preempt_to_resume_p50_ms": pct(M["p2r"], 50), "preempt_to_resume_p99_ms": pct(M["p2r"], 99),
+        "arrivals": {"process": args.arrivals, "rate_per_s": args.rate if args.arrivals == "poisson" else None,
+                     "seed": "7 + pair" if args.arrivals == "poisson" else "1234 + device",
+                     "frac_preempting": main_s.get("frac_preempting"), "reparks": main_s.get("reparks"),
+                     "inference_device_us_p50": pct(main_s.get("device_us", []), 50)},
+        "chase": {"desc": "closed loop: every request preempts the running job; next request after its resume",
+                  "p50_ms": pct(Cc["lat"], 50), "p99_ms": pct(Cc["lat"], 99),
+                  "preempt_latency_p50_ms": pct(Cc["pre"], 50), "preempt_latency_p99_ms": pct(Cc["pre"], 99),
+                  "preempt_to_resume_p50_ms": pct(Cc["p2r"], 50),
+                  "preempt_to_resume_p99_ms": pct(Cc["p2r"], 99)},
         "migration": {"live_bytes_mean": float(byts.mean()) if len(byts) else None,
                       "pack_us_mean": float(pack_us[ok].mean()) if ok.any() else None,
                       "pack_gbs": pack_achieved,
@@ -570,7 +680,7 @@ def main():
         "e2e": {"value": pct(E, 99), "unit": UNIT, "h2d_bytes_per_step": 2048 * 4,
                 "d2h_bytes_per_step": 1000 * 4, "p50_ms": pct(E, 50)},
         "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),
-        "clocks": m0["clocks"],
+        "clocks": main_s["clocks"],
     }
     if not args.no_cpu_baseline:
         o = oracle_sample(args, args.steps)

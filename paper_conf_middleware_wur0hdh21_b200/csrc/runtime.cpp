@@ -1052,6 +1052,10 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     }
     if (e != cudaSuccess) return cuda_fail(e, "unpack");
     cudaEventRecord(J.ev_c[dst], D.s_train);
+    // Hold no device token while the swap-in lands: a request arriving during the H2D runs
+    // at once instead of queueing behind a resumed subgraph that waits for the copy; the
+    // driver then re-parks (no copy: nothing ran) if requests are pending.
+    if ((e = spin_event(J.ev_c[dst])) != cudaSuccess) return cuda_fail(e, "swap-in wait");
     lk.lock();
     J.dev = dst;
   } else {
@@ -1096,6 +1100,8 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     // (a cross-device event wait when the slots are different GPUs)
     e = cudaStreamWaitEvent(T.s_train, J.ev_b[src], 0);
     if (e != cudaSuccess) return cuda_fail(e, "stream wait");
+    // as for the host tier: relaunch only once the state has landed on the target
+    if ((e = spin_event(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
     if (rt->cfg.poison_released) {
       if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
     }
