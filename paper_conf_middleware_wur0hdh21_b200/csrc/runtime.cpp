@@ -197,6 +197,7 @@ struct Job {
   std::thread driver;
   std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
   std::vector<cudaEvent_t> ev_ring;  // [slot * kMaxInflight + i]: in-flight subgraph ends
+  std::vector<cudaEvent_t> ev_ck;    // [slot * 2 + i]: host-tier copy chunks in flight
 };
 
 }  // namespace
@@ -857,6 +858,7 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
   J.ev_r.assign(n, nullptr);
   J.ev_ring.assign(n * kMaxInflight, nullptr);
+  J.ev_ck.assign(n * 2, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
   for (size_t s = 0; s < n; ++s) {
@@ -866,6 +868,8 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
     SF_CK(cudaEventCreateWithFlags(&J.ev_r[s], cudaEventDisableTiming));
     for (int i = 0; i < kMaxInflight; ++i)
       SF_CK(cudaEventCreateWithFlags(&J.ev_ring[s * kMaxInflight + i], cudaEventDisableTiming));
+    for (int i = 0; i < 2; ++i)
+      SF_CK(cudaEventCreateWithFlags(&J.ev_ck[s * 2 + i], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
     SF_CK(cudaEventCreate(&J.ev_b[s]));
     SF_CK(cudaEventCreate(&J.ev_c[s]));
@@ -878,6 +882,17 @@ cudaError_t spin_event(cudaEvent_t ev) {
   for (;;) {
     cudaError_t e = cudaEventQuery(ev);
     if (e != cudaErrorNotReady) return e;
+  }
+}
+
+// Millisecond-scale waits (host-tier D2H / H2D, peer stores) poll with short sleeps: a
+// tight cudaEventQuery loop on this thread contends for the CUDA driver's locks with the
+// dispatcher's kernel launches and stretches the preempter's launch chain.
+cudaError_t wait_event_relaxed(cudaEvent_t ev) {
+  for (;;) {
+    cudaError_t e = cudaEventQuery(ev);
+    if (e != cudaErrorNotReady) return e;
+    std::this_thread::sleep_for(std::chrono::microseconds(20));
   }
 }
 
@@ -913,6 +928,45 @@ cudaError_t poison(Binding& b, cudaStream_t st) {
   for (auto [off, len] : b.poison_ranges) {
     cudaError_t e = sfk::launch_fill(b.arena + off, len, 0xFF, st);
     if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+
+// Host-tier transfer that yields to inference: copy-engine traffic over PCIe slows a
+// concurrent batch-1 forward by ~45% on B200 (scripts/infer_bench.py COPY=d2h: 50 -> 74 us),
+// so the staging moves in 2 MB chunks, at most two in flight, and no chunk is issued while a
+// request is queued or running on the slot.  Returns once every chunk has completed.
+cudaError_t yielding_copy(Job& J, Slot& S, int slot, void* dst, const void* src, size_t bytes,
+                          cudaMemcpyKind kind, cudaStream_t st) {
+  constexpr size_t kChunk = size_t(2) << 20;
+  size_t off = 0;
+  int head = 0, n_inflight = 0;  // ring of 2 events
+  auto busy = [&] {
+    const int o = S.owner.load(std::memory_order_acquire);
+    return S.qn.load(std::memory_order_acquire) > 0 || o == kInferOwner;
+  };
+  while (off < bytes || n_inflight > 0) {
+    if (off < bytes && n_inflight < 2 && !busy()) {
+      const size_t n = std::min(kChunk, bytes - off);
+      cudaError_t e = cudaMemcpyAsync(static_cast<uint8_t*>(dst) + off, static_cast<const uint8_t*>(src) + off,
+                                      n, kind, st);
+      if (e == cudaSuccess) e = cudaEventRecord(J.ev_ck[slot * 2 + (head + n_inflight) % 2], st);
+      if (e != cudaSuccess) return e;
+      ++n_inflight;
+      off += n;
+      continue;
+    }
+    if (n_inflight > 0) {
+      const cudaError_t q = cudaEventQuery(J.ev_ck[slot * 2 + head]);
+      if (q == cudaSuccess) {
+        head = (head + 1) % 2;
+        --n_inflight;
+        continue;
+      }
+      if (q != cudaErrorNotReady) return q;
+    }
+    for (int i = 0; i < 64; ++i) cpu_relax();
   }
   return cudaSuccess;
 }
@@ -989,16 +1043,18 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       const CopyList& L = B.pack[k];
       e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, J.it, S.s_mig, S.tstamp);
       cudaEventRecord(J.ev_b[src], S.s_mig);
-      if (e == cudaSuccess)
-        e = cudaMemcpyAsync(B.host_staging, B.staging, g.staging_total[k], cudaMemcpyDeviceToHost, S.s_mig);
     }
     if (e != cudaSuccess) return cuda_fail(e, "pack");
-    cudaEventRecord(J.ev_c[src], S.s_mig);
     lk.lock();
     J.mig_enqueued = true;
     rt->cv.notify_all();
     lk.unlock();
-    if ((e = spin_event(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
+    if (!repark && !zc &&
+        (e = yielding_copy(J, S, src, B.host_staging, B.staging, g.staging_total[k], cudaMemcpyDeviceToHost,
+                           S.s_mig)) != cudaSuccess)
+      return cuda_fail(e, "D2H");
+    cudaEventRecord(J.ev_c[src], S.s_mig);
+    if ((e = wait_event_relaxed(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
     float pack_us = repark ? 0.f : static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
     if (pack_us < 0.f) pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
     const float d2h_us = repark ? 0.f : elapsed_us(J.ev_b[src], J.ev_c[src]);
@@ -1042,8 +1098,8 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     } else if (!BD.staging) {
       e = cudaErrorInvalidValue;
     } else {
-      e = cudaMemcpyAsync(BD.staging, B.host_staging, g.staging_total[k], cudaMemcpyHostToDevice,
-                          D.s_train);
+      e = yielding_copy(J, D, dst, BD.staging, B.host_staging, g.staging_total[k], cudaMemcpyHostToDevice,
+                        D.s_train);
       cudaEventRecord(J.ev_b[dst], D.s_train);
       if (e == cudaSuccess) {
         const CopyList& L = BD.unpack[k];
@@ -1055,7 +1111,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     // Hold no device token while the swap-in lands: a request arriving during the H2D runs
     // at once instead of queueing behind a resumed subgraph that waits for the copy; the
     // driver then re-parks (no copy: nothing ran) if requests are pending.
-    if ((e = spin_event(J.ev_c[dst])) != cudaSuccess) return cuda_fail(e, "swap-in wait");
+    if ((e = wait_event_relaxed(J.ev_c[dst])) != cudaSuccess) return cuda_fail(e, "swap-in wait");
     lk.lock();
     J.dev = dst;
   } else {
@@ -1078,7 +1134,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     Slot& T = slot_of(rt, target);
     if (T.remote) {
       // process-per-GPU handoff: the copy must be complete before the partner adopts the job
-      if ((e = spin_event(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
+      if ((e = wait_event_relaxed(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
       const float us = static_cast<float>(tstamp_us(S.tstamp));
       if (rt->cfg.poison_released) {
         if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
@@ -1101,7 +1157,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     e = cudaStreamWaitEvent(T.s_train, J.ev_b[src], 0);
     if (e != cudaSuccess) return cuda_fail(e, "stream wait");
     // as for the host tier: relaunch only once the state has landed on the target
-    if ((e = spin_event(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
+    if ((e = wait_event_relaxed(J.ev_b[src])) != cudaSuccess) return cuda_fail(e, "peer store wait");
     if (rt->cfg.poison_released) {
       if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
     }
@@ -1542,6 +1598,7 @@ void sf_destroy(sf_runtime* rt) {
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_r[s]);
       for (int i = 0; i < kMaxInflight; ++i) cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
+    for (int i = 0; i < 2; ++i) cudaEventDestroy(J->ev_ck[s * 2 + i]);
       cudaEventDestroy(J->ev_a[s]);
       cudaEventDestroy(J->ev_b[s]);
       cudaEventDestroy(J->ev_c[s]);

@@ -10,12 +10,41 @@ rt = Runtime([0], dispatch_spin_us=int(os.environ.get("SPIN", "0")))
 ghi = rt.register(gi, 1); ghi.partition(); ghi.bind(0, staging=False); ghi.load(0, arrs_i)
 x = torch.rand(1, 2048, device="cuda"); out = torch.empty(1, 1000, device="cuda")
 lat, pre, dev = [], [], []
+gap = float(os.environ.get("GAP_MS", "0")) * 1e-3
+if os.environ.get("COPY"):  # background copy-engine traffic like a host-tier migration
+    import threading
+    dsrc = torch.empty(227 << 20, dtype=torch.uint8, device="cuda")
+    hdst = torch.empty(227 << 20, dtype=torch.uint8).pin_memory()
+    cs = torch.cuda.Stream()
+    stop_copy = False
+    def bg():
+        while not globals()["stop_copy"]:
+            with torch.cuda.stream(cs):
+                if os.environ.get("COPY") == "h2d":
+                    dsrc.copy_(hdst, non_blocking=True)
+                else:
+                    hdst.copy_(dsrc, non_blocking=True)
+            cs.synchronize()
+    th = threading.Thread(target=bg, daemon=True)
+    th.start()
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if os.environ.get("FLUSH") else None
+import time
 for i in range(int(sys.argv[1]) if len(sys.argv) > 1 else 300):
+    if flush is not None:
+        flush.fill_(i & 255)
+        torch.cuda.synchronize()
+    if gap:
+        t_end = time.perf_counter() + gap
+        while time.perf_counter() < t_end:
+            pass
     r = rt.submit(ghi, 0, x.data_ptr(), out.data_ptr()); tm = rt.wait(r, 300)
     if i >= 20:
         lat.append((tm["end_ns"] - tm["arrival_ns"]) * 1e-6)
         pre.append((tm["start_ns"] - tm["arrival_ns"]) * 1e-6)
         dev.append(tm["device_us"] * 1e-3)
+if os.environ.get("COPY"):
+    stop_copy = True
+    th.join()
 rt.close()
 print(json.dumps({"p50_ms": float(np.median(lat)), "p99_ms": float(np.percentile(lat, 99)),
                   "min_ms": float(np.min(lat)), "wake_p50_ms": float(np.median(pre)),
