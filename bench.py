@@ -610,6 +610,16 @@ def main():
         if args.arrivals == "poisson" else main_s
     e2e_steps = max(20, args.steps // 2)
     e2e_s = arm(args, local, e2e_steps, 3, host_io=True, measure=False)
+    hi_rate = None
+    if args.arrivals == "poisson" and not args.no_baselines:
+        r0 = args.rate
+        args.rate = 1000.0  # lambda in {100, 1000} req/s
+        hr = run_poisson_arm(args, local, max(100, args.steps), 10, host_io=False, measure=False)
+        args.rate = r0
+        hi_rate = {"rate_per_s": 1000.0, "n": len(hr["lat"]), "p50_ms": pct(hr["lat"], 50),
+                   "p95_ms": pct(hr["lat"], 95), "p99_ms": pct(hr["lat"], 99),
+                   "preempt_latency_p99_ms": pct(hr["pre"], 99), "frac_preempting": hr["frac_preempting"],
+                   "reparks": hr["reparks"], "training_iterations_done": hr["iters_done"]}
     base = {}
     if not args.no_baselines:
         nb = max(20, args.steps // 2)
@@ -679,6 +689,7 @@ def main():
                      "seed": "7 + pair" if args.arrivals == "poisson" else "1234 + device",
                      "frac_preempting": main_s.get("frac_preempting"), "reparks": main_s.get("reparks"),
                      "inference_device_us_p50": pct(main_s.get("device_us", []), 50)},
+        "poisson_1000": hi_rate,
         "chase": {"desc": "closed loop: every request preempts the running job; next request after its resume",
                   "p50_ms": pct(Cc["lat"], 50), "p99_ms": pct(Cc["lat"], 99),
                   "preempt_latency_p50_ms": pct(Cc["pre"], 50), "preempt_latency_p99_ms": pct(Cc["pre"], 99),
