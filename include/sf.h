@@ -156,6 +156,11 @@ typedef struct sf_config {
                                     their estimated device time (EMA of observed subgraph
                                     durations) stays within this budget, bounding what a
                                     preemption drains; 0 = window limit only */
+  int32_t migrate_home;          /* 1: a job moved to a peer slot by a higher-priority job or
+                                    an inference request migrates back to the slot it started
+                                    on at its first boundary after that slot is free again (no
+                                    queued inference, no present job of priority >= its own);
+                                    0 (paper): it stays on the target */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,
@@ -169,8 +174,14 @@ const char* sf_last_error(void);
 int32_t sf_abi_version(void);
 
 /* Validate and copy a graph (shapes, dtypes, op arity, read-before-write).
- * priority > 0 marks an inference (preempter) graph.  SF_EUNSUPPORTED for ops outside
- * the fixed set; SF_EINVAL for malformed graphs. */
+ * priority: larger = more important.  Inference requests always rank
+ * above every training job (reading Q13).  Between training jobs (PAPER.md:1184-1222,
+ * Fig. 7 scenario): a job of a higher-priority graph started on a slot is "allowed to start
+ * immediately after submission" — every lower-priority job on that slot
+ * stops at its next subgraph boundary and migrates to its auto_target (peer slot: resumes
+ * there at once; SF_TARGET_HOST: parked, swapped back in once no higher-priority job is
+ * present on the slot), or, when its auto_target is the slot itself, waits in place.
+ * SF_EUNSUPPORTED for ops outside the fixed set; SF_EINVAL for malformed graphs. */
 sf_status sf_register_graph(sf_runtime* rt, const sf_graph_desc* g, int32_t priority,
                             sf_graph_id* out);
 
@@ -245,6 +256,9 @@ typedef struct sf_job_info {
   int64_t n_reparks;            /* host-tier preemptions that found the parked copy of the
                                    same cut still current (nothing ran since the swap-in) and
                                    re-parked without pack / D2H */
+  uint64_t submit_ns;           /* CLOCK_MONOTONIC at sf_start_training / sf_adopt_job */
+  int32_t priority;             /* the graph's registered priority */
+  int32_t home;                 /* slot the job started on */
 } sf_job_info;
 
 typedef struct sf_cut_info {

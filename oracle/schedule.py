@@ -20,6 +20,13 @@ trace or the GPU runtime's recorded one):
       arrival and before the inference starts (subgraphs already dispatched to the GPU are
       allowed to finish); events may carry "launch" (dispatch time),
       else t0 is the dispatch time.
+  I5  training priority ("a high priority job is allowed to start
+      immediately after submission"; "upon the arrival of a high
+      priority model, the low priority one is preempted and migrated"): on a device, from a
+      job's submission there until its last subgraph there ends, no training subgraph of a
+      lower-priority job is DISPATCHED there; and the high-priority job's first subgraph
+      starts within ``window`` x (longest lower-priority subgraph on the device) + slack of
+      its submission (the outstanding subgraphs drain, nothing more).
 
 Event dicts: {"dev", "job", "kind": "train"|"infer", "iter", "k", "t0", "t1",
 "arrival" (infer only)}; times in any consistent unit.
@@ -106,6 +113,29 @@ def check_cut_rule(events: Sequence[dict]) -> None:
                                          f"inference at {r['t0']}")
 
 
+def check_priority(events: Sequence[dict], prio: Dict[int, int],
+                   submit: Dict[int, tuple], slack: float = 0.0, window: int = 1) -> None:
+    """I5: ``prio[job]`` = priority, ``submit[job]`` = (device, submission time)."""
+    trains = [e for e in events if e["kind"] == "train"]
+    for hj, (dev, ts) in submit.items():
+        mine = sorted((e for e in trains if e["job"] == hj and e["dev"] == dev),
+                      key=lambda e: e["t0"])
+        if not mine:
+            continue
+        end = mine[-1]["t1"]
+        lower = [e for e in trains if e["dev"] == dev and prio[e["job"]] < prio[hj]]
+        for e in lower:
+            if ts <= e.get("launch", e["t0"]) < end:
+                raise InvariantError(
+                    f"dev {dev}: job {e['job']} (prio {prio[e['job']]}) dispatched "
+                    f"({e['iter']},{e['k']}) at {e.get('launch', e['t0'])} while job {hj} "
+                    f"(prio {prio[hj]}) was present [{ts},{end})")
+        longest = max([e["t1"] - e["t0"] for e in lower], default=0.0)
+        if mine[0]["t0"] - ts > window * longest + slack:
+            raise InvariantError(f"dev {dev}: job {hj} started {mine[0]['t0'] - ts} after "
+                                 f"submission > {window} x {longest} + {slack}")
+
+
 def check_all(events: Sequence[dict], n_sub: Dict[int, int], slack: float = 0.0) -> None:
     check_no_corun(events)
     check_job_order(events, n_sub)
@@ -174,4 +204,56 @@ def simulate(durations: Sequence[float], iters: int, arrivals: Sequence[float],
         ev.append({"dev": 0, "job": 1, "kind": "infer", "iter": 0, "k": 0, "t0": s,
                    "t1": s + infer_dur, "arrival": a})
         free0 = s + infer_dur
+    return ev
+
+
+def simulate_priority(dur_lo: Sequence[float], iters_lo: int, dur_hi: Sequence[float],
+                      iters_hi: int, t_hi: float, tier: str = "host", swap_out: float = 0.0,
+                      swap_in: float = 0.0, home: bool = False) -> List[dict]:
+    """Discrete-event model of the Fig. 7 scenario: job 0 (low
+    priority) trains on device 0; job 1 (high priority) is submitted on device 0 at
+    ``t_hi``.  Job 0 stops at its first boundary >= t_hi (the subgraph running at t_hi
+    finishes); job 1 starts right then and runs to completion on
+    device 0.  Host tier: job 0's state goes out (``swap_out``, concurrent with job 1) and
+    comes back (``swap_in``) once job 1 finished, then job 0 continues on device 0.  Peer
+    tier: job 0 resumes on device 1 at cut + swap_out (reading Q7: it stays there), or
+    with ``home`` migrates back to device 0 at its first boundary after job 1 finished
+    (another ``swap_out``)."""
+    ev: List[dict] = []
+    n_lo = len(dur_lo)
+    t, dev, it, k = 0.0, 0, 0, 0
+    hi_end = None
+    moved_home = False
+    while it < iters_lo:
+        if hi_end is None and t >= t_hi:
+            # cut: job 1 runs its whole job on device 0 from here
+            cut = t
+            s = cut
+            for i in range(iters_hi):
+                for j, d in enumerate(dur_hi):
+                    ev.append({"dev": 0, "job": 1, "kind": "train", "iter": i, "k": j,
+                               "t0": s, "t1": s + d})
+                    s += d
+            hi_end = s
+            if tier == "host":
+                t = max(hi_end, cut + swap_out) + swap_in
+            else:
+                dev, t = 1, cut + swap_out
+            continue
+        if home and dev == 1 and hi_end is not None and t >= hi_end and not moved_home:
+            dev, t, moved_home = 0, t + swap_out, True
+            continue
+        ev.append({"dev": dev, "job": 0, "kind": "train", "iter": it, "k": k, "t0": t,
+                   "t1": t + dur_lo[k]})
+        t += dur_lo[k]
+        k += 1
+        if k == n_lo:
+            it, k = it + 1, 0
+    if hi_end is None:  # job 0 finished before job 1 arrived
+        s = max(t, t_hi)
+        for i in range(iters_hi):
+            for j, d in enumerate(dur_hi):
+                ev.append({"dev": 0, "job": 1, "kind": "train", "iter": i, "k": j,
+                           "t0": s, "t1": s + d})
+                s += d
     return ev

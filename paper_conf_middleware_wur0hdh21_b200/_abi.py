@@ -53,7 +53,7 @@ class sf_config(C.Structure):
                 ("poison_released", C.c_int32), ("trace_capacity", C.c_int32),
                 ("max_inflight", C.c_int32), ("defer_migration", C.c_int32),
                 ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
-                ("inflight_budget_us", C.c_int32)]
+                ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):
@@ -71,7 +71,8 @@ class sf_job_info(C.Structure):
                 ("n_preemptions", C.c_int32), ("migrated_bytes", C.c_uint64),
                 ("last_pack_us", C.c_double), ("last_xfer_us", C.c_double),
                 ("last_unpack_us", C.c_double), ("last_stop_ns", C.c_uint64),
-                ("last_resume_ns", C.c_uint64), ("n_reparks", C.c_int64)]
+                ("last_resume_ns", C.c_uint64), ("n_reparks", C.c_int64),
+                ("submit_ns", C.c_uint64), ("priority", C.c_int32), ("home", C.c_int32)]
 
 
 class sf_cut_info(C.Structure):

@@ -168,6 +168,8 @@ struct Job {
   int dev;
   int64_t iters;
   int auto_target;
+  int home = 0;           // slot the job started on (migrate_home policy)
+  uint64_t t_submit = 0;  // CLOCK_MONOTONIC at sf_start_training / sf_adopt_job
   int64_t it = 0;
   int k = 0;
   int state = SF_JOB_RUNNING;
@@ -907,6 +909,26 @@ float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
 
 bool slot_has_inference(sf_runtime* rt, int s) { return !slot_of(rt, s).q.empty(); }
 
+// A training job of priority > min_prio (>= when or_equal) is present on slot s: running or
+// waiting for the device there, or parked from s on the host tier (it swaps back into s).
+// Jobs moving to a peer, explicitly parked (sf_preempt) or finished are not present.
+const Job* present_job(sf_runtime* rt, int s, const Job* me, int min_prio, bool or_equal) {
+  for (const auto& Jp : rt->jobs) {
+    const Job& o = *Jp;
+    if (&o == me || o.dev != s) continue;
+    const int p = o.g->priority;
+    if (or_equal ? p < min_prio : p <= min_prio) continue;
+    if (o.state == SF_JOB_RUNNING || o.state == SF_JOB_STOPPING ||
+        (o.state == SF_JOB_MIGRATING && o.preempt_target == SF_TARGET_HOST))
+      return &o;
+  }
+  return nullptr;
+}
+// Higher-priority training on J's slot (the Fig. 7 preempter).
+const Job* higher_training(sf_runtime* rt, const Job& J, int s) {
+  return present_job(rt, s, &J, J.g->priority, false);
+}
+
 // Device-side kernel duration stamps (globaltimer): reset {start, end} = {~0, 0}.
 cudaError_t tstamp_reset(unsigned long long* t, cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(t, 0xFF, sizeof(unsigned long long), st);
@@ -1078,9 +1100,11 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       dst = J.resume_dev;
       J.resume_req = false;
     } else {
-      // swap back in once the device's inference queue drained (reading Q4/Q13)
+      // swap back in once the device's inference queue drained (reading Q4/Q13) and no
+      // higher-priority training job is present on it
       rt->cv.wait(lk, [&] {
-        return rt->shutting_down || (!slot_has_inference(rt, src) && S.owner != kInferOwner);
+        return rt->shutting_down || (!slot_has_inference(rt, src) && S.owner != kInferOwner &&
+                                     !higher_training(rt, J, src));
       });
     }
     Slot& D = slot_of(rt, dst);
@@ -1242,10 +1266,21 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         J.t_req = now_ns();
         ++J.sched_pos;
       }
-      const bool has_inf = slot_has_inference(rt, J.dev);
+      // the device is wanted by queued inference (always first, Q13) or by a present
+      // higher-priority training job
+      const bool req_inf = slot_has_inference(rt, J.dev);
+      const Job* hp = req_inf ? nullptr : higher_training(rt, J, J.dev);
+      const bool has_inf = req_inf || hp != nullptr;
       const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu && has_inf &&
                              J.auto_target != J.dev;
-      const bool want_cut = J.preempt_req || (auto_want && at_cut_ok);
+      // migrate_home: back to the start slot once it is free (no inference queued there, no
+      // present job of priority >= ours); a peer move like any other
+      const bool home_want = rt->cfg.migrate_home && !has_inf && J.dev != J.home &&
+                             g.bind[J.home] && !g.bind[J.home]->remote &&
+                             g.bind[J.dev]->peer.count(J.home) && !slot_has_inference(rt, J.home) &&
+                             !present_job(rt, J.home, &J, J.g->priority, true) &&
+                             (!rt->cfg.iteration_granularity || J.k == 0);
+      const bool want_cut = J.preempt_req || (auto_want && at_cut_ok) || home_want;
       // without a migration, yield the device to queued inference at this boundary (unless the
       // session-slicing baseline keeps it for the rest of the iteration)
       const bool yield_to_inf = rt->cfg.exclusive_gpu && has_inf && !(auto_want && !at_cut_ok);
@@ -1254,8 +1289,9 @@ void driver_main(sf_runtime* rt, Job* Jp) {
           release();
           if (!J.preempt_req) {
             J.preempt_park = false;
-            J.preempt_target = J.auto_target;
-            J.t_req = slot_of(rt, J.dev).q.front()->arrival;
+            J.preempt_target = home_want ? J.home : J.auto_target;
+            J.t_req = req_inf ? slot_of(rt, J.dev).q.front()->arrival
+                              : hp ? hp->t_submit : now_ns();
           }
           const int src = J.dev;
           const bool peer = J.preempt_target != SF_TARGET_HOST;
@@ -1875,6 +1911,8 @@ static sf_status start_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t
   J->dev = dev;
   J->iters = iters;
   J->auto_target = auto_target;
+  J->home = dev;
+  J->t_submit = now_ns();
   J->it = it0;
   J->k = k0;
   J->stamp_resume = it0 > 0 || k0 > 0;  // an adopted job: its first launch is the resume
@@ -1905,6 +1943,7 @@ static sf_status start_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t
   Job* jp = J.get();
   rt->jobs.push_back(std::move(J));
   jp->driver = std::thread(driver_main, rt, jp);
+  rt->cv.notify_all();  // lower-priority jobs on dev re-check their boundary gate
   *out = jp->id;
   return SF_OK;
 }
@@ -2048,6 +2087,9 @@ sf_status sf_job_query(sf_runtime* rt, sf_job_id jid, sf_job_info* out) {
   out->last_stop_ns = J->last_stop;
   out->last_resume_ns = J->last_resume;
   out->n_reparks = J->n_repark;
+  out->submit_ns = J->t_submit;
+  out->priority = J->g->priority;
+  out->home = J->home;
   if (J->state == SF_JOB_FAILED) return fail(SF_ECUDA, J->error);
   return SF_OK;
 }

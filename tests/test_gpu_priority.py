@@ -1,0 +1,195 @@
+"""GPU tests of training-preempts-training (the Fig. 7 scenario,
+PAPER.md:1184-1222): a high-priority training job submitted on a slot preempts the
+low-priority job running there, which migrates to its auto_target and resumes there
+(peer slot), or parks on the host tier until the slot is free again.
+
+Bars (north_star): each job's final state is bit-identical to its own unpreempted GPU run
+and within 1e-4 of the CPU oracle; the recorded trace satisfies I1 (no co-run), I2 (per-job
+order, no work lost) and I5 (priority: no lower-priority dispatch while the high-priority
+job is present; it starts within the drain of the outstanding subgraphs) of
+oracle/schedule.py.
+"""
+import time
+
+import numpy as np
+import pytest
+
+from oracle import graph as OG, runner as R, schedule as SC
+from sf_inputs import data as D, graphs as G
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+HOST = -1
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-30))
+
+
+@pytest.fixture(scope="module")
+def P():
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_middleware_wur0hdh21_b200 import runtime as RT, _abi as A
+    return RT, A
+
+
+LO_SEED, HI_SEED = 3, 13
+
+
+def _graphs():
+    g_lo = G.mlp_train()
+    g_hi = G.mlp_train((784, 128, 10), batch=32)
+    return g_lo, g_hi
+
+
+def _setup(RT, g, rt, prio, slots, seed):
+    gh = rt.register(g, priority=prio)
+    gh.partition()
+    st, ds = D.init_state(g, seed=seed), D.datasets(g)
+    for s in range(slots):
+        gh.bind(s, staging=True, host_staging=True)
+        gh.load(s, ds)
+    gh.load(0, st)
+    return gh, st
+
+
+def _solo(P, g, iters, seed):
+    RT, _ = P
+    with RT.Runtime([0]) as rt:
+        gh, st = _setup(RT, g, rt, 0, 1, seed)
+        j = rt.start_training(gh, 0, iters, HOST)
+        rt.wait_job(j, 300)
+        return {i: gh.read(0, i) for i in st}
+
+
+def _wait_iter(rt, job, it, timeout=60.0):
+    t0 = time.time()
+    while rt.job_info(job)["iter"] < it:
+        assert time.time() - t0 < timeout
+        time.sleep(0.0005)
+
+
+@pytest.mark.parametrize("tier,home,W", [("host", False, 1), ("peer", False, 1),
+                                         ("peer", True, 1), ("host", False, 2)])
+def test_training_preempts_training(P, tier, home, W):
+    RT, A = P
+    g_lo, g_hi = _graphs()
+    it_lo, it_hi = 40, 5  # the low-priority job outlives the high-priority one
+    base_lo = _solo(P, g_lo, it_lo, LO_SEED)
+    base_hi = _solo(P, g_hi, it_hi, HI_SEED)
+    slots = 2 if tier == "peer" else 1
+    with RT.Runtime([0] * slots, poison=True, max_inflight=W, migrate_home=home) as rt:
+        gl, st_lo = _setup(RT, g_lo, rt, 0, slots, LO_SEED)
+        gH, st_hi = _setup(RT, g_hi, rt, 1, 1, HI_SEED)
+        jl = rt.start_training(gl, 0, it_lo, 1 if tier == "peer" else HOST)
+        _wait_iter(rt, jl, 5)
+        jh = rt.start_training(gH, 0, it_hi, 0)  # high priority: nowhere to go (waits in place)
+        rt.wait_job(jh, 120)
+        rt.wait_job(jl, 120)
+        il, ih = rt.job_info(jl), rt.job_info(jh)
+        trace = rt.trace()
+        got_lo = {i: gl.read(il["dev"], i) for i in st_lo}
+        got_hi = {i: gH.read(0, i) for i in st_hi}
+    assert ih["priority"] == 1 and il["priority"] == 0
+    assert il["n_preemptions"] >= 1, il
+    if tier == "peer":
+        assert il["dev"] == (0 if home else 1), il
+        assert il["n_preemptions"] == (2 if home else 1), il
+    for i in st_lo:
+        assert got_lo[i].tobytes() == base_lo[i].tobytes(), g_lo.tensors[i].name
+    for i in st_hi:
+        assert got_hi[i].tobytes() == base_hi[i].tobytes(), g_hi.tensors[i].name
+    ref_lo = R.run(g_lo, it_lo, st_lo, D.datasets(g_lo), keep_stagings=False)
+    ref_hi = R.run(g_hi, it_hi, st_hi, D.datasets(g_hi), keep_stagings=False)
+    for got, ref, g in ((got_lo, ref_lo, g_lo), (got_hi, ref_hi, g_hi)):
+        for i in ref.state:
+            if ref.state[i].dtype == np.float32:
+                assert rel(got[i], ref.state[i]) <= TOL, g.tensors[i].name
+    n = {jl: len(OG.partition(g_lo)), jh: len(OG.partition(g_hi))}
+    trains = [e for e in trace if e["kind"] == "train"]
+    SC.check_no_corun(trains)
+    SC.check_job_order(trains, n, start={jl: (0, 0), jh: (0, 0)})
+    # host-observed boundaries: 2 ms of host slack as for I3
+    SC.check_priority(trains, {jl: 0, jh: 1}, {jh: (0, ih["submit_ns"])}, slack=2e6, window=W)
+    # the low-priority job ran on slot 0 both before and (host tier / home) after the
+    # high-priority job, and on the peer in between (peer tier)
+    hi_evs = [e for e in trains if e["job"] == jh]
+    during = [e for e in trains if e["job"] == jl and hi_evs[0]["t0"] <= e["t0"] < hi_evs[-1]["t1"]]
+    if tier == "host":
+        assert not during
+    else:
+        assert during and all(e["dev"] == 1 for e in during)
+
+
+def test_equal_priority_jobs_share_a_slot_at_subgraph_granularity(P):
+    """Two jobs of equal priority on one slot take turns at subgraph boundaries (the
+    device token): both finish, bit-identical to their solo runs, and
+    their subgraphs never overlap (I1)."""
+    RT, A = P
+    g_lo, g_hi = _graphs()
+    base_a = _solo(P, g_lo, 15, LO_SEED)
+    base_b = _solo(P, g_hi, 15, HI_SEED)
+    with RT.Runtime([0], poison=True) as rt:
+        ga, st_a = _setup(RT, g_lo, rt, 0, 1, LO_SEED)
+        gb, st_b = _setup(RT, g_hi, rt, 0, 1, HI_SEED)
+        ja = rt.start_training(ga, 0, 15, 0)
+        jb = rt.start_training(gb, 0, 15, 0)
+        rt.wait_job(ja, 120)
+        rt.wait_job(jb, 120)
+        trace = rt.trace()
+        got_a = {i: ga.read(0, i) for i in st_a}
+        got_b = {i: gb.read(0, i) for i in st_b}
+    for got, base in ((got_a, base_a), (got_b, base_b)):
+        for i in base:
+            assert got[i].tobytes() == base[i].tobytes()
+    trains = [e for e in trace if e["kind"] == "train"]
+    SC.check_no_corun(trains)
+    SC.check_job_order(trains, {ja: len(OG.partition(g_lo)), jb: len(OG.partition(g_hi))},
+                       start={ja: (0, 0), jb: (0, 0)})
+
+
+def test_inference_still_preempts_both_priorities(P):
+    """Inference ranks above every training job (reading Q13): with a high-priority job
+    running and the low-priority one parked, requests still cut the high-priority job."""
+    RT, A = P
+    import torch
+    g_lo, g_hi = _graphs()
+    gi = G.mlp_infer()
+    sti = D.init_state(gi, seed=D.SEED_INFER)
+    xs = D.infer_inputs(gi, 8)
+    base_lo = _solo(P, g_lo, 20, LO_SEED)
+    base_hi = _solo(P, g_hi, 400, HI_SEED)
+    with RT.Runtime([0], poison=True) as rt:
+        gl, st_lo = _setup(RT, g_lo, rt, 0, 1, LO_SEED)
+        gH, st_hi = _setup(RT, g_hi, rt, 1, 1, HI_SEED)
+        ghi = rt.register(gi, priority=2)
+        ghi.partition()
+        ghi.bind(0, staging=False)
+        ghi.load(0, sti)
+        jl = rt.start_training(gl, 0, 20, HOST)
+        _wait_iter(rt, jl, 3)
+        jh = rt.start_training(gH, 0, 400, HOST)
+        _wait_iter(rt, jh, 2)
+        xin = torch.from_numpy(xs).cuda()
+        out = torch.zeros(8, 1, 10, device="cuda")
+        tim = []
+        for r in range(8):
+            time.sleep(0.002)
+            tim.append(rt.wait(rt.submit(ghi, 0, xin[r].data_ptr(), out[r].data_ptr()), 30))
+        rt.wait_job(jh, 120)
+        rt.wait_job(jl, 120)
+        ih = rt.job_info(jh)
+        got_lo = {i: gl.read(0, i) for i in st_lo}
+        got_hi = {i: gH.read(0, i) for i in st_hi}
+        trace = rt.trace()
+    assert ih["n_preemptions"] >= 4, ih
+    assert sum(t["preempted_job"] == jh for t in tim) >= 4
+    for r in range(8):
+        assert rel(out[r].cpu().numpy(), R.run_inference(gi, sti, xs[r])) <= TOL
+    for got, base in ((got_lo, base_lo), (got_hi, base_hi)):
+        for i in base:
+            assert got[i].tobytes() == base[i].tobytes()
+    SC.check_no_corun(trace)

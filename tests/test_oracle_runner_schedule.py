@@ -133,3 +133,56 @@ def test_model_closed_form_single_arrival():
     evs = SC.simulate(dur, 2, [5.0], 1.0, tier="peer", swap_out=0.5)
     nxt = [e for e in evs if e["kind"] == "train" and e["t0"] >= 8.0][0]
     assert (nxt["dev"], nxt["k"], nxt["t0"]) == (1, 2, 8.5)
+
+
+# ---- I5: training priority (Fig. 7 scenario) ---------------
+
+def test_priority_checker_rejects_lower_dispatch_and_late_start():
+    prio = {0: 0, 1: 1}
+    ok = [_ev(0, 0, "train", 0, 2), _ev(0, 0, "train", 2, 4, k=1),   # S_1 running at 3
+          _ev(0, 1, "train", 4, 5), _ev(0, 1, "train", 5, 6, k=1),
+          _ev(0, 0, "train", 6, 8, it=1)]
+    SC.check_priority(ok, prio, {1: (0, 3)})
+    SC.check_no_corun(ok)
+    # a low-priority subgraph dispatched at 4.5 while job 1 is present on device 0
+    bad = ok[:3] + [_ev(0, 0, "train", 4.5, 4.9, it=1)] + ok[3:4]
+    with pytest.raises(SC.InvariantError):
+        SC.check_priority(bad, prio, {1: (0, 3)})
+    # ... but on another device (the peer it migrated to) it may run
+    SC.check_priority(ok[:3] + [_ev(1, 0, "train", 4.5, 4.9, it=1)] + ok[3:4], prio, {1: (0, 3)})
+    # job 1 waited 5 > one outstanding low subgraph (2) after submission
+    late = [_ev(0, 0, "train", 0, 2), _ev(0, 0, "train", 2, 4, k=1),
+            _ev(0, 1, "train", 8, 9), _ev(0, 1, "train", 9, 10, k=1)]
+    with pytest.raises(SC.InvariantError):
+        SC.check_priority(late, prio, {1: (0, 3)})
+    SC.check_priority(late, prio, {1: (0, 3)}, window=3)
+
+
+def test_priority_model_closed_form():
+    lo, hi = [2.0, 2.0], [1.0, 1.0]
+    # job 1 submitted at 3 while S_1 of job 0 runs [2, 4): cut at 4, job 1 runs [4, 8)
+    evs = SC.simulate_priority(lo, 3, hi, 2, 3.0, tier="host", swap_out=0.5, swap_in=1.5)
+    h = [e for e in evs if e["job"] == 1]
+    assert (h[0]["t0"], h[-1]["t1"]) == (4.0, 8.0)
+    nxt = [e for e in evs if e["job"] == 0 and e["t0"] >= 4.0][0]
+    assert (nxt["dev"], nxt["iter"], nxt["k"], nxt["t0"]) == (0, 1, 0, 9.5)  # max(8, 4.5) + 1.5
+    evs = SC.simulate_priority(lo, 3, hi, 2, 3.0, tier="peer", swap_out=0.5)
+    nxt = [e for e in evs if e["job"] == 0 and e["t0"] >= 4.0][0]
+    assert (nxt["dev"], nxt["iter"], nxt["k"], nxt["t0"]) == (1, 1, 0, 4.5)
+    # migrate-back: the first job-0 boundary after 8 is 8.5 on device 1 -> device 0 at 9.0
+    evs = SC.simulate_priority(lo, 4, hi, 2, 3.0, tier="peer", swap_out=0.5, home=True)
+    back = [e for e in evs if e["job"] == 0 and e["t0"] >= 8.0]
+    assert (back[0]["dev"], back[0]["t0"]) == (0, 9.0)
+
+
+def test_priority_model_satisfies_invariants():
+    lo, hi = [0.7, 1.3, 0.4, 2.1], [0.5, 0.9, 1.1]
+    for tier, home in (("host", False), ("peer", False), ("peer", True)):
+        for t_hi in (0.0, 3.3, 7.0, 100.0):
+            evs = SC.simulate_priority(lo, 6, hi, 4, t_hi, tier=tier, swap_out=0.3,
+                                       swap_in=0.3, home=home)
+            SC.check_no_corun(evs)
+            SC.check_job_order(evs, {0: len(lo), 1: len(hi)})
+            SC.check_priority(evs, {0: 0, 1: 1}, {1: (0, t_hi)}, slack=1e-9)
+            assert len([e for e in evs if e["job"] == 0]) == 6 * len(lo)
+            assert len([e for e in evs if e["job"] == 1]) == 4 * len(hi)
