@@ -126,6 +126,13 @@ typedef uint64_t sf_req_id;
 #define SF_HOST_ZC 1 /* zero-copy: pack kernel stores straight into mapped pinned memory,
                         unpack kernel reads it back over PCIe */
 
+/* Migration engine. */
+#define SF_MIG_SM 0 /* descriptor-walk kernels: pack / unpack / fused peer store (default) */
+#define SF_MIG_CE 1 /* copy engines only, zero SM work: one cudaMemcpyBatchAsync per ~2 MB of
+                       live tensors, arena -> pinned staging payloads (the CPU writes header and
+                       zero padding: same staging bytes as a pack), staging -> arena, or
+                       arena -> peer arena; host_mode is ignored */
+
 typedef struct sf_config {
   int32_t n_devices;             /* logical device slots */
   const int32_t* cuda_ordinals;  /* host array [n_devices]: CUDA device of each slot, or -1
@@ -161,6 +168,7 @@ typedef struct sf_config {
                                     on at its first boundary after that slot is free again (no
                                     queued inference, no present job of priority >= its own);
                                     0 (paper): it stays on the target */
+  int32_t migration_engine;      /* SF_MIG_SM (default) or SF_MIG_CE */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,

@@ -22,6 +22,8 @@ SF_EUNSUPPORTED = -7
 SF_TARGET_HOST = -1
 SF_HOST_CE = 0
 SF_HOST_ZC = 1
+SF_MIG_SM = 0
+SF_MIG_CE = 1
 SF_PART_PER_LAYER_PHASE = 0
 SF_PART_MAX_OPS = 1
 JOB_STATES = {0: "running", 1: "stopping", 2: "migrating", 3: "preempted", 4: "done", 5: "failed",
@@ -53,7 +55,8 @@ class sf_config(C.Structure):
                 ("poison_released", C.c_int32), ("trace_capacity", C.c_int32),
                 ("max_inflight", C.c_int32), ("defer_migration", C.c_int32),
                 ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
-                ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32)]
+                ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32),
+                ("migration_engine", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):

@@ -955,28 +955,71 @@ cudaError_t poison(Binding& b, cudaStream_t st) {
 }
 
 
-// Host-tier transfer that yields to inference: copy-engine traffic over PCIe slows a
-// concurrent batch-1 forward by ~45% on B200 (scripts/infer_bench.py COPY=d2h: 50 -> 74 us),
-// so the staging moves in 2 MB chunks, at most two in flight, and no chunk is issued while a
-// request is queued or running on the slot.  Returns once every chunk has completed.
-cudaError_t yielding_copy(Job& J, Slot& S, int slot, void* dst, const void* src, size_t bytes,
-                          cudaMemcpyKind kind, cudaStream_t st) {
+// Copy-engine transfers.  A segment list is issued in ~2 MB batches (large segments split),
+// one cudaMemcpyBatchAsync per batch (per-segment cudaMemcpyAsync where the batch API is
+// unavailable), so no SM runs for the copy.  With `yield`, at most two batches are in flight
+// and none is issued while a request is queued or running on the slot: copy-engine traffic
+// over PCIe slows a concurrent batch-1 forward by ~45% on B200 (scripts/infer_bench.py
+// COPY=d2h: 50 -> 74 us; reading Q22).  Returns once every batch has been issued and (yield)
+// has completed.
+struct Seg {
+  void* dst;
+  const void* src;
+  size_t n;
+};
+
+cudaError_t issue_batch(std::vector<void*>& d, std::vector<void*>& s, std::vector<size_t>& n,
+                        cudaStream_t st) {
+  static std::atomic<bool> batch_ok{!(std::getenv("SF_CE_NOBATCH") && std::getenv("SF_CE_NOBATCH")[0] == '1')};
+  if (d.size() > 1 && batch_ok.load(std::memory_order_relaxed)) {
+    cudaMemcpyAttributes attr{};
+    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+    size_t idx = 0, fail_idx = 0;
+    const cudaError_t e =
+        cudaMemcpyBatchAsync(d.data(), s.data(), n.data(), d.size(), &attr, &idx, 1, &fail_idx, st);
+    if (e == cudaSuccess) return e;
+    if (e != cudaErrorNotSupported && e != cudaErrorInvalidValue) return e;
+    cudaGetLastError();
+    batch_ok = false;  // fall back to one copy per segment from now on
+  }
+  for (size_t i = 0; i < d.size(); ++i) {
+    const cudaError_t e = cudaMemcpyAsync(d[i], s[i], n[i], cudaMemcpyDefault, st);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+cudaError_t ce_segments(Job& J, Slot& S, int slot, const std::vector<Seg>& segs, cudaStream_t st,
+                        bool yield) {
   constexpr size_t kChunk = size_t(2) << 20;
-  size_t off = 0;
+  size_t si = 0, so = 0;  // cursor: segment, offset inside it
   int head = 0, n_inflight = 0;  // ring of 2 events
+  std::vector<void*> bd, bs;
+  std::vector<size_t> bn;
   auto busy = [&] {
     const int o = S.owner.load(std::memory_order_acquire);
     return S.qn.load(std::memory_order_acquire) > 0 || o == kInferOwner;
   };
-  while (off < bytes || n_inflight > 0) {
-    if (off < bytes && n_inflight < 2 && !busy()) {
-      const size_t n = std::min(kChunk, bytes - off);
-      cudaError_t e = cudaMemcpyAsync(static_cast<uint8_t*>(dst) + off, static_cast<const uint8_t*>(src) + off,
-                                      n, kind, st);
-      if (e == cudaSuccess) e = cudaEventRecord(J.ev_ck[slot * 2 + (head + n_inflight) % 2], st);
+  while (si < segs.size() || n_inflight > 0) {
+    if (si < segs.size() && (!yield || (n_inflight < 2 && !busy()))) {
+      bd.clear(); bs.clear(); bn.clear();
+      size_t got = 0;
+      while (si < segs.size() && got < kChunk) {
+        const Seg& g = segs[si];
+        const size_t n = std::min(kChunk - got, g.n - so);
+        if (n > 0) {
+          bd.push_back(static_cast<uint8_t*>(g.dst) + so);
+          bs.push_back(const_cast<uint8_t*>(static_cast<const uint8_t*>(g.src) + so));
+          bn.push_back(n);
+        }
+        got += n;
+        so += n;
+        if (so == g.n) { ++si; so = 0; }
+      }
+      cudaError_t e = issue_batch(bd, bs, bn, st);
+      if (e == cudaSuccess && yield) e = cudaEventRecord(J.ev_ck[slot * 2 + (head + n_inflight) % 2], st);
       if (e != cudaSuccess) return e;
-      ++n_inflight;
-      off += n;
+      if (yield) ++n_inflight;
       continue;
     }
     if (n_inflight > 0) {
@@ -991,6 +1034,39 @@ cudaError_t yielding_copy(Job& J, Slot& S, int slot, void* dst, const void* src,
     for (int i = 0; i < 64; ++i) cpu_relax();
   }
   return cudaSuccess;
+}
+
+cudaError_t yielding_copy(Job& J, Slot& S, int slot, void* dst, const void* src, size_t bytes,
+                          cudaStream_t st) {
+  return ce_segments(J, S, slot, {Seg{dst, src, bytes}}, st, true);
+}
+
+// Copy-engine-only migration (SF_MIG_CE): the per-tensor segments of cut k.
+//   to_host: arena -> pinned staging payloads; from_host: staging payloads -> arena;
+//   peer: arena -> peer arena (same offsets).
+std::vector<Seg> cut_segments(const Graph& g, int k, uint8_t* arena, uint8_t* other, int dir) {
+  std::vector<Seg> v;
+  v.reserve(g.live[k].size());
+  for (size_t e = 0; e < g.live[k].size(); ++e) {
+    const Tensor& t = g.T[g.live[k][e]];
+    if (dir == 0) v.push_back({other + g.payload_off[k][e], arena + t.offset, t.nbytes});
+    else if (dir == 1) v.push_back({arena + t.offset, other + g.payload_off[k][e], t.nbytes});
+    else v.push_back({other + t.offset, arena + t.offset, t.nbytes});
+  }
+  return v;
+}
+
+// The staging header of cut k (iter patched) and zero padding, written by the CPU straight
+// into pinned staging (the copy engines write only the payloads): byte-identical to a pack.
+void write_host_header(const Graph& g, int k, int64_t iter, uint8_t* stg) {
+  std::memcpy(stg, g.header[k].data(), g.header[k].size());
+  std::memcpy(stg + 16, &iter, sizeof(iter));
+  const auto& off = g.payload_off[k];
+  for (size_t e = 0; e < off.size(); ++e) {
+    const uint64_t end = off[e] + g.T[g.live[k][e]].nbytes;
+    const uint64_t next = e + 1 < off.size() ? off[e + 1] : g.staging_total[k];
+    if (next > end) std::memset(stg + end, 0, next - end);
+  }
 }
 
 // Preempt J at its current boundary (rt->m held on entry and on return).
@@ -1051,10 +1127,16 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
                       J.parked_iter == J.it && J.parked_k == k;
   if (target == SF_TARGET_HOST) {
     // ---- host tier: pack (+ D2H), park, swap back in ------------------------------
-    const bool zc = rt->cfg.host_mode == SF_HOST_ZC || B.staging == nullptr;
+    // SF_MIG_CE: no pack kernel; the CPU writes the header, the copy engines the payloads
+    const bool ce = rt->cfg.migration_engine == SF_MIG_CE;
+    const bool zc = !ce && (rt->cfg.host_mode == SF_HOST_ZC || B.staging == nullptr);
     tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
     if (repark) {
+      cudaEventRecord(J.ev_b[src], S.s_mig);
+      e = cudaSuccess;
+    } else if (ce) {
+      write_host_header(g, k, J.it, B.host_staging);
       cudaEventRecord(J.ev_b[src], S.s_mig);
       e = cudaSuccess;
     } else if (zc) {
@@ -1072,12 +1154,13 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     rt->cv.notify_all();
     lk.unlock();
     if (!repark && !zc &&
-        (e = yielding_copy(J, S, src, B.host_staging, B.staging, g.staging_total[k], cudaMemcpyDeviceToHost,
-                           S.s_mig)) != cudaSuccess)
+        (e = ce ? ce_segments(J, S, src, cut_segments(g, k, B.arena, B.host_staging, 0), S.s_mig, true)
+                : yielding_copy(J, S, src, B.host_staging, B.staging, g.staging_total[k], S.s_mig)) !=
+            cudaSuccess)
       return cuda_fail(e, "D2H");
     cudaEventRecord(J.ev_c[src], S.s_mig);
     if ((e = wait_event_relaxed(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
-    float pack_us = repark ? 0.f : static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
+    float pack_us = repark || ce ? 0.f : static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
     if (pack_us < 0.f) pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
     const float d2h_us = repark ? 0.f : elapsed_us(J.ev_b[src], J.ev_c[src]);
     if (rt->cfg.poison_released) {
@@ -1115,15 +1198,17 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     // the parked bytes live in the source binding's pinned staging; a ZC swap-in reads
     // them in place when resuming on the same slot, otherwise H2D + unpack
     tstamp_reset(D.tstamp + 2, D.s_train);
-    if (zc && dst == src) {
+    if (ce) {
+      e = ce_segments(J, D, dst, cut_segments(g, k, BD.arena, B.host_staging, 1), D.s_train, true);
+      cudaEventRecord(J.ev_b[dst], D.s_train);
+    } else if (zc && dst == src) {
       const CopyList& L = BD.unpack_zc[k];
       e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
       cudaEventRecord(J.ev_b[dst], D.s_train);
     } else if (!BD.staging) {
       e = cudaErrorInvalidValue;
     } else {
-      e = yielding_copy(J, D, dst, BD.staging, B.host_staging, g.staging_total[k], cudaMemcpyHostToDevice,
-                        D.s_train);
+      e = yielding_copy(J, D, dst, BD.staging, B.host_staging, g.staging_total[k], D.s_train);
       cudaEventRecord(J.ev_b[dst], D.s_train);
       if (e == cudaSuccess) {
         const CopyList& L = BD.unpack[k];
@@ -1152,7 +1237,10 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     const CopyList& L = it->second[k];
     tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
-    e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S.s_mig, S.tstamp);
+    if (rt->cfg.migration_engine == SF_MIG_CE)  // copy engines over NVLink, no SM work
+      e = ce_segments(J, S, src, cut_segments(g, k, B.arena, g.bind[target]->arena, 2), S.s_mig, false);
+    else
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S.s_mig, S.tstamp);
     if (e != cudaSuccess) return cuda_fail(e, "peer store");
     cudaEventRecord(J.ev_b[src], S.s_mig);
     Slot& T = slot_of(rt, target);

@@ -133,13 +133,13 @@ class Runtime:
                  host_mode: int = A.SF_HOST_CE, poison: bool = False, budget_bytes: int = 0,
                  trace_capacity: int = 0, defer_migration: bool = False, max_inflight: int = 1,
                  dispatch_spin_us: int = 0, inflight_budget_us: int = 0,
-                 migrate_home: bool = False):
+                 migrate_home: bool = False, migration_engine: int = 0):
         self.ordinals = list(ordinals)
         arr = (C.c_int32 * len(self.ordinals))(*self.ordinals)
         cfg = A.sf_config(len(self.ordinals), arr, int(exclusive), int(auto_preempt),
                           int(iteration_granularity), host_mode, int(poison), trace_capacity,
                           max_inflight, int(defer_migration), budget_bytes, dispatch_spin_us,
-                          inflight_budget_us, int(migrate_home))
+                          inflight_budget_us, int(migrate_home), migration_engine)
         h = C.c_void_p()
         check(lib().sf_create(C.byref(cfg), C.byref(h)), "sf_create")
         self.h = h

@@ -53,16 +53,16 @@ def state_graph(sizes):
     return g
 
 
-def c5(reps=4):
+def c5(reps=4, engine=0, totals=None, mixes=None):
     out = []
-    totals = [1 << 20, 4 << 20, 16 << 20, 64 << 20, 256 << 20, 1 << 30, 2 << 30, 4 << 30, 8 << 30]
-    for mix in ("single", "resnet_hist", "uniform_1MB", "all_4KB"):
+    totals = totals or [1 << 20, 4 << 20, 16 << 20, 64 << 20, 256 << 20, 1 << 30, 2 << 30, 4 << 30, 8 << 30]
+    for mix in mixes or ("single", "resnet_hist", "uniform_1MB", "all_4KB"):
         for tot in totals:
             if mix == "all_4KB" and tot > (512 << 20):
                 continue
             sizes = sizes_for(tot, mix)
             g = state_graph(sizes)
-            with Runtime([0, 0]) as rt:
+            with Runtime([0, 0], migration_engine=engine) as rt:
                 gh = rt.register(g)
                 gh.partition()
                 gh.bind(0, staging=False)
@@ -83,11 +83,46 @@ def c5(reps=4):
                 ji = rt.job_info(job)
                 live = gh.live_set(0)[1]
             t = float(np.median([x for x in times if x > 0])) if times else float("nan")
-            out.append({"mix": mix, "bytes": live, "tensors": len(sizes) + 1, "kernel_us": t,
+            out.append({"engine": ["sm", "ce"][engine], "mix": mix, "bytes": live, "tensors": len(sizes) + 1, "kernel_us": t,
                         "gbs_2x": 2 * live / (t * 1e-6) / 1e9, "frac_hbm": 2 * live / (t * 1e-6) / 1e9 / PEAK,
                         "preemptions": ji["n_preemptions"]})
             print(json.dumps(out[-1]), flush=True)
     return out
+
+
+def c5ce():
+    """Copy-engine-only peer migration (cudaMemcpyBatchAsync, no SM work) vs the SM
+    descriptor walk on the same live sets (same GPU: HBM -> HBM)."""
+    totals = [1 << 20, 16 << 20, 256 << 20, 1 << 30]
+    mixes = ("single", "resnet_hist", "all_4KB")
+    return {"sm": c5(engine=0, totals=totals, mixes=mixes), "ce": c5(engine=1, totals=totals, mixes=mixes)}
+
+
+def c2host():
+    """C2-shaped job (ResNet-50 state, batch 8) parked on the host tier at several cuts:
+    SM engine (pack kernel + one D2H of the staging; H2D + unpack kernel) vs CE engine
+    (per-tensor batched D2H / H2D, no SM work)."""
+    g = G.resnet50_forest(batch=8)
+    st, ds = D.init_state(g), D.datasets(g)
+    rows = []
+    for engine in (0, 1):
+        with Runtime([0], migration_engine=engine) as rt:
+            gh = rt.register(g)
+            gh.partition(policy="max_ops", max_ops=1, update_chunks=8)
+            gh.bind(0, host_staging=True)
+            gh.load(0, {**st, **ds})
+            n = gh.n_subgraphs
+            cuts = [0, n // 3, 2 * n // 3, n - 1]
+            for c, k in enumerate(cuts):
+                job = rt.start_training(gh, 0, 3, HOST, schedule=[(1, k, HOST)])
+                rt.wait_job(job, 120)
+                ji = rt.job_info(job)
+                rows.append({"engine": ["sm", "ce"][engine], "k": k, "live_bytes": gh.live_set(k)[1],
+                             "tensors": len(gh.live_set(k)[0]), "pack_us": ji["last_pack_us"],
+                             "d2h_h2d_us": ji["last_xfer_us"], "unpack_us": ji["last_unpack_us"],
+                             "preempt_to_resume_ms": (ji["last_resume_ns"] - ji["last_stop_ns"]) * 1e-6})
+                print(json.dumps(rows[-1]), flush=True)
+    return rows
 
 
 def c3():

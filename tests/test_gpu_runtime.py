@@ -550,3 +550,55 @@ def test_open_loop_requests_during_swap_in_are_bitwise(P, defer):
     assert info["n_preemptions"] >= 5, info
     print("preemptions", info["n_preemptions"], "re-parks", info["n_reparks"])
     assert_bitwise(base, got)
+
+
+# ---- copy-engine-only migration (SF_MIG_CE) ----------------------
+
+def test_ce_migration_staging_bytes_equal_oracle_pack(P):
+    """The CE host tier writes the same staging bytes as the pack kernel: the CPU writes
+    header + zero padding, the copy engines the payloads (cut 0: exact oracle pack)."""
+    RT, A = P
+    g = G.mlp_train()
+    st = D.init_state(g)
+    _, _, _, _, hs = run_gpu(P, g, 1, schedule=[(0, 0, HOST)], slots=1,
+                             migration_engine=A.SF_MIG_CE)
+    L = OG.live_set(g, OG.partition(g), 0)
+    expect = S.pack(g, L, st, 0, 0)
+    assert hs[:len(expect)].tobytes() == expect
+    # a mid cut after a different cut dirtied the staging: header + padding still exact
+    ds = D.datasets(g)
+    _, _, _, _, hs = run_gpu(P, g, 4, schedule=[(1, 4, HOST), (3, 3, HOST)], slots=1,
+                             migration_engine=A.SF_MIG_CE)
+    ref = R.run(g, 4, st, ds, schedule=[(1, 4, R.HOST), (3, 3, R.HOST)])
+    buf = ref.stagings[-1][3]
+    hdr, ents = S.parse(buf)
+    ps = -(-(32 + 24 * len(ents)) // 256) * 256
+    gb = hs[:len(buf)].tobytes()
+    assert gb[:ps] == buf[:ps]
+    for (tid, dt, off, nb) in ents:
+        pad = -(-nb // 256) * 256
+        assert not any(gb[off + nb:off + pad])
+
+
+@pytest.mark.parametrize("W", [1, 2])
+def test_ce_migration_host_and_peer_bitwise(P, W):
+    """Copy-engine-only migration on both tiers, every cut, poisoned released arenas:
+    bit-identical to the unpreempted run; resnet prefix (many small tensors) as well."""
+    RT, A = P
+    g = G.mlp_train()
+    base, _, _, _, _ = run_gpu(P, g, 30, max_inflight=W)
+    n = len(OG.partition(g))
+    sched = sorted([(5, k, HOST) for k in range(n)] + [(8, k, 1 - (k % 2)) for k in range(1, n)]
+                   + [(12, 0, 0), (15, 2, 1), (16, 3, HOST), (20, 1, 0)])
+    got, _, info, _, _ = run_gpu(P, g, 30, schedule=sched, poison=True, max_inflight=W,
+                                 migration_engine=A.SF_MIG_CE)
+    assert info["n_preemptions"] >= 10
+    assert_bitwise(base, got)
+    gr = G.resnet50_forest(batch=1, spatial_div=4, max_layers=12)
+    nr = len(OG.partition(gr))
+    sched = D.preemption_schedule(3, nr, 10, targets=[1, 0, HOST], seed=5)
+    base, _, _, _, _ = run_gpu(P, gr, 3)
+    got, _, info, _, _ = run_gpu(P, gr, 3, schedule=sched, poison=True,
+                                 migration_engine=A.SF_MIG_CE)
+    assert info["n_preemptions"] >= 4
+    assert_bitwise(base, got)
