@@ -66,11 +66,16 @@ enum sf_tensor_kind {
   SF_LABEL = 5, SF_ACT = 6, SF_GRAD = 7, SF_OUTPUT = 8
 };
 
-/* The fixed op set of BASELINE.json north_star.  Operand conventions:
+/* The fixed op set of BASELINE.json north_star (+ GELU).  Operand
+ * conventions:
  *  GEMM         in[A,B] out[C]        C = op(A) op(B) (+C if SF_GEMM_ACC); op = transpose
  *                                     if SF_GEMM_TA / SF_GEMM_TB; fp32-accurate (3xTF32)
- *  BIAS_ACT     in[z,b1(,b2,b3)] out[h]  h = act(z + b1 + b2 + b3), act = ReLU if SF_ACT_RELU
- *  BIAS_ACT_BWD in[dh,h] out[dz,db]   dz = dh * [h > 0]; db = column sum of dz
+ *  BIAS_ACT     in[z,b1(,b2,b3)] out[h(,u)]  u = z + b1 + b2 + b3; h = act(u): ReLU if
+ *                                     SF_ACT_RELU, GELU (exact erf form) if SF_ACT_GELU, else
+ *                                     identity; out[1] = u (GELU only: the backward needs it)
+ *  BIAS_ACT_BWD in[dh,h] out[dz,db]   ReLU: dz = dh * [h > 0];
+ *               in[dh,u] (SF_ACT_GELU) GELU: dz = dh * (Phi(u) + u phi(u));
+ *                                     db = column sum of dz
  *  COLSUM       in[x] out[s]          s = column sum of x (s is [1, cols])
  *  SOFTMAX_CE   in[logits,labels] out[loss,dlogits]  mean sparse CE; (softmax-onehot)/B
  *  SOFTMAX      in[logits] out[probs]
@@ -88,6 +93,7 @@ enum sf_op_type {
 #define SF_GEMM_TB 2
 #define SF_GEMM_ACC 4
 #define SF_ACT_RELU 1
+#define SF_ACT_GELU 2 /* gelu(u) = u Phi(u) = 0.5 u (1 + erf(u / sqrt 2)) (BERT's activation) */
 
 typedef struct sf_tensor_desc {
   int32_t rows, cols; /* 2-D row-major */
@@ -413,10 +419,14 @@ sf_status sf_debug_chain_trace(void* dev_buf);
 sf_status sf_op_mlp_chain(const float* x, int32_t M, int32_t n_layers, const int32_t* widths,
                           const float* const* W, const float* const* b, const int32_t* relu,
                           float* const* h, float* probs, void* stream);
+/* act: 0 identity, SF_ACT_RELU, SF_ACT_GELU. */
 sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
-                         float* h, int32_t rows, int32_t cols, int32_t relu, void* stream);
+                         float* h, int32_t rows, int32_t cols, int32_t act, void* stream);
 sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* db,
                              int32_t rows, int32_t cols, void* stream);
+/* GELU backward fused with the bias gradient: dz = dh * gelu'(u); db = column sum of dz. */
+sf_status sf_op_gelu_bwd(const float* dh, const float* u, float* dz, float* db, int32_t rows,
+                         int32_t cols, void* stream);
 sf_status sf_op_colsum(const float* x, float* s, int32_t rows, int32_t cols, void* stream);
 sf_status sf_op_softmax_ce(const float* logits, const int32_t* labels, float* loss,
                            float* dlogits, int32_t rows, int32_t cols, void* stream);

@@ -29,7 +29,7 @@ from __future__ import annotations
 from typing import List, Tuple
 
 from sf_inputs.ir import (ACC, ADAM, BIAS_ACT, BIAS_ACT_BWD, COLSUM, DATASET, F32, FEED,
-                          GEMM, I32, INPUT, LABEL, OUTPUT, PERSISTENT_KINDS, SGD_MOM,
+                          GELU, GEMM, I32, RELU, INPUT, LABEL, OUTPUT, PERSISTENT_KINDS, SGD_MOM,
                           SOFTMAX, SOFTMAX_CE, STEP_INC, TA, TB, Graph)
 
 OPTIMIZER_OPS = (SGD_MOM, ADAM, STEP_INC)
@@ -76,9 +76,12 @@ def validate(g: Graph) -> None:
             chk(K == K2 and C.rows == M and C.cols == N, f"op {j}: gemm shape mismatch")
             chk(A.dtype == B.dtype == C.dtype == F32, f"op {j}: gemm dtype")
         elif op.type == BIAS_ACT:
-            chk(2 <= len(op.ins) <= 4 and len(op.outs) == 1, f"op {j}: bias_act arity")
-            z, h = T[op.ins[0]], T[op.outs[0]]
-            chk((z.rows, z.cols) == (h.rows, h.cols), f"op {j}: bias_act shape")
+            n_out = (1, 2) if op.flags & GELU else (1,)
+            chk(2 <= len(op.ins) <= 4 and len(op.outs) in n_out, f"op {j}: bias_act arity")
+            chk(not (op.flags & RELU and op.flags & GELU), f"op {j}: one activation")
+            z = T[op.ins[0]]
+            for o in op.outs:
+                chk((z.rows, z.cols) == (T[o].rows, T[o].cols), f"op {j}: bias_act shape")
             for b in op.ins[1:]:
                 chk((T[b].rows, T[b].cols) == (1, z.cols), f"op {j}: bias shape")
         elif op.type == BIAS_ACT_BWD:

@@ -15,7 +15,9 @@ from __future__ import annotations
 
 import numpy as np
 
-from sf_inputs.ir import (ACC, ADAM, BIAS_ACT, BIAS_ACT_BWD, COLSUM, FEED, GEMM, RELU,
+from scipy.special import erf
+
+from sf_inputs.ir import (ACC, ADAM, BIAS_ACT, BIAS_ACT_BWD, COLSUM, FEED, GELU, GEMM, RELU,
                           SGD_MOM, SOFTMAX, SOFTMAX_CE, STEP_INC, TA, TB)
 
 
@@ -58,6 +60,31 @@ def bias_act(z, biases, relu, exact=False):
     if relu:
         s = np.maximum(s, 0.0)
     return _out(s, exact)
+
+
+def gelu(u, exact=False):
+    """GELU, exact erf form (Hendrycks & Gimpel; BERT's activation; TF gelu with
+    approximate=False): gelu(u) = u Phi(u) = 0.5 u (1 + erf(u / sqrt 2))."""
+    x = _f(u, exact)
+    return _out(0.5 * x * (1.0 + erf(x / np.sqrt(2.0))), exact)
+
+
+def bias_gelu(z, biases, exact=False):
+    """u = z + b1 [+ b2 + b3]; h = gelu(u).  Returns (h, u): u is kept for the backward."""
+    s = _f(z, exact).copy()
+    for b in biases:
+        s = s + _f(b, exact)
+    u = _out(s, exact)
+    return gelu(u, exact), u
+
+
+def gelu_bwd(dh, u, exact=False):
+    """dz = dh * gelu'(u), gelu'(u) = Phi(u) + u phi(u) (product rule on u Phi(u));
+    db = column sum of dz."""
+    x = _f(u, exact)
+    d = 0.5 * (1.0 + erf(x / np.sqrt(2.0))) + x * np.exp(-0.5 * x * x) / np.sqrt(2.0 * np.pi)
+    dz = _f(dh, exact) * d
+    return _out(dz, exact), _out(dz.sum(axis=0, keepdims=True), exact)
 
 
 def bias_act_bwd(dh, h, exact=False):
@@ -142,8 +169,15 @@ def apply_op(op, T, shapes, exact=False):
     t, ins, outs = op.type, op.ins, op.outs
     if t == GEMM:
         T[outs[0]] = gemm(T[ins[0]], T[ins[1]], T.get(outs[0]), op.flags, exact)
+    elif t == BIAS_ACT and op.flags & GELU:
+        h, u = bias_gelu(T[ins[0]], [T[i] for i in ins[1:]], exact)
+        T[outs[0]] = h
+        if len(outs) > 1:
+            T[outs[1]] = u
     elif t == BIAS_ACT:
         T[outs[0]] = bias_act(T[ins[0]], [T[i] for i in ins[1:]], bool(op.flags & RELU), exact)
+    elif t == BIAS_ACT_BWD and op.flags & GELU:
+        T[outs[0]], T[outs[1]] = gelu_bwd(T[ins[0]], T[ins[1]], exact)
     elif t == BIAS_ACT_BWD:
         T[outs[0]], T[outs[1]] = bias_act_bwd(T[ins[0]], T[ins[1]], exact)
     elif t == COLSUM:

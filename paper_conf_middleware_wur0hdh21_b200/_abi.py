@@ -154,6 +154,7 @@ PROTOTYPES = {
                               _P(C.c_int32), _P(_vp), _vp, _vp]),
     "sf_op_bias_act": (_st, [_vp, _vp, _vp, _vp, _vp, C.c_int32, C.c_int32, C.c_int32, _vp]),
     "sf_op_bias_act_bwd": (_st, [_vp, _vp, _vp, _vp, C.c_int32, C.c_int32, _vp]),
+    "sf_op_gelu_bwd": (_st, [_vp, _vp, _vp, _vp, C.c_int32, C.c_int32, _vp]),
     "sf_op_colsum": (_st, [_vp, _vp, C.c_int32, C.c_int32, _vp]),
     "sf_op_softmax_ce": (_st, [_vp, _vp, _vp, _vp, C.c_int32, C.c_int32, _vp]),
     "sf_op_softmax": (_st, [_vp, _vp, C.c_int32, C.c_int32, _vp]),

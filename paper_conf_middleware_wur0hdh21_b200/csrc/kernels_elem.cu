@@ -28,9 +28,30 @@ __device__ __forceinline__ float warp_max(float v) {
 }
 
 // ---- bias + activation ----------------------------------------------------------------
+// act: 0 identity, 1 ReLU, 2 GELU (exact erf form, gelu(u) = 0.5 u (1 + erf(u / sqrt 2)));
+// pre (optional) receives u = z + biases (the GELU backward reads it).
+__device__ __forceinline__ float act_fwd(int act, float v) {
+  if (act == 1) return fmaxf(v, 0.f);
+  if (act == 2) return 0.5f * v * (1.f + erff(v * 0.70710678118654752f));
+  return v;
+}
+// Backward of the activation given the mask operand m: ReLU (m = h): [m > 0]; GELU (m = u):
+// gelu'(u) = Phi(u) + u phi(u).
+__device__ __forceinline__ float act_bwd(int mode, float v, float m) {
+  if (mode == 1) return m > 0.f ? v : 0.f;
+  const float cdf = 0.5f * (1.f + erff(m * 0.70710678118654752f));
+  const float pdf = 0.3989422804014327f * expf(-0.5f * m * m);
+  return v * (cdf + m * pdf);
+}
+__device__ __forceinline__ float4 act_bwd4(int mode, float4 v, float4 m) {
+  return make_float4(act_bwd(mode, v.x, m.x), act_bwd(mode, v.y, m.y), act_bwd(mode, v.z, m.z),
+                     act_bwd(mode, v.w, m.w));
+}
+
 __global__ void bias_act_kernel(const float* __restrict__ z, const float* __restrict__ b1,
                                 const float* __restrict__ b2, const float* __restrict__ b3,
-                                float* __restrict__ h, int rows, int cols, int relu, int vec) {
+                                float* __restrict__ h, float* __restrict__ pre, int rows, int cols,
+                                int relu, int vec) {
   sfdev::griddep_wait();
   sfdev::griddep_launch();
   const uint64_t total = static_cast<uint64_t>(rows) * cols;
@@ -44,7 +65,8 @@ __global__ void bias_act_kernel(const float* __restrict__ z, const float* __rest
       v.x += b.x; v.y += b.y; v.z += b.z; v.w += b.w;
       if (b2) { b = *reinterpret_cast<const float4*>(b2 + c); v.x += b.x; v.y += b.y; v.z += b.z; v.w += b.w; }
       if (b3) { b = *reinterpret_cast<const float4*>(b3 + c); v.x += b.x; v.y += b.y; v.z += b.z; v.w += b.w; }
-      if (relu) { v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f); }
+      if (pre) reinterpret_cast<float4*>(pre)[q] = v;
+      v.x = act_fwd(relu, v.x); v.y = act_fwd(relu, v.y); v.z = act_fwd(relu, v.z); v.w = act_fwd(relu, v.w);
       reinterpret_cast<float4*>(h)[q] = v;
     }
     return;
@@ -55,8 +77,8 @@ __global__ void bias_act_kernel(const float* __restrict__ z, const float* __rest
     float v = z[i] + b1[c];
     if (b2) v += b2[c];
     if (b3) v += b3[c];
-    if (relu) v = fmaxf(v, 0.f);
-    h[i] = v;
+    if (pre) pre[i] = v;
+    h[i] = act_fwd(relu, v);
   }
 }
 
@@ -77,7 +99,7 @@ ColsumPlan plan_colsum(int rows, int cols) {
 __global__ void __launch_bounds__(256)
 colsum_kernel(const float* __restrict__ x, const float* __restrict__ mask, float* __restrict__ dz,
               float* __restrict__ s, int rows, int cols, int rper, int rsplit, float* ws,
-              unsigned* counters) {
+              unsigned* counters, int mode) {
   const int lane = threadIdx.x & 31, rl = threadIdx.x >> 5;
   const int col = blockIdx.x * 32 + lane;
   const int z = blockIdx.y;
@@ -88,7 +110,7 @@ colsum_kernel(const float* __restrict__ x, const float* __restrict__ mask, float
       const size_t i = static_cast<size_t>(r) * cols + col;
       float v = x[i];
       if (mask) {
-        v = mask[i] > 0.f ? v : 0.f;
+        v = act_bwd(mode, v, mask[i]);
         dz[i] = v;
       }
       acc += v;
@@ -139,7 +161,7 @@ Colsum4Plan plan_colsum4(int rows, int cols) {
 __global__ void __launch_bounds__(256)
 colsum4_kernel(const float* __restrict__ x, const float* __restrict__ mask, float* __restrict__ dz,
                float* __restrict__ s, int rows, int cols, int rper, int rsplit, float* ws,
-               unsigned* counters) {
+               unsigned* counters, int mode) {
   const int cq = threadIdx.x & 15, rl = threadIdx.x >> 4;
   const int quad = blockIdx.x * 16 + cq;
   const int nq = cols / 4;
@@ -159,9 +181,7 @@ colsum4_kernel(const float* __restrict__ x, const float* __restrict__ mask, floa
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const size_t i = static_cast<size_t>(r + 16 * u) * nq + quad;
-          const float4 mk = __ldcs(m4 + i);
-          v[u].x = mk.x > 0.f ? v[u].x : 0.f; v[u].y = mk.y > 0.f ? v[u].y : 0.f;
-          v[u].z = mk.z > 0.f ? v[u].z : 0.f; v[u].w = mk.w > 0.f ? v[u].w : 0.f;
+          v[u] = act_bwd4(mode, v[u], __ldcs(m4 + i));
           d4[i] = v[u];
         }
       }
@@ -174,9 +194,7 @@ colsum4_kernel(const float* __restrict__ x, const float* __restrict__ mask, floa
       const size_t i = static_cast<size_t>(r) * nq + quad;
       float4 v = __ldcs(x4 + i);
       if (mask) {
-        const float4 mk = __ldcs(m4 + i);
-        v.x = mk.x > 0.f ? v.x : 0.f; v.y = mk.y > 0.f ? v.y : 0.f;
-        v.z = mk.z > 0.f ? v.z : 0.f; v.w = mk.w > 0.f ? v.w : 0.f;
+        v = act_bwd4(mode, v, __ldcs(m4 + i));
         d4[i] = v;
       }
       acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
@@ -514,15 +532,15 @@ unsigned grid_for(uint64_t work_items, uint64_t per_item_min, unsigned cap) {
 }  // namespace
 
 cudaError_t launch_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
-                            float* h, int rows, int cols, bool relu, cudaStream_t st) {
+                            float* h, int rows, int cols, int act, cudaStream_t st, float* pre) {
   const uint64_t total = static_cast<uint64_t>(rows) * cols;
   if (total == 0) return cudaSuccess;
   auto al = [](const void* p) { return p == nullptr || reinterpret_cast<uintptr_t>(p) % 16 == 0; };
-  const int vec = (cols % 4 == 0) && al(z) && al(b1) && al(b2) && al(b3) && al(h);
+  const int vec = (cols % 4 == 0) && al(z) && al(b1) && al(b2) && al(b3) && al(h) && al(pre);
   const unsigned blocks = grid_for(vec ? total / 4 : total, 256 * 4, 148 * 8);
   count_launch();
-  return launch_k(bias_act_kernel, dim3(blocks), dim3(256), 0, st, z, b1, b2, b3, h, rows, cols,
-                  relu ? 1 : 0, vec);
+  return launch_k(bias_act_kernel, dim3(blocks), dim3(256), 0, st, z, b1, b2, b3, h, pre, rows,
+                  cols, act, vec);
 }
 
 uint64_t colsum_ws_floats(int rows, int cols) {
@@ -536,14 +554,15 @@ uint64_t colsum_counter_slots(int rows, int cols) {
 }
 
 cudaError_t launch_colsum(const float* x, const float* mask, float* dz, float* s, int rows,
-                          int cols, float* ws, unsigned* counters, cudaStream_t st) {
+                          int cols, float* ws, unsigned* counters, cudaStream_t st, int mode) {
   if (cols <= 0) return cudaSuccess;
   auto al = [](const void* p) { return p == nullptr || reinterpret_cast<uintptr_t>(p) % 16 == 0; };
   if (cols % 4 == 0 && rows > 0 && al(x) && al(mask) && al(dz) && al(s) && al(ws)) {
     Colsum4Plan q = plan_colsum4(rows, cols);
     if (q.rsplit > 1 && (!ws || !counters)) return cudaErrorInvalidValue;
     dim3 grid(q.col_tiles, q.rsplit);
-    colsum4_kernel<<<grid, 256, 0, st>>>(x, mask, dz, s, rows, cols, q.rper, q.rsplit, ws, counters);
+    colsum4_kernel<<<grid, 256, 0, st>>>(x, mask, dz, s, rows, cols, q.rper, q.rsplit, ws, counters,
+                                         mode);
     count_launch();
     return cudaGetLastError();
   }
@@ -554,7 +573,7 @@ cudaError_t launch_colsum(const float* x, const float* mask, float* dz, float* s
   }
   if (p.rsplit > 1 && (!ws || !counters)) return cudaErrorInvalidValue;
   dim3 grid(p.col_tiles, p.rsplit);
-  colsum_kernel<<<grid, 256, 0, st>>>(x, mask, dz, s, rows, cols, p.rper, p.rsplit, ws, counters);
+  colsum_kernel<<<grid, 256, 0, st>>>(x, mask, dz, s, rows, cols, p.rper, p.rsplit, ws, counters, mode);
   count_launch();
   return cudaGetLastError();
 }

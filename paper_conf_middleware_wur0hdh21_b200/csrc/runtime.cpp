@@ -267,9 +267,16 @@ sf_status validate(const Graph& g) {
         break;
       }
       case SF_OP_BIAS_ACT: {
-        if ((s = chk(o.n_in >= 2 && o.n_in <= 4 && o.n_out == 1, SF_EINVAL, at + "bias_act arity"))) return s;
+        const bool gelu = o.flags & SF_ACT_GELU;
+        if ((s = chk(o.n_in >= 2 && o.n_in <= 4 && (o.n_out == 1 || (gelu && o.n_out == 2)), SF_EINVAL,
+                     at + "bias_act arity")))
+          return s;
+        if ((s = chk(!(gelu && (o.flags & SF_ACT_RELU)), SF_EINVAL, at + "one activation"))) return s;
         const Tensor &z = T(o.in[0]), &h = T(o.out[0]);
         if ((s = chk(z.rows == h.rows && z.cols == h.cols, SF_EINVAL, at + "bias_act shape"))) return s;
+        if (o.n_out == 2 && (s = chk(T(o.out[1]).rows == z.rows && T(o.out[1]).cols == z.cols, SF_EINVAL,
+                                     at + "bias_act pre-activation shape")))
+          return s;
         for (int i = 1; i < o.n_in; ++i)
           if ((s = chk(T(o.in[i]).rows == 1 && T(o.in[i]).cols == z.cols, SF_EINVAL, at + "bias shape")))
             return s;
@@ -575,7 +582,7 @@ int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
     L.K = A.cols; L.N = C.cols;
     int y = o.out[0], used = 1;
     if (i + 1 < e && g.ops[i + 1].type == SF_OP_BIAS_ACT && g.ops[i + 1].in[0] == o.out[0] &&
-        C.kind != SF_OUTPUT && readers(o.out[0]) == 1) {
+        !(g.ops[i + 1].flags & SF_ACT_GELU) && C.kind != SF_OUTPUT && readers(o.out[0]) == 1) {
       const sf_op_desc& ba = g.ops[i + 1];
       for (int q = 1; q < ba.n_in; ++q) L.b[q - 1] = c.f(ba.in[q]);
       L.relu = ba.flags & SF_ACT_RELU;
@@ -740,7 +747,8 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         // Fuse a following BIAS_ACT into the GEMV epilogue when the GEMM output has no other
         // reader (same arithmetic order as the unfused pair, so results are bit-identical).
         if (j + 1 < e && !ga.acc && g.ops[j + 1].type == SF_OP_BIAS_ACT && g.ops[j + 1].in[0] == o.out[0] &&
-            C.kind != SF_OUTPUT && sfk::gemm_can_fuse_bias(ga.M, ga.N, ga.K, ga.ta, ga.tb, ga.ldb)) {
+            !(g.ops[j + 1].flags & SF_ACT_GELU) && C.kind != SF_OUTPUT &&
+            sfk::gemm_can_fuse_bias(ga.M, ga.N, ga.K, ga.ta, ga.tb, ga.ldb)) {
           int readers = 0;
           for (const auto& q : g.ops)
             for (int t : op_reads(q)) readers += (t == o.out[0]);
@@ -763,13 +771,14 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         const Tensor& z = g.T[o.in[0]];
         err = sfk::launch_bias_act(c.f(o.in[0]), c.f(o.in[1]), o.n_in > 2 ? c.f(o.in[2]) : nullptr,
                                    o.n_in > 3 ? c.f(o.in[3]) : nullptr, c.f(o.out[0]), z.rows, z.cols,
-                                   o.flags & SF_ACT_RELU, c.st);
+                                   (o.flags & SF_ACT_GELU) ? 2 : (o.flags & SF_ACT_RELU) ? 1 : 0, c.st,
+                                   o.n_out > 1 ? c.f(o.out[1]) : nullptr);
         break;
       }
       case SF_OP_BIAS_ACT_BWD: {
         const Tensor& x = g.T[o.in[0]];
         err = sfk::launch_colsum(c.f(o.in[0]), c.f(o.in[1]), c.f(o.out[0]), c.f(o.out[1]), x.rows,
-                                 x.cols, c.b.ws, c.b.counters, c.st);
+                                 x.cols, c.b.ws, c.b.counters, c.st, (o.flags & SF_ACT_GELU) ? 2 : 1);
         break;
       }
       case SF_OP_COLSUM: {
@@ -2392,14 +2401,15 @@ sf_status sf_op_gemm_bias_act(const float* A, const float* B, float* C, int32_t 
 }
 
 sf_status sf_op_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
-                         float* h, int32_t rows, int32_t cols, int32_t relu, void* stream) {
+                         float* h, int32_t rows, int32_t cols, int32_t act, void* stream) {
   if (!z || !b1 || !h) return fail(SF_EINVAL, "bias_act args");
-  SF_CK(sfk::launch_bias_act(z, b1, b2, b3, h, rows, cols, relu != 0, as_stream(stream)));
+  if (act < 0 || act > SF_ACT_GELU) return fail(SF_EINVAL, "bias_act: act must be 0, RELU or GELU");
+  SF_CK(sfk::launch_bias_act(z, b1, b2, b3, h, rows, cols, act, as_stream(stream)));
   return SF_OK;
 }
 
 static sf_status colsum_common(const float* x, const float* mask, float* dz, float* s, int rows,
-                               int cols, cudaStream_t st) {
+                               int cols, cudaStream_t st, int mode = 1) {
   const uint64_t wsf = sfk::colsum_ws_floats(rows, cols);
   const uint64_t cs = sfk::colsum_counter_slots(rows, cols);
   void* ws = nullptr;
@@ -2410,7 +2420,7 @@ static sf_status colsum_common(const float* x, const float* mask, float* dz, flo
     SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
   }
   SF_CK(sfk::launch_colsum(x, mask, dz, s, rows, cols, static_cast<float*>(ws),
-                           static_cast<unsigned*>(cnt), st));
+                           static_cast<unsigned*>(cnt), st, mode));
   if (ws) {
     SF_CK(cudaFreeAsync(ws, st));
     SF_CK(cudaFreeAsync(cnt, st));
@@ -2422,6 +2432,12 @@ sf_status sf_op_bias_act_bwd(const float* dh, const float* h, float* dz, float* 
                              int32_t cols, void* stream) {
   if (!dh || !h || !dz || !db) return fail(SF_EINVAL, "bias_act_bwd args");
   return colsum_common(dh, h, dz, db, rows, cols, as_stream(stream));
+}
+
+sf_status sf_op_gelu_bwd(const float* dh, const float* u, float* dz, float* db, int32_t rows,
+                         int32_t cols, void* stream) {
+  if (!dh || !u || !dz || !db) return fail(SF_EINVAL, "gelu_bwd args");
+  return colsum_common(dh, u, dz, db, rows, cols, as_stream(stream), 2);
 }
 
 sf_status sf_op_colsum(const float* x, float* s, int32_t rows, int32_t cols, void* stream) {

@@ -94,10 +94,14 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
 // Elementwise / reduction ops (deterministic).  ws / counters sized by *_ws().
 uint64_t colsum_ws_floats(int rows, int cols);
 uint64_t colsum_counter_slots(int rows, int cols);
+// act: 0 identity, 1 ReLU, 2 GELU; pre (optional): u = z + biases
 cudaError_t launch_bias_act(const float* z, const float* b1, const float* b2, const float* b3,
-                            float* h, int rows, int cols, bool relu, cudaStream_t st);
+                            float* h, int rows, int cols, int act, cudaStream_t st,
+                            float* pre = nullptr);
+// s = colsum(dz); with a mask operand dz = act'(mask) * x: mode 1 ReLU (mask = h > 0),
+// mode 2 GELU (mask = u)
 cudaError_t launch_colsum(const float* x, const float* h_mask, float* dz, float* s, int rows,
-                          int cols, float* ws, unsigned* counters, cudaStream_t st);
+                          int cols, float* ws, unsigned* counters, cudaStream_t st, int mode = 1);
 uint64_t softmax_ce_ws_floats(int rows);
 cudaError_t launch_softmax_ce(const float* logits, const int32_t* labels, float* loss,
                               float* dlogits, int rows, int cols, float* ws, unsigned* counter,

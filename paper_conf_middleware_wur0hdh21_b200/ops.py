@@ -63,11 +63,18 @@ def mlp_chain(x: torch.Tensor, Ws: Sequence[torch.Tensor], bs: Sequence[Optional
           "sf_op_mlp_chain")
 
 
-def bias_act(z, biases: Sequence[torch.Tensor], h, relu: bool, stream=None) -> None:
+def bias_act(z, biases: Sequence[torch.Tensor], h, relu, stream=None) -> None:
+    """relu: False / True, or the act code (0 identity, 1 ReLU, 2 GELU)."""
     bs = list(biases) + [None] * (3 - len(biases))
     _need_cuda(z, h, *bs)
     check(lib().sf_op_bias_act(_p(z), _p(bs[0]), _p(bs[1]), _p(bs[2]), _p(h), z.shape[0], z.shape[1],
                                int(relu), _s(stream)), "sf_op_bias_act")
+
+
+def gelu_bwd(dh, u, dz, db, stream=None) -> None:
+    _need_cuda(dh, u, dz, db)
+    check(lib().sf_op_gelu_bwd(_p(dh), _p(u), _p(dz), _p(db), dh.shape[0], dh.shape[1],
+                               _s(stream)), "sf_op_gelu_bwd")
 
 
 def bias_act_bwd(dh, h, dz, db, stream=None) -> None:

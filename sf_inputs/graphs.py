@@ -20,7 +20,7 @@ from __future__ import annotations
 
 from typing import List, Sequence, Tuple
 
-from .ir import (ACC, ADAM, BIAS_ACT, BIAS_ACT_BWD, COLSUM, DATASET, F32, FEED, GEMM,
+from .ir import (ACC, ADAM, BIAS_ACT, BIAS_ACT_BWD, COLSUM, DATASET, F32, FEED, GELU, GEMM,
                  GRAD, I32, INPUT, LABEL, OUTPUT, PARAM, RELU, SCALAR_STATE, SGD_MOM,
                  SLOT, SOFTMAX, SOFTMAX_CE, STEP_INC, TA, TB, ACT, Graph)
 
@@ -36,8 +36,11 @@ ADAM_EPS = 1e-8
 # C1: MLP training graph (generalised to any widths for tiny test graphs)
 # ---------------------------------------------------------------------------------
 def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int = 16,
-              lr: float = SGD_LR, mu: float = SGD_MU, name: str = "mlp") -> Graph:
-    """Training graph of an MLP with ReLU hidden layers and softmax-CE loss.
+              lr: float = SGD_LR, mu: float = SGD_MU, name: str = "mlp",
+              act: str = "relu") -> Graph:
+    """Training graph of an MLP with ReLU (or GELU: ``act="gelu"``) hidden layers and
+    softmax-CE loss.  A GELU layer's BIAS_ACT also writes its pre-activation u_i, which
+    its BIAS_ACT_BWD reads.
 
     For widths (784, 256, 10) this is exactly SURVEY.md 8(c) step 1 (o1..o11) with
     FEED ops for x, y in front (data cursor = step, reading Q3/Q11) and STEP_INC
@@ -64,6 +67,8 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
     # forward
     h_prev = x
     hs: List[int] = []
+    us: List[int] = []
+    gelu = act == "gelu"
     for i in range(L):
         ph = i
         if i == 0:
@@ -73,7 +78,13 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
         g.op(GEMM, [h_prev, W[i]], [z], phase=ph)
         last = i == L - 1
         h = g.add("logits" if last else f"h{i+1}", batch, widths[i + 1], F32, ACT)
-        g.op(BIAS_ACT, [z, b[i]], [h], flags=0 if last else RELU, phase=ph)
+        if gelu and not last:
+            u = g.add(f"u{i+1}", batch, widths[i + 1], F32, ACT)
+            g.op(BIAS_ACT, [z, b[i]], [h, u], flags=GELU, phase=ph)
+            us.append(u)
+        else:
+            g.op(BIAS_ACT, [z, b[i]], [h], flags=0 if last else RELU, phase=ph)
+            us.append(h)
         hs.append(h)
         h_prev = h
     loss = g.add("loss", 1, 1, F32, OUTPUT)
@@ -95,7 +106,7 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
         else:
             dz = g.add(f"dz{i+1}", batch, widths[i + 1], F32, GRAD)
             dbi = g.add(f"db{i+1}", 1, widths[i + 1], F32, GRAD)
-            g.op(BIAS_ACT_BWD, [d_out, hs[i]], [dz, dbi], phase=ph)
+            g.op(BIAS_ACT_BWD, [d_out, us[i]], [dz, dbi], flags=GELU if gelu else 0, phase=ph)
             dWi = g.add(f"dW{i+1}", widths[i], widths[i + 1], F32, GRAD)
             g.op(GEMM, [inp, dz], [dWi], flags=TA, phase=ph)
             d_out = dz
@@ -264,8 +275,11 @@ def resnet50_forest(batch: int = 8, spatial_div: int = 1, lr: float = SGD_LR,
 def bert_chain(layers: int = 24, hidden: int = 1024, inter: int = 4096, vocab: int = 30522,
                tokens: int = 512, positions: int = 512, lr: float = ADAM_LR,
                b1: float = ADAM_B1, b2: float = ADAM_B2, eps: float = ADAM_EPS,
-               name: str = "bert_chain") -> Graph:
+               name: str = "bert_chain", act: str = "relu") -> Graph:
     """BERT-large variables (391 tensors, 335,141,888 params at defaults) + Adam.
+
+    ``act="gelu"``: the FFN intermediate Linear uses GELU (where BERT has it; its
+    pre-activation is kept for the backward), the other Linears stay ReLU.
 
     Compute (reading Q16): x0 = pos[:tokens] + embLN_gamma + embLN_beta (requires
     tokens == positions); per layer six Linear+ReLU (q, k, v, o with LN1 gamma/beta as
@@ -326,8 +340,13 @@ def bert_chain(layers: int = 24, hidden: int = 1024, inter: int = 4096, vocab: i
             if nm == "out":
                 bs += [L[l]["g2"], L[l]["be2"]]
             hn = g.add(f"l{l}_{nm}_h", tokens, kout, F32, ACT)
-            g.op(BIAS_ACT, [z] + bs, [hn], flags=RELU, phase=l)
-            rec.append((h, hn, L[l]["W" + nm], bs))
+            if act == "gelu" and nm == "i":
+                u = g.add(f"l{l}_{nm}_u", tokens, kout, F32, ACT)
+                g.op(BIAS_ACT, [z] + bs, [hn, u], flags=GELU, phase=l)
+                rec.append((h, u, L[l]["W" + nm], bs, GELU))
+            else:
+                g.op(BIAS_ACT, [z] + bs, [hn], flags=RELU, phase=l)
+                rec.append((h, hn, L[l]["W" + nm], bs, 0))
             h = hn
         acts.append(rec)
     ph = layers
@@ -361,11 +380,11 @@ def bert_chain(layers: int = 24, hidden: int = 1024, inter: int = 4096, vocab: i
         ph = layers + 2 + (layers - 1 - l)
         for j in range(len(lin_names) - 1, -1, -1):
             nm = lin_names[j]
-            inp, out, Wt, bs = acts[l][j]
+            inp, out, Wt, bs, fl = acts[l][j]
             kin, kout = dims[nm]
             dz = g.add(f"l{l}_{nm}_dz", tokens, kout, F32, GRAD)
             gb = g.add(f"l{l}_{nm}_bias_grad", 1, kout, F32, GRAD)
-            g.op(BIAS_ACT_BWD, [dh, out], [dz, gb], phase=ph)
+            g.op(BIAS_ACT_BWD, [dh, out], [dz, gb], flags=fl, phase=ph)
             for bt in bs:
                 grads[bt] = gb  # additive biases share the column-sum gradient
             gW = g.add(f"l{l}_{nm}_kernel_grad", kin, kout, F32, GRAD)

@@ -43,8 +43,8 @@ PERSISTENT_KINDS = (PARAM, SLOT, SCALAR_STATE)
 
 # ---- op types (include/sf.h: sf_op_type) --------------------------------------
 GEMM = 1          # ins [A, B]; outs [C]; flags TA|TB|ACC
-BIAS_ACT = 2      # ins [z, b1, (b2), (b3)]; outs [h]; flags RELU
-BIAS_ACT_BWD = 3  # ins [dh, h]; outs [dz, db]   (ReLU backward + bias grad)
+BIAS_ACT = 2      # ins [z, b1, (b2), (b3)]; outs [h] (GELU: [h, u]); flags RELU | GELU
+BIAS_ACT_BWD = 3  # ins [dh, h] (GELU: [dh, u]); outs [dz, db]   (act backward + bias grad)
 COLSUM = 4        # ins [x]; outs [s]
 SOFTMAX_CE = 5    # ins [logits, labels]; outs [loss, dlogits]
 SOFTMAX = 6       # ins [logits]; outs [probs]
@@ -62,6 +62,7 @@ TB = 2
 ACC = 4
 # BIAS_ACT flags
 RELU = 1
+GELU = 2          # BIAS_ACT / BIAS_ACT_BWD flag: exact-erf GELU
 
 
 @dataclass

@@ -65,6 +65,7 @@ def test_enum_values_match_workload_codes():
     defs = dict(re.findall(r"#define\s+(SF_\w+)\s+\(?(-?\d+)\)?", src))
     assert int(defs["SF_GEMM_TA"]) == ir.TA and int(defs["SF_GEMM_TB"]) == ir.TB
     assert int(defs["SF_GEMM_ACC"]) == ir.ACC and int(defs["SF_ACT_RELU"]) == ir.RELU
+    assert int(defs["SF_ACT_GELU"]) == ir.GELU
 
 
 def test_struct_layouts_match_c(built):

@@ -243,6 +243,25 @@ def test_gemm_plain_tf32_would_fail_the_bar(ops):
 
 
 # ---- elementwise / reductions -------------------------------------------------------------
+@pytest.mark.parametrize("rows,cols,nb", [(64, 256, 1), (512, 4096, 2), (5, 7, 3), (1001, 64, 1)])
+def test_bias_gelu_and_backward(ops, rows, cols, nb):
+    """GELU: erff/expf kernels vs the fp64 oracle at 1e-4."""
+    rng = np.random.default_rng(rows + 3 * cols)
+    z = (rng.standard_normal((rows, cols)) * 2).astype(np.float32)
+    bs = [rng.standard_normal((1, cols)).astype(np.float32) for _ in range(nb)]
+    h = torch.empty(rows, cols, device="cuda")
+    ops.bias_act(cu(z), [cu(b) for b in bs], h, 2)
+    rh, ru = O.bias_gelu(z, bs)
+    assert rel(h.cpu().numpy(), rh) <= TOL
+    dh = rng.standard_normal((rows, cols)).astype(np.float32)
+    dz = torch.empty(rows, cols, device="cuda")
+    db = torch.empty(1, cols, device="cuda")
+    ops.gelu_bwd(cu(dh), cu(ru), dz, db)
+    rdz, rdb = O.gelu_bwd(dh, ru)
+    assert rel(dz.cpu().numpy(), rdz) <= TOL
+    assert rel(db.cpu().numpy(), rdb) <= TOL
+
+
 @pytest.mark.parametrize("rows,cols,nb,relu", [(64, 256, 1, True), (64, 10, 1, False),
                                                 (1001, 64, 3, False), (5, 7, 2, True)])
 def test_bias_act(ops, rows, cols, nb, relu):

@@ -306,13 +306,15 @@ def test_live_sets_match_oracle(P, U):
     rt.close()
 
 
-def _bert_mini():
-    return G.bert_chain(layers=2, hidden=64, inter=128, vocab=301, tokens=32, positions=32)
+def _bert_mini(act="relu"):
+    return G.bert_chain(layers=2, hidden=64, inter=128, vocab=301, tokens=32, positions=32, act=act)
 
 
-def test_c3_mini_vs_oracle_and_mid_cut_bitwise(P):
-    """BERT-shaped chain with Adam (misaligned vocab 301 -> padded GEMM operands)."""
-    g = _bert_mini()
+@pytest.mark.parametrize("act", ["relu", "gelu"])
+def test_c3_mini_vs_oracle_and_mid_cut_bitwise(P, act):
+    """BERT-shaped chain with Adam (misaligned vocab 301 -> padded GEMM operands); with
+    act="gelu" the FFN intermediate is GELU."""
+    g = _bert_mini(act)
     st, ds = D.init_state(g), D.datasets(g)
     base, bo, _, _, _ = run_gpu(P, g, 3)
     ref = R.run(g, 3, st, ds, keep_stagings=False)
@@ -601,4 +603,28 @@ def test_ce_migration_host_and_peer_bitwise(P, W):
     got, _, info, _, _ = run_gpu(P, gr, 3, schedule=sched, poison=True,
                                  migration_engine=A.SF_MIG_CE)
     assert info["n_preemptions"] >= 4
+    assert_bitwise(base, got)
+
+
+# ---- GELU layers ----------------------------------------------------
+
+def test_gelu_mlp_trajectory_vs_oracle_and_preempted_bitwise(P):
+    """A GELU MLP (u_i kept for the backward, so it is live across the cuts between the
+    layer's forward and its backward): 20 iterations vs the oracle at 1e-4, and preempted at
+    every cut (host + peer, poisoned arenas) bit-identical to the unpreempted GPU run."""
+    g = G.mlp_train(act="gelu")
+    st, ds = D.init_state(g), D.datasets(g)
+    got, outs, _, _, _ = run_gpu(P, g, 20)
+    ref = R.run(g, 20, st, ds, keep_stagings=False)
+    for i in ref.state:
+        if ref.state[i].dtype == np.float32:
+            assert rel(got[i], ref.state[i]) <= TOL, g.tensors[i].name
+    assert rel(outs["loss"], ref.outputs[-1]["loss"]) <= TOL
+    n = len(OG.partition(g))
+    u1 = g.tid("u1")
+    assert any(u1 in OG.live_set(g, OG.partition(g), k) for k in range(n))
+    sched = sorted([(5, k, HOST) for k in range(n)] + [(8, k, 1 - (k % 2)) for k in range(1, n)])
+    base, _, _, _, _ = run_gpu(P, g, 12)
+    got, _, info, _, _ = run_gpu(P, g, 12, schedule=sched, poison=True)
+    assert info["n_preemptions"] >= 8
     assert_bitwise(base, got)

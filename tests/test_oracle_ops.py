@@ -13,6 +13,9 @@
       w_t = w_0 - sum_{s=1..t} lr g sqrt(1-b2^s) / (|g| sqrt(1-b2^s) + eps);
   g = 0 leaves w bitwise unchanged.
 - ReLU backward at h = 0 passes no gradient (reading Q10, TF ReluGrad).
+- GELU (exact erf form): torch.nn.functional.gelu(approximate="none") in fp64 and its
+  autograd derivative; identities gelu(0) = 0, gelu(u) - gelu(-u) = u (Phi(u) + Phi(-u)
+  = 1), gelu'(0) = 1/2; the whole-MLP finite differences run with GELU layers too.
 """
 import math
 
@@ -108,9 +111,10 @@ def _fwd_bwd(g, T, parts, exact=True, with_bwd=True):
             O.apply_op(op, T, shapes, exact)
 
 
+@pytest.mark.parametrize("act", ["relu", "gelu"])
 @pytest.mark.parametrize("widths,batch", [((2, 3, 2), 4), ((5, 7, 3), 6), ((4, 6, 5, 3), 5)])
-def test_finite_difference_whole_mlp(widths, batch):
-    g = G.mlp_train(widths, batch=batch, pool=1)
+def test_finite_difference_whole_mlp(widths, batch, act):
+    g = G.mlp_train(widths, batch=batch, pool=1, act=act)
     OG.validate(g)
     parts = OG.partition(g)
     st = D.init_state(g, seed=21)
@@ -192,3 +196,26 @@ def test_feed_cycles_through_pool():
     assert O.feed(pool, np.array([[0]]), 2).tolist() == [[0, 1], [2, 3]]
     assert O.feed(pool, np.array([[4]]), 2).tolist() == [[4.0, 5.0], [6.0, 7.0]]
     assert O.feed(pool, np.array([[5]]), 2).tolist() == [[8.0, 9.0], [10.0, 11.0]]
+
+
+def test_gelu_vs_torch_and_identities():
+    rng = np.random.default_rng(8)
+    u = (rng.standard_normal((7, 11)) * 3).astype(np.float32)
+    ut = torch.tensor(u, dtype=torch.float64, requires_grad=True)
+    ref = torch.nn.functional.gelu(ut, approximate="none")
+    h = O.gelu(u)
+    np.testing.assert_allclose(h, ref.detach().numpy(), rtol=1e-6, atol=1e-7)
+    assert np.array_equal(h, ref.detach().numpy().astype(np.float32))  # one rounding
+    dh = rng.standard_normal((7, 11)).astype(np.float32)
+    ref.backward(torch.tensor(dh, dtype=torch.float64))
+    dz, db = O.gelu_bwd(dh, u)
+    np.testing.assert_allclose(dz, ut.grad.numpy(), rtol=1e-6, atol=1e-7)
+    np.testing.assert_allclose(db[0], ut.grad.numpy().sum(axis=0), rtol=1e-6, atol=1e-6)
+    x = np.linspace(-6, 6, 101)
+    e = O.gelu(x, exact=True) - O.gelu(-x, exact=True)
+    np.testing.assert_allclose(e, x, atol=1e-14)
+    assert O.gelu(np.zeros((1, 1)), exact=True)[0, 0] == 0.0
+    d0, _ = O.gelu_bwd(np.ones((1, 1)), np.zeros((1, 1)), exact=True)
+    assert d0[0, 0] == 0.5
+    h, uu = O.bias_gelu(np.zeros((2, 3), np.float32), [np.full((1, 3), 10.0, np.float32)])
+    assert np.all(uu == 10.0) and np.all(h == 10.0)
