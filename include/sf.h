@@ -175,6 +175,11 @@ typedef struct sf_config {
                                     queued inference, no present job of priority >= its own);
                                     0 (paper): it stays on the target */
   int32_t migration_engine;      /* SF_MIG_SM (default) or SF_MIG_CE */
+  int32_t host_stage_inline;     /* 1: a job's host input stage runs on its driver thread while
+                                    the job holds the device (with iteration_granularity = 1:
+                                    session-based time slicing, the Gandiva-like baseline of
+                                    PAPER.md:1385-1392); 0: feeds prefetch on their own thread
+                                    (CPU executors scheduled freely) */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,
@@ -342,6 +347,56 @@ sf_status sf_import_arena(sf_runtime* rt, sf_graph_id g, int32_t slot, const sf_
 sf_status sf_adopt_job(sf_runtime* rt, sf_graph_id g, int32_t dev, int64_t iters, int64_t iter,
                        int32_t k, int32_t auto_target, sf_job_id* out);
 
+/* ---- host input stages: interleaving and input reuse ------
+ * The paper's CPU executor (data loading + preprocessing) of a job: "executors
+ * on different devices can be scheduled freely ... any CPU executor [may] run while a GPU is
+ * occupied", overlapping one job's preprocessing with another job's GPU subgraphs.  A feed runs
+ * a host stage callback that writes iteration `iter`'s fed tensors (INPUT / LABEL tensors no op
+ * writes) into pinned buffers, prefetching up to `depth` iterations on a runtime thread that
+ * never holds a device.  At S_0 of each iteration the job copies them into its arena on its
+ * training stream (they then migrate like any in-flight tensor).
+ * Shared feed (input reuse, Fig. 5): one host stage feeds several graphs;
+ * each batch is copied once into an immutable device buffer ("an immutable copy of the tensor in
+ * GPU global memory ... public to all GPU executors sharing the tensor") and the members run
+ * their iterations in lockstep round-robin (member 0's iteration i, member 1's iteration i,
+ * ..., then batch i+1).  Members are the graphs attached to the feed, in attach order; they
+ * must run the same number of iterations and start at iteration 0. */
+typedef uint32_t sf_feed_id;
+/* Host stage: fill dst[i] (pinned host, bytes[i] bytes) for iteration `iter`; return 0 on
+ * success (non-zero fails the job).  Called from one runtime thread at a time per feed. */
+typedef int32_t (*sf_host_stage_fn)(void* user, int64_t iter, void* const* dst,
+                                    const uint64_t* bytes, int32_t n);
+typedef struct sf_feed_desc {
+  sf_host_stage_fn fn;
+  void* user;              /* passed to fn; caller-owned, valid until sf_destroy */
+  int32_t n;               /* fed tensors per iteration, 1..8 */
+  const uint64_t* bytes;   /* host [n], copied */
+  int32_t depth;           /* prefetch ring slots 1..8 (0 -> 2) */
+  int32_t shared;          /* 1: input-reuse group (immutable device copy, lockstep members) */
+  int32_t dev;             /* shared: slot whose device holds the immutable copy */
+  int32_t pad;
+} sf_feed_desc;
+sf_status sf_create_feed(sf_runtime* rt, const sf_feed_desc* d, sf_feed_id* out);
+/* Feed graph g's tensors tensor_ids[0..n) (host array; INPUT / LABEL tensors no op writes, byte
+ * sizes equal to the feed's) from feed f.  Before sf_start_training; a non-shared feed takes one
+ * graph.  SF_EINVAL on size / kind mismatch. */
+sf_status sf_attach_feed(sf_runtime* rt, sf_graph_id g, sf_feed_id f, const uint32_t* tensor_ids);
+
+/* Built-in host stage (synthetic image pipeline, reading Q27): batch b = iter mod P of
+ * a u8 image pool [P * batch][cols] is decoded to fp32 x = u8 / 255 with a seeded horizontal
+ * flip per sample (row r of the pool flips when the low bit of the (r+1)-th splitmix64 output of
+ * `seed` is set; images are img_w pixels wide), labels copied; dst = {x [batch][cols] f32,
+ * y [batch][1] i32}.  user = const sf_u8_stage*. */
+typedef struct sf_u8_stage {
+  const uint8_t* images;   /* host [pool_rows][cols] */
+  const int32_t* labels;   /* host [pool_rows] */
+  int64_t pool_rows;       /* multiple of batch */
+  int32_t batch, cols, img_w;
+  uint32_t seed;
+} sf_u8_stage;
+int32_t sf_stage_u8_normalize(void* user, int64_t iter, void* const* dst, const uint64_t* bytes,
+                              int32_t n);
+
 /* ---- inference (the preempter) --------------------------------------------------- */
 typedef struct sf_timing {
   uint64_t arrival_ns;   /* scheduled arrival (CLOCK_MONOTONIC) */
@@ -366,7 +421,9 @@ sf_status sf_submit_inference(sf_runtime* rt, sf_graph_id g, int32_t dev, const 
 sf_status sf_wait(sf_runtime* rt, sf_req_id req, int64_t timeout_ns, sf_timing* timing);
 
 /* ---- trace (schedule invariants; oracle/schedule.py checks it) ------------------- */
-enum sf_event_kind { SF_EV_TRAIN = 0, SF_EV_INFER = 1, SF_EV_MIGRATE = 2 };
+enum sf_event_kind { SF_EV_TRAIN = 0, SF_EV_INFER = 1, SF_EV_MIGRATE = 2,
+                     SF_EV_HOST = 3 /* host stage of a feed: dev = -1 - feed id (prefetch
+                                       thread) or the job's slot (inline), k = -1 */ };
 typedef struct sf_trace_event {
   int32_t dev, job, kind, k;   /* job: training job id, or 1<<20 | request for inference */
   int64_t iter;

@@ -11,6 +11,7 @@ rounding to fp32 per op output) of what the B200 hot path computes:
 * runner.py    — sequential execution of the partitioned graph for T iterations
                  under a preemption schedule with simulated devices whose arenas are
                  poisoned before unpack; batch-1 inference.
+* feed.py      — the workload's host input stage (u8 image decode + seeded flip).
 * schedule.py  — discrete-event schedule simulation and the invariant checker
                  (no two models' subgraphs overlap on a device; per-job order; stop
                  latency bounded by the in-flight subgraph).

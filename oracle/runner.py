@@ -24,7 +24,7 @@ cut k of several iterations (tiny MLPs, C1, a C2 prefix); GPU-free trajectory sa
 from __future__ import annotations
 
 from dataclasses import dataclass, field
-from typing import Dict, List, Optional, Sequence, Tuple
+from typing import Callable, Dict, List, Optional, Sequence, Tuple
 
 import numpy as np
 
@@ -65,9 +65,13 @@ def run(g: Graph, iters: int, state0: Dict[int, np.ndarray], data: Dict[int, np.
         schedule: Sequence[Tuple[int, int, int]] = (), parts=None, n_devices: int = 2,
         home: int = 0, exact: bool = False, keep_stagings: bool = True,
         omit: Sequence[int] = (),
-        inference: Optional[Tuple[Graph, Dict[int, np.ndarray], np.ndarray]] = None
+        inference: Optional[Tuple[Graph, Dict[int, np.ndarray], np.ndarray]] = None,
+        feeds: Optional[Callable[[int], Dict[int, np.ndarray]]] = None
         ) -> Trajectory:
     """Run ``iters`` iterations; ``schedule`` = [(iter, k, target)] cuts (target or HOST).
+
+    ``feeds(it)`` -> {tensor id: array}: externally fed INPUT / LABEL tensors written
+    into the current device at the start of S_0 of iteration ``it`` (host input stage).
 
     ``omit`` drops tensor ids from every migrated live set (minimality pin only).
     """
@@ -108,6 +112,9 @@ def run(g: Graph, iters: int, state0: Dict[int, np.ndarray], data: Dict[int, np.
                 for i, arr in got.items():
                     devs[dst][i] = arr.astype(np.float64) if exact and arr.dtype == np.float32 else arr
                 cur = dst
+            if k == 0 and feeds is not None:
+                for i, arr in feeds(it).items():
+                    devs[cur][i] = np.array(arr, copy=True)
             for j in range(a, b):
                 O.apply_op(g.ops[j], devs[cur], shapes, exact)
             tr.trace.append((cur, it, k))

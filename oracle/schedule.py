@@ -136,6 +136,26 @@ def check_priority(events: Sequence[dict], prio: Dict[int, int],
                                  f"submission > {window} x {longest} + {slack}")
 
 
+def check_lockstep(events: Sequence[dict], members: Sequence[int]) -> None:
+    """I6, input reuse ("all models should finish processing an input
+    tensor before moving onto the next input batch ... each model's GPU executor in a
+    round-robin manner"): ordered by start time, the training subgraphs of the member jobs
+    form contiguous blocks (iteration i of member m) in the order (i, m) = (0, 0), (0, 1),
+    ..., (1, 0), ... — a member absent from the tail (it finished) is skipped."""
+    order = {j: m for m, j in enumerate(members)}
+    ev = sorted((e for e in events if e["kind"] == "train" and e["job"] in order),
+                key=lambda e: e["t0"])
+    blocks = []
+    for e in ev:
+        key = (e["iter"], order[e["job"]])
+        if not blocks or blocks[-1] != key:
+            blocks.append(key)
+    if len(set(blocks)) != len(blocks):
+        raise InvariantError(f"lockstep: a (iteration, member) block is split: {blocks}")
+    if blocks != sorted(blocks):
+        raise InvariantError(f"lockstep: blocks out of round-robin order: {blocks}")
+
+
 def check_all(events: Sequence[dict], n_sub: Dict[int, int], slack: float = 0.0) -> None:
     check_no_corun(events)
     check_job_order(events, n_sub)

@@ -28,7 +28,7 @@ SF_PART_PER_LAYER_PHASE = 0
 SF_PART_MAX_OPS = 1
 JOB_STATES = {0: "running", 1: "stopping", 2: "migrating", 3: "preempted", 4: "done", 5: "failed",
               6: "migrated_out"}
-EV_TRAIN, EV_INFER, EV_MIGRATE = 0, 1, 2
+EV_TRAIN, EV_INFER, EV_MIGRATE, EV_HOST = 0, 1, 2, 3
 INFER_JOB_FLAG = 1 << 20
 
 
@@ -56,7 +56,7 @@ class sf_config(C.Structure):
                 ("max_inflight", C.c_int32), ("defer_migration", C.c_int32),
                 ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
                 ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32),
-                ("migration_engine", C.c_int32)]
+                ("migration_engine", C.c_int32), ("host_stage_inline", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):
@@ -105,6 +105,18 @@ class sf_ipc_arena(C.Structure):
                 ("cuda_ordinal", C.c_int32), ("pad", C.c_int32)]
 
 
+class sf_feed_desc(C.Structure):
+    _fields_ = [("fn", C.c_void_p), ("user", C.c_void_p), ("n", C.c_int32),
+                ("bytes", C.POINTER(C.c_uint64)), ("depth", C.c_int32), ("shared", C.c_int32),
+                ("dev", C.c_int32), ("pad", C.c_int32)]
+
+
+class sf_u8_stage(C.Structure):
+    _fields_ = [("images", C.c_void_p), ("labels", C.c_void_p), ("pool_rows", C.c_int64),
+                ("batch", C.c_int32), ("cols", C.c_int32), ("img_w", C.c_int32),
+                ("seed", C.c_uint32)]
+
+
 class sf_copy_desc(C.Structure):
     _fields_ = [("src", C.c_void_p), ("dst", C.c_void_p), ("nbytes", C.c_uint64),
                 ("span", C.c_uint64)]
@@ -136,6 +148,9 @@ PROTOTYPES = {
     "sf_adopt_job": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int64, C.c_int64, C.c_int32, C.c_int32,
                            _P(C.c_uint32)]),
     "sf_resume": (_st, [_vp, C.c_uint32, C.c_int32]),
+    "sf_create_feed": (_st, [_vp, _P(sf_feed_desc), _P(C.c_uint32)]),
+    "sf_attach_feed": (_st, [_vp, C.c_uint32, C.c_uint32, _P(C.c_uint32)]),
+    "sf_stage_u8_normalize": (C.c_int32, [_vp, C.c_int64, _P(_vp), _P(C.c_uint64), C.c_int32]),
     "sf_job_query": (_st, [_vp, C.c_uint32, _P(sf_job_info)]),
     "sf_wait_job": (_st, [_vp, C.c_uint32, C.c_int64]),
     "sf_stop_job": (_st, [_vp, C.c_uint32]),

@@ -12,6 +12,8 @@
 //  * invariant 1: no co-running GPU executors .......... PAPER.md:794-806 (s.3.4)
 //  * preempter starts immediately after submission ..... PAPER.md:808-814 (s.3.4)
 //  * atomic-flag executor sync, 1-LOC priority ......... PAPER.md:904-909, 920-923 (s.4)
+//  * CPU executors scheduled freely (host feeds) ....... PAPER.md:816-826 (s.3.4)
+//  * input reuse: immutable shared copy, lockstep ...... PAPER.md:828-896 (s.3.4, Fig. 5)
 // B200 choices are described in DESIGN.md: cut at subgraph boundaries with in-flight
 // activations (reading Q1), one multi-tensor pack / unpack / peer-store launch per cut,
 // stream-ordered resume of a pre-instantiated CUDA graph on the target.
@@ -112,8 +114,13 @@ struct Binding {
   std::vector<void*> dev_allocs;
 };
 
+struct Feed;
+
 struct Graph {
   std::string name;
+  Feed* feed = nullptr;              // host input stage feeding this graph (sf_attach_feed)
+  std::vector<uint32_t> feed_tids;   // fed tensor of each feed buffer
+  int feed_member = -1;              // shared feed: member index (attach order)
   int priority = 0;
   std::vector<Tensor> T;
   std::vector<sf_op_desc> ops;
@@ -202,6 +209,35 @@ struct Job {
   std::vector<cudaEvent_t> ev_ck;    // [slot * 2 + i]: host-tier copy chunks in flight
 };
 
+// Host input stage (sf_create_feed).  Ring slot s holds iteration slot_iter[s]; states:
+// 0 free, 1 being filled, 2 ready (pinned host bytes, shared: also the immutable device copy).
+// A slot returns to free once every consumer's S_0 (which copies it into the arena) retired.
+struct Feed {
+  sf_feed_id id = 0;
+  sf_host_stage_fn fn = nullptr;
+  void* user = nullptr;
+  int n = 0, depth = 2, dev = -1;
+  bool shared = false;
+  std::vector<uint64_t> bytes, off;  // per fed buffer: size, offset inside a ring slot
+  uint64_t stride = 0;
+  uint8_t* host = nullptr;   // pinned [depth][stride]
+  uint8_t* dbuf = nullptr;   // shared: device [depth][stride], the immutable copies
+  cudaStream_t st = nullptr;
+  cudaEvent_t ev = nullptr;
+  std::vector<int64_t> slot_iter;
+  std::vector<int> slot_state;
+  std::vector<uint32_t> consumed;  // shared: bit m = member m copied the slot (S_0 retired)
+  std::vector<Graph*> members;
+  std::vector<Job*> member_jobs;
+  int64_t next_iter = 0;
+  bool active = false, inline_mode = false, failed = false;
+  std::string error;
+  int64_t turn_it = 0;  // shared: lockstep cursor (iteration, member)
+  int turn_m = 0;
+  uint64_t gen = 0;     // bumped when a job (re)starts the feed: stale fills are discarded
+  std::thread stager;
+};
+
 }  // namespace
 
 struct sf_runtime {
@@ -209,6 +245,7 @@ struct sf_runtime {
   std::vector<std::unique_ptr<Slot>> slots;
   std::vector<std::unique_ptr<Graph>> graphs;
   std::vector<std::unique_ptr<Job>> jobs;
+  std::vector<std::unique_ptr<Feed>> feeds;
   std::unordered_map<sf_req_id, std::unique_ptr<Request>> reqs;
   sf_req_id next_req = 1;
   std::mutex m;
@@ -1301,6 +1338,106 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
   return SF_OK;
 }
 
+// ---- host feeds (rt->m held) -----------------------------------------------------------
+// A shared-feed member takes part in the lockstep until its job finished; a member whose job
+// has not started yet is waited for.
+bool member_active(const Feed& F, int m) {
+  const Job* j = F.member_jobs[m];
+  if (!j) return true;
+  if (j->state == SF_JOB_DONE || j->state == SF_JOB_FAILED || j->state == SF_JOB_MIGRATED_OUT) return false;
+  return !(j->k == 0 && (j->it >= j->iters || j->stop_req));
+}
+// Shared slots whose batch every active member has copied become free for the next batch.
+void feed_release_drained(Feed& F) {
+  if (!F.shared) return;
+  const uint32_t all = F.members.size() >= 32 ? ~0u : (1u << F.members.size()) - 1;
+  uint32_t inactive = 0;
+  for (size_t m = 0; m < F.members.size(); ++m)
+    if (!member_active(F, static_cast<int>(m))) inactive |= 1u << m;
+  for (int s = 0; s < F.depth; ++s)
+    if (F.slot_state[s] == 2 && (F.consumed[s] | inactive) == all) F.slot_state[s] = 0;
+}
+// Lockstep round-robin: member 0's iteration i, member 1's, ..., then i + 1.
+void feed_advance_turn(Feed& F) {
+  const int M = static_cast<int>(F.members.size());
+  for (int i = 0; i < M; ++i) {
+    if (++F.turn_m == M) { F.turn_m = 0; ++F.turn_it; }
+    if (member_active(F, F.turn_m)) return;
+  }
+}
+// S_0 of iteration `it` retired: its copy of the slot into the arena has executed.
+void feed_consumed(Feed& F, int64_t it, int member) {
+  const int s = static_cast<int>(it % F.depth);
+  if (F.slot_iter[s] != it || F.slot_state[s] != 2) return;
+  if (!F.shared) {
+    F.slot_state[s] = 0;
+  } else {
+    F.consumed[s] |= 1u << member;
+    feed_release_drained(F);
+  }
+}
+void push_host_event(sf_runtime* rt, const Feed& F, int job, int64_t it, uint64_t t0, uint64_t t1) {
+  sf_trace_event ev{};
+  ev.dev = -1 - static_cast<int32_t>(F.id);
+  ev.job = job;
+  ev.kind = SF_EV_HOST;
+  ev.k = -1;
+  ev.iter = it;
+  ev.t0_ns = t0;
+  ev.t1_ns = t1;
+  ev.arrival_ns = t0;
+  push_trace(rt, ev);
+}
+// Run the host stage for iteration `it` into ring slot s (rt->m NOT held); "" on success.
+std::string feed_fill(sf_runtime* rt, Feed& F, int s, int64_t it) {
+  std::vector<void*> dst(F.n);
+  for (int i = 0; i < F.n; ++i) dst[i] = F.host + s * F.stride + F.off[i];
+  if (F.fn(F.user, it, dst.data(), F.bytes.data(), F.n) != 0) return "host stage returned an error";
+  if (F.shared) {  // the immutable device copy every member reads
+    cudaError_t e = cudaSetDevice(rt->slots[F.dev]->cuda);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(F.dbuf + s * F.stride, F.host + s * F.stride, F.stride, cudaMemcpyHostToDevice, F.st);
+    if (e == cudaSuccess) e = cudaEventRecord(F.ev, F.st);
+    if (e == cudaSuccess) e = cudaEventSynchronize(F.ev);
+    if (e != cudaSuccess) return std::string("feed H2D: ") + cudaGetErrorString(e);
+  }
+  return "";
+}
+
+// The feed's CPU executor: prefetches up to `depth` iterations, never holding a device.
+void stager_main(sf_runtime* rt, Feed* Fp) {
+  Feed& F = *Fp;
+  std::unique_lock<std::mutex> lk(rt->m);
+  while (true) {
+    rt->cv.wait(lk, [&] {
+      return rt->shutting_down || F.failed ||
+             (F.active && !F.inline_mode && F.slot_state[F.next_iter % F.depth] == 0);
+    });
+    if (rt->shutting_down || F.failed) break;
+    const int64_t it = F.next_iter;
+    const int s = static_cast<int>(it % F.depth);
+    const uint64_t gen = F.gen;
+    F.slot_state[s] = 1;
+    F.slot_iter[s] = it;
+    F.consumed[s] = 0;
+    ++F.next_iter;
+    lk.unlock();
+    const uint64_t t0 = now_ns();
+    const std::string err = feed_fill(rt, F, s, it);
+    const uint64_t t1 = now_ns();
+    lk.lock();
+    if (!err.empty()) {
+      F.failed = true;
+      F.error = err;
+      rt->cv.notify_all();
+      break;
+    }
+    F.slot_state[s] = gen == F.gen ? 2 : 0;  // a restart meanwhile discards the fill
+    push_host_event(rt, F, static_cast<int>((1u << 21) | F.id), it, t0, t1);
+    rt->cv.notify_all();
+  }
+}
+
 // Job driver.  J.it / J.k is the LAUNCH cursor (the next subgraph not yet launched); up to
 // max_inflight subgraphs are queued on the device back to back (no host gap between them).
 // When a preemption is requested or a request is queued on the device, launching stops,
@@ -1349,6 +1486,16 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       if (q.empty()) {
         release();
         J.state = SF_JOB_DONE;
+        if (g.feed) {
+          Feed& F = *g.feed;
+          bool any = false;
+          if (F.shared) {  // leave the lockstep
+            if (F.turn_m == g.feed_member) feed_advance_turn(F);
+            for (size_t m = 0; m < F.members.size(); ++m) any |= member_active(F, static_cast<int>(m));
+          }
+          if (!any) F.active = false;  // the stage stops prefetching
+          else feed_release_drained(F);
+        }
         rt->cv.notify_all();
         break;
       }
@@ -1405,7 +1552,30 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         }
       } else {
         Slot& S = slot_of(rt, J.dev);
-        if (rt->cfg.exclusive_gpu && !J.holds_token) {
+        // host feed: S_0 needs its iteration's inputs (shared feed: also its lockstep turn);
+        // until then the job leaves the device to others — one job's CPU stage overlaps
+        // another job's GPU subgraphs
+        bool feed_ok = true;
+        if (g.feed && J.k == 0) {
+          Feed& F = *g.feed;
+          if (F.failed) {
+            release();
+            J.error = "host stage: " + F.error;
+            J.state = SF_JOB_FAILED;
+            rt->cv.notify_all();
+            break;
+          }
+          const int s = static_cast<int>(J.it % F.depth);
+          if (F.shared && !(F.turn_it == J.it && F.turn_m == g.feed_member)) feed_ok = false;
+          else if (!F.inline_mode && !(F.slot_state[s] == 2 && F.slot_iter[s] == J.it)) feed_ok = false;
+        }
+        if (!feed_ok) {
+          if (q.empty()) {
+            release();
+            rt->cv.wait(lk);
+            continue;
+          }
+        } else if (rt->cfg.exclusive_gpu && !J.holds_token) {
           // invariant 1: no other model's subgraph on this device
           if (S.owner != -1) {
             if (q.empty()) {
@@ -1417,7 +1587,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
             J.holds_token = true;
           }
         }
-        launch = (!rt->cfg.exclusive_gpu || J.holds_token) && static_cast<int>(q.size()) < W &&
+        launch = feed_ok && (!rt->cfg.exclusive_gpu || J.holds_token) && static_cast<int>(q.size()) < W &&
                  (q.empty() || budget_us <= 0.0 || queued_us() + est_us[J.k] <= budget_us);
       }
     }
@@ -1427,6 +1597,27 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       const int64_t it = J.it;
       cudaGraphExec_t ver = g.bind[dev]->versions[k];
       sfk::count_launch(g.bind[dev]->version_kernels[k]);
+      Feed* F = k == 0 ? g.feed : nullptr;
+      const int fslot = F ? static_cast<int>(it % F->depth) : -1;
+      if (F && F->inline_mode && !(F->slot_state[fslot] == 2 && F->slot_iter[fslot] == it)) {
+        // session-slicing baseline: the CPU stage runs now, while the job holds the device
+        F->slot_state[fslot] = 1;
+        F->slot_iter[fslot] = it;
+        lk.unlock();
+        const uint64_t h0 = now_ns();
+        const std::string err = feed_fill(rt, *F, fslot, it);
+        const uint64_t h1 = now_ns();
+        lk.lock();
+        if (!err.empty()) {
+          release();
+          J.error = "host stage: " + err;
+          J.state = SF_JOB_FAILED;
+          rt->cv.notify_all();
+          break;
+        }
+        F->slot_state[fslot] = 2;
+        push_host_event(rt, *F, static_cast<int>(J.id), it, h0, h1);
+      }
       const bool stamp = J.stamp_resume;
       J.stamp_resume = false;
       const int ev = ev_next;
@@ -1437,6 +1628,13 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
       // wait on the peer store) has executed when this event completes on the device
       cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
+      if (e == cudaSuccess && F) {  // this iteration's fed tensors into the arena, then S_0
+        const uint8_t* src = (F->shared ? F->dbuf : F->host) + fslot * F->stride;
+        uint8_t* arena = g.bind[dev]->arena;
+        for (int i = 0; e == cudaSuccess && i < F->n; ++i)
+          e = cudaMemcpyAsync(arena + g.T[g.feed_tids[i]].offset, src + F->off[i], F->bytes[i],
+                              cudaMemcpyDefault, S.s_train);
+      }
       if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
       if (e == cudaSuccess) e = cudaEventRecord(J.ev_ring[dev * kMaxInflight + ev], S.s_train);
       lk.lock();
@@ -1448,7 +1646,14 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         break;
       }
       q.push_back({it, k, dev, ev, t0, stamp});
-      if (++J.k == n) { J.k = 0; ++J.it; }
+      if (++J.k == n) {
+        J.k = 0;
+        ++J.it;
+        if (g.feed && g.feed->shared) {  // the next member's turn on this batch
+          feed_advance_turn(*g.feed);
+          rt->cv.notify_all();
+        }
+      }
       continue;
     }
     if (q.empty()) {  // nothing launched and nothing in flight: wait for a state change
@@ -1487,6 +1692,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     lk.lock();
     q.pop_front();
+    if (f.k == 0 && g.feed) feed_consumed(*g.feed, f.it, g.feed_member);
     if (f.stamp) {
       J.last_resume = t_res;  // host-observed device resume (CLOCK_MONOTONIC)
       if (unpack_us >= 0.f) { J.unpack_us = unpack_us; J.xfer_us += std::max(h2d_us, 0.f); }
@@ -1703,6 +1909,18 @@ void sf_destroy(sf_runtime* rt) {
     if (J->driver.joinable()) J->driver.join();
   for (auto& S : rt->slots)
     if (S->dispatcher.joinable()) S->dispatcher.join();
+  for (auto& F : rt->feeds)
+    if (F->stager.joinable()) F->stager.join();
+  for (auto& F : rt->feeds) {
+    if (F->shared) {
+      cudaSetDevice(rt->slots[F->dev]->cuda);
+      cudaStreamSynchronize(F->st);
+      cudaFree(F->dbuf);
+      cudaStreamDestroy(F->st);
+      cudaEventDestroy(F->ev);
+    }
+    cudaFreeHost(F->host);
+  }
   for (auto& S : rt->slots) {
     if (S->remote) continue;
     cudaSetDevice(S->cuda);
@@ -2037,7 +2255,25 @@ static sf_status start_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t
     J->sched.push_back(c);
   }
   if (sf_status s = ensure_events(rt, *J)) return s;
+  if (g->feed) {
+    Feed& F = *g->feed;
+    if (F.shared) {
+      if (it0 != 0 || k0 != 0) return fail(SF_EUNSUPPORTED, "shared-feed members start at iteration 0");
+      if (F.member_jobs[g->feed_member] && F.member_jobs[g->feed_member]->state != SF_JOB_DONE)
+        return fail(SF_EBUSY, "a job of this feed member is running");
+    } else {
+      // (re)start the pipeline at the job's first un-fed iteration; in-flight fills are stale
+      ++F.gen;
+      for (int s = 0; s < F.depth; ++s)
+        if (F.slot_state[s] != 1) F.slot_state[s] = 0;
+      F.next_iter = it0 + (k0 > 0 ? 1 : 0);
+      F.inline_mode = rt->cfg.host_stage_inline != 0;
+    }
+    F.failed = false;
+    F.active = true;
+  }
   Job* jp = J.get();
+  if (g->feed) g->feed->member_jobs[g->feed_member] = jp;
   rt->jobs.push_back(std::move(J));
   jp->driver = std::thread(driver_main, rt, jp);
   rt->cv.notify_all();  // lower-priority jobs on dev re-check their boundary gate
@@ -2054,6 +2290,107 @@ sf_status sf_start_training(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_
 sf_status sf_adopt_job(sf_runtime* rt, sf_graph_id gid, int32_t dev, int64_t iters, int64_t iter,
                        int32_t k, int32_t auto_target, sf_job_id* out) {
   return start_job(rt, gid, dev, iters, auto_target, nullptr, 0, iter, k, out);
+}
+
+sf_status sf_create_feed(sf_runtime* rt, const sf_feed_desc* d, sf_feed_id* out) {
+  if (!rt || !d || !out || !d->fn || d->n < 1 || d->n > 8 || !d->bytes || d->depth < 0 || d->depth > 8)
+    return fail(SF_EINVAL, "bad feed descriptor");
+  std::lock_guard<std::mutex> lk(rt->m);
+  auto F = std::make_unique<Feed>();
+  F->id = static_cast<sf_feed_id>(rt->feeds.size());
+  F->fn = d->fn;
+  F->user = d->user;
+  F->n = d->n;
+  F->depth = d->depth ? d->depth : 2;
+  F->shared = d->shared != 0;
+  F->dev = d->dev;
+  for (int i = 0; i < F->n; ++i) {
+    if (d->bytes[i] == 0) return fail(SF_EINVAL, "empty fed tensor");
+    F->off.push_back(F->stride);
+    F->bytes.push_back(d->bytes[i]);
+    F->stride += round_up(d->bytes[i], kAlign);
+  }
+  F->slot_iter.assign(F->depth, -1);
+  F->slot_state.assign(F->depth, 0);
+  F->consumed.assign(F->depth, 0);
+  if (F->shared) {
+    if (F->dev < 0 || F->dev >= static_cast<int>(rt->slots.size()) || rt->slots[F->dev]->remote)
+      return fail(SF_EINVAL, "shared feed: dev is not a local slot");
+    SF_CK(cudaSetDevice(rt->slots[F->dev]->cuda));
+    SF_CK(cudaMalloc(&F->dbuf, F->stride * F->depth));
+    SF_CK(cudaStreamCreateWithFlags(&F->st, cudaStreamNonBlocking));
+    SF_CK(cudaEventCreateWithFlags(&F->ev, cudaEventDisableTiming));
+  }
+  SF_CK(cudaHostAlloc(&F->host, F->stride * F->depth, cudaHostAllocPortable));
+  Feed* fp = F.get();
+  rt->feeds.push_back(std::move(F));
+  fp->stager = std::thread(stager_main, rt, fp);
+  *out = fp->id;
+  return SF_OK;
+}
+
+sf_status sf_attach_feed(sf_runtime* rt, sf_graph_id gid, sf_feed_id fid, const uint32_t* tids) {
+  if (!rt || !tids) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g) return fail(SF_EINVAL, "bad graph id");
+  if (fid >= rt->feeds.size()) return fail(SF_EINVAL, "bad feed id");
+  Feed& F = *rt->feeds[fid];
+  if (g->feed) return fail(SF_ESTATE, "graph already has a feed");
+  if (!F.shared && !F.members.empty()) return fail(SF_EBUSY, "a non-shared feed takes one graph");
+  if (F.members.size() >= 32) return fail(SF_EINVAL, "at most 32 members per shared feed");
+  for (int i = 0; i < F.n; ++i) {
+    if (tids[i] >= g->T.size()) return fail(SF_EINVAL, "fed tensor id out of range");
+    const Tensor& t = g->T[tids[i]];
+    if ((t.kind != SF_INPUT && t.kind != SF_LABEL) || g->op_written[tids[i]])
+      return fail(SF_EINVAL, "fed tensors are INPUT / LABEL tensors no op writes");
+    if (t.nbytes != F.bytes[i]) return fail(SF_EINVAL, "fed tensor size differs from the feed's");
+  }
+  for (const auto& J : rt->jobs)
+    if (J->g == g && J->state != SF_JOB_DONE && J->state != SF_JOB_FAILED)
+      return fail(SF_ESTATE, "attach before starting the graph's jobs");
+  g->feed = &F;
+  g->feed_tids.assign(tids, tids + F.n);
+  g->feed_member = static_cast<int>(F.members.size());
+  F.members.push_back(g);
+  F.member_jobs.push_back(nullptr);
+  return SF_OK;
+}
+
+// Built-in host stage (sf.h: sf_stage_u8_normalize).  splitmix64 (Steele, Lea, Flood 2014):
+// output n (1-based) of a generator seeded with s is fin(s + n * 0x9E3779B97F4A7C15).
+static uint64_t splitmix64_out(uint64_t seed, uint64_t n) {
+  uint64_t z = seed + n * 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+int32_t sf_stage_u8_normalize(void* user, int64_t iter, void* const* dst, const uint64_t* bytes,
+                              int32_t n) {
+  const sf_u8_stage* u = static_cast<const sf_u8_stage*>(user);
+  if (!u || !dst || n != 2 || u->batch <= 0 || u->cols <= 0 || u->img_w <= 0 || u->cols % u->img_w ||
+      u->pool_rows < u->batch || u->pool_rows % u->batch || iter < 0)
+    return -1;
+  if (bytes[0] != static_cast<uint64_t>(u->batch) * u->cols * 4 || bytes[1] != static_cast<uint64_t>(u->batch) * 4)
+    return -1;
+  const int64_t b = iter % (u->pool_rows / u->batch);
+  float* x = static_cast<float*>(dst[0]);
+  int32_t* y = static_cast<int32_t*>(dst[1]);
+  const int W = u->img_w, H = u->cols / u->img_w;
+  for (int r = 0; r < u->batch; ++r) {
+    const int64_t row = b * u->batch + r;
+    const uint8_t* src = u->images + row * u->cols;
+    float* xr = x + static_cast<int64_t>(r) * u->cols;
+    if (splitmix64_out(u->seed, static_cast<uint64_t>(row) + 1) & 1) {
+      for (int yy = 0; yy < H; ++yy)
+        for (int xx = 0; xx < W; ++xx) xr[yy * W + xx] = static_cast<float>(src[yy * W + (W - 1 - xx)]) / 255.0f;
+    } else {
+      for (int c = 0; c < u->cols; ++c) xr[c] = static_cast<float>(src[c]) / 255.0f;
+    }
+    y[r] = u->labels[row];
+  }
+  return 0;
 }
 
 sf_status sf_export_arena(sf_runtime* rt, sf_graph_id gid, int32_t dev, sf_ipc_arena* out) {

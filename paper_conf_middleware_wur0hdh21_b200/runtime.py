@@ -124,6 +124,11 @@ class GraphHandle:
     def arena_bytes(self, slot: int) -> torch.Tensor:
         return self.mem[slot]["arena"]
 
+    def attach_feed(self, feed: int, tensor_ids: Sequence[int]) -> None:
+        """Feed these INPUT / LABEL tensors from host feed ``feed`` (sf_attach_feed)."""
+        arr = (C.c_uint32 * len(tensor_ids))(*tensor_ids)
+        check(lib().sf_attach_feed(self.rt.h, self.gid, feed, arr), "sf_attach_feed")
+
 
 class Runtime:
     """One sf_runtime: logical device slots mapped onto CUDA devices."""
@@ -133,17 +138,20 @@ class Runtime:
                  host_mode: int = A.SF_HOST_CE, poison: bool = False, budget_bytes: int = 0,
                  trace_capacity: int = 0, defer_migration: bool = False, max_inflight: int = 1,
                  dispatch_spin_us: int = 0, inflight_budget_us: int = 0,
-                 migrate_home: bool = False, migration_engine: int = 0):
+                 migrate_home: bool = False, migration_engine: int = 0,
+                 host_stage_inline: bool = False):
         self.ordinals = list(ordinals)
         arr = (C.c_int32 * len(self.ordinals))(*self.ordinals)
         cfg = A.sf_config(len(self.ordinals), arr, int(exclusive), int(auto_preempt),
                           int(iteration_granularity), host_mode, int(poison), trace_capacity,
                           max_inflight, int(defer_migration), budget_bytes, dispatch_spin_us,
-                          inflight_budget_us, int(migrate_home), migration_engine)
+                          inflight_budget_us, int(migrate_home), migration_engine,
+                          int(host_stage_inline))
         h = C.c_void_p()
         check(lib().sf_create(C.byref(cfg), C.byref(h)), "sf_create")
         self.h = h
         self.graphs: List[GraphHandle] = []
+        self._keep: list = []  # host-stage user data referenced by the library
 
     def close(self) -> None:
         if self.h:
@@ -164,6 +172,27 @@ class Runtime:
         gh = GraphHandle(self, gid.value, g, priority)
         self.graphs.append(gh)
         return gh
+
+    # ---- host input stages (sf_create_feed) ---------------------------------------------------
+    def create_feed(self, fn_ptr: int, user_ptr: int, nbytes: Sequence[int], depth: int = 2,
+                    shared: bool = False, dev: int = 0) -> int:
+        b = (C.c_uint64 * len(nbytes))(*nbytes)
+        d = A.sf_feed_desc(fn_ptr, user_ptr, len(nbytes), b, depth, int(shared), dev, 0)
+        f = C.c_uint32()
+        check(lib().sf_create_feed(self.h, C.byref(d), C.byref(f)), "sf_create_feed")
+        return f.value
+
+    def u8_feed(self, images: np.ndarray, labels: np.ndarray, batch: int, img_w: int, seed: int,
+                depth: int = 2, shared: bool = False, dev: int = 0) -> int:
+        """Feed driven by the built-in host stage sf_stage_u8_normalize (x f32, y i32)."""
+        images = np.ascontiguousarray(images, dtype=np.uint8)
+        labels = np.ascontiguousarray(labels, dtype=np.int32).reshape(-1)
+        st = A.sf_u8_stage(images.ctypes.data, labels.ctypes.data, images.shape[0], batch,
+                           images.shape[1], img_w, seed)
+        self._keep += [images, labels, st]
+        fn = C.cast(lib().sf_stage_u8_normalize, C.c_void_p).value
+        return self.create_feed(fn, C.addressof(st), [batch * images.shape[1] * 4, batch * 4],
+                                depth, shared, dev)
 
     # ---- jobs -----------------------------------------------------------------------------
     def start_training(self, gh: GraphHandle, slot: int, iters: int, auto_target: int,
@@ -238,7 +267,7 @@ class Runtime:
         out = []
         for i in range(n.value):
             e = buf[i]
-            kind = {A.EV_TRAIN: "train", A.EV_INFER: "infer"}.get(e.kind, "migrate")
+            kind = {A.EV_TRAIN: "train", A.EV_INFER: "infer", A.EV_HOST: "host"}.get(e.kind, "migrate")
             d = {"dev": e.dev, "job": e.job, "kind": kind, "iter": e.iter, "k": e.k,
                  "t0": e.t0_ns, "t1": e.t1_ns}
             if kind == "infer":

@@ -105,3 +105,11 @@ def poisson_arrivals(n: int, rate_per_s: float, seed: int = 7) -> np.ndarray:
     """Open-loop Poisson arrival offsets in seconds."""
     rng = np.random.Generator(np.random.PCG64(seed))
     return np.cumsum(rng.exponential(1.0 / rate_per_s, size=n))
+
+
+def u8_images(n: int, cols: int, classes: int, seed: int = SEED_DATA):
+    """Synthetic u8 image pool for the host input stage (reading Q27): pixels U{0..255},
+    labels U{0..classes-1}."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    return (rng.integers(0, 256, size=(n, cols), dtype=np.uint8),
+            rng.integers(0, classes, size=(n, 1), dtype=np.int32))

@@ -37,10 +37,11 @@ ADAM_EPS = 1e-8
 # ---------------------------------------------------------------------------------
 def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int = 16,
               lr: float = SGD_LR, mu: float = SGD_MU, name: str = "mlp",
-              act: str = "relu") -> Graph:
+              act: str = "relu", host_fed: bool = False) -> Graph:
     """Training graph of an MLP with ReLU (or GELU: ``act="gelu"``) hidden layers and
     softmax-CE loss.  A GELU layer's BIAS_ACT also writes its pre-activation u_i, which
-    its BIAS_ACT_BWD reads.
+    its BIAS_ACT_BWD reads.  ``host_fed``: x, y come from a host
+    input stage (sf_attach_feed) instead of FEED ops over DATASET pools.
 
     For widths (784, 256, 10) this is exactly SURVEY.md 8(c) step 1 (o1..o11) with
     FEED ops for x, y in front (data cursor = step, reading Q3/Q11) and STEP_INC
@@ -59,8 +60,9 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
         aW.append(g.add(f"aW{i+1}", widths[i], widths[i + 1], F32, SLOT))
         ab.append(g.add(f"ab{i+1}", 1, widths[i + 1], F32, SLOT))
     step = g.add("step", 1, 1, I32, SCALAR_STATE)
-    xpool = g.add("X_pool", pool * batch, widths[0], F32, DATASET)
-    ypool = g.add("Y_pool", pool * batch, 1, I32, DATASET)
+    if not host_fed:
+        xpool = g.add("X_pool", pool * batch, widths[0], F32, DATASET)
+        ypool = g.add("Y_pool", pool * batch, 1, I32, DATASET)
     x = g.add("x", batch, widths[0], F32, INPUT)
     y = g.add("y", batch, 1, I32, LABEL)
 
@@ -71,7 +73,7 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
     gelu = act == "gelu"
     for i in range(L):
         ph = i
-        if i == 0:
+        if i == 0 and not host_fed:
             g.op(FEED, [xpool, step], [x], phase=ph)
             g.op(FEED, [ypool, step], [y], phase=ph)
         z = g.add(f"z{i+1}", batch, widths[i + 1], F32, ACT)

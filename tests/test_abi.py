@@ -71,7 +71,7 @@ def test_enum_values_match_workload_codes():
 def test_struct_layouts_match_c(built):
     structs = ["sf_tensor_desc", "sf_op_desc", "sf_graph_desc", "sf_config", "sf_partition_opts",
                "sf_partition_info", "sf_job_info", "sf_cut_info", "sf_timing", "sf_trace_event",
-               "sf_cut_request", "sf_copy_desc"]
+               "sf_cut_request", "sf_copy_desc", "sf_feed_desc", "sf_u8_stage"]
     lines = ['#include <stdio.h>', '#include <stddef.h>', f'#include "{HEADER}"', "int main(){"]
     for s in structs:
         lines.append(f'printf("{s} %zu\\n", sizeof({s}));')
@@ -107,3 +107,22 @@ def test_create_without_gpu_reports_cuda_error(built):
     from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
     with pytest.raises(built.SFError):
         Runtime([0])
+
+
+def test_builtin_host_stage_equals_oracle(built):
+    """sf_stage_u8_normalize (host code, no GPU) is bit-identical to oracle/feed.py."""
+    import numpy as np
+    from oracle import feed as FD
+    from sf_inputs import data as D
+    imgs, labels = D.u8_images(96, 28 * 28, 10, seed=3)
+    st = built.sf_u8_stage(imgs.ctypes.data, labels.ctypes.data, 96, 32, 784, 28, 77)
+    x = np.empty((32, 784), np.float32)
+    y = np.empty((32, 1), np.int32)
+    dst = (ctypes.c_void_p * 2)(x.ctypes.data, y.ctypes.data)
+    nb = (ctypes.c_uint64 * 2)(x.nbytes, y.nbytes)
+    for it in (0, 1, 2, 5):
+        assert built.lib().sf_stage_u8_normalize(ctypes.addressof(st), it, dst, nb, 2) == 0
+        rx, ry = FD.u8_stage(imgs, labels, it, 32, 28, seed=77)
+        assert x.tobytes() == rx.tobytes() and y.tobytes() == ry.tobytes()
+    nb[0] = 4  # size mismatch is an error, not a buffer overrun
+    assert built.lib().sf_stage_u8_normalize(ctypes.addressof(st), 0, dst, nb, 2) != 0
