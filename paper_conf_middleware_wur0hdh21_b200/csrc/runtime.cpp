@@ -223,7 +223,7 @@ struct Feed {
   uint8_t* host = nullptr;   // pinned [depth][stride]
   uint8_t* dbuf = nullptr;   // shared: device [depth][stride], the immutable copies
   cudaStream_t st = nullptr;
-  cudaEvent_t ev = nullptr;
+  std::vector<cudaEvent_t> ev;  // shared: per ring slot, its H2D into dbuf completed
   std::vector<int64_t> slot_iter;
   std::vector<int> slot_state;
   std::vector<uint32_t> consumed;  // shared: bit m = member m copied the slot (S_0 retired)
@@ -1393,12 +1393,12 @@ std::string feed_fill(sf_runtime* rt, Feed& F, int s, int64_t it) {
   std::vector<void*> dst(F.n);
   for (int i = 0; i < F.n; ++i) dst[i] = F.host + s * F.stride + F.off[i];
   if (F.fn(F.user, it, dst.data(), F.bytes.data(), F.n) != 0) return "host stage returned an error";
-  if (F.shared) {  // the immutable device copy every member reads
+  if (F.shared) {  // the immutable device copy every member reads (members' training streams
+                   // wait for ev[s]; the slot is refilled only after all of them consumed it)
     cudaError_t e = cudaSetDevice(rt->slots[F.dev]->cuda);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(F.dbuf + s * F.stride, F.host + s * F.stride, F.stride, cudaMemcpyHostToDevice, F.st);
-    if (e == cudaSuccess) e = cudaEventRecord(F.ev, F.st);
-    if (e == cudaSuccess) e = cudaEventSynchronize(F.ev);
+    if (e == cudaSuccess) e = cudaEventRecord(F.ev[s], F.st);
     if (e != cudaSuccess) return std::string("feed H2D: ") + cudaGetErrorString(e);
   }
   return "";
@@ -1631,6 +1631,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       if (e == cudaSuccess && F) {  // this iteration's fed tensors into the arena, then S_0
         const uint8_t* src = (F->shared ? F->dbuf : F->host) + fslot * F->stride;
         uint8_t* arena = g.bind[dev]->arena;
+        if (F->shared) e = cudaStreamWaitEvent(S.s_train, F->ev[fslot], 0);
         for (int i = 0; e == cudaSuccess && i < F->n; ++i)
           e = cudaMemcpyAsync(arena + g.T[g.feed_tids[i]].offset, src + F->off[i], F->bytes[i],
                               cudaMemcpyDefault, S.s_train);
@@ -1917,7 +1918,7 @@ void sf_destroy(sf_runtime* rt) {
       cudaStreamSynchronize(F->st);
       cudaFree(F->dbuf);
       cudaStreamDestroy(F->st);
-      cudaEventDestroy(F->ev);
+      for (auto e : F->ev) cudaEventDestroy(e);
     }
     cudaFreeHost(F->host);
   }
@@ -2319,7 +2320,8 @@ sf_status sf_create_feed(sf_runtime* rt, const sf_feed_desc* d, sf_feed_id* out)
     SF_CK(cudaSetDevice(rt->slots[F->dev]->cuda));
     SF_CK(cudaMalloc(&F->dbuf, F->stride * F->depth));
     SF_CK(cudaStreamCreateWithFlags(&F->st, cudaStreamNonBlocking));
-    SF_CK(cudaEventCreateWithFlags(&F->ev, cudaEventDisableTiming));
+    F->ev.assign(F->depth, nullptr);
+    for (auto& e : F->ev) SF_CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   }
   SF_CK(cudaHostAlloc(&F->host, F->stride * F->depth, cudaHostAllocPortable));
   Feed* fp = F.get();
