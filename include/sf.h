@@ -180,6 +180,14 @@ typedef struct sf_config {
                                     session-based time slicing, the Gandiva-like baseline of
                                     PAPER.md:1385-1392); 0: feeds prefetch on their own thread
                                     (CPU executors scheduled freely) */
+  int32_t pad0;
+  uint64_t infer_l2_persist_bytes; /* > 0: reserve this much of each device's L2 (clamped to
+                                    cudaDevAttrMaxPersistingL2CacheSize) as a persisting
+                                    set-aside for the inference graphs' weights: their request
+                                    kernels carry an access-policy window over the arena and
+                                    tag weight TMA loads evict_last, so the collocated training
+                                    job's streaming traffic cannot evict them (Q29);
+                                    0 = off */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,

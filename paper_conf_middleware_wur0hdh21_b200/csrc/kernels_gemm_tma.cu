@@ -22,7 +22,9 @@
 #include <algorithm>
 #include <cstdlib>
 #include <atomic>
+#include <map>
 #include <mutex>
+#include <tuple>
 
 #include "sf_device.cuh"
 #include "sf_kernels.h"
@@ -567,7 +569,8 @@ __global__ void __cluster_dims__(kGvCluster, 1, 1) __launch_bounds__(288)
 gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict__ X,
                 float* __restrict__ Y, int M, int N, int K, int ldx, int ldy, int kper, int acc,
                 const float* __restrict__ b1, const float* __restrict__ b2,
-                const float* __restrict__ b3, int relu, int b_const) {
+                const float* __restrict__ b3, int relu, int b_const, int l2_keep,
+                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
   using Cfg = GvCfg<MR, BC>;
   constexpr int QW = Cfg::QW, RL = Cfg::RL, S = Cfg::S;
   extern __shared__ __align__(1024) unsigned char gv_smem[];
@@ -605,12 +608,17 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
   if (warp == 8) {
     if ((tid & 31) == 0) {
       if (!b_const) sfdev::griddep_wait();  // W may be written by the predecessor
+      const uint64_t pol = sfdev::policy_evict_last();
       for (int i = 0; i < nbox; ++i) {
         const int slot = i % S;
         if (i >= S) sfdev::mbar_wait(&empty[slot], ((i / S) - 1) & 1);
         expect_tx(&full[slot], Cfg::BOX);
-        tma_load_2d(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]), c0,
-                    k0 + i * kGvRows);
+        if (l2_keep)  // resident inference weights: keep them in the persisting L2 set-aside
+          sfdev::tma_load_2d_hint(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]),
+                                  c0, k0 + i * kGvRows, pol);
+        else
+          tma_load_2d(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]), c0,
+                      k0 + i * kGvRows);
       }
     }
     __syncwarp();
@@ -676,6 +684,46 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
         if (relu) v = fmaxf(v, 0.f);
         o[j] = v;
       }
+    }
+  }
+  if (sm_out != nullptr && rank == 0) {
+    // fused row softmax: the last column block to publish its outputs normalises all rows
+    // (threadfence-reduction pattern; fixed-order reductions, so results are deterministic)
+    __shared__ int sm_last;
+    __shared__ float sm_red[9];
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x / kGvCluster - 1;
+    __syncthreads();
+    if (sm_last) {
+      __threadfence();
+      const int lane = tid & 31;
+      for (int m = 0; m < M; ++m) {
+        const float* yr = Y + static_cast<size_t>(m) * ldy;
+        float mx = -INFINITY;
+        for (int n = tid; n < N; n += 288) mx = fmaxf(mx, __ldcg(yr + n));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        if (lane == 0) sm_red[warp] = mx;
+        __syncthreads();
+        mx = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 9; ++w) mx = fmaxf(mx, sm_red[w]);
+        __syncthreads();
+        float s = 0.f;
+        for (int n = tid; n < N; n += 288) s += expf(__ldcg(yr + n) - mx);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        if (lane == 0) sm_red[warp] = s;
+        __syncthreads();
+        s = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 9; ++w) s += sm_red[w];
+        __syncthreads();
+        float* orow = sm_out + static_cast<size_t>(m) * sm_ldo;
+        for (int n = tid; n < N; n += 288) orow[n] = expf(__ldcg(yr + n) - mx) / s;
+      }
+      if (tid == 0) *sm_counter = 0u;
     }
   }
   cluster.sync();
@@ -795,7 +843,8 @@ cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cud
   count_launch();
   return launch_k(kern, dim3(grid), dim3(288), smem, st, w, a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc,
                   kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
-                  a.b_const ? 1 : 0);
+                  a.b_const ? 1 : 0, a.b_const && l2_keep_enabled() ? 1 : 0, a.sm_out, a.sm_ldo,
+                  a.sm_counter);
 }
 
 template <int BC>
@@ -821,6 +870,12 @@ bool gemv_tma_eligible(const GemmArgs& a) {
   return (a.K + kGvCluster - 1) / kGvCluster <= kGvMaxKper;
 }
 
+bool gemv_softmax_fusable(const GemmArgs& a) {
+  static const char gemv_path = std::getenv("SF_GEMV") ? std::getenv("SF_GEMV")[0] : 't';
+  static const bool off = std::getenv("SF_FUSE_SOFTMAX") && std::getenv("SF_FUSE_SOFTMAX")[0] == '0';
+  return !off && gemv_path == 't' && !a.acc && gemv_tma_eligible(a);
+}
+
 cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st) {
   // widest column block that still puts one CTA on every SM
   int bc = 32;
@@ -828,9 +883,28 @@ cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st) {
     if ((a.N + c - 1) / c * kGvCluster >= 148) { bc = c; break; }
   int kper = (a.K + kGvCluster - 1) / kGvCluster;
   kper = (kper + kGvRows - 1) / kGvRows * kGvRows;
+  // the weight maps of an inference graph never change: encode once per (W, shape, box)
+  struct Key {
+    const void* p; int n, k, ld, bc;
+    bool operator<(const Key& o) const {
+      return std::tie(p, n, k, ld, bc) < std::tie(o.p, o.n, o.k, o.ld, o.bc);
+    }
+  };
+  static std::mutex mu;
+  static std::map<Key, CUtensorMap> cache;
+  const Key key{a.B, a.N, a.K, a.ldb, bc};
   CUtensorMap w;
-  if (!map2d(&w, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, bc, kGvRows, CU_TENSOR_MAP_SWIZZLE_NONE))
-    return cudaErrorInvalidValue;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = a.b_const ? cache.find(key) : cache.end();
+    if (it != cache.end()) {
+      w = it->second;
+    } else {
+      if (!map2d(&w, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, bc, kGvRows, CU_TENSOR_MAP_SWIZZLE_NONE))
+        return cudaErrorInvalidValue;
+      if (a.b_const && cache.size() < 4096) cache[key] = w;
+    }
+  }
   if (bc == 128) return dispatch_gemv_mr<128>(w, a, kper, st);
   if (bc == 64) return dispatch_gemv_mr<64>(w, a, kper, st);
   return dispatch_gemv_mr<32>(w, a, kper, st);

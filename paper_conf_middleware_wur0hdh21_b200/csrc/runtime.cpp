@@ -163,6 +163,7 @@ struct Slot {
   cudaEvent_t ev_i0 = nullptr;  // timing: request chain start (ev_infer marks its end)
   unsigned long long* tstamp = nullptr;  // device {start, end} x 2 (pack/peer, unpack)
   std::atomic<int> owner{-1};  // device token (atomic: the spinning dispatcher polls it)
+  size_t l2_setaside = 0, l2_max_window = 0;  // persisting L2 for inference weights
   std::deque<Request*> q;
   std::atomic<int> qn{0};       // q.size(), readable without the runtime lock
   std::thread dispatcher;
@@ -563,6 +564,7 @@ sf_status do_partition(Graph& g, const sf_partition_opts& o) {
       g.ws_floats = std::max(g.ws_floats, sfk::softmax_ce_ws_floats(g.T[op.in[0]].rows));
     }
   }
+  g.counter_slots += 1;  // the last slot: completion counter of a GEMV with fused softmax
   g.partitioned = true;
   return SF_OK;
 }
@@ -576,7 +578,16 @@ struct Capture {
   cudaStream_t st;
   bool dry;                          // prepare pass: upload descriptor arrays, launch nothing
   std::map<int, void*>* prepared;    // first op index of an optimizer group -> device array
-  uint8_t* ptr(int t) const { return b.arena + g.T[t].offset; }
+  // request I/O in place (direct inference launches): the INPUT tensor is read from, and the
+  // OUTPUT tensor written to, the caller's buffers instead of arena copies
+  int redir_in = -1, redir_out = -1;
+  uint8_t* in_ptr = nullptr;
+  uint8_t* out_ptr = nullptr;
+  uint8_t* ptr(int t) const {
+    if (t == redir_in) return in_ptr;
+    if (t == redir_out) return out_ptr;
+    return b.arena + g.T[t].offset;
+  }
   float* f(int t) const { return reinterpret_cast<float*>(ptr(t)); }
 };
 
@@ -795,9 +806,19 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
             for (int i = 1; i < ba.n_in; ++i) ga.bias[i - 1] = c.f(ba.in[i]);
             ga.relu = ba.flags & SF_ACT_RELU;
             ga.ldc = g.T[ba.out[0]].cols;
+            // ... and a following SOFTMAX of that output (the inference head) into the same
+            // kernel: the last column block normalises the rows
+            int used = 2;
+            if (j + 2 < e && g.ops[j + 2].type == SF_OP_SOFTMAX && g.ops[j + 2].in[0] == ba.out[0] &&
+                sfk::gemv_softmax_fusable(ga)) {
+              ga.sm_out = c.f(g.ops[j + 2].out[0]);
+              ga.sm_ldo = g.T[g.ops[j + 2].out[0]].cols;
+              ga.sm_counter = c.b.counters + (g.counter_slots - 1);
+              used = 3;
+            }
             err = sfk::launch_gemm(ga, c.st);
             if (err != cudaSuccess) return fail(SF_ECUDA, "op " + std::to_string(j) + ": " + cudaGetErrorString(err));
-            j += 2;
+            j += used;
             continue;
           }
         }
@@ -1770,8 +1791,16 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     static const bool use_pdl = !(std::getenv("SF_PDL") && std::getenv("SF_PDL")[0] == '0');
     std::string op_err;
     if (direct) sfk::set_pdl(use_pdl);
+    if (direct && S->l2_setaside > 0) {  // weights stay in the persisting L2 set-aside
+      const size_t win = std::min<size_t>(g.arena_bytes, S->l2_max_window);
+      sfk::set_l2_keep(true, B->arena, win, std::min(1.0f, static_cast<float>(S->l2_setaside) / win));
+    }
+    // the kernels read the request's input and write its output in place (UVA: device or
+    // pinned host buffers), saving the two copy kernels of the I/O staging
+    static const bool redirect = !(std::getenv("SF_INFER_REDIRECT") && std::getenv("SF_INFER_REDIRECT")[0] == '0');
+    const bool in_place = direct && aligned && redirect;
     e = cudaEventRecord(S->ev_i0, S->s_infer);
-    if (e != cudaSuccess) {
+    if (e != cudaSuccess || in_place) {
     } else if (aligned) {
       e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
     } else {
@@ -1780,6 +1809,12 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
+        if (in_place) {
+          c.redir_in = g.input_tid;
+          c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(r->in));
+          c.redir_out = g.output_tid;
+          c.out_ptr = static_cast<uint8_t*>(r->out);
+        }
         if (launch_subgraph_ops(c, static_cast<int>(k)) != SF_OK) {
           op_err = g_err;
           e = cudaErrorUnknown;
@@ -1789,11 +1824,12 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
         sfk::count_launch(B->version_kernels[k]);
       }
     }
-    if (e == cudaSuccess) {
+    if (e == cudaSuccess && !in_place) {
       if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
       else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
     }
     sfk::set_pdl(false);
+    sfk::set_l2_keep(false);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
     if (e == cudaSuccess) e = spin_event(S->ev_infer);
     const uint64_t t1 = now_ns();
@@ -1868,6 +1904,14 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
     SF_CK(cudaEventCreate(&S->ev_infer));
     SF_CK(cudaEventCreate(&S->ev_i0));
     SF_CK(cudaMalloc(&S->tstamp, 4 * sizeof(unsigned long long)));
+    if (cfg->infer_l2_persist_bytes > 0) {
+      int mx = 0, mw = 0;
+      SF_CK(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, c));
+      SF_CK(cudaDeviceGetAttribute(&mw, cudaDevAttrMaxAccessPolicyWindowSize, c));
+      S->l2_setaside = std::min<size_t>(cfg->infer_l2_persist_bytes, static_cast<size_t>(mx));
+      S->l2_max_window = static_cast<size_t>(mw);
+      SF_CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, S->l2_setaside));
+    }
     rt->slots.push_back(std::move(S));
   }
   // peer access between distinct physical devices (NVLink / NVSwitch)

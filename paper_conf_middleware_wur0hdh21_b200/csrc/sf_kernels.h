@@ -43,12 +43,24 @@ struct GemmArgs {
   // B is not written by any kernel that may still be running (inference weights): the GEMV
   // may stream it before griddep_wait() under programmatic dependent launch
   bool b_const = false;
+  // optional fused row softmax of the (epilogued) output into sm_out (TMA GEMV path only, see
+  // gemv_softmax_fusable): the last column block to finish normalises every row; sm_counter is
+  // a zeroed device counter the kernel leaves zeroed
+  float* sm_out = nullptr;
+  int sm_ldo = 0;
+  unsigned* sm_counter = nullptr;
 };
+bool gemv_softmax_fusable(const GemmArgs& a);
 // True when launch_gemm can fuse a following BIAS_ACT into this GEMM's epilogue.
 // Programmatic dependent launch for the launches this host thread makes (thread-local;
 // the inference dispatcher enables it around a request's kernel chain).
 void set_pdl(bool on);
 bool pdl_enabled();
+// Inference launches of this host thread tag constant weights (GEMV TMA loads) evict_last, and
+// launch_k attaches the thread's access-policy window (persisting L2 set-aside), if any.
+void set_l2_keep(bool on, const void* base = nullptr, size_t bytes = 0, float hit_ratio = 0.f);
+bool l2_keep_enabled();
+const cudaAccessPolicyWindow* l2_window();
 bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb);
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);

@@ -6,7 +6,8 @@ from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
 g, gi = bench.build_workload(8, 1)
 arrs, arrs_i = bench.workload_arrays(g, gi, (8, 1))
 import os
-rt = Runtime([0], dispatch_spin_us=int(os.environ.get("SPIN", "0")))
+rt = Runtime([0], dispatch_spin_us=int(os.environ.get("SPIN", "0")),
+             infer_l2_persist_bytes=int(float(os.environ.get("L2P_MB", "0")) * (1 << 20)))
 ghi = rt.register(gi, 1); ghi.partition(); ghi.bind(0, staging=False); ghi.load(0, arrs_i)
 x = torch.rand(1, 2048, device="cuda"); out = torch.empty(1, 1000, device="cuda")
 lat, pre, dev = [], [], []
@@ -46,6 +47,9 @@ if os.environ.get("COPY"):
     stop_copy = True
     th.join()
 rt.close()
-print(json.dumps({"p50_ms": float(np.median(lat)), "p99_ms": float(np.percentile(lat, 99)),
+print(json.dumps({"l2p_mb": os.environ.get("L2P_MB", "0"), "flush": bool(flush is not None),
+                  "max_persist_mb": torch.cuda.get_device_properties(0).persisting_l2_cache_max_size / 2**20
+                  if hasattr(torch.cuda.get_device_properties(0), "persisting_l2_cache_max_size") else None,
+                  "p50_ms": float(np.median(lat)), "p99_ms": float(np.percentile(lat, 99)),
                   "min_ms": float(np.min(lat)), "wake_p50_ms": float(np.median(pre)),
                   "device_p50_ms": float(np.median(dev))}))
