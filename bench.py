@@ -109,7 +109,10 @@ class ClockSampler:
 def build_workload(batch: int, spatial_div: int):
     from sf_inputs import graphs as G
     g = G.resnet50_forest(batch=batch, spatial_div=spatial_div)
-    gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M")
+    # SF_BENCH_WT=1: output-major weights ([N][K], GEMM TB, row-streaming GEMV); measured
+    # slower than the [K][N] TMA cluster GEMV on this workload (reading Q30)
+    gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M",
+                     wt=os.environ.get("SF_BENCH_WT", "0") == "1")
     return g, gi
 
 
@@ -666,6 +669,23 @@ def main():
     except Exception:
         pass
     m0 = chase_s
+    # the box's pinned-memory copy peak per direction (host tier vs PCIe)
+    link = {}
+    try:
+        hb = torch.empty(256 << 20, dtype=torch.uint8).pin_memory()
+        db = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+        for name, (dst, src) in (("h2d", (db, hb)), ("d2h", (hb, db))):
+            best = 0.0
+            for _ in range(4):
+                e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+                e0.record(); dst.copy_(src, non_blocking=True); e1.record(); e1.synchronize()
+                best = max(best, hb.numel() / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+            link[name] = best
+        del hb, db
+    except Exception:
+        link = {}
+    dev_us = pct(main_s.get("device_us", []), 50)
+    w_bytes = (2048 * 4096 + 4096 * 4096 + 4096 * 1000 + 4096 + 4096 + 1000) * 4
     line = {
         "metric": METRIC, "value": pct(M["lat"], 99), "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
@@ -700,6 +720,9 @@ def main():
                       "pack_gbs": pack_achieved,
                       "d2h_plus_h2d_us_mean": float(xfer[ok].mean()) if ok.any() else None,
                       "host_link_gbs": migr_gbs,
+                      "host_link_peak_gbs": link or None,
+                      "host_link_frac": (migr_gbs / (0.5 * (link["h2d"] + link["d2h"])))
+                      if link and migr_gbs else None,
                       "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},
         "training_subgraph_ms_mean": m0["sub_ms"], "n_subgraphs": m0["n_subgraphs"],
         "training_iteration_ms_median": m0["iter_ms"],
@@ -709,6 +732,12 @@ def main():
                      "frac": (pack_achieved / hbm) if pack_achieved else None,
                      "traffic": traffic, "peak_source": peak_src,
                      "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
+        "inference_roofline": {"kernel": "request chain (3 TMA cluster GEMVs, fused bias/ReLU, "
+                                         "fused softmax; device time p50)",
+                               "bound": "hbm", "algorithmic_bytes": w_bytes,
+                               "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
+                               "peak": hbm, "unit": "GB/s",
+                               "frac": (w_bytes / (dev_us * 1e-6) / 1e9 / hbm) if dev_us else None},
         "e2e": {"value": pct(E, 99), "unit": UNIT, "h2d_bytes_per_step": 2048 * 4,
                 "d2h_bytes_per_step": 1000 * 4, "p50_ms": pct(E, 50)},
         "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),

@@ -416,6 +416,8 @@ typedef struct sf_timing {
   int32_t cut_k;
   float device_us;       /* device time of the request's kernel chain (input copy .. output
                             copy), CUDA events on the inference stream */
+  float launch_us;       /* host time the dispatcher took to issue the chain (first event
+                            record .. last launch returned) */
 } sf_timing;
 
 /* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).

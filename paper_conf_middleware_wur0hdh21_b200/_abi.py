@@ -88,7 +88,8 @@ class sf_cut_info(C.Structure):
 class sf_timing(C.Structure):
     _fields_ = [("arrival_ns", C.c_uint64), ("start_ns", C.c_uint64), ("end_ns", C.c_uint64),
                 ("dev", C.c_int32), ("preempted_job", C.c_int32), ("cut_iter", C.c_int64),
-                ("cut_k", C.c_int32), ("device_us", C.c_float)]
+                ("cut_k", C.c_int32), ("device_us", C.c_float),
+                ("launch_us", C.c_float)]
 
 
 class sf_trace_event(C.Structure):

@@ -34,21 +34,7 @@ thread_local bool t_pdl = false;
 }
 void set_pdl(bool on) { t_pdl = on; }
 bool pdl_enabled() { return t_pdl; }
-thread_local bool t_l2_keep = false;
-thread_local cudaAccessPolicyWindow t_apw{};
-void set_l2_keep(bool on, const void* base, size_t bytes, float hit_ratio) {
-  t_l2_keep = on;
-  t_apw = cudaAccessPolicyWindow{};
-  if (on && base && bytes) {
-    t_apw.base_ptr = const_cast<void*>(base);
-    t_apw.num_bytes = bytes;
-    t_apw.hitRatio = hit_ratio;
-    t_apw.hitProp = cudaAccessPropertyPersisting;
-    t_apw.missProp = cudaAccessPropertyStreaming;
-  }
-}
-bool l2_keep_enabled() { return t_l2_keep; }
-const cudaAccessPolicyWindow* l2_window() { return t_l2_keep && t_apw.num_bytes ? &t_apw : nullptr; }
+
 
 constexpr int kCopyThreads = 256;
 constexpr int kCopyUnroll = SF_COPY_UNROLL;

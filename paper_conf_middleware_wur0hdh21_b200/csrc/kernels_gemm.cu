@@ -671,6 +671,7 @@ uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
 
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0) return cudaSuccess;
+  if (gemv_rows_eligible(a)) return launch_gemv_rows(a, st);
   if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)))
     return cudaErrorInvalidValue;  // fused epilogue only exists on the GEMV path
   // M <= 8 paths: SF_GEMV = tma (default: TMA-streamed cluster GEMV) | cluster (register-

@@ -569,7 +569,7 @@ __global__ void __cluster_dims__(kGvCluster, 1, 1) __launch_bounds__(288)
 gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict__ X,
                 float* __restrict__ Y, int M, int N, int K, int ldx, int ldy, int kper, int acc,
                 const float* __restrict__ b1, const float* __restrict__ b2,
-                const float* __restrict__ b3, int relu, int b_const, int l2_keep,
+                const float* __restrict__ b3, int relu, int b_const, int l2_hint,
                 float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
   using Cfg = GvCfg<MR, BC>;
   constexpr int QW = Cfg::QW, RL = Cfg::RL, S = Cfg::S;
@@ -608,12 +608,12 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
   if (warp == 8) {
     if ((tid & 31) == 0) {
       if (!b_const) sfdev::griddep_wait();  // W may be written by the predecessor
-      const uint64_t pol = sfdev::policy_evict_last();
+      const uint64_t pol = sfdev::l2_policy(l2_hint);
       for (int i = 0; i < nbox; ++i) {
         const int slot = i % S;
         if (i >= S) sfdev::mbar_wait(&empty[slot], ((i / S) - 1) & 1);
         expect_tx(&full[slot], Cfg::BOX);
-        if (l2_keep)  // resident inference weights: keep them in the persisting L2 set-aside
+        if (l2_hint)  // keep (persisting set-aside) / stream (evict first) the weights
           sfdev::tma_load_2d_hint(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]),
                                   c0, k0 + i * kGvRows, pol);
         else
@@ -727,6 +727,265 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
     }
   }
   cluster.sync();
+}
+
+// ---- row-contiguous GEMV (M <= 8, B stored [N][K]: the inference weight layout) ---------
+// y[m][n] = act(sum_k x[m][k] B[n][k] + biases): every output is the dot product of x with one
+// contiguous row of B, so each CTA's work is ONE contiguous span of rows [r0, r1) streamed
+// sequentially by 1-D bulk copies (one row per ring slot) — the DRAM access pattern of a pure
+// read stream, no split-K, no cluster reduction.  Warp 8 lane 0 is the producer; ring slot s
+// is always consumed by warp s % NW (NW = min(8, slots)), which takes its rows in order, so
+// no consumer can run a phase ahead on a slot (lane j: float4 j, j + 32, ...; shuffle-tree
+// reduce, fixed order, deterministic).  Weights that no running kernel writes (b_const) stream before
+// griddep_wait(), so under PDL a layer's rows arrive while its predecessor drains; one CTA per
+// SM leaves room for the next layer's CTA.  Optional fused row softmax as in gemv_tma_kernel.
+constexpr int kGrRing = 96 * 1024;   // bytes of rows in flight per CTA
+constexpr int kGrMaxRow = 32 * 1024;  // K <= 8192
+constexpr int kGrMaxX = 64 * 1024;    // M * K * 4: x staged in smem
+
+template <int MR>
+__global__ void __launch_bounds__(288)
+gemv_rows_kernel(const float* __restrict__ Bm, const float* __restrict__ X, float* __restrict__ Y,
+                 int M, int N, int K, int ldb, int ldx, int ldy, int slots,
+                 const float* __restrict__ b1, const float* __restrict__ b2,
+                 const float* __restrict__ b3, int relu, int b_const, int l2_hint,
+                 float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
+  extern __shared__ __align__(1024) unsigned char gr_smem[];
+  const int rowf = K;                        // floats per row (K % 4 == 0)
+  const uint32_t row_bytes = static_cast<uint32_t>(K) * 4;
+  const int slot_f = (rowf + 31) / 32 * 32;  // 128-B aligned slots
+  float* ring = reinterpret_cast<float*>(gr_smem);
+  float* xs = ring + static_cast<size_t>(slots) * slot_f;
+  uint64_t* full = reinterpret_cast<uint64_t*>(xs + static_cast<size_t>(MR) * K);
+  uint64_t* empty = full + slots;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  // balanced contiguous row span of this CTA
+  const int r0 = static_cast<int>(static_cast<int64_t>(N) * blockIdx.x / gridDim.x);
+  const int r1 = static_cast<int>(static_cast<int64_t>(N) * (blockIdx.x + 1) / gridDim.x);
+  const int nrows = r1 - r0;
+  if (tid == 0) {
+    for (int i = 0; i < slots; ++i) {
+      sfdev::mbar_init(&full[i], 1);
+      sfdev::mbar_init(&empty[i], 1);
+    }
+    sfdev::mbar_fence_init();
+  }
+  __syncthreads();
+  sfdev::griddep_launch();  // the next layer may start streaming its own rows now
+  if (warp == 8) {
+    if (lane == 0) {
+      if (!b_const) sfdev::griddep_wait();  // B may be written by the predecessor
+      const uint64_t pol = sfdev::l2_policy(l2_hint);
+      for (int i = 0; i < nrows; ++i) {
+        const int s = i % slots;
+        if (i >= slots) sfdev::mbar_wait(&empty[s], ((i / slots) - 1) & 1);
+        expect_tx(&full[s], row_bytes);
+        const uint32_t dst = sfdev::smem_u32(ring + static_cast<size_t>(s) * slot_f);
+        const float* src = Bm + static_cast<size_t>(r0 + i) * ldb;
+        if (l2_hint) sfdev::bulk_load_1d_hint(dst, src, row_bytes, sfdev::smem_u32(&full[s]), pol);
+        else sfdev::bulk_load_1d(dst, src, row_bytes, sfdev::smem_u32(&full[s]));
+      }
+    }
+    __syncwarp();
+  } else {
+    sfdev::griddep_wait();  // x is the predecessor's output
+    for (int i = tid; i < MR * K; i += 256) {
+      const int m = i / K, k = i % K;
+      xs[i] = m < M ? X[static_cast<size_t>(m) * ldx + k] : 0.f;
+    }
+    asm volatile("bar.sync 1, 256;" ::: "memory");
+    const int nq = K / 4;
+    const float4* x4 = reinterpret_cast<const float4*>(xs);
+    const int nw = slots < 8 ? slots : 8;
+    for (int i = 0; i < nrows; ++i) {
+      const int s = i % slots;
+      if (s % nw != warp) continue;
+      sfdev::mbar_wait(&full[s], (i / slots) & 1);
+      const float4* w4 = reinterpret_cast<const float4*>(ring + static_cast<size_t>(s) * slot_f);
+      float acc[MR];
+#pragma unroll
+      for (int m = 0; m < MR; ++m) acc[m] = 0.f;
+#pragma unroll 4
+      for (int q = lane; q < nq; q += 32) {
+        const float4 w = w4[q];
+#pragma unroll
+        for (int m = 0; m < MR; ++m) {
+          const float4 xv = x4[m * nq + q];
+          acc[m] = fmaf(xv.x, w.x, acc[m]);
+          acc[m] = fmaf(xv.y, w.y, acc[m]);
+          acc[m] = fmaf(xv.z, w.z, acc[m]);
+          acc[m] = fmaf(xv.w, w.w, acc[m]);
+        }
+      }
+      __syncwarp();
+      if (lane == 0) sfdev::mbar_arrive(&empty[s]);
+#pragma unroll
+      for (int m = 0; m < MR; ++m)
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) acc[m] += __shfl_xor_sync(0xffffffffu, acc[m], o);
+      if (lane < MR && lane < M) {
+        float v = 0.f;
+#pragma unroll
+        for (int m = 0; m < MR; ++m)
+          if (m == lane) v = acc[m];
+        const int n = r0 + i;
+        if (b1) v += b1[n];
+        if (b2) v += b2[n];
+        if (b3) v += b3[n];
+        if (relu) v = fmaxf(v, 0.f);
+        Y[static_cast<size_t>(lane) * ldy + n] = v;
+      }
+    }
+  }
+  if (sm_out != nullptr) {
+    // fused row softmax: the last CTA to publish its rows normalises every output row
+    __shared__ int sm_last;
+    __shared__ float sm_red[9];
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (sm_last) {
+      __threadfence();
+      for (int m = 0; m < M; ++m) {
+        const float* yr = Y + static_cast<size_t>(m) * ldy;
+        float mx = -INFINITY;
+        for (int n = tid; n < N; n += 288) mx = fmaxf(mx, __ldcg(yr + n));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        if (lane == 0) sm_red[warp] = mx;
+        __syncthreads();
+        mx = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 9; ++w) mx = fmaxf(mx, sm_red[w]);
+        __syncthreads();
+        float sum = 0.f;
+        for (int n = tid; n < N; n += 288) sum += expf(__ldcg(yr + n) - mx);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+        if (lane == 0) sm_red[warp] = sum;
+        __syncthreads();
+        sum = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 9; ++w) sum += sm_red[w];
+        __syncthreads();
+        float* orow = sm_out + static_cast<size_t>(m) * sm_ldo;
+        for (int n = tid; n < N; n += 288) orow[n] = expf(__ldcg(yr + n) - mx) / sum;
+      }
+      if (tid == 0) *sm_counter = 0u;
+    }
+  }
+}
+
+// Same contraction with plain vectorised loads (no smem ring): warp w of the grid takes rows
+// w, w + #warps, ...; lane j loads float4 j, j + 32, ... of the row, 8 loads in flight, with
+// an L2 cache-policy hint (ld.global.nc.L2::cache_hint) so kept weights land in the persisting
+// set-aside (TMA bulk copies do not honour it on B200, Q29).  SF_GEMV_ROWS=ldg.
+template <int MR>
+__global__ void __launch_bounds__(256)
+gemv_rows_ldg_kernel(const float* __restrict__ Bm, const float* __restrict__ X, float* __restrict__ Y,
+                     int M, int N, int K, int ldb, int ldx, int ldy,
+                     const float* __restrict__ b1, const float* __restrict__ b2,
+                     const float* __restrict__ b3, int relu, int l2_hint,
+                     float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
+  extern __shared__ __align__(16) float gl_xs[];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  sfdev::griddep_launch();
+  sfdev::griddep_wait();
+  for (int i = tid; i < MR * K; i += 256) {
+    const int m = i / K, k = i % K;
+    gl_xs[i] = m < M ? X[static_cast<size_t>(m) * ldx + k] : 0.f;
+  }
+  __syncthreads();
+  const uint64_t pol = sfdev::l2_policy(l2_hint ? l2_hint : 2);
+  const int nq = K / 4;
+  const float4* x4 = reinterpret_cast<const float4*>(gl_xs);
+  const int nwarps = gridDim.x * 8;
+  for (int n = blockIdx.x * 8 + warp; n < N; n += nwarps) {
+    const float4* w4 = reinterpret_cast<const float4*>(Bm + static_cast<size_t>(n) * ldb);
+    float acc[MR];
+#pragma unroll
+    for (int m = 0; m < MR; ++m) acc[m] = 0.f;
+    int q = lane;
+    for (; q + 7 * 32 < nq; q += 8 * 32) {
+      float4 w[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) w[u] = sfdev::ldg4_hint(w4 + q + 32 * u, pol);
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+#pragma unroll
+        for (int m = 0; m < MR; ++m) {
+          const float4 xv = x4[m * nq + q + 32 * u];
+          acc[m] = fmaf(xv.x, w[u].x, acc[m]);
+          acc[m] = fmaf(xv.y, w[u].y, acc[m]);
+          acc[m] = fmaf(xv.z, w[u].z, acc[m]);
+          acc[m] = fmaf(xv.w, w[u].w, acc[m]);
+        }
+    }
+    for (; q < nq; q += 32) {
+      const float4 w = sfdev::ldg4_hint(w4 + q, pol);
+#pragma unroll
+      for (int m = 0; m < MR; ++m) {
+        const float4 xv = x4[m * nq + q];
+        acc[m] = fmaf(xv.x, w.x, acc[m]);
+        acc[m] = fmaf(xv.y, w.y, acc[m]);
+        acc[m] = fmaf(xv.z, w.z, acc[m]);
+        acc[m] = fmaf(xv.w, w.w, acc[m]);
+      }
+    }
+#pragma unroll
+    for (int m = 0; m < MR; ++m)
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) acc[m] += __shfl_xor_sync(0xffffffffu, acc[m], o);
+    if (lane < MR && lane < M) {
+      float v = 0.f;
+#pragma unroll
+      for (int m = 0; m < MR; ++m)
+        if (m == lane) v = acc[m];
+      if (b1) v += b1[n];
+      if (b2) v += b2[n];
+      if (b3) v += b3[n];
+      if (relu) v = fmaxf(v, 0.f);
+      Y[static_cast<size_t>(lane) * ldy + n] = v;
+    }
+  }
+  if (sm_out != nullptr) {
+    __shared__ int sm_last;
+    __shared__ float sm_red[8];
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (sm_last) {
+      __threadfence();
+      for (int m = 0; m < M; ++m) {
+        const float* yr = Y + static_cast<size_t>(m) * ldy;
+        float mx = -INFINITY;
+        for (int n = tid; n < N; n += 256) mx = fmaxf(mx, __ldcg(yr + n));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        if (lane == 0) sm_red[warp] = mx;
+        __syncthreads();
+        mx = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 8; ++w) mx = fmaxf(mx, sm_red[w]);
+        __syncthreads();
+        float sum = 0.f;
+        for (int n = tid; n < N; n += 256) sum += expf(__ldcg(yr + n) - mx);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+        if (lane == 0) sm_red[warp] = sum;
+        __syncthreads();
+        sum = sm_red[0];
+#pragma unroll
+        for (int w = 1; w < 8; ++w) sum += sm_red[w];
+        __syncthreads();
+        float* orow = sm_out + static_cast<size_t>(m) * sm_ldo;
+        for (int n = tid; n < N; n += 256) orow[n] = expf(__ldcg(yr + n) - mx) / sum;
+      }
+      if (tid == 0) *sm_counter = 0u;
+    }
+  }
 }
 
 // ---- host: tensor maps ------------------------------------------------------------------
@@ -843,7 +1102,7 @@ cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cud
   count_launch();
   return launch_k(kern, dim3(grid), dim3(288), smem, st, w, a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc,
                   kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
-                  a.b_const ? 1 : 0, a.b_const && l2_keep_enabled() ? 1 : 0, a.sm_out, a.sm_ldo,
+                  a.b_const ? 1 : 0, a.l2_hint, a.sm_out, a.sm_ldo,
                   a.sm_counter);
 }
 
@@ -870,10 +1129,80 @@ bool gemv_tma_eligible(const GemmArgs& a) {
   return (a.K + kGvCluster - 1) / kGvCluster <= kGvMaxKper;
 }
 
+bool gemv_rows_eligible(const GemmArgs& a) {
+  auto al = [](const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; };
+  static const bool off = std::getenv("SF_GEMV_ROWS") && std::getenv("SF_GEMV_ROWS")[0] == '0';
+  if (off || a.M < 1 || a.M > 8 || a.ta || !a.tb || a.acc) return false;
+  if (a.K % 4 || a.ldb % 4 || a.K * 4 > kGrMaxRow || a.M * a.K * 4 > kGrMaxX || !al(a.B)) return false;
+  return a.N > 0 && a.K > 0;
+}
+
+template <int MR>
+cudaError_t launch_gemv_rows_ldg_t(const GemmArgs& a, cudaStream_t st) {
+  auto kern = gemv_rows_ldg_kernel<MR>;
+  const size_t smem = static_cast<size_t>(MR) * a.K * 4;
+  static std::atomic<uint64_t> configured{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (!(configured.load() & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kGrMaxX);
+    if (e != cudaSuccess) return e;
+    configured.fetch_or(bit);
+  }
+  // 2 CTAs (16 warps) per SM, capped by one warp per row
+  const int grid = std::max(1, std::min((a.N + 7) / 8, 2 * 148));
+  count_launch();
+  return launch_k(kern, dim3(grid), dim3(256), smem, st, a.B, a.A, a.C, a.M, a.N, a.K, a.ldb, a.lda,
+                  a.ldc, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0, a.l2_hint, a.sm_out,
+                  a.sm_ldo, a.sm_counter);
+}
+
+template <int MR>
+cudaError_t launch_gemv_rows_t(const GemmArgs& a, cudaStream_t st) {
+  static const bool ldg = std::getenv("SF_GEMV_ROWS") && std::getenv("SF_GEMV_ROWS")[0] == 'l';
+  if (ldg) return launch_gemv_rows_ldg_t<MR>(a, st);
+  auto kern = gemv_rows_kernel<MR>;
+  const int slot_f = (a.K + 31) / 32 * 32;
+  const int slots = std::max(2, std::min(16, kGrRing / (slot_f * 4)));
+  const size_t smem = static_cast<size_t>(slots) * slot_f * 4 + static_cast<size_t>(MR) * a.K * 4 +
+                      2 * slots * 8 + 64;
+  static std::atomic<uint64_t> configured{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = 1ull << (dev & 63);
+  if (!(configured.load() & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         kGrRing + kGrMaxRow + kGrMaxX + 2 * 16 * 8 + 64);
+    if (e != cudaSuccess) return e;
+    configured.fetch_or(bit);
+  }
+  static int n_sms = [] {
+    int d = 0, n = 148;
+    cudaGetDevice(&d);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, d);
+    return n;
+  }();
+  const int grid = std::min(a.N, n_sms);  // one CTA per SM: the next layer's CTA fits beside it
+  count_launch();
+  return launch_k(kern, dim3(grid), dim3(288), smem, st, a.B, a.A, a.C, a.M, a.N, a.K, a.ldb, a.lda,
+                  a.ldc, slots, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0, a.b_const ? 1 : 0,
+                  a.l2_hint, a.sm_out, a.sm_ldo, a.sm_counter);
+}
+
 bool gemv_softmax_fusable(const GemmArgs& a) {
   static const char gemv_path = std::getenv("SF_GEMV") ? std::getenv("SF_GEMV")[0] : 't';
   static const bool off = std::getenv("SF_FUSE_SOFTMAX") && std::getenv("SF_FUSE_SOFTMAX")[0] == '0';
-  return !off && gemv_path == 't' && !a.acc && gemv_tma_eligible(a);
+  if (off || a.acc) return false;
+  if (a.tb) return gemv_rows_eligible(a);
+  return gemv_path == 't' && gemv_tma_eligible(a);
+}
+
+cudaError_t launch_gemv_rows(const GemmArgs& a, cudaStream_t st) {
+  if (a.M == 1) return launch_gemv_rows_t<1>(a, st);
+  if (a.M == 2) return launch_gemv_rows_t<2>(a, st);
+  if (a.M <= 4) return launch_gemv_rows_t<4>(a, st);
+  return launch_gemv_rows_t<8>(a, st);
 }
 
 cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st) {

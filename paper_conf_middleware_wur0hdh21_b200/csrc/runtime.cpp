@@ -30,6 +30,7 @@
 #include <map>
 #include <memory>
 #include <mutex>
+#include <set>
 #include <string>
 #include <thread>
 #include <unordered_map>
@@ -106,6 +107,8 @@ struct Binding {
   // TMA tensor-map requirement); refreshed from the arena at sf_start_training
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
   std::map<int, void*> prepared;  // optimizer group first op -> uploaded descriptor array
+  std::set<int> l2_keep;          // inference weights kept in the persisting L2 set-aside
+  bool l2_planned = false;
   std::map<int, std::pair<float*, unsigned*>> chain_bufs;  // chain first op -> (ws, counters)
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
   // refreshed inside the version graph (copy2d before / after the GEMM)
@@ -152,6 +155,7 @@ struct Request {
   int64_t cut_iter = -1;
   int cut_k = -1;
   float device_us = -1.f;
+  float launch_us = -1.f;
   std::string error;
 };
 
@@ -578,6 +582,7 @@ struct Capture {
   cudaStream_t st;
   bool dry;                          // prepare pass: upload descriptor arrays, launch nothing
   std::map<int, void*>* prepared;    // first op index of an optimizer group -> device array
+  const std::set<int>* l2_keep = nullptr;  // weights held in the persisting L2 set-aside
   // request I/O in place (direct inference launches): the INPUT tensor is read from, and the
   // OUTPUT tensor written to, the caller's buffers instead of arena copies
   int redir_in = -1, redir_out = -1;
@@ -762,6 +767,7 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         ga.lda = A.cols; ga.ldb = B.cols; ga.ldc = C.cols;
         ga.ws = c.b.ws; ga.counters = c.b.counters;
         ga.b_const = !g.op_written[o.in[1]];
+        if (c.l2_keep) ga.l2_hint = c.l2_keep->count(o.in[1]) ? 1 : 2;
         auto sa = c.b.shadow.find(o.in[0]);
         if (sa != c.b.shadow.end()) { ga.A = sa->second.first; ga.lda = sa->second.second; }
         auto sb = c.b.shadow.find(o.in[1]);
@@ -796,7 +802,7 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         // reader (same arithmetic order as the unfused pair, so results are bit-identical).
         if (j + 1 < e && !ga.acc && g.ops[j + 1].type == SF_OP_BIAS_ACT && g.ops[j + 1].in[0] == o.out[0] &&
             !(g.ops[j + 1].flags & SF_ACT_GELU) && C.kind != SF_OUTPUT &&
-            sfk::gemm_can_fuse_bias(ga.M, ga.N, ga.K, ga.ta, ga.tb, ga.ldb)) {
+            (sfk::gemm_can_fuse_bias(ga.M, ga.N, ga.K, ga.ta, ga.tb, ga.ldb) || sfk::gemv_rows_eligible(ga))) {
           int readers = 0;
           for (const auto& q : g.ops)
             for (int t : op_reads(q)) readers += (t == o.out[0]);
@@ -1791,14 +1797,34 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     static const bool use_pdl = !(std::getenv("SF_PDL") && std::getenv("SF_PDL")[0] == '0');
     std::string op_err;
     if (direct) sfk::set_pdl(use_pdl);
-    if (direct && S->l2_setaside > 0) {  // weights stay in the persisting L2 set-aside
-      const size_t win = std::min<size_t>(g.arena_bytes, S->l2_max_window);
-      sfk::set_l2_keep(true, B->arena, win, std::min(1.0f, static_cast<float>(S->l2_setaside) / win));
+    if (direct && S->l2_setaside > 0 && !B->l2_planned) {
+      // persisting L2 set-aside: keep whole weight tensors, largest first, within the set-aside
+      // (a cyclic stream larger than the set-aside would thrash it); the rest is streamed
+      // evict-first so it cannot displace them (reading Q29)
+      std::vector<std::pair<uint64_t, int>> ws;
+      for (const auto& o : g.ops)
+        if (o.type == SF_OP_GEMM && !g.op_written[o.in[1]] && g.T[o.out[0]].rows <= 8)
+          ws.push_back({g.T[o.in[1]].nbytes, o.in[1]});
+      std::sort(ws.rbegin(), ws.rend());
+      uint64_t used = 0;
+      for (auto [nb, t] : ws)
+        if (used + nb <= S->l2_setaside) { B->l2_keep.insert(t); used += nb; }
+      B->l2_planned = true;
     }
-    // the kernels read the request's input and write its output in place (UVA: device or
-    // pinned host buffers), saving the two copy kernels of the I/O staging
+    // device-resident request buffers are read / written in place by the kernels (saving the
+    // two copy kernels of the I/O staging); pinned host buffers keep the SM copy kernels, which
+    // move them in one coalesced pass instead of every GEMV CTA reading its x slice over PCIe
     static const bool redirect = !(std::getenv("SF_INFER_REDIRECT") && std::getenv("SF_INFER_REDIRECT")[0] == '0');
-    const bool in_place = direct && aligned && redirect;
+    auto on_device = [](const void* p) {
+      cudaPointerAttributes a{};
+      if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+      }
+      return a.type == cudaMemoryTypeDevice;
+    };
+    const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
+    const uint64_t tl0 = now_ns();
     e = cudaEventRecord(S->ev_i0, S->s_infer);
     if (e != cudaSuccess || in_place) {
     } else if (aligned) {
@@ -1809,6 +1835,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
+        if (S->l2_setaside > 0) c.l2_keep = &B->l2_keep;
         if (in_place) {
           c.redir_in = g.input_tid;
           c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(r->in));
@@ -1828,8 +1855,8 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
       else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
     }
+    const uint64_t tl1 = now_ns();
     sfk::set_pdl(false);
-    sfk::set_l2_keep(false);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
     if (e == cudaSuccess) e = spin_event(S->ev_infer);
     const uint64_t t1 = now_ns();
@@ -1842,6 +1869,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     r->start = t0;
     r->end = t1;
     r->device_us = dev_ms >= 0.f ? dev_ms * 1e3f : -1.f;
+    r->launch_us = static_cast<float>((tl1 - tl0) * 1e-3);
     if (e != cudaSuccess) r->error = op_err.empty() ? cudaGetErrorString(e) : op_err;
     r->done = true;
     S->q.pop_front();
@@ -2643,6 +2671,7 @@ sf_status sf_wait(sf_runtime* rt, sf_req_id id, int64_t timeout_ns, sf_timing* t
     t->cut_iter = r->cut_iter;
     t->cut_k = r->cut_k;
     t->device_us = r->device_us;
+    t->launch_us = r->launch_us;
   }
   std::string err = r->error;
   rt->reqs.erase(it);
@@ -2696,7 +2725,7 @@ static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, in
   sfk::GemmArgs ga{A, B, C, M, N, K, lda, ldb, ldc, (flags & SF_GEMM_TA) != 0,
                    (flags & SF_GEMM_TB) != 0, (flags & SF_GEMM_ACC) != 0, nullptr, nullptr};
   const bool epi = b1 || relu;
-  const bool fuse = epi && sfk::gemm_can_fuse_bias(M, N, K, ga.ta, ga.tb, ldb);
+  const bool fuse = epi && (sfk::gemm_can_fuse_bias(M, N, K, ga.ta, ga.tb, ldb) || sfk::gemv_rows_eligible(ga));
   if (fuse) {
     ga.bias[0] = b1; ga.bias[1] = b2; ga.bias[2] = b3;
     ga.relu = relu;

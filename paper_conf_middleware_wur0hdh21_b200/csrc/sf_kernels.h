@@ -49,18 +49,21 @@ struct GemmArgs {
   float* sm_out = nullptr;
   int sm_ldo = 0;
   unsigned* sm_counter = nullptr;
+  // L2 policy of the GEMV weight stream: 0 default, 1 keep (evict_last: held in the persisting
+  // L2 set-aside across requests), 2 stream (evict_first: do not displace kept weights)
+  int l2_hint = 0;
 };
 bool gemv_softmax_fusable(const GemmArgs& a);
+// M <= 8 with B stored [N][K] (TB, the inference weight layout): row-contiguous streaming GEMV
+// with the same fused epilogue / softmax (kernels_gemm_tma.cu).
+bool gemv_rows_eligible(const GemmArgs& a);
+cudaError_t launch_gemv_rows(const GemmArgs& a, cudaStream_t st);
 // True when launch_gemm can fuse a following BIAS_ACT into this GEMM's epilogue.
 // Programmatic dependent launch for the launches this host thread makes (thread-local;
 // the inference dispatcher enables it around a request's kernel chain).
 void set_pdl(bool on);
 bool pdl_enabled();
-// Inference launches of this host thread tag constant weights (GEMV TMA loads) evict_last, and
-// launch_k attaches the thread's access-policy window (persisting L2 set-aside), if any.
-void set_l2_keep(bool on, const void* base = nullptr, size_t bytes = 0, float hit_ratio = 0.f);
-bool l2_keep_enabled();
-const cudaAccessPolicyWindow* l2_window();
+
 bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb);
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);

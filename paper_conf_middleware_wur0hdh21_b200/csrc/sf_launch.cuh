@@ -15,20 +15,13 @@ inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute at[2];
-  unsigned na = 0;
+  cudaLaunchAttribute at[1];
   if (pdl_enabled()) {
-    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[na].val.programmaticStreamSerializationAllowed = 1;
-    ++na;
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
   }
-  if (const cudaAccessPolicyWindow* w = l2_window()) {
-    at[na].id = cudaLaunchAttributeAccessPolicyWindow;
-    at[na].val.accessPolicyWindow = *w;
-    ++na;
-  }
-  cfg.attrs = na ? at : nullptr;
-  cfg.numAttrs = na;
   return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
 }
 

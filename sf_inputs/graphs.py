@@ -127,19 +127,24 @@ def mlp_train(widths: Sequence[int] = (784, 256, 10), batch: int = 64, pool: int
 
 
 def mlp_infer(widths: Sequence[int] = (784, 256, 10), batch: int = 1,
-              name: str = "mlp_infer") -> Graph:
-    """Batch-1 inference forward: GEMM -> bias+ReLU -> ... -> softmax."""
+              name: str = "mlp_infer", wt: bool = False) -> Graph:
+    """Batch-1 inference forward: GEMM -> bias+ReLU -> ... -> softmax.
+
+    ``wt``: weights stored output-major, W_i as [N][K] with GEMM flag TB (z = h W_i^T) — the
+    serving layout in which every output is a dot product with one contiguous weight row
+    (reading Q30)."""
     L = len(widths) - 1
     g = Graph(name)
     W, b = [], []
     for i in range(L):
-        W.append(g.add(f"W{i+1}", widths[i], widths[i + 1], F32, PARAM))
+        shape = (widths[i + 1], widths[i]) if wt else (widths[i], widths[i + 1])
+        W.append(g.add(f"W{i+1}", *shape, F32, PARAM))
         b.append(g.add(f"b{i+1}", 1, widths[i + 1], F32, PARAM))
     x = g.add("x", batch, widths[0], F32, INPUT)
     h = x
     for i in range(L):
         z = g.add(f"z{i+1}", batch, widths[i + 1], F32, ACT)
-        g.op(GEMM, [h, W[i]], [z])
+        g.op(GEMM, [h, W[i]], [z], flags=TB if wt else 0)
         last = i == L - 1
         hn = g.add("logits" if last else f"h{i+1}", batch, widths[i + 1], F32, ACT)
         g.op(BIAS_ACT, [z, b[i]], [hn], flags=0 if last else RELU)

@@ -83,6 +83,10 @@ GEMM_SHAPES = [
     # GEMV paths (M <= 8): cluster kernel incl. empty K ranks, K tails, ACC; K/8 > 512 falls back
     (8, 4096, 4096, 0), (4, 12, 13, 0), (1, 4, 1, 0), (5, 1024, 999, ACC), (2, 1000, 4100, 0),
     (3, 516, 64, 0), (1, 2048, 20000, 0),
+    # row-contiguous GEMV (M <= 8, TB): ragged rows per CTA, N < #SMs, K*4 = 32 KB, K % 4 != 0 and
+    # M*K*4 > 64 KB fall back to the tiled path
+    (1, 4096, 2048, TB), (8, 1000, 2048, TB), (3, 17, 8, TB), (1, 1, 4096, TB), (2, 300, 8192, TB),
+    (4, 100, 13, TB), (5, 30, 8192, TB), (1, 1000, 4096, TB | ACC),
 ]
 
 
@@ -122,6 +126,26 @@ def test_gemm_bias_act_vs_oracle(ops, M, N, K, nb, relu):
     assert rel(C.cpu().numpy(), ref) <= TOL
     C2 = torch.full((M, N), 7.0, device="cuda")
     ops.gemm_bias_act(cu(A), cu(B), C2, [cu(b) for b in bs], relu)
+    assert torch.equal(C, C2)
+
+
+GEMV_ROWS_EPI = [(1, 4096, 2048, 1, True), (1, 1000, 4096, 1, False), (8, 260, 784, 3, True),
+                 (2, 7, 1024, 2, True)]
+
+
+@pytest.mark.parametrize("M,N,K,nb,relu", GEMV_ROWS_EPI)
+def test_gemv_rows_bias_act_vs_oracle(ops, M, N, K, nb, relu):
+    """Row-contiguous GEMV (weights [N][K], TB) with the fused bias / ReLU epilogue."""
+    rng = np.random.default_rng(M + 3 * N + K + nb)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    Bt = rng.standard_normal((N, K)).astype(np.float32)
+    bs = [rng.standard_normal((1, N)).astype(np.float32) for _ in range(nb)]
+    ref = O.bias_act(O.gemm(A, Bt, None, TB), bs, relu)
+    C = torch.full((M, N), 7.0, device="cuda")
+    ops.gemm_bias_act(cu(A), cu(Bt), C, [cu(b) for b in bs], relu, TB)
+    assert rel(C.cpu().numpy(), ref) <= TOL
+    C2 = torch.full((M, N), 7.0, device="cuda")
+    ops.gemm_bias_act(cu(A), cu(Bt), C2, [cu(b) for b in bs], relu, TB)
     assert torch.equal(C, C2)
 
 

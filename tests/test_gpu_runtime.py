@@ -464,12 +464,12 @@ def test_remote_slot_errors(P):
 
 
 _INFER_CHILD = r"""
-import sys, numpy as np, torch
+import os, sys, numpy as np, torch
 sys.path.insert(0, '.')
 from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
 from sf_inputs import data as D, graphs as G
 g = G.mlp_train()
-gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths")
+gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths", wt=os.environ.get("WT") == "1")
 rt = Runtime([0], dispatch_spin_us=int(sys.argv[2]))
 gh = rt.register(g); gh.partition(); gh.bind(0, staging=True, host_staging=True)
 gh.load(0, {**D.init_state(g), **D.datasets(g)})
@@ -494,10 +494,14 @@ np.save(sys.argv[1], out.cpu().numpy())
 """
 
 
-@pytest.mark.parametrize("env,spin", [({"SF_CHAIN": "1"}, -1), ({"SF_CHAIN": "1", "SF_PDL": "0"}, 0),
+@pytest.mark.parametrize("env,spin", [({}, -1), ({"SF_CHAIN": "1"}, -1), ({"SF_CHAIN": "1", "SF_PDL": "0"}, 0),
                                       ({"SF_INFER_DIRECT": "0"}, 0), ({"SF_GEMV": "split"}, 2000),
-                                      ({"SF_GEMV": "cluster", "SF_INFER_DIRECT": "0"}, -1)],
-                         ids=["chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv"])
+                                      ({"SF_GEMV": "cluster", "SF_INFER_DIRECT": "0"}, -1),
+                                      ({"WT": "1"}, -1), ({"WT": "1", "SF_INFER_DIRECT": "0"}, 0),
+                                      ({"WT": "1", "SF_FUSE_SOFTMAX": "0", "SF_INFER_REDIRECT": "0",
+                                        "SF_PDL": "0"}, 0)],
+                         ids=["default", "chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv",
+                              "rows", "rows-graphs", "rows-unfused"])
 def test_inference_paths_vs_oracle(env, spin, tmp_path):
     """Every inference launch path (fused chain, PDL direct launches, captured graphs, the
     GEMV variants; device and pinned-host request buffers; spinning and blocking dispatcher)
@@ -508,7 +512,7 @@ def test_inference_paths_vs_oracle(env, spin, tmp_path):
     subprocess.run([sys.executable, "-c", _INFER_CHILD, str(f), str(spin)], cwd=root,
                    env=dict(os.environ, **env), check=True, timeout=240)
     got = np.load(f)
-    gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths")
+    gi = G.mlp_infer((256, 512, 516, 128), name="infer_paths", wt=env.get("WT") == "1")
     sti = D.init_state(gi, seed=D.SEED_INFER)
     xs = D.infer_inputs(gi, 6)
     for r in range(6):

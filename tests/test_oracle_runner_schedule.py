@@ -186,3 +186,15 @@ def test_priority_model_satisfies_invariants():
             SC.check_priority(evs, {0: 0, 1: 1}, {1: (0, t_hi)}, slack=1e-9)
             assert len([e for e in evs if e["job"] == 0]) == 6 * len(lo)
             assert len([e for e in evs if e["job"] == 1]) == 4 * len(hi)
+
+
+def test_inference_weight_layouts_agree():
+    """mlp_infer(wt=True) stores W_i as [N][K] (GEMM TB): with W^T it computes the same forward
+    pass as the [K][N] layout (one rounding per op, so bit-identical)."""
+    g0 = G.mlp_infer((9, 6, 4))
+    g1 = G.mlp_infer((9, 6, 4), wt=True)
+    p0 = D.init_state(g0, seed=2)
+    p1 = {g1.tid(g0.tensors[i].name): (a.T.copy() if g0.tensors[i].name.startswith("W") else a)
+          for i, a in p0.items()}
+    x = D.infer_inputs(g0, 1)[0]
+    assert R.run_inference(g0, p0, x).tobytes() == R.run_inference(g1, p1, x).tobytes()
