@@ -249,7 +249,9 @@ def test_inference_vs_oracle_and_auto_preemption_invariants(P, W):
     SC.check_no_corun(evs)
     SC.check_job_order([e for e in evs if e["kind"] == "train"], {0: n}, start={0: (0, 0)})
     SC.check_cut_rule(evs)
-    SC.check_preempt_latency(evs, slack=2e6)  # ns: host-observed boundaries + gate
+    # ns: host-observed boundaries + gate; the slack absorbs OS scheduling outliers of the
+    # driver / dispatcher threads (typical waits are tens of us)
+    SC.check_preempt_latency(evs, slack=5e6)
 
 
 def test_error_paths(P):
