@@ -127,7 +127,7 @@ def workload_arrays(g, gi, key):
 
 
 def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclusive=True,
-            iteration_granularity=False, measure=True, defer=None):
+            iteration_granularity=False, measure=True, defer=None, duplex=None):
     """One runtime instance: training job + one request per step.  Returns samples."""
     import torch
     from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
@@ -138,7 +138,8 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
                  iteration_granularity=iteration_granularity, max_inflight=args.max_inflight,
                  defer_migration=args.defer if defer is None else defer,
                  dispatch_spin_us=args.dispatch_spin_us,
-                 inflight_budget_us=args.inflight_budget_us)
+                 inflight_budget_us=args.inflight_budget_us,
+                 host_duplex=bool(args.duplex if duplex is None else duplex))
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
                         update_chunks=args.update_chunks)
@@ -252,7 +253,7 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
 
 
 def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
-                    iteration_granularity=False, measure=True, defer=None):
+                    iteration_granularity=False, measure=True, defer=None, duplex=None):
     """C4 as specified: an OPEN-LOOP Poisson request stream (rate args.rate
     req/s, arrival seed 7 + pair) against the running training job.  Each request is submitted
     at its scheduled arrival time (passed to sf_submit_inference, so any host delay counts
@@ -267,7 +268,8 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
                  iteration_granularity=iteration_granularity, max_inflight=args.max_inflight,
                  defer_migration=args.defer if defer is None else defer,
                  dispatch_spin_us=args.dispatch_spin_us,
-                 inflight_budget_us=args.inflight_budget_us)
+                 inflight_budget_us=args.inflight_budget_us,
+                 host_duplex=bool(args.duplex if duplex is None else duplex))
     gh = rt.register(g)
     gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
@@ -578,6 +580,9 @@ def main():
     ap.add_argument("--rate", type=float, default=100.0, help="Poisson arrival rate, req/s")
     ap.add_argument("--defer", type=int, default=1,
                     help="1: migrate after the preempter drained (default); 0: concurrently")
+    ap.add_argument("--duplex", type=int, default=1,
+                    help="1: full-duplex host round trip when nothing waits for the device "
+                         "(default); 0: D2H, then H2D")
     args = ap.parse_args()
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))
@@ -629,10 +634,17 @@ def main():
         co = arm(args, local, nb, 3, host_io=False, exclusive=False, measure=False)
         itg = arm(args, local, nb, 3, host_io=False, iteration_granularity=True, measure=False)
         alt = arm(args, local, nb, 3, host_io=False, measure=False, defer=not args.defer)
+        # the other host round-trip order, per preemption cycle (closed loop, every request preempts)
+        seq = run_arm(args, local, nb, 3, host_io=False, measure=False, duplex=not args.duplex)
         base = {"arrivals": args.arrivals,
                 "free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
                 ("concurrent" if args.defer else "deferred") + "_migration_p99_ms": pct(alt["lat"], 99),
                 ("concurrent" if args.defer else "deferred") + "_migration_p50_ms": pct(alt["lat"], 50),
+                ("sequential" if args.duplex else "duplex") + "_host_round_trip": {
+                    "preempt_to_resume_p50_ms": pct(seq["p2r"], 50),
+                    "preempt_to_resume_p99_ms": pct(seq["p2r"], 99),
+                    "d2h_plus_h2d_us_mean": float(np.mean([x for x in seq["xfer_us"] if x > 0]))
+                    if any(x > 0 for x in seq["xfer_us"]) else None},
                 "iteration_slicing_p99_ms": pct(itg["lat"], 99),
                 "iteration_slicing_p50_ms": pct(itg["lat"], 50)}
 
@@ -721,8 +733,13 @@ def main():
                       "d2h_plus_h2d_us_mean": float(xfer[ok].mean()) if ok.any() else None,
                       "host_link_gbs": migr_gbs,
                       "host_link_peak_gbs": link or None,
-                      "host_link_frac": (migr_gbs / (0.5 * (link["h2d"] + link["d2h"])))
-                      if link and migr_gbs else None,
+                      # roofline time of the round trip over the measured per-direction
+                      # peaks (duplex: the slower direction; sequential: both) / measured
+                      "host_link_frac": (((max if args.duplex else (lambda a, b: a + b))(
+                          1.0 / link["d2h"], 1.0 / link["h2d"]) * byts[ok].mean() / 1e9)
+                          / (xfer[ok].mean() * 1e-6)) if link and migr_gbs else None,
+                      "host_round_trip": "full duplex (chunk c returns H2D as soon as its D2H "
+                      "landed)" if args.duplex else "sequential (D2H, then H2D)",
                       "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},
         "training_subgraph_ms_mean": m0["sub_ms"], "n_subgraphs": m0["n_subgraphs"],
         "training_iteration_ms_median": m0["iter_ms"],

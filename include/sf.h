@@ -180,7 +180,13 @@ typedef struct sf_config {
                                     session-based time slicing, the Gandiva-like baseline of
                                     PAPER.md:1385-1392); 0: feeds prefetch on their own thread
                                     (CPU executors scheduled freely) */
-  int32_t pad0;
+  int32_t host_duplex;           /* 1: a host-tier park that nothing waits for (the device's
+                                    inference queue drained, no higher-priority job present,
+                                    not an explicit sf_preempt) runs its round trip full
+                                    duplex: each 2 MB chunk of the packed staging comes back
+                                    H2D as soon as its D2H landed, so both PCIe directions run
+                                    at once (max(S/d2h, S/h2d) instead of the sum); 0: D2H,
+                                    then H2D */
   uint64_t infer_l2_persist_bytes; /* > 0: reserve this much of each device's L2 (clamped to
                                     cudaDevAttrMaxPersistingL2CacheSize) as a persisting
                                     set-aside for the inference graphs' weights: their request

@@ -57,7 +57,7 @@ class sf_config(C.Structure):
                 ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
                 ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32),
                 ("migration_engine", C.c_int32), ("host_stage_inline", C.c_int32),
-                ("pad0", C.c_int32), ("infer_l2_persist_bytes", C.c_uint64)]
+                ("host_duplex", C.c_int32), ("infer_l2_persist_bytes", C.c_uint64)]
 
 
 class sf_partition_opts(C.Structure):

@@ -142,6 +142,7 @@ struct Graph {
 
 constexpr int kInferOwner = 1 << 20;
 constexpr int kMaxInflight = 4;
+constexpr int kCkEvents = 8;  // per slot: [0, 4) D2H chunk ring, [4, 8) H2D chunk ring
 
 struct Request {
   sf_req_id id;
@@ -211,7 +212,7 @@ struct Job {
   std::thread driver;
   std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
   std::vector<cudaEvent_t> ev_ring;  // [slot * kMaxInflight + i]: in-flight subgraph ends
-  std::vector<cudaEvent_t> ev_ck;    // [slot * 2 + i]: host-tier copy chunks in flight
+  std::vector<cudaEvent_t> ev_ck;    // [slot * kCkEvents + i]: host-tier copy chunks in flight
 };
 
 // Host input stage (sf_create_feed).  Ring slot s holds iteration slot_iter[s]; states:
@@ -933,7 +934,7 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
   J.ev_r.assign(n, nullptr);
   J.ev_ring.assign(n * kMaxInflight, nullptr);
-  J.ev_ck.assign(n * 2, nullptr);
+  J.ev_ck.assign(n * kCkEvents, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
   for (size_t s = 0; s < n; ++s) {
@@ -943,8 +944,8 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
     SF_CK(cudaEventCreateWithFlags(&J.ev_r[s], cudaEventDisableTiming));
     for (int i = 0; i < kMaxInflight; ++i)
       SF_CK(cudaEventCreateWithFlags(&J.ev_ring[s * kMaxInflight + i], cudaEventDisableTiming));
-    for (int i = 0; i < 2; ++i)
-      SF_CK(cudaEventCreateWithFlags(&J.ev_ck[s * 2 + i], cudaEventDisableTiming));
+    for (int i = 0; i < kCkEvents; ++i)
+      SF_CK(cudaEventCreateWithFlags(&J.ev_ck[s * kCkEvents + i], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
     SF_CK(cudaEventCreate(&J.ev_b[s]));
     SF_CK(cudaEventCreate(&J.ev_c[s]));
@@ -1090,13 +1091,13 @@ cudaError_t ce_segments(Job& J, Slot& S, int slot, const std::vector<Seg>& segs,
         if (so == g.n) { ++si; so = 0; }
       }
       cudaError_t e = issue_batch(bd, bs, bn, st);
-      if (e == cudaSuccess && yield) e = cudaEventRecord(J.ev_ck[slot * 2 + (head + n_inflight) % 2], st);
+      if (e == cudaSuccess && yield) e = cudaEventRecord(J.ev_ck[slot * kCkEvents + (head + n_inflight) % 2], st);
       if (e != cudaSuccess) return e;
       if (yield) ++n_inflight;
       continue;
     }
     if (n_inflight > 0) {
-      const cudaError_t q = cudaEventQuery(J.ev_ck[slot * 2 + head]);
+      const cudaError_t q = cudaEventQuery(J.ev_ck[slot * kCkEvents + head]);
       if (q == cudaSuccess) {
         head = (head + 1) % 2;
         --n_inflight;
@@ -1112,6 +1113,76 @@ cudaError_t ce_segments(Job& J, Slot& S, int slot, const std::vector<Seg>& segs,
 cudaError_t yielding_copy(Job& J, Slot& S, int slot, void* dst, const void* src, size_t bytes,
                           cudaStream_t st) {
   return ce_segments(J, S, slot, {Seg{dst, src, bytes}}, st, true);
+}
+
+// Full-duplex host round trip (cfg.host_duplex): when nothing waits for the device at the
+// park, the job need not stay parked, so each 2 MB chunk of the packed staging goes D2H on the
+// migration stream and comes back H2D on the training stream as soon as it landed in pinned
+// memory (a stream-ordered event wait, no host sync).  Both PCIe directions then run at once
+// and the round trip costs max(S/d2h, S/h2d) instead of S/d2h + S/h2d.  With `poison_chunks`
+// each device staging chunk is filled with 0xFF between its D2H and its H2D, so a chunk that
+// does not come back from pinned memory shows up in the unpacked state.  Yields like
+// ce_segments: at most two chunks in flight per direction, none issued while a request is
+// queued or running on the slot.  Returns once every chunk is back in device staging.
+cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t* hstg, size_t total,
+                              bool poison_chunks) {
+  static const size_t kChunk = std::getenv("SF_DUPLEX_CHUNK_KB")
+                                   ? size_t(std::atoi(std::getenv("SF_DUPLEX_CHUNK_KB"))) << 10
+                                   : size_t(2) << 20;
+  static const size_t kDepth = std::getenv("SF_DUPLEX_DEPTH")
+                                   ? size_t(std::max(1, std::min(2, std::atoi(std::getenv("SF_DUPLEX_DEPTH")))))
+                                   : 2;
+  constexpr int R = 4;  // event ring per direction (kCkEvents / 2)
+  const size_t nch = (total + kChunk - 1) / kChunk;
+  size_t nd = 0, nh = 0, cd = 0, ch = 0;  // D2H / H2D issued, D2H / H2D completed
+  cudaEvent_t* evd = &J.ev_ck[slot * kCkEvents];
+  cudaEvent_t* evh = evd + R;
+  auto busy = [&] {
+    const int o = S.owner.load(std::memory_order_acquire);
+    return S.qn.load(std::memory_order_acquire) > 0 || o == kInferOwner;
+  };
+  static const bool quiet = !(std::getenv("SF_DUPLEX_QUIET") && std::getenv("SF_DUPLEX_QUIET")[0] == '0');
+  while (ch < nch) {
+    bool progressed = false;
+    if (quiet && busy()) {
+      // a request is queued or running: no CUDA calls from this thread (driver-lock
+      // contention stretches the dispatcher's launch chain); in-flight chunks drain alone
+      std::this_thread::sleep_for(std::chrono::microseconds(10));
+      continue;
+    }
+    if (!busy()) {
+      if (nd < nch && nd - cd < kDepth && nd - nh < static_cast<size_t>(R)) {
+        const size_t off = nd * kChunk, n = std::min(kChunk, total - off);
+        cudaError_t e = cudaMemcpyAsync(hstg + off, dstg + off, n, cudaMemcpyDeviceToHost, S.s_mig);
+        if (e == cudaSuccess && poison_chunks) e = sfk::launch_fill(dstg + off, n, 0xFF, S.s_mig);
+        if (e == cudaSuccess) e = cudaEventRecord(evd[nd % R], S.s_mig);
+        if (e != cudaSuccess) return e;
+        ++nd;
+        progressed = true;
+      }
+      if (nh < nd && nh - ch < kDepth) {
+        const size_t off = nh * kChunk, n = std::min(kChunk, total - off);
+        cudaError_t e = cudaStreamWaitEvent(S.s_train, evd[nh % R], 0);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(dstg + off, hstg + off, n, cudaMemcpyHostToDevice, S.s_train);
+        if (e == cudaSuccess) e = cudaEventRecord(evh[nh % R], S.s_train);
+        if (e != cudaSuccess) return e;
+        ++nh;
+        progressed = true;
+      }
+    }
+    if (cd < nd) {
+      const cudaError_t q = cudaEventQuery(evd[cd % R]);
+      if (q == cudaSuccess) { ++cd; progressed = true; }
+      else if (q != cudaErrorNotReady) return q;
+    }
+    if (ch < nh) {
+      const cudaError_t q = cudaEventQuery(evh[ch % R]);
+      if (q == cudaSuccess) { ++ch; progressed = true; }
+      else if (q != cudaErrorNotReady) return q;
+    }
+    if (!progressed) for (int i = 0; i < 64; ++i) cpu_relax();
+  }
+  return cudaSuccess;
 }
 
 // Copy-engine-only migration (SF_MIG_CE): the per-tensor segments of cut k.
@@ -1225,18 +1296,36 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     lk.lock();
     J.mig_enqueued = true;
     rt->cv.notify_all();
+    // nothing waits for the device (its queue drained, no higher-priority job present): the
+    // swap-in may start at once, chunk by chunk, while the rest is still going out
+    const bool duplex = rt->cfg.host_duplex && !expl && !repark && !ce && !zc && B.staging &&
+                        !slot_has_inference(rt, src) && S.owner != kInferOwner &&
+                        !higher_training(rt, J, src);
     lk.unlock();
-    if (!repark && !zc &&
-        (e = ce ? ce_segments(J, S, src, cut_segments(g, k, B.arena, B.host_staging, 0), S.s_mig, true)
-                : yielding_copy(J, S, src, B.host_staging, B.staging, g.staging_total[k], S.s_mig)) !=
-            cudaSuccess)
-      return cuda_fail(e, "D2H");
-    cudaEventRecord(J.ev_c[src], S.s_mig);
+    if (duplex) {
+      if ((e = duplex_round_trip(J, S, src, B.staging, B.host_staging, g.staging_total[k],
+                                 rt->cfg.poison_released != 0)) != cudaSuccess)
+        return cuda_fail(e, "duplex D2H/H2D");
+      if (rt->cfg.poison_released) {  // the released arena, before the unpack reads staging
+        if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
+      }
+      cudaEventRecord(J.ev_sub[src], S.s_mig);
+      cudaStreamWaitEvent(S.s_train, J.ev_sub[src], 0);
+      cudaEventRecord(J.ev_c[src], S.s_train);  // round trip complete
+    } else {
+      if (!repark && !zc &&
+          (e = ce ? ce_segments(J, S, src, cut_segments(g, k, B.arena, B.host_staging, 0), S.s_mig, true)
+                  : yielding_copy(J, S, src, B.host_staging, B.staging, g.staging_total[k], S.s_mig)) !=
+              cudaSuccess)
+        return cuda_fail(e, "D2H");
+      cudaEventRecord(J.ev_c[src], S.s_mig);
+    }
     if ((e = wait_event_relaxed(J.ev_c[src])) != cudaSuccess) return cuda_fail(e, "pack wait");
     float pack_us = repark || ce ? 0.f : static_cast<float>(tstamp_us(S.tstamp));  // kernel-only duration
     if (pack_us < 0.f) pack_us = elapsed_us(J.ev_a[src], J.ev_b[src]);
+    // duplex: the whole round trip (both directions overlapped), else the D2H alone
     const float d2h_us = repark ? 0.f : elapsed_us(J.ev_b[src], J.ev_c[src]);
-    if (rt->cfg.poison_released) {
+    if (rt->cfg.poison_released && !duplex) {
       if ((e = poison(B, S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison");
       if ((e = cudaStreamSynchronize(S.s_mig)) != cudaSuccess) return cuda_fail(e, "poison sync");
     }
@@ -1255,7 +1344,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       if (!J.resume_req) { J.state = SF_JOB_DONE; rt->cv.notify_all(); return SF_OK; }
       dst = J.resume_dev;
       J.resume_req = false;
-    } else {
+    } else if (!duplex) {
       // swap back in once the device's inference queue drained (reading Q4/Q13) and no
       // higher-priority training job is present on it
       rt->cv.wait(lk, [&] {
@@ -1271,7 +1360,11 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     // the parked bytes live in the source binding's pinned staging; a ZC swap-in reads
     // them in place when resuming on the same slot, otherwise H2D + unpack
     tstamp_reset(D.tstamp + 2, D.s_train);
-    if (ce) {
+    if (duplex) {  // the H2D already ran (its time is in xfer_us): unpack only
+      cudaEventRecord(J.ev_b[dst], D.s_train);
+      const CopyList& L = BD.unpack[k];
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
+    } else if (ce) {
       e = ce_segments(J, D, dst, cut_segments(g, k, BD.arena, B.host_staging, 1), D.s_train, true);
       cudaEventRecord(J.ev_b[dst], D.s_train);
     } else if (zc && dst == src) {
@@ -2022,7 +2115,7 @@ void sf_destroy(sf_runtime* rt) {
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_r[s]);
       for (int i = 0; i < kMaxInflight; ++i) cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
-    for (int i = 0; i < 2; ++i) cudaEventDestroy(J->ev_ck[s * 2 + i]);
+      for (int i = 0; i < kCkEvents; ++i) cudaEventDestroy(J->ev_ck[s * kCkEvents + i]);
       cudaEventDestroy(J->ev_a[s]);
       cudaEventDestroy(J->ev_b[s]);
       cudaEventDestroy(J->ev_c[s]);

@@ -403,6 +403,26 @@ def test_host_modes_and_deferred_migration_bitwise(P, host_mode, defer):
     assert_bitwise(base, got)
 
 
+@pytest.mark.parametrize("defer", [0, 1])
+def test_duplex_host_round_trip_bitwise(P, defer):
+    """Full-duplex host round trip (host_duplex): chunk c comes back H2D as soon as its D2H
+    landed, with the device staging chunk poisoned in between and the released arena
+    poisoned before the unpack.  A ~70 MB live set spans ~35 chunks.  The trajectory equals
+    the unpreempted run bit for bit, and the parked pinned bytes equal those of a sequential
+    (D2H, then H2D) round trip of the same schedule."""
+    g = G.mlp_train((2048, 4096, 10), batch=64, pool=4)
+    base, _, _, _, _ = run_gpu(P, g, 8, slots=1)
+    sched = [(2, k, HOST) for k in range(5)] + [(5, 2, HOST)]
+    got, _, info, _, hs = run_gpu(P, g, 8, schedule=sched, slots=1, poison=True,
+                                  defer_migration=bool(defer), host_duplex=True)
+    assert info["n_preemptions"] == 6
+    assert_bitwise(base, got)
+    _, _, info_s, _, hs_s = run_gpu(P, g, 8, schedule=sched, slots=1, poison=True,
+                                    defer_migration=bool(defer), host_duplex=False)
+    assert info_s["n_preemptions"] == 6
+    assert hs.tobytes() == hs_s.tobytes()  # same parks in the same order: same pinned bytes
+
+
 def _run_with_requests(P, g, gi, n_req, **kw):
     RT, A = P
     rt, gh, st, ds = setup(P, g, slots=1, **kw)
@@ -521,8 +541,8 @@ def test_inference_paths_vs_oracle(env, spin, tmp_path):
         assert rel(got[r], R.run_inference(gi, sti, xs[r])) <= TOL, (env, r)
 
 
-@pytest.mark.parametrize("defer", [True, False])
-def test_open_loop_requests_during_swap_in_are_bitwise(P, defer):
+@pytest.mark.parametrize("defer,duplex", [(True, False), (False, False), (True, True)])
+def test_open_loop_requests_during_swap_in_are_bitwise(P, defer, duplex):
     """Open-loop request stream (arrivals independent of the job's state): requests land
     while the parked state is being swapped back in, so the job is re-preempted before it
     ran anything (re-park without pack / D2H) or while its H2D + unpack is still in flight
@@ -532,7 +552,8 @@ def test_open_loop_requests_during_swap_in_are_bitwise(P, defer):
     iters = 12
     base = run_gpu(P, g, iters, slots=1)[0]
     RT, A = P
-    rt, gh, st, ds = setup(P, g, slots=1, poison=True, defer_migration=defer, dispatch_spin_us=-1)
+    rt, gh, st, ds = setup(P, g, slots=1, poison=True, defer_migration=defer, dispatch_spin_us=-1,
+                           host_duplex=duplex)
     gi = G.mlp_infer((256, 512, 12))
     ghi = rt.register(gi, priority=1)
     ghi.partition()
