@@ -127,7 +127,8 @@ def workload_arrays(g, gi, key):
 
 
 def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclusive=True,
-            iteration_granularity=False, measure=True, defer=None, duplex=None):
+            iteration_granularity=False, measure=True, defer=None, duplex=None,
+            early=None):
     """One runtime instance: training job + one request per step.  Returns samples."""
     import torch
     from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
@@ -139,7 +140,8 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
                  defer_migration=args.defer if defer is None else defer,
                  dispatch_spin_us=args.dispatch_spin_us,
                  inflight_budget_us=args.inflight_budget_us,
-                 host_duplex=bool(args.duplex if duplex is None else duplex))
+                 host_duplex=bool(args.duplex if duplex is None else duplex),
+                 early_launch=bool(args.early if early is None else early))
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
                         update_chunks=args.update_chunks)
@@ -253,7 +255,8 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
 
 
 def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
-                    iteration_granularity=False, measure=True, defer=None, duplex=None):
+                    iteration_granularity=False, measure=True, defer=None, duplex=None,
+            early=None):
     """C4 as specified: an OPEN-LOOP Poisson request stream (rate args.rate
     req/s, arrival seed 7 + pair) against the running training job.  Each request is submitted
     at its scheduled arrival time (passed to sf_submit_inference, so any host delay counts
@@ -269,7 +272,8 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
                  defer_migration=args.defer if defer is None else defer,
                  dispatch_spin_us=args.dispatch_spin_us,
                  inflight_budget_us=args.inflight_budget_us,
-                 host_duplex=bool(args.duplex if duplex is None else duplex))
+                 host_duplex=bool(args.duplex if duplex is None else duplex),
+                 early_launch=bool(args.early if early is None else early))
     gh = rt.register(g)
     gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
@@ -353,7 +357,26 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
             print(f"[diag] {name:15s} n={len(sel):4d} wait us p50/p99 {np.median(w):7.1f}/{np.percentile(w, 99):7.1f}"
                   f"  device us p50/p99 {np.median(dv):6.1f}/{np.percentile(dv, 99):6.1f}"
                   f"  total p50/p99 {np.median(tot):6.1f}/{np.percentile(tot, 99):6.1f}", file=sys.stderr)
+    # where a request's latency goes: wait for the device (drain of the preempted job's
+    # in-flight subgraphs, or an earlier request), device time of the chain, host overhead
+    # (dispatch decision .. first event on the device, last kernel .. completion observed)
+    bd = {}
+    for name, sel in (("preempting", [t for t in T if t["preempted_job"] == job]),
+                      ("not_preempting", [t for t in T if t["preempted_job"] != job])):
+        sel = [t for t in sel if t["device_us"] > 0]
+        if not sel:
+            continue
+        w = np.array([(t["start_ns"] - t["arrival_ns"]) * 1e-3 for t in sel])
+        dv = np.array([t["device_us"] for t in sel])
+        ho = np.array([(t["end_ns"] - t["start_ns"]) * 1e-3 - t["device_us"] for t in sel])
+        lu = np.array([t["launch_us"] for t in sel])
+        du = np.array([t["dispatch_us"] for t in sel])
+        bd[name] = {"n": len(sel), **{f"{k}_p{q}": round(float(np.percentile(v, q)), 2)
+                                       for k, v in (("wait", w), ("device", dv), ("host_overhead", ho),
+                                                    ("launch", lu), ("dispatch", du))
+                                       for q in (50, 99)}}
     return {"lat": lat, "pre": pre, "p2r": p2r, "frac_preempting": len(pre) / max(1, len(T)),
+            "breakdown": bd,
             "device_us": dev_us, "region_ms": ev0.elapsed_time(ev1), "wall_s": wall,
             "launches": launches, "clocks": sampler.summary() if sampler else None,
             "reparks": info_j["n_reparks"], "iters_done": len(per_it)}
@@ -583,6 +606,9 @@ def main():
     ap.add_argument("--duplex", type=int, default=1,
                     help="1: full-duplex host round trip when nothing waits for the device "
                          "(default); 0: D2H, then H2D")
+    ap.add_argument("--early", type=int, default=1,
+                    help="1: a preempting request is enqueued behind a device-side wait on the "
+                         "job's in-flight subgraphs (default); 0: launched after the drain")
     args = ap.parse_args()
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))
@@ -636,6 +662,8 @@ def main():
         alt = arm(args, local, nb, 3, host_io=False, measure=False, defer=not args.defer)
         # the other host round-trip order, per preemption cycle (closed loop, every request preempts)
         seq = run_arm(args, local, nb, 3, host_io=False, measure=False, duplex=not args.duplex)
+        # the other preempter launch policy (same arrivals)
+        lat_other = arm(args, local, nb, 3, host_io=False, measure=False, early=not args.early)
         base = {"arrivals": args.arrivals,
                 "free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
                 ("concurrent" if args.defer else "deferred") + "_migration_p99_ms": pct(alt["lat"], 99),
@@ -645,6 +673,9 @@ def main():
                     "preempt_to_resume_p99_ms": pct(seq["p2r"], 99),
                     "d2h_plus_h2d_us_mean": float(np.mean([x for x in seq["xfer_us"] if x > 0]))
                     if any(x > 0 for x in seq["xfer_us"]) else None},
+                ("launch_after_drain" if args.early else "early_launch"): {
+                    "p99_ms": pct(lat_other["lat"], 99), "p50_ms": pct(lat_other["lat"], 50),
+                    "preempt_latency_p99_ms": pct(lat_other["pre"], 99)},
                 "iteration_slicing_p99_ms": pct(itg["lat"], 99),
                 "iteration_slicing_p50_ms": pct(itg["lat"], 50)}
 
@@ -693,7 +724,28 @@ def main():
                 e0.record(); dst.copy_(src, non_blocking=True); e1.record(); e1.synchronize()
                 best = max(best, hb.numel() / (e0.elapsed_time(e1) * 1e-3) / 1e9)
             link[name] = best
-        del hb, db
+        # both directions at once (two streams): the platform's full-duplex total
+        hb2 = torch.empty_like(hb).pin_memory()
+        db2 = torch.empty_like(db)
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        best = 0.0
+        for _ in range(4):
+            torch.cuda.synchronize()
+            e0, e1, e2 = torch.cuda.Event(True), torch.cuda.Event(True), torch.cuda.Event(True)
+            e0.record()
+            s1.wait_event(e0)
+            s2.wait_event(e0)
+            with torch.cuda.stream(s1):
+                db.copy_(hb, non_blocking=True)
+                e1.record(s1)
+            with torch.cuda.stream(s2):
+                hb2.copy_(db2, non_blocking=True)
+                e2.record(s2)
+            e1.synchronize(); e2.synchronize()
+            t = max(e0.elapsed_time(e1), e0.elapsed_time(e2)) * 1e-3
+            best = max(best, 2 * hb.numel() / t / 1e9)
+        link["duplex_total"] = best
+        del hb, db, hb2, db2
     except Exception:
         link = {}
     dev_us = pct(main_s.get("device_us", []), 50)
@@ -711,6 +763,7 @@ def main():
                    "max_inflight": args.max_inflight,
                    "dispatch_spin_us": args.dispatch_spin_us,
                    "inflight_budget_us": args.inflight_budget_us,
+                   "early_launch": bool(args.early), "host_duplex": bool(args.duplex),
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets > 126 MB L2 (no flush needed)"},
@@ -720,7 +773,8 @@ def main():
         "arrivals": {"process": args.arrivals, "rate_per_s": args.rate if args.arrivals == "poisson" else None,
                      "seed": "7 + pair" if args.arrivals == "poisson" else "1234 + device",
                      "frac_preempting": main_s.get("frac_preempting"), "reparks": main_s.get("reparks"),
-                     "inference_device_us_p50": pct(main_s.get("device_us", []), 50)},
+                     "inference_device_us_p50": pct(main_s.get("device_us", []), 50),
+                     "latency_breakdown_us": main_s.get("breakdown")},
         "poisson_1000": hi_rate,
         "chase": {"desc": "closed loop: every request preempts the running job; next request after its resume",
                   "p50_ms": pct(Cc["lat"], 50), "p99_ms": pct(Cc["lat"], 99),
@@ -735,9 +789,11 @@ def main():
                       "host_link_peak_gbs": link or None,
                       # roofline time of the round trip over the measured per-direction
                       # peaks (duplex: the slower direction; sequential: both) / measured
-                      "host_link_frac": (((max if args.duplex else (lambda a, b: a + b))(
-                          1.0 / link["d2h"], 1.0 / link["h2d"]) * byts[ok].mean() / 1e9)
-                          / (xfer[ok].mean() * 1e-6)) if link and migr_gbs else None,
+                      "host_link_frac": ((max(1.0 / link["d2h"], 1.0 / link["h2d"],
+                                              2.0 / link["duplex_total"]) if args.duplex
+                                          else 1.0 / link["d2h"] + 1.0 / link["h2d"])
+                                         * byts[ok].mean() / 1e9 / (xfer[ok].mean() * 1e-6))
+                      if link and migr_gbs else None,
                       "host_round_trip": "full duplex (chunk c returns H2D as soon as its D2H "
                       "landed)" if args.duplex else "sequential (D2H, then H2D)",
                       "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},

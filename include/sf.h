@@ -194,6 +194,16 @@ typedef struct sf_config {
                                     tag weight TMA loads evict_last, so the collocated training
                                     job's streaming traffic cannot evict them (Q29);
                                     0 = off */
+  int32_t early_launch;          /* 1: a request that preempts the job owning the device is
+                                    enqueued as soon as the job's driver can dispatch nothing
+                                    more, behind a stream-ordered wait on the job's newest
+                                    in-flight subgraph: the host launches overlap the drain
+                                    and the chain starts on the GPU the moment the dispatched
+                                    kernels finish; trace events of such
+                                    requests carry the job in `iter` (invariant 1 through the
+                                    device dependency); ignored with iteration_granularity;
+                                    0: launch after the drain was observed on the host */
+  int32_t pad1;
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,
@@ -424,6 +434,7 @@ typedef struct sf_timing {
                             copy), CUDA events on the inference stream */
   float launch_us;       /* host time the dispatcher took to issue the chain (first event
                             record .. last launch returned) */
+  float dispatch_us;     /* host time from the dispatch decision to the first enqueue */
 } sf_timing;
 
 /* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).
@@ -446,6 +457,8 @@ typedef struct sf_trace_event {
   uint64_t t0_ns, t1_ns;       /* host CLOCK_MONOTONIC: launch .. completion observed */
   uint64_t arrival_ns;         /* inference: scheduled arrival; train: host dispatch time
                                   (<= t0 when queued behind an in-flight predecessor) */
+  /* inference: iter = -1, or the training job whose subgraphs dispatched before t0 this
+     request was ordered after on the device (early_launch); t0 is then its dispatch time */
 } sf_trace_event;
 sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* n_out);
 uint64_t sf_now_ns(void); /* CLOCK_MONOTONIC */

@@ -29,7 +29,9 @@ trace or the GPU runtime's recorded one):
       its submission (the outstanding subgraphs drain, nothing more).
 
 Event dicts: {"dev", "job", "kind": "train"|"infer", "iter", "k", "t0", "t1",
-"arrival" (infer only)}; times in any consistent unit.
+"arrival" (infer only), "after" (infer only, optional: the training job it was ordered
+after on the device), "launch" (train only, optional: dispatch time)}; times in any
+consistent unit.
 
 Pins (tests/test_oracle_schedule.py): hand-built violating traces for I1..I4 are
 rejected; the discrete-event model's traces satisfy them; closed-form latencies of
@@ -45,17 +47,36 @@ class InvariantError(AssertionError):
     pass
 
 
+def _device_ordered(a: dict, b: dict) -> bool:
+    """True when one of two overlapping HOST intervals is an inference event that the GPU
+    ran after the other, a training subgraph: the request carries ``after`` = that job
+    (its chain waited, on the device, for the job's newest subgraph dispatched before the
+    request's own dispatch t0 — stream order covers every earlier one) and the subgraph
+    was dispatched ("launch", else t0) no later than the request.  Host intervals are
+    supersets of device execution, so only such a dependency makes an overlap legal."""
+    for r, t in ((a, b), (b, a)):
+        if (r["kind"] == "infer" and t["kind"] == "train" and r.get("after") == t["job"]
+                and t.get("launch", t["t0"]) <= r["t0"]):
+            return True
+    return False
+
+
 def check_no_corun(events: Sequence[dict]) -> None:
-    """I1: per device, intervals of different jobs never overlap."""
+    """I1: per device, intervals of different jobs never overlap (unless device-ordered,
+    see _device_ordered)."""
     by_dev: Dict[int, List[dict]] = {}
     for e in events:
         by_dev.setdefault(e["dev"], []).append(e)
     for d, evs in by_dev.items():
         evs = sorted(evs, key=lambda e: (e["t0"], e["t1"]))
-        for a, b in zip(evs, evs[1:]):
-            if a["job"] != b["job"] and b["t0"] < a["t1"]:
-                raise InvariantError(f"dev {d}: job {a['job']} [{a['t0']},{a['t1']}) overlaps "
-                                     f"job {b['job']} [{b['t0']},{b['t1']})")
+        active: List[dict] = []
+        for b in evs:
+            active = [a for a in active if a["t1"] > b["t0"]]
+            for a in active:
+                if a["job"] != b["job"] and not _device_ordered(a, b):
+                    raise InvariantError(f"dev {d}: job {a['job']} [{a['t0']},{a['t1']}) overlaps "
+                                         f"job {b['job']} [{b['t0']},{b['t1']})")
+            active.append(b)
 
 
 def check_job_order(events: Sequence[dict], n_sub: Dict[int, int],

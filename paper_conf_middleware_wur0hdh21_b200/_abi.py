@@ -57,7 +57,8 @@ class sf_config(C.Structure):
                 ("device_budget_bytes", C.c_uint64), ("dispatch_spin_us", C.c_int32),
                 ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32),
                 ("migration_engine", C.c_int32), ("host_stage_inline", C.c_int32),
-                ("host_duplex", C.c_int32), ("infer_l2_persist_bytes", C.c_uint64)]
+                ("host_duplex", C.c_int32), ("infer_l2_persist_bytes", C.c_uint64),
+                ("early_launch", C.c_int32), ("pad1", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):
@@ -89,7 +90,7 @@ class sf_timing(C.Structure):
     _fields_ = [("arrival_ns", C.c_uint64), ("start_ns", C.c_uint64), ("end_ns", C.c_uint64),
                 ("dev", C.c_int32), ("preempted_job", C.c_int32), ("cut_iter", C.c_int64),
                 ("cut_k", C.c_int32), ("device_us", C.c_float),
-                ("launch_us", C.c_float)]
+                ("launch_us", C.c_float), ("dispatch_us", C.c_float)]
 
 
 class sf_trace_event(C.Structure):

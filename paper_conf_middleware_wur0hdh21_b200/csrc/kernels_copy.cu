@@ -153,7 +153,10 @@ cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
   static const uint64_t min_chunks =
       std::getenv("SF_COPY_MINCHUNKS") ? std::atoll(std::getenv("SF_COPY_MINCHUNKS")) : 2048;
   uint64_t blocks = (total_chunks + min_chunks - 1) / min_chunks;
-  blocks = std::min<uint64_t>(blocks, 148ull * bps);
+  // waves > 1: CTAs are short-lived, so a higher-priority stream's kernel (a preempter
+  // arriving mid-migration) gets SMs after one wave instead of after the whole walk
+  static const int waves = std::getenv("SF_COPY_WAVES") ? std::max(1, std::atoi(std::getenv("SF_COPY_WAVES"))) : 1;
+  blocks = std::min<uint64_t>(blocks, 148ull * bps * waves);
   blocks = std::max<uint64_t>(blocks, 1);
   const uint64_t per_block = (total_chunks + blocks - 1) / blocks;
   blocks = (total_chunks + per_block - 1) / per_block;

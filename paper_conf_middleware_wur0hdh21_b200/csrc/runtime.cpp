@@ -157,6 +157,7 @@ struct Request {
   int cut_k = -1;
   float device_us = -1.f;
   float launch_us = -1.f;
+  float dispatch_us = -1.f;  // dispatch decision .. first enqueue (host)
   std::string error;
 };
 
@@ -194,6 +195,12 @@ struct Job {
   bool cut_ready = false;
   bool mig_enqueued = false;
   bool holds_token = false;
+  // early launch (cfg.early_launch): the driver is between its gate check and the
+  // registration of a launched subgraph (runtime lock released); last_ev = completion event
+  // of the newest in-flight subgraph, n_inflight = subgraphs on the device
+  bool launching = false;
+  cudaEvent_t last_ev = nullptr;
+  int n_inflight = 0;
   sf_cut_info cut{};
   bool resume_req = false;
   int resume_dev = -1;
@@ -1719,6 +1726,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       sfk::count_launch(g.bind[dev]->version_kernels[k]);
       Feed* F = k == 0 ? g.feed : nullptr;
       const int fslot = F ? static_cast<int>(it % F->depth) : -1;
+      J.launching = true;  // until the launch below is registered (early-launch handshake)
       if (F && F->inline_mode && !(F->slot_state[fslot] == 2 && F->slot_iter[fslot] == it)) {
         // session-slicing baseline: the CPU stage runs now, while the job holds the device
         F->slot_state[fslot] = 1;
@@ -1729,6 +1737,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         const uint64_t h1 = now_ns();
         lk.lock();
         if (!err.empty()) {
+          J.launching = false;
           release();
           J.error = "host stage: " + err;
           J.state = SF_JOB_FAILED;
@@ -1759,6 +1768,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
       if (e == cudaSuccess) e = cudaEventRecord(J.ev_ring[dev * kMaxInflight + ev], S.s_train);
       lk.lock();
+      J.launching = false;
       if (e != cudaSuccess) {
         release();
         J.error = std::string("subgraph launch: ") + cudaGetErrorString(e);
@@ -1767,6 +1777,9 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         break;
       }
       q.push_back({it, k, dev, ev, t0, stamp});
+      J.last_ev = J.ev_ring[dev * kMaxInflight + ev];
+      J.n_inflight = static_cast<int>(q.size());
+      if (S.qn.load(std::memory_order_acquire) > 0) rt->cv.notify_all();  // a waiting dispatcher
       if (++J.k == n) {
         J.k = 0;
         ++J.it;
@@ -1813,6 +1826,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     lk.lock();
     q.pop_front();
+    J.n_inflight = static_cast<int>(q.size());
     if (f.k == 0 && g.feed) feed_consumed(*g.feed, f.it, g.feed_member);
     if (f.stamp) {
       J.last_resume = t_res;  // host-observed device resume (CLOCK_MONOTONIC)
@@ -1854,14 +1868,33 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     const int o = S->owner.load(std::memory_order_acquire);
     return !excl || o == -1 || o == kInferOwner;
   };
-  auto ready = [&] { return rt->shutting_down || (!S->q.empty() && free_for_inference()); };
+  // Early launch (cfg.early_launch): the request need not wait on the host for the training
+  // job's in-flight subgraphs to drain.  Once the job's driver can dispatch nothing more (its
+  // boundary gate sees the queued request, and it is not inside a launch), the dispatcher
+  // takes the device token and enqueues the chain behind a stream-ordered wait on the job's
+  // newest in-flight subgraph: the GPU starts the preempter the moment the preemptee's
+  // dispatched kernels finish, and the launches overlap that drain ("the preparation of the
+  // new job overlaps the abort of the preempted one").  No subgraph of the
+  // two models co-runs on the device (invariant 1 holds through the device dependency; the
+  // trace records it, oracle/schedule.py I1).  Not with iteration-granularity slicing.
+  const bool early = excl && rt->cfg.early_launch && !rt->cfg.iteration_granularity;
+  auto steal_from = [&]() -> Job* {  // rt->m held
+    if (!early) return nullptr;
+    const int o = S->owner.load(std::memory_order_acquire);
+    if (o < 0 || o >= kInferOwner || static_cast<size_t>(o) >= rt->jobs.size()) return nullptr;
+    Job* J = rt->jobs[o].get();
+    return J && !J->launching && J->dev == S->id ? J : nullptr;
+  };
+  auto ready = [&] {
+    return rt->shutting_down || (!S->q.empty() && (free_for_inference() || steal_from() != nullptr));
+  };
   while (true) {
     if (!ready() && spin_us != 0) {
       // busy-poll (no futex wake-up on the request path) for dispatch_spin_us, -1 = forever
       const uint64_t deadline = spin_us < 0 ? ~0ull : now_ns() + static_cast<uint64_t>(spin_us) * 1000;
       lk.unlock();
       while (!rt->stop_spin.load(std::memory_order_relaxed) && now_ns() < deadline) {
-        if (S->qn.load(std::memory_order_acquire) > 0 && free_for_inference()) break;
+        if (S->qn.load(std::memory_order_acquire) > 0 && (early || free_for_inference())) break;
         for (int i = 0; i < 32; ++i) cpu_relax();
       }
       lk.lock();
@@ -1869,8 +1902,19 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     rt->cv.wait(lk, ready);
     if (S->q.empty() && rt->shutting_down) break;
     if (S->q.empty()) continue;
-    if (rt->cfg.exclusive_gpu) S->owner = kInferOwner;
     Request* r = S->q.front();
+    Job* dep = free_for_inference() ? nullptr : steal_from();
+    cudaEvent_t dep_ev = nullptr;
+    if (dep) {
+      dep_ev = dep->n_inflight > 0 ? dep->last_ev : nullptr;
+      dep->holds_token = false;  // the job re-acquires the token before its next launch
+      if (r->preempted_job < 0) {
+        r->preempted_job = static_cast<int>(dep->id);
+        r->cut_iter = dep->it;  // the launch cursor: where the job stops
+        r->cut_k = dep->k;
+      }
+    }
+    if (rt->cfg.exclusive_gpu) S->owner = kInferOwner;
     Graph& g = *r->g;
     Binding* B = g.bind[S->id].get();
     const uint64_t t0 = now_ns();
@@ -1918,7 +1962,10 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     };
     const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
     const uint64_t tl0 = now_ns();
-    e = cudaEventRecord(S->ev_i0, S->s_infer);
+    // early launch: the chain (and its start event) wait on the device for the job's
+    // dispatched subgraphs; the driver dispatches nothing more while the request is queued
+    if (dep_ev) e = cudaStreamWaitEvent(S->s_infer, dep_ev, 0);
+    if (e == cudaSuccess) e = cudaEventRecord(S->ev_i0, S->s_infer);
     if (e != cudaSuccess || in_place) {
     } else if (aligned) {
       e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
@@ -1959,10 +2006,13 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       cudaGetLastError();
     }
     lk.lock();
-    r->start = t0;
+    // an early-launched chain starts on the device when the job's drain completes: its start
+    // is taken as completion - device time (never earlier than the true device start)
+    r->start = dep && dev_ms >= 0.f ? std::max(t0, t1 - static_cast<uint64_t>(dev_ms * 1e6f)) : t0;
     r->end = t1;
     r->device_us = dev_ms >= 0.f ? dev_ms * 1e3f : -1.f;
     r->launch_us = static_cast<float>((tl1 - tl0) * 1e-3);
+    r->dispatch_us = static_cast<float>((tl0 - t0) * 1e-3);
     if (e != cudaSuccess) r->error = op_err.empty() ? cudaGetErrorString(e) : op_err;
     r->done = true;
     S->q.pop_front();
@@ -1970,6 +2020,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     sf_trace_event ev{};
     ev.dev = S->id; ev.job = static_cast<int32_t>(kInferOwner | (r->id & 0xFFFFF)); ev.kind = SF_EV_INFER;
     ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
+    ev.iter = dep ? static_cast<int64_t>(dep->id) : -1;  // device-ordered after that job's dispatched subgraphs
     push_trace(rt, ev);
     if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
     rt->cv.notify_all();
@@ -2765,6 +2816,7 @@ sf_status sf_wait(sf_runtime* rt, sf_req_id id, int64_t timeout_ns, sf_timing* t
     t->cut_k = r->cut_k;
     t->device_us = r->device_us;
     t->launch_us = r->launch_us;
+    t->dispatch_us = r->dispatch_us;
   }
   std::string err = r->error;
   rt->reqs.erase(it);

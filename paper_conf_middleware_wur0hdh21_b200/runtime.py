@@ -140,14 +140,15 @@ class Runtime:
                  dispatch_spin_us: int = 0, inflight_budget_us: int = 0,
                  migrate_home: bool = False, migration_engine: int = 0,
                  host_stage_inline: bool = False, infer_l2_persist_bytes: int = 0,
-                 host_duplex: bool = False):
+                 host_duplex: bool = False, early_launch: bool = False):
         self.ordinals = list(ordinals)
         arr = (C.c_int32 * len(self.ordinals))(*self.ordinals)
         cfg = A.sf_config(len(self.ordinals), arr, int(exclusive), int(auto_preempt),
                           int(iteration_granularity), host_mode, int(poison), trace_capacity,
                           max_inflight, int(defer_migration), budget_bytes, dispatch_spin_us,
                           inflight_budget_us, int(migrate_home), migration_engine,
-                          int(host_stage_inline), int(host_duplex), infer_l2_persist_bytes)
+                          int(host_stage_inline), int(host_duplex), infer_l2_persist_bytes,
+                          int(early_launch), 0)
         h = C.c_void_p()
         check(lib().sf_create(C.byref(cfg), C.byref(h)), "sf_create")
         self.h = h
@@ -273,6 +274,8 @@ class Runtime:
                  "t0": e.t0_ns, "t1": e.t1_ns}
             if kind == "infer":
                 d["arrival"] = e.arrival_ns
+                if e.iter >= 0:
+                    d["after"] = e.iter  # device-ordered after that job's dispatched subgraphs
             elif kind == "train":
                 d["launch"] = e.arrival_ns
             out.append(d)

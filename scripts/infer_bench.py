@@ -10,7 +10,7 @@ rt = Runtime([0], dispatch_spin_us=int(os.environ.get("SPIN", "0")),
              infer_l2_persist_bytes=int(float(os.environ.get("L2P_MB", "0")) * (1 << 20)))
 ghi = rt.register(gi, 1); ghi.partition(); ghi.bind(0, staging=False); ghi.load(0, arrs_i)
 x = torch.rand(1, 2048, device="cuda"); out = torch.empty(1, 1000, device="cuda")
-lat, pre, dev = [], [], []
+lat, pre, dev, ho, lu = [], [], [], [], []
 gap = float(os.environ.get("GAP_MS", "0")) * 1e-3
 if os.environ.get("COPY"):  # background copy-engine traffic like a host-tier migration
     import threading
@@ -18,14 +18,20 @@ if os.environ.get("COPY"):  # background copy-engine traffic like a host-tier mi
     hdst = torch.empty(227 << 20, dtype=torch.uint8).pin_memory()
     cs = torch.cuda.Stream()
     stop_copy = False
+    cs2 = torch.cuda.Stream()
+    dsrc2 = torch.empty_like(dsrc)
+    hdst2 = torch.empty_like(hdst).pin_memory()
     def bg():
         while not globals()["stop_copy"]:
-            with torch.cuda.stream(cs):
-                if os.environ.get("COPY") == "h2d":
+            mode = os.environ.get("COPY")
+            if mode in ("h2d", "duplex"):
+                with torch.cuda.stream(cs):
                     dsrc.copy_(hdst, non_blocking=True)
-                else:
-                    hdst.copy_(dsrc, non_blocking=True)
+            if mode in ("d2h", "duplex"):
+                with torch.cuda.stream(cs2):
+                    hdst2.copy_(dsrc2, non_blocking=True)
             cs.synchronize()
+            cs2.synchronize()
     th = threading.Thread(target=bg, daemon=True)
     th.start()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if os.environ.get("FLUSH") else None
@@ -43,6 +49,8 @@ for i in range(int(sys.argv[1]) if len(sys.argv) > 1 else 300):
         lat.append((tm["end_ns"] - tm["arrival_ns"]) * 1e-6)
         pre.append((tm["start_ns"] - tm["arrival_ns"]) * 1e-6)
         dev.append(tm["device_us"] * 1e-3)
+        ho.append((tm["end_ns"] - tm["start_ns"]) * 1e-3 - tm["device_us"])
+        lu.append(tm["launch_us"])
 if os.environ.get("COPY"):
     stop_copy = True
     th.join()
@@ -52,4 +60,7 @@ print(json.dumps({"l2p_mb": os.environ.get("L2P_MB", "0"), "flush": bool(flush i
                   if hasattr(torch.cuda.get_device_properties(0), "persisting_l2_cache_max_size") else None,
                   "p50_ms": float(np.median(lat)), "p99_ms": float(np.percentile(lat, 99)),
                   "min_ms": float(np.min(lat)), "wake_p50_ms": float(np.median(pre)),
-                  "device_p50_ms": float(np.median(dev))}))
+                  "device_p50_ms": float(np.median(dev)), "device_p99_ms": float(np.percentile(dev, 99)),
+                  "copy": os.environ.get("COPY"), "spin": os.environ.get("SPIN", "0"),
+                  "host_overhead_us_p50": float(np.median(ho)), "host_overhead_us_p99": float(np.percentile(ho, 99)),
+                  "launch_us_p50": float(np.median(lu))}))

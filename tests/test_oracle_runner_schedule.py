@@ -67,6 +67,31 @@ def test_checker_rejects_corun():
     SC.check_no_corun([_ev(0, 0, "train", 0, 10), _ev(1, 1, "infer", 5, 7, arrival=4)])
 
 
+def test_checker_device_ordered_overlap():
+    """An early-launched request (dispatched while job 0's subgraph was still in flight,
+    ordered after it on the device) may overlap that subgraph's host interval; a subgraph
+    of the job dispatched after the request, or another job's, may not."""
+    tr = _ev(0, 0, "train", 0, 10)
+    tr["launch"] = 0
+    r = _ev(0, 1 << 20, "infer", 5, 30, arrival=4)
+    r["after"] = 0
+    SC.check_no_corun([tr, r])
+    late = dict(tr, t0=6, t1=12, launch=6, k=1)  # dispatched after the request
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun([tr, r, late])
+    other = dict(tr, job=2)
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun([other, r])
+    plain = dict(r)
+    del plain["after"]
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun([tr, plain])
+    # a non-adjacent overlap (long subgraph, short one inside) is still found
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun([_ev(0, 0, "train", 0, 100), _ev(0, 0, "train", 1, 2, k=1),
+                           _ev(0, 3, "train", 50, 60)])
+
+
 def test_checker_rejects_order_gap_and_duplicate():
     ok = [_ev(0, 0, "train", i, i + 1, it=i // 3, k=i % 3) for i in range(7)]
     SC.check_job_order(ok, {0: 3})
