@@ -556,6 +556,7 @@ constexpr int kGvCluster = 8;
 constexpr int kGvRows = 32;            // rows per TMA box
 constexpr int kGvRing = 64 * 1024;     // bytes of W in flight per CTA
 constexpr int kGvMaxKper = 1024;       // x slice staged in smem (K <= 8192)
+constexpr int kGvPrefetch = 8;         // l2_hint flag: prefetch the W slice into L2 up front
 
 template <int MR, int BC>
 struct GvCfg {
@@ -608,12 +609,18 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
   if (warp == 8) {
     if ((tid & 31) == 0) {
       if (!b_const) sfdev::griddep_wait();  // W may be written by the predecessor
-      const uint64_t pol = sfdev::l2_policy(l2_hint);
+      const int hint = l2_hint & 3;
+      const uint64_t pol = sfdev::l2_policy(hint);
+      if (l2_hint & kGvPrefetch) {
+        // the whole slice beyond the ring goes to L2 now: DRAM works ahead of the ring (and,
+        // under PDL, while the predecessor layer drains); the ring's loads then hit L2
+        for (int i = S; i < nbox; ++i) sfdev::tma_prefetch_2d(&tmW, c0, k0 + i * kGvRows);
+      }
       for (int i = 0; i < nbox; ++i) {
         const int slot = i % S;
         if (i >= S) sfdev::mbar_wait(&empty[slot], ((i / S) - 1) & 1);
         expect_tx(&full[slot], Cfg::BOX);
-        if (l2_hint)  // keep (persisting set-aside) / stream (evict first) the weights
+        if (hint)  // keep (persisting set-aside) / stream (evict first) the weights
           sfdev::tma_load_2d_hint(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]),
                                   c0, k0 + i * kGvRows, pol);
         else
@@ -1084,6 +1091,13 @@ cudaError_t dispatch_major(bool a_mn, bool b_mn, const CUtensorMap& a, const CUt
 }
 
 
+// SF_GEMV_PF=1: prefetch each CTA's weight slice into L2 up front (measured: 46 -> 50 us on
+// the C4 chain with a dirty cold L2, 38.4 -> 40 us warm; off by default, Q33)
+bool gemv_prefetch() {
+  static const bool on = std::getenv("SF_GEMV_PF") && std::getenv("SF_GEMV_PF")[0] == '1';
+  return on;
+}
+
 template <int MR, int BC>
 cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cudaStream_t st) {
   auto kern = gemv_tma_kernel<MR, BC>;
@@ -1102,7 +1116,7 @@ cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cud
   count_launch();
   return launch_k(kern, dim3(grid), dim3(288), smem, st, w, a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc,
                   kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
-                  a.b_const ? 1 : 0, a.l2_hint, a.sm_out, a.sm_ldo,
+                  a.b_const ? 1 : 0, a.l2_hint | (gemv_prefetch() ? kGvPrefetch : 0), a.sm_out, a.sm_ldo,
                   a.sm_counter);
 }
 

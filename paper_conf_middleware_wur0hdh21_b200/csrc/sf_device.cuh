@@ -152,6 +152,11 @@ __device__ __forceinline__ float4 ldg4_hint(const float4* p, uint64_t policy) {
                : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(policy));
   return v;
 }
+// 2-D tensor tile -> L2 only (no smem, no completion): warms L2 ahead of the TMA loads.
+__device__ __forceinline__ void tma_prefetch_2d(const void* tmap, int x, int y) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];"
+               :: "l"(reinterpret_cast<uint64_t>(tmap)), "r"(x), "r"(y) : "memory");
+}
 // 0 -> no hint; 1 -> evict_last; 2 -> evict_first
 __device__ __forceinline__ uint64_t l2_policy(int hint) {
   return hint == 1 ? policy_evict_last() : policy_evict_first();

@@ -122,7 +122,12 @@ class RuntimeOps:
 
     def request(self) -> dict:
         import time
-        self._poll(lambda i: i["state_name"] == "running", "job not running")
+        i0 = self._poll(lambda i: i["state_name"] == "running", "job not running")
+        # the job holds the device once its launch cursor moved (a request arriving before
+        # that finds the device free and preempts nothing)
+        key0 = (i0["iter"], i0["k"])
+        self._poll(lambda i: i["state_name"] == "running" and (i["iter"], i["k"]) != key0,
+                   "job not advancing")
         t_arr = time.perf_counter() + self.rng.uniform(0.2, 1.0) * self.sub_ms * 2e-3
         while time.perf_counter() < t_arr:
             pass

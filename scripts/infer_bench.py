@@ -35,9 +35,13 @@ if os.environ.get("COPY"):  # background copy-engine traffic like a host-tier mi
     th = threading.Thread(target=bg, daemon=True)
     th.start()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if os.environ.get("FLUSH") else None
+rflush = torch.ones(512 << 20, dtype=torch.uint8, device="cuda") if os.environ.get("FLUSH") == "r" else None
 import time
 for i in range(int(sys.argv[1]) if len(sys.argv) > 1 else 300):
-    if flush is not None:
+    if rflush is not None:  # clean cold L2: read-only sweep of 512 MB
+        rflush.view(torch.int64).sum()
+        torch.cuda.synchronize()
+    elif flush is not None:  # dirty cold L2: 256 MB of writes
         flush.fill_(i & 255)
         torch.cuda.synchronize()
     if gap:
@@ -55,7 +59,7 @@ if os.environ.get("COPY"):
     stop_copy = True
     th.join()
 rt.close()
-print(json.dumps({"l2p_mb": os.environ.get("L2P_MB", "0"), "flush": bool(flush is not None),
+print(json.dumps({"l2p_mb": os.environ.get("L2P_MB", "0"), "flush": os.environ.get("FLUSH"),
                   "max_persist_mb": torch.cuda.get_device_properties(0).persisting_l2_cache_max_size / 2**20
                   if hasattr(torch.cuda.get_device_properties(0), "persisting_l2_cache_max_size") else None,
                   "p50_ms": float(np.median(lat)), "p99_ms": float(np.percentile(lat, 99)),
