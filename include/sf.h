@@ -477,7 +477,9 @@ typedef struct sf_copy_desc {
 /* descs: HOST array [n].  patch_iter >= 0: overwrite bytes [16, 24) of descriptor 0's
  * destination with patch_iter (the staging header's iter field). */
 sf_status sf_op_mtcopy(const sf_copy_desc* descs, int32_t n, int64_t patch_iter, void* stream);
-/* C = op(A) op(B) (+C); lda/ldb/ldc = row strides (elements) of the stored matrices. */
+/* C = op(A) op(B) (+C); lda/ldb/ldc = row strides (elements) of the stored matrices.
+ * Split-K shapes use a runtime-owned workspace cached per (device, stream) and grown on
+ * demand (never freed before process exit); calls on one stream share it in stream order. */
 sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N,
                      int32_t K, int32_t lda, int32_t ldb, int32_t ldc, int32_t flags,
                      void* stream);

@@ -309,9 +309,16 @@ struct Plan {
   int bn, splits, kb_per_split, tiles_n, tiles_m;
 };
 
-Plan plan_gemm(int M, int N, int K) {
+// SF_GEMM_BN256=1: 128x256 tiles (TMA path) for N >= 256 — half the A-operand smem reads per
+// flop of the 3 MMAs; 2 pipeline stages fit (96 KB per stage)
+bool gemm_bn256() {
+  static const bool on = std::getenv("SF_GEMM_BN256") && std::getenv("SF_GEMM_BN256")[0] == '1';
+  return on;
+}
+
+Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
   Plan pl;
-  pl.bn = N <= 64 ? 64 : 128;
+  pl.bn = force_bn ? force_bn : N <= 64 ? 64 : 128;
   pl.tiles_n = (N + pl.bn - 1) / pl.bn;
   pl.tiles_m = (M + BM - 1) / BM;
   const int tiles = pl.tiles_n * pl.tiles_m;
@@ -660,7 +667,12 @@ uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb) {
     return g.splits > 1 ? static_cast<uint64_t>(g.splits) * M * N : 0;
   }
   Plan pl = plan_gemm(M, N, K);
-  return pl.splits > 1 ? static_cast<uint64_t>(pl.splits) * M * N : 0;
+  uint64_t w = pl.splits > 1 ? static_cast<uint64_t>(pl.splits) * M * N : 0;
+  if (gemm_bn256() && N >= 256) {
+    const Plan p2 = plan_gemm(M, N, K, 256);
+    if (p2.splits > 1) w = std::max<uint64_t>(w, static_cast<uint64_t>(p2.splits) * M * N);
+  }
+  return w;
 }
 
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
@@ -752,6 +764,11 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   // explicitly masked hi on B200, scripts/rawhi_check.py); SF_GEMM_RAWHI=0 masks explicitly.
   static const bool raw_hi = !(std::getenv("SF_GEMM_RAWHI") && std::getenv("SF_GEMM_RAWHI")[0] == '0');
   const bool legacy = path && std::string(path) == "legacy";
+  if (!legacy && raw_hi && gemm_bn256() && a.N >= 256) {
+    const Plan p2 = plan_gemm(a.M, a.N, a.K, 256);
+    if ((p2.splits == 1 || (a.ws && a.counters)) && gemm_tma_eligible(a, p2.splits))
+      return launch_gemm_tma(a, 256, p2.splits, p2.kb_per_split, p2.tiles_n, p2.tiles_m, raw_hi, st);
+  }
   if (!legacy && gemm_tma_eligible(a, pl.splits))
     return launch_gemm_tma(a, pl.bn, pl.splits, pl.kb_per_split, pl.tiles_n, pl.tiles_m, raw_hi, st);
   Params p;

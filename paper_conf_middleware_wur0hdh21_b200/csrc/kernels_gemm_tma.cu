@@ -41,7 +41,7 @@ constexpr int kThreads = 10 * 32;
 
 template <int BN>
 struct TCfg {
-  static constexpr int STAGES = BN == 64 ? 4 : 3;
+  static constexpr int STAGES = BN == 64 ? 4 : BN == 128 ? 3 : 2;
   static constexpr int A_BYTES = BM * BK * 4;
   static constexpr int B_BYTES = BN * BK * 4;
   static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
@@ -1282,7 +1282,7 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   // persistent CTAs (double-buffered TMEM) measured equal to per-tile CTAs on the forest
   // shapes (profiles/r01_ncu_summary.md); opt in with SF_GEMM_PERSISTENT=1
   static const bool persistent = std::getenv("SF_GEMM_PERSISTENT") && std::getenv("SF_GEMM_PERSISTENT")[0] == '1';
-  if (persistent && raw_hi) {
+  if (persistent && raw_hi && bn != 256) {
     PParams pp{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, tiles_n, tiles_m,
                tiles_n * tiles_m * splits, a.C};
     e = bn == 64 ? dispatch_persistent<64>(a_mn, b_mn, ma, mb, mc, pp, st)
@@ -1290,6 +1290,8 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   } else if (bn == 64)
     e = raw_hi ? dispatch_major<64, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<64, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
+  else if (bn == 256)
+    e = dispatch_major<256, true>(a_mn, b_mn, ma, mb, mc, p, grid, st);
   else
     e = raw_hi ? dispatch_major<128, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<128, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);

@@ -1149,6 +1149,9 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
     return S.qn.load(std::memory_order_acquire) > 0 || o == kInferOwner;
   };
   static const bool quiet = !(std::getenv("SF_DUPLEX_QUIET") && std::getenv("SF_DUPLEX_QUIET")[0] == '0');
+  // SF_DUPLEX_HOSTORDER=1: issue H2D(c) once the host saw D2H(c) complete (no cross-engine
+  // event wait on the device)
+  static const bool host_order = std::getenv("SF_DUPLEX_HOSTORDER") && std::getenv("SF_DUPLEX_HOSTORDER")[0] == '1';
   while (ch < nch) {
     bool progressed = false;
     if (quiet && busy()) {
@@ -1167,9 +1170,9 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
         ++nd;
         progressed = true;
       }
-      if (nh < nd && nh - ch < kDepth) {
+      if (nh < (host_order ? cd : nd) && nh - ch < kDepth) {
         const size_t off = nh * kChunk, n = std::min(kChunk, total - off);
-        cudaError_t e = cudaStreamWaitEvent(S.s_train, evd[nh % R], 0);
+        cudaError_t e = host_order ? cudaSuccess : cudaStreamWaitEvent(S.s_train, evd[nh % R], 0);
         if (e == cudaSuccess) e = cudaMemcpyAsync(dstg + off, hstg + off, n, cudaMemcpyHostToDevice, S.s_train);
         if (e == cudaSuccess) e = cudaEventRecord(evh[nh % R], S.s_train);
         if (e != cudaSuccess) return e;
@@ -2878,19 +2881,30 @@ static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, in
   cudaStream_t st = as_stream(stream);
   const uint64_t wsf = sfk::gemm_workspace_floats(M, N, K, ga.ta, ga.tb);
   const uint64_t cs = sfk::gemm_counter_slots(M, N, K, ga.ta, ga.tb);
-  void* ws = nullptr;
-  void* cnt = nullptr;
   if (wsf) {
-    SF_CK(cudaMallocAsync(&ws, wsf * 4, st));
-    SF_CK(cudaMallocAsync(&cnt, cs * 4, st));
-    SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
-    ga.ws = static_cast<float*>(ws);
-    ga.counters = static_cast<unsigned*>(cnt);
-  }
-  SF_CK(sfk::launch_gemm(ga, st));
-  if (ws) {
-    SF_CK(cudaFreeAsync(ws, st));
-    SF_CK(cudaFreeAsync(cnt, st));
+    // split-K workspace + reduction counters cached per (device, stream) and grown on demand
+    // (stream-ordered free of the old buffers); the counters reset themselves after every
+    // reduction, so they are zeroed once, at allocation
+    struct OpWs { float* ws = nullptr; unsigned* cnt = nullptr; uint64_t wsf = 0, cs = 0; };
+    static std::mutex m;
+    static std::map<std::pair<int, cudaStream_t>, OpWs> cache;
+    int dev = 0;
+    SF_CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> g(m);
+    OpWs& w = cache[{dev, st}];
+    if (w.wsf < wsf || w.cs < cs) {
+      if (w.ws) { SF_CK(cudaFreeAsync(w.ws, st)); SF_CK(cudaFreeAsync(w.cnt, st)); }
+      w.wsf = std::max(w.wsf, wsf);
+      w.cs = std::max(w.cs, cs);
+      SF_CK(cudaMallocAsync(reinterpret_cast<void**>(&w.ws), w.wsf * 4, st));
+      SF_CK(cudaMallocAsync(reinterpret_cast<void**>(&w.cnt), w.cs * 4, st));
+      SF_CK(cudaMemsetAsync(w.cnt, 0, w.cs * 4, st));
+    }
+    ga.ws = w.ws;
+    ga.counters = w.cnt;
+    SF_CK(sfk::launch_gemm(ga, st));
+  } else {
+    SF_CK(sfk::launch_gemm(ga, st));
   }
   if (epi && !fuse) {
     if (ldc != N) return fail(SF_EINVAL, "unfused gemm epilogue needs ldc == N");
