@@ -157,8 +157,8 @@ def c1():
     g = G.mlp_train()
     st, ds = D.init_state(g), D.datasets(g)
     rows = []
-    for k in range(5):
-        with Runtime([0]) as rt:
+    for k, dx in [(k, dx) for dx in (False, True) for k in range(5)]:
+        with Runtime([0], host_duplex=dx) as rt:
             gh = rt.register(g)
             gh.partition()
             gh.bind(0, host_staging=True)
@@ -166,7 +166,7 @@ def c1():
             job = rt.start_training(gh, 0, 60, HOST, schedule=[(50, k, HOST)])
             rt.wait_job(job, 60)
             ji = rt.job_info(job)
-            rows.append({"k": k, "live_bytes": gh.live_set(k)[1], "pack_us": ji["last_pack_us"],
+            rows.append({"k": k, "host_duplex": dx, "live_bytes": gh.live_set(k)[1], "pack_us": ji["last_pack_us"],
                          "d2h_h2d_us": ji["last_xfer_us"], "unpack_us": ji["last_unpack_us"],
                          "preempt_to_resume_us": (ji["last_resume_ns"] - ji["last_stop_ns"]) * 1e-3})
     print(json.dumps({"c1": rows}), flush=True)
