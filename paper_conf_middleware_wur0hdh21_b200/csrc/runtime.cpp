@@ -971,11 +971,19 @@ cudaError_t spin_event(cudaEvent_t ev) {
 // Millisecond-scale waits (host-tier D2H / H2D, peer stores) poll with short sleeps: a
 // tight cudaEventQuery loop on this thread contends for the CUDA driver's locks with the
 // dispatcher's kernel launches and stretches the preempter's launch chain.
+// The first ~100 us are polled with short pauses: a sleep costs the OS timer slack (tens of
+// us, often more), which dominated the preempt-to-resume of small live sets (C1: two relaxed
+// waits per host round trip).
 cudaError_t wait_event_relaxed(cudaEvent_t ev) {
+  const uint64_t spin_until = now_ns() + 100000;
   for (;;) {
     cudaError_t e = cudaEventQuery(ev);
     if (e != cudaErrorNotReady) return e;
-    std::this_thread::sleep_for(std::chrono::microseconds(20));
+    if (now_ns() < spin_until) {
+      for (int i = 0; i < 256; ++i) cpu_relax();
+    } else {
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+    }
   }
 }
 
