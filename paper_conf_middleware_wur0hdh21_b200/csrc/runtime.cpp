@@ -1595,16 +1595,25 @@ void driver_main(sf_runtime* rt, Job* Jp) {
   std::deque<Inflight> q;
   // device-time estimate per subgraph (EMA of host-observed busy intervals); with
   // inflight_budget_us > 0 a subgraph is queued behind others only while the queued work
-  // stays within the budget, which bounds the drain a preemption waits for
+  // stays within the budget, which bounds the drain a preemption waits for.  The budget is
+  // time-aware: the front subgraph counts only its estimated REMAINING time (it started at
+  // front_start, when its predecessor was seen to finish, or at its dispatch), so the next one
+  // is queued while the front still runs instead of after a host round trip.
   std::vector<double> est_us(n, 0.0);
   const double budget_us = rt->cfg.inflight_budget_us;
+  uint64_t front_start = 0;  // host estimate of the front's device start (0: unknown)
   auto queued_us = [&] {
     double t = 0.0;
     for (const auto& f : q) t += est_us[f.k];
+    if (!q.empty() && front_start) {
+      const double el = (now_ns() - front_start) * 1e-3;
+      t -= std::min(est_us[q.front().k], std::max(0.0, el));
+    }
     return t;
   };
   int ev_next = 0;
   uint64_t last_t1 = 0;
+  int64_t broke_for = -1;  // front (it * n + k) whose wait was left early once
   std::unique_lock<std::mutex> lk(rt->m);
   bool pending_peer_stats = false;
   int stats_slot = -1;
@@ -1787,6 +1796,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         rt->cv.notify_all();
         break;
       }
+      if (q.empty()) front_start = t0;
       q.push_back({it, k, dev, ev, t0, stamp});
       J.last_ev = J.ev_ring[dev * kMaxInflight + ev];
       J.n_inflight = static_cast<int>(q.size());
@@ -1808,16 +1818,34 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     // retire the oldest in-flight subgraph
     const Inflight f = q.front();
     Slot& S = slot_of(rt, f.dev);
+    // time-aware budget: leave the wait (once per front) when the next subgraph fits the
+    // budget while the front is still running; the gate at the top decides under the lock
+    const bool may_break = budget_us > 0.0 && static_cast<int>(q.size()) < W && !J.preempt_req &&
+                           J.it < J.iters && !J.stop_req && !(g.feed && J.k == 0) &&
+                           broke_for != (f.it * n + f.k);
     lk.unlock();
     cudaSetDevice(S.cuda);
     uint64_t t_res = 0;
     cudaError_t e = cudaSuccess;
+    bool broke = false;
     for (;;) {
       if (f.stamp && !t_res && cudaEventQuery(J.ev_r[f.dev]) == cudaSuccess) t_res = now_ns();
       const cudaError_t qq = cudaEventQuery(J.ev_ring[f.dev * kMaxInflight + f.ev]);
-      if (qq == cudaErrorNotReady) continue;
+      if (qq == cudaErrorNotReady) {
+        if (may_break && S.qn.load(std::memory_order_relaxed) == 0 &&
+            queued_us() + est_us[J.k] <= budget_us) {
+          broke = true;
+          break;
+        }
+        continue;
+      }
       e = qq;
       break;
+    }
+    if (broke) {
+      broke_for = f.it * n + f.k;
+      lk.lock();
+      continue;
     }
     const uint64_t t1 = now_ns();
     if (f.stamp && !t_res) t_res = t1;
@@ -1862,6 +1890,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     tev.arrival_ns = f.t0;  // train events: host dispatch (launch) time
     last_t1 = t1;
+    front_start = q.empty() ? 0 : std::max(q.front().t0, t1);
     push_trace(rt, tev);
     // iteration-granularity (session time slicing baseline) keeps the device for the whole
     // iteration; otherwise an empty window is a scheduling point
