@@ -51,7 +51,7 @@ struct TCfg {
 
 struct TParams {
   int M, N, K, ldc;
-  int splits, kb_per_split, acc, dbg;
+  int splits, kb_per_split, acc, dbg, stages;
   float* C;
   float* ws;
   unsigned* counters;
@@ -112,13 +112,14 @@ __global__ void __launch_bounds__(kThreads, 1)
 gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, TParams p) {
   using C = TCfg<BN>;
+  const int NS = p.stages;  // ring depth (<= C::STAGES; 2 for short K: two CTAs per SM)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~static_cast<uintptr_t>(1023));
-  uint64_t* tma_full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
-  uint64_t* conv_full = tma_full + C::STAGES;
-  uint64_t* empty = conv_full + C::STAGES;
-  uint64_t* done = empty + C::STAGES;
+  uint64_t* tma_full = reinterpret_cast<uint64_t*>(smem + NS * C::STAGE_BYTES);
+  uint64_t* conv_full = tma_full + NS;
+  uint64_t* empty = conv_full + NS;
+  uint64_t* done = empty + NS;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(done + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -128,7 +129,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   const int nkb = max(0, min(nkb_total, kb_begin + p.kb_per_split) - kb_begin);
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < C::STAGES; ++s) {
+    for (int s = 0; s < NS; ++s) {
       sfdev::mbar_init(&tma_full[s], 1);
       sfdev::mbar_init(&conv_full[s], kConvWarps);
       sfdev::mbar_init(&empty[s], 1);
@@ -148,7 +149,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   if (warp == 0) {
     if (lane == 0) {
       for (int i = 0; i < nkb; ++i) {
-        const int s = i % C::STAGES, round = i / C::STAGES;
+        const int s = i % NS, round = i / NS;
         if (round > 0) sfdev::mbar_wait(&empty[s], (round - 1) & 1);
         const uint32_t st = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
         const uint32_t bar = sfdev::smem_u32(&tma_full[s]);
@@ -172,8 +173,8 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   } else if (warp <= kConvWarps) {
     const int t = threadIdx.x - 32;  // 0..255
     for (int i = 0; i < nkb; ++i) {
-      const int s = i % C::STAGES;
-      sfdev::mbar_wait(&tma_full[s], (i / C::STAGES) & 1);
+      const int s = i % NS;
+      sfdev::mbar_wait(&tma_full[s], (i / NS) & 1);
       uint8_t* st = smem + s * C::STAGE_BYTES;
       float4* a = reinterpret_cast<float4*>(st);
       float4* alo = reinterpret_cast<float4*>(st + C::A_BYTES);
@@ -191,8 +192,8 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
                                ((B_MN ? 1u : 0u) << 16) | (uint32_t(BN >> 3) << 17) |
                                (uint32_t(BM >> 4) << 24);
     for (int i = 0; i < nkb; ++i) {
-      const int s = i % C::STAGES;
-      sfdev::mbar_wait(&conv_full[s], (i / C::STAGES) & 1);
+      const int s = i % NS;
+      sfdev::mbar_wait(&conv_full[s], (i / NS) & 1);
       sfdev::tc_fence_after();
       if (lane == 0) {
         const uint32_t base = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
@@ -1048,7 +1049,8 @@ cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUten
     if (e != cudaSuccess) return e;
     configured.fetch_or(bit);
   }
-  kern<<<grid, kThreads, TCfg<BN>::SMEM, st>>>(a, b, c, p);
+  const int smem = p.stages * TCfg<BN>::STAGE_BYTES + 1024 + 256;
+  kern<<<grid, kThreads, smem, st>>>(a, b, c, p);
   count_launch();
   return cudaGetLastError();
 }
@@ -1276,7 +1278,16 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
                           : map3d_ws(&mc, a.ws, a.N, a.M, splits));
   if (!ok) return cudaErrorInvalidValue;
   static const int dbg = std::getenv("SF_GEMM_DEBUG") ? std::atoi(std::getenv("SF_GEMM_DEBUG")) : 0;
-  TParams p{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, dbg, a.C, a.ws, a.counters};
+  // ring depth: with more 128x64 tiles than SMs (no split-K), 2 stages let two CTAs share an SM, so
+  // the grid runs in half the waves and one CTA's prologue / epilogue overlaps the other's
+  // loads (tall forest GEMMs: 100352x64x148 41.9 -> 29.7 us, 25088x64x576 33.7 -> 27.6 us;
+  // split-K shapes keep the deep ring).  SF_GEMM_STAGES overrides.
+  static const int stages_env = std::getenv("SF_GEMM_STAGES") ? std::atoi(std::getenv("SF_GEMM_STAGES")) : -1;
+  const int max_stages = bn == 64 ? TCfg<64>::STAGES : bn == 128 ? TCfg<128>::STAGES : TCfg<256>::STAGES;
+  int stages = max_stages;
+  if (stages_env > 0) stages = std::min(stages_env, max_stages);
+  else if (bn == 64 && splits == 1 && tiles_n * tiles_m > 148) stages = 2;  // 2 x 97 KB fit an SM
+  TParams p{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, dbg, stages, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;
   // persistent CTAs (double-buffered TMEM) measured equal to per-tile CTAs on the forest
