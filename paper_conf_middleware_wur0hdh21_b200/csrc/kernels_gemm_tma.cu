@@ -180,8 +180,10 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       float4* alo = reinterpret_cast<float4*>(st + C::A_BYTES);
       float4* b = reinterpret_cast<float4*>(st + 2 * C::A_BYTES);
       float4* blo = reinterpret_cast<float4*>(st + 2 * C::A_BYTES + C::B_BYTES);
-      split_tile<C::A_BYTES / 16 / 256, RAW_HI>(a, alo, t);
-      split_tile<C::B_BYTES / 16 / 256, RAW_HI>(b, blo, t);
+      if (!(p.dbg & 2)) {  // dbg bit 1 (probe only, wrong results): skip the split
+        split_tile<C::A_BYTES / 16 / 256, RAW_HI>(a, alo, t);
+        split_tile<C::B_BYTES / 16 / 256, RAW_HI>(b, blo, t);
+      }
       sfdev::fence_proxy_async_smem();
       __syncwarp();
       if (lane == 0) sfdev::mbar_arrive(&conv_full[s]);
@@ -205,9 +207,11 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
           const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
           auto da = [&](uint32_t x) { return A_MN ? desc_mn(x + ao) : desc_k(x + ao); };
           auto db = [&](uint32_t x) { return B_MN ? desc_mn(x + bo) : desc_k(x + bo); };
-          sfdev::mma_tf32(tmem, da(a_lo), db(b_hi), idesc, (i | kk) != 0);
-          sfdev::mma_tf32(tmem, da(a_hi), db(b_lo), idesc, 1u);
-          sfdev::mma_tf32(tmem, da(a_hi), db(b_hi), idesc, 1u);
+          if (!(p.dbg & 4)) {  // dbg bit 2 (probe only, wrong results): hi.hi MMA alone
+            sfdev::mma_tf32(tmem, da(a_lo), db(b_hi), idesc, (i | kk) != 0);
+            sfdev::mma_tf32(tmem, da(a_hi), db(b_lo), idesc, 1u);
+          }
+          sfdev::mma_tf32(tmem, da(a_hi), db(b_hi), idesc, (p.dbg & 4) ? ((i | kk) != 0) : 1u);
         }
         sfdev::mma_commit(&empty[s]);
       }
