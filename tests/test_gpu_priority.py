@@ -160,9 +160,12 @@ def test_equal_priority_jobs_share_a_slot_at_subgraph_granularity(P):
                        start={ja: (0, 0), jb: (0, 0)})
 
 
-def test_inference_still_preempts_both_priorities(P):
+@pytest.mark.parametrize("early,W", [(False, 1), (True, 2)])
+def test_inference_still_preempts_both_priorities(P, early, W):
     """Inference ranks above every training job (reading Q13): with a high-priority job
-    running and the low-priority one parked, requests still cut the high-priority job."""
+    running and the low-priority one parked, requests still cut the high-priority job.
+    With early_launch the requests are enqueued behind the job's in-flight subgraphs on the
+    device; the trace must still show no co-running except through that dependency."""
     RT, A = P
     import torch
     g_lo, g_hi = _graphs()
@@ -171,7 +174,7 @@ def test_inference_still_preempts_both_priorities(P):
     xs = D.infer_inputs(gi, 8)
     base_lo = _solo(P, g_lo, 20, LO_SEED)
     base_hi = _solo(P, g_hi, 400, HI_SEED)
-    with RT.Runtime([0], poison=True) as rt:
+    with RT.Runtime([0], poison=True, early_launch=early, max_inflight=W) as rt:
         gl, st_lo = _setup(RT, g_lo, rt, 0, 1, LO_SEED)
         gH, st_hi = _setup(RT, g_hi, rt, 1, 1, HI_SEED)
         ghi = rt.register(gi, priority=2)
