@@ -665,3 +665,49 @@ def test_gelu_mlp_trajectory_vs_oracle_and_preempted_bitwise(P):
     got, _, info, _, _ = run_gpu(P, g, 12, schedule=sched, poison=True)
     assert info["n_preemptions"] >= 8
     assert_bitwise(base, got)
+
+
+@pytest.mark.parametrize("early", [False, True])
+def test_requests_chase_peer_migrations_bitwise(P, early):
+    """Auto-preemption to a peer slot: requests are submitted to the slot the job runs on.
+    The first one migrates the job to slot 1 through the peer-store walk (poisoned released
+    arena); it stays there, so later requests cut it at a boundary and it
+    yields in place.  With early_launch the chain waits on the device for the job's
+    dispatched subgraphs.  Final state bit-identical to the unpreempted run; requests within
+    1e-4 of the oracle; invariant 1 on the trace."""
+    import time
+    g = G.mlp_train((784, 512, 10), batch=64, pool=4)
+    gi = G.mlp_infer()
+    iters = 1500
+    base = run_gpu(P, g, iters, slots=1)[0]
+    RT, A = P
+    rt, gh, st, ds = setup(P, g, slots=2, poison=True, early_launch=early, max_inflight=2,
+                           dispatch_spin_us=-1)
+    ghi = rt.register(gi, priority=1)
+    ghi.partition()
+    sti = D.init_state(gi, seed=D.SEED_INFER)
+    for s in range(2):
+        ghi.bind(s, staging=False)
+        ghi.load(s, sti)
+    xs = D.infer_inputs(gi, 6)
+    xin = torch.from_numpy(xs).cuda()
+    out = torch.zeros(6, 1, 10, device="cuda")
+    job = rt.start_training(gh, 0, iters, 1)
+    tims = []
+    for r in range(6):
+        time.sleep(0.002)
+        info = rt.job_info(job)
+        if info["state_name"] != "running":
+            break
+        tims.append(rt.wait(rt.submit(ghi, info["dev"], xin[r].data_ptr(), out[r].data_ptr()), 30))
+    rt.wait_job(job, 120)
+    info = rt.job_info(job)
+    got = {i: gh.read(info["dev"], i) for i in st}
+    trace = [e for e in rt.trace() if e["kind"] in ("train", "infer")]
+    rt.close()
+    assert info["n_preemptions"] >= 1 and info["dev"] == 1, info
+    assert_bitwise(base, got)
+    assert len(tims) >= 3
+    for r in range(len(tims)):
+        assert rel(out[r].cpu().numpy(), R.run_inference(gi, sti, xs[r])) <= TOL
+    SC.check_no_corun(trace)
