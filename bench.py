@@ -128,7 +128,7 @@ def workload_arrays(g, gi, key):
 
 def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclusive=True,
             iteration_granularity=False, measure=True, defer=None, duplex=None,
-            early=None):
+            early=None, target=HOST):
     """One runtime instance: training job + one request per step.  Returns samples."""
     import torch
     from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
@@ -162,7 +162,7 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
         x_t = torch.from_numpy(xs).to(dev)
         out_t = torch.zeros(len(xs), 1, 1000, device=dev)
     rng = np.random.default_rng(1234 + local_dev)
-    job = rt.start_training(gh, 0, 1 << 40, HOST)
+    job = rt.start_training(gh, 0, 1 << 40, target)
     # estimate the mean training-subgraph duration from the trace (for arrival jitter)
     time.sleep(0.3)
     tr = [e for e in rt.trace() if e["kind"] == "train"]
@@ -256,7 +256,7 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
 
 def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
                     iteration_granularity=False, measure=True, defer=None, duplex=None,
-            early=None):
+            early=None, target=HOST):
     """C4 as specified: an OPEN-LOOP Poisson request stream (rate args.rate
     req/s, arrival seed 7 + pair) against the running training job.  Each request is submitted
     at its scheduled arrival time (passed to sf_submit_inference, so any host delay counts
@@ -292,7 +292,7 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
     else:
         x_t = torch.from_numpy(xs).to(dev)
         out_t = torch.zeros(len(xs), 1, 1000, device=dev)
-    job = rt.start_training(gh, 0, 1 << 40, HOST)
+    job = rt.start_training(gh, 0, 1 << 40, target)
     time.sleep(0.3)
     rng = np.random.default_rng(7 + args.rank // 2)
     gaps_ns = (rng.exponential(1.0 / args.rate, n_in) * 1e9).astype(np.int64)
@@ -664,6 +664,9 @@ def main():
         seq = run_arm(args, local, nb, 3, host_io=False, measure=False, duplex=not args.duplex)
         # the other preempter launch policy (same arrivals)
         lat_other = arm(args, local, nb, 3, host_io=False, measure=False, early=not args.early)
+        # no migration at all: the job stops at the boundary and waits in place (what the host
+        # tier costs the requests that arrive during its round trip)
+        inplace = arm(args, local, nb, 3, host_io=False, measure=False, target=0)
         base = {"arrivals": args.arrivals,
                 "free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
                 ("concurrent" if args.defer else "deferred") + "_migration_p99_ms": pct(alt["lat"], 99),
@@ -676,6 +679,8 @@ def main():
                 ("launch_after_drain" if args.early else "early_launch"): {
                     "p99_ms": pct(lat_other["lat"], 99), "p50_ms": pct(lat_other["lat"], 50),
                     "preempt_latency_p99_ms": pct(lat_other["pre"], 99)},
+                "no_migration_wait_in_place": {"p99_ms": pct(inplace["lat"], 99),
+                                               "p50_ms": pct(inplace["lat"], 50)},
                 "iteration_slicing_p99_ms": pct(itg["lat"], 99),
                 "iteration_slicing_p50_ms": pct(itg["lat"], 50)}
 
