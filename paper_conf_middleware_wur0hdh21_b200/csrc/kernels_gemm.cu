@@ -328,7 +328,8 @@ Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
     // fill the 148 SMs in ONE wave: floor, never a small second wave
     splits = std::max(1, 148 / tiles);
     splits = std::min(splits, std::max(1, nkb / 2));
-    splits = std::min(splits, 64);
+    static const int max_split = std::getenv("SF_GEMM_MAXSPLIT") ? std::max(1, std::atoi(std::getenv("SF_GEMM_MAXSPLIT"))) : 64;
+    splits = std::min(splits, max_split);
   }
   pl.kb_per_split = (nkb + splits - 1) / splits;
   pl.splits = (nkb + pl.kb_per_split - 1) / pl.kb_per_split;

@@ -89,21 +89,32 @@ __device__ __forceinline__ float tf32_trunc(float x) {
   return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
 }
 
+__device__ __forceinline__ float4 lds128(uint32_t a) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts128(uint32_t a, float4 v) {
+  asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" :: "r"(a), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
+}
+
 // Split NQ float4 of a tile (thread stride 256): lo = tf32(x - trunc_tf32(x)) into `lo`;
-// unless RAW_HI, also overwrite x with trunc_tf32(x).  All loads are issued first.
+// unless RAW_HI, also overwrite x with trunc_tf32(x).  All loads are issued first; explicit
+// shared-space accesses (LDS/STS.128, not generic LD/ST).
 template <int NQ, bool RAW_HI>
 __device__ __forceinline__ void split_tile(float4* __restrict__ x, float4* __restrict__ lo, int t) {
+  const uint32_t xs = sfdev::smem_u32(x) + 16u * t, ls = sfdev::smem_u32(lo) + 16u * t;
   float4 v[NQ];
 #pragma unroll
-  for (int i = 0; i < NQ; ++i) v[i] = x[t + 256 * i];
+  for (int i = 0; i < NQ; ++i) v[i] = lds128(xs + 4096u * i);
 #pragma unroll
   for (int i = 0; i < NQ; ++i) {
     float4 h, l;
     h.x = tf32_trunc(v[i].x); h.y = tf32_trunc(v[i].y); h.z = tf32_trunc(v[i].z); h.w = tf32_trunc(v[i].w);
     l.x = tf32_trunc(v[i].x - h.x); l.y = tf32_trunc(v[i].y - h.y);
     l.z = tf32_trunc(v[i].z - h.z); l.w = tf32_trunc(v[i].w - h.w);
-    lo[t + 256 * i] = l;
-    if (!RAW_HI) x[t + 256 * i] = h;
+    sts128(ls + 4096u * i, l);
+    if (!RAW_HI) sts128(xs + 4096u * i, h);
   }
 }
 
