@@ -31,6 +31,13 @@
 #include "sf_launch.cuh"
 
 namespace sfk {
+// SF_GEMM_DUAL=1: split-K shapes with 128x64 tiles plan two CTAs per SM (2-stage ring,
+// 2 x 148 slots).  Measured: dW 148x64x100352 42.3 -> 40.3 us, 256x64x6272 20.8 -> 27.0 us
+// (the co-resident CTAs share the SM's TMA / smem / tensor issue), so off by default.
+bool gemm_dual64() {
+  static const bool on = std::getenv("SF_GEMM_DUAL") && std::getenv("SF_GEMM_DUAL")[0] == '1';
+  return on;
+}
 namespace {
 
 constexpr int BM = 128;
@@ -324,9 +331,12 @@ Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
   const int tiles = pl.tiles_n * pl.tiles_m;
   const int nkb = std::max(1, (K + BK - 1) / BK);
   int splits = 1;
-  if (tiles < 148) {
-    // fill the 148 SMs in ONE wave: floor, never a small second wave
-    splits = std::max(1, 148 / tiles);
+  // CTA slots of one wave: 128x64 tiles run two CTAs per SM (2-stage ring, ~97 KB each; the
+  // k-block rate is a per-CTA bound, so split-K shapes scale with the CTA count)
+  const int slots = pl.bn == 64 && gemm_dual64() ? 2 * 148 : 148;
+  if (tiles < slots) {
+    // fill the slots in ONE wave: floor, never a small second wave
+    splits = std::max(1, slots / tiles);
     splits = std::min(splits, std::max(1, nkb / 2));
     static const int max_split = std::getenv("SF_GEMM_MAXSPLIT") ? std::max(1, std::atoi(std::getenv("SF_GEMM_MAXSPLIT"))) : 64;
     splits = std::min(splits, max_split);

@@ -1301,7 +1301,7 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   const int max_stages = bn == 64 ? TCfg<64>::STAGES : bn == 128 ? TCfg<128>::STAGES : TCfg<256>::STAGES;
   int stages = max_stages;
   if (stages_env > 0) stages = std::min(stages_env, max_stages);
-  else if (bn == 64 && splits == 1 && tiles_n * tiles_m > 148) stages = 2;  // 2 x 97 KB fit an SM
+  else if (bn == 64 && (splits == 1 ? tiles_n * tiles_m > 148 : gemm_dual64())) stages = 2;  // 2 x 97 KB fit an SM
   TParams p{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, dbg, stages, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;

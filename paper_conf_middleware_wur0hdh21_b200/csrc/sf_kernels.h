@@ -103,6 +103,7 @@ cudaError_t launch_chain(const ChainArgs& a, cudaStream_t st);
 void set_chain_trace(void* dev_buf);
 void* chain_trace_buffer();
 cudaError_t launch_gemv_tma(const GemmArgs& a, cudaStream_t st);
+bool gemm_dual64();  // 128x64 GEMM tiles: two CTAs per SM (split planner + ring depth)
 cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_split, int tiles_n,
                             int tiles_m, bool raw_hi, cudaStream_t st);
 
