@@ -557,7 +557,7 @@ def test_open_loop_requests_during_swap_in_are_bitwise(P, defer, duplex, early):
     (the pack must wait for it).  With released arenas poisoned, any ordering mistake turns
     into NaN; the final state must equal the unpreempted GPU run bit for bit."""
     g = G.mlp_train((2048, 4096, 10), batch=64, pool=4)
-    iters = 12
+    iters = 24 if early else 12  # early launch + duplex park less: run longer for enough cuts
     base = run_gpu(P, g, iters, slots=1)[0]
     RT, A = P
     rt, gh, st, ds = setup(P, g, slots=1, poison=True, defer_migration=defer, dispatch_spin_us=-1,
