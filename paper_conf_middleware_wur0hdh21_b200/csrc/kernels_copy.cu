@@ -146,7 +146,8 @@ mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t total, uint64_t per_b
 }
 
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
-                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp) {
+                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp,
+                          int waves_arg) {
   if (n <= 0 || total_chunks == 0) return cudaSuccess;
   // Grid: a multiple of the 148 SMs, enough bytes per CTA to amortise the search.
   static const int bps = std::getenv("SF_COPY_BPS") ? std::atoi(std::getenv("SF_COPY_BPS")) : 8;
@@ -155,7 +156,8 @@ cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
   uint64_t blocks = (total_chunks + min_chunks - 1) / min_chunks;
   // waves > 1: CTAs are short-lived, so a higher-priority stream's kernel (a preempter
   // arriving mid-migration) gets SMs after one wave instead of after the whole walk
-  static const int waves = std::getenv("SF_COPY_WAVES") ? std::max(1, std::atoi(std::getenv("SF_COPY_WAVES"))) : 1;
+  static const int waves_env = std::getenv("SF_COPY_WAVES") ? std::max(1, std::atoi(std::getenv("SF_COPY_WAVES"))) : 1;
+  const int waves = waves_arg > 0 ? waves_arg : waves_env;
   blocks = std::min<uint64_t>(blocks, 148ull * bps * waves);
   blocks = std::max<uint64_t>(blocks, 1);
   const uint64_t per_block = (total_chunks + blocks - 1) / blocks;

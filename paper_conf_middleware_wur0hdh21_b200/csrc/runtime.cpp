@@ -108,6 +108,9 @@ struct Binding {
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
   std::map<int, void*> prepared;  // optimizer group first op -> uploaded descriptor array
   std::set<int> l2_keep;          // inference weights kept in the persisting L2 set-aside
+  // inference: the whole request chain (PDL edges kept) captured once per (in, out) request
+  // buffer pair and replayed with one graph launch (SF_INFER_GRAPH)
+  std::map<std::pair<const void*, void*>, std::pair<cudaGraphExec_t, uint64_t>> chain_graphs;
   bool l2_planned = false;
   std::map<int, std::pair<float*, unsigned*>> chain_bufs;  // chain first op -> (ws, counters)
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
@@ -1231,6 +1234,13 @@ void write_host_header(const Graph& g, int k, int64_t iter, uint8_t* stg) {
   }
 }
 
+// Host-tier swap-in unpack grid in waves (SF_UNPACK_WAVES, default 1): short-lived CTAs let a
+// request that arrives during the unpack get SMs after one wave instead of after the walk.
+int unpack_waves() {
+  static const int w = std::getenv("SF_UNPACK_WAVES") ? std::max(1, std::atoi(std::getenv("SF_UNPACK_WAVES"))) : 1;
+  return w;
+}
+
 // Preempt J at its current boundary (rt->m held on entry and on return).
 sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
   Graph& g = *J.g;
@@ -1381,7 +1391,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     if (duplex) {  // the H2D already ran (its time is in xfer_us): unpack only
       cudaEventRecord(J.ev_b[dst], D.s_train);
       const CopyList& L = BD.unpack[k];
-      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2, unpack_waves());
     } else if (ce) {
       e = ce_segments(J, D, dst, cut_segments(g, k, BD.arena, B.host_staging, 1), D.s_train, true);
       cudaEventRecord(J.ev_b[dst], D.s_train);
@@ -1396,7 +1406,7 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       cudaEventRecord(J.ev_b[dst], D.s_train);
       if (e == cudaSuccess) {
         const CopyList& L = BD.unpack[k];
-        e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2);
+        e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, D.s_train, D.tstamp + 2, unpack_waves());
       }
     }
     if (e != cudaSuccess) return cuda_fail(e, "unpack");
@@ -2012,7 +2022,50 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
-    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
+    // one graph launch for the whole chain when it was captured for this buffer pair
+    static const bool use_graph = std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1';
+    bool graphed = false;
+    if (e == cudaSuccess && direct && in_place && use_graph && S->l2_setaside == 0) {
+      auto key = std::make_pair(r->in, r->out);
+      auto it = B->chain_graphs.find(key);
+      if (it == B->chain_graphs.end() && B->chain_graphs.size() < 64) {
+        // capture the chain (direct launches, PDL) on a private stream into one graph
+        cudaStream_t cap = nullptr;
+        cudaGraph_t graph = nullptr;
+        cudaGraphExec_t exec = nullptr;
+        const uint64_t l0 = sfk::launches();
+        cudaError_t ce = cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking);
+        if (ce == cudaSuccess) ce = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
+        bool ok = ce == cudaSuccess;
+        for (size_t k = 0; ok && k < B->versions.size(); ++k) {
+          Capture c{g, *B, cap, false, &B->prepared};
+          c.redir_in = g.input_tid;
+          c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(r->in));
+          c.redir_out = g.output_tid;
+          c.out_ptr = static_cast<uint8_t*>(r->out);
+          ok = launch_subgraph_ops(c, static_cast<int>(k)) == SF_OK;
+        }
+        if (cap) {
+          const cudaError_t ee = cudaStreamEndCapture(cap, &graph);
+          ok = ok && ee == cudaSuccess && graph;
+        }
+        const uint64_t nk = sfk::launches() - l0;
+        sfk::count_launch(uint64_t(0) - nk);  // captured, not launched
+        if (ok && cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess) {
+          it = B->chain_graphs.emplace(key, std::make_pair(exec, nk)).first;
+        } else {
+          cudaGetLastError();
+        }
+        if (graph) cudaGraphDestroy(graph);
+        if (cap) cudaStreamDestroy(cap);
+      }
+      if (it != B->chain_graphs.end()) {
+        e = cudaGraphLaunch(it->second.first, S->s_infer);
+        sfk::count_launch(it->second.second);
+        graphed = true;
+      }
+    }
+    for (size_t k = 0; !graphed && e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
         if (S->l2_setaside > 0) c.l2_keep = &B->l2_keep;
@@ -2195,6 +2248,7 @@ void sf_destroy(sf_runtime* rt) {
       }
       cudaSetDevice(rt->slots[B->slot]->cuda);
       for (auto v : B->versions) cudaGraphExecDestroy(v);
+      for (auto& cg : B->chain_graphs) cudaGraphExecDestroy(cg.second.first);
       for (void* d : B->dev_allocs) cudaFree(d);
       if (B->ws) cudaFree(B->ws);
       if (B->counters) cudaFree(B->counters);

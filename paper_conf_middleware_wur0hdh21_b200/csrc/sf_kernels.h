@@ -22,7 +22,7 @@ struct DCopy {
 // tstamp (optional, device): {earliest CTA start, latest CTA end} in %globaltimer ns; the
 // caller initialises it to {~0, 0}.
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
-                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp = nullptr);
+                          int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp = nullptr, int waves = 0);
 cudaError_t launch_fill(void* dst, uint64_t n, uint8_t value, cudaStream_t st);
 cudaError_t launch_copy2d(const void* src, uint64_t spitch, void* dst, uint64_t dpitch, uint64_t rows,
                           uint64_t width, cudaStream_t st);
