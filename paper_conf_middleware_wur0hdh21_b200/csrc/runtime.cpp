@@ -1150,6 +1150,11 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
   static const size_t kDepth = std::getenv("SF_DUPLEX_DEPTH")
                                    ? size_t(std::max(1, std::min(2, std::atoi(std::getenv("SF_DUPLEX_DEPTH")))))
                                    : 2;
+  // D2H traffic delays a concurrent request's command / completion traffic the most
+  // (reading Q34): SF_DUPLEX_DEPTH_D2H caps the D2H chunks in flight separately
+  static const size_t kDepthD2H = std::getenv("SF_DUPLEX_DEPTH_D2H")
+                                      ? size_t(std::max(1, std::min(2, std::atoi(std::getenv("SF_DUPLEX_DEPTH_D2H")))))
+                                      : kDepth;
   constexpr int R = 4;  // event ring per direction (kCkEvents / 2)
   const size_t nch = (total + kChunk - 1) / kChunk;
   size_t nd = 0, nh = 0, cd = 0, ch = 0;  // D2H / H2D issued, D2H / H2D completed
@@ -1172,7 +1177,7 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
       continue;
     }
     if (!busy()) {
-      if (nd < nch && nd - cd < kDepth && nd - nh < static_cast<size_t>(R)) {
+      if (nd < nch && nd - cd < kDepthD2H && nd - nh < static_cast<size_t>(R)) {
         const size_t off = nd * kChunk, n = std::min(kChunk, total - off);
         cudaError_t e = cudaMemcpyAsync(hstg + off, dstg + off, n, cudaMemcpyDeviceToHost, S.s_mig);
         if (e == cudaSuccess && poison_chunks) e = sfk::launch_fill(dstg + off, n, 0xFF, S.s_mig);
