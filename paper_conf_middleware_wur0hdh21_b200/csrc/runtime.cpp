@@ -111,6 +111,8 @@ struct Binding {
   // inference: the whole request chain (PDL edges kept) captured once per (in, out) request
   // buffer pair and replayed with one graph launch (SF_INFER_GRAPH)
   std::map<std::pair<const void*, void*>, std::pair<cudaGraphExec_t, uint64_t>> chain_graphs;
+  std::set<std::pair<const void*, void*>> chain_pending;  // queued for the builder
+  std::mutex chain_m;
   bool l2_planned = false;
   std::map<int, std::pair<float*, unsigned*>> chain_bufs;  // chain first op -> (ws, counters)
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
@@ -271,6 +273,13 @@ struct sf_runtime {
   std::vector<sf_trace_event> trace;
   size_t trace_cap = 1 << 16;
   size_t trace_dropped = 0;
+  // background builder of per-buffer-pair inference chain graphs (SF_INFER_GRAPH=1)
+  struct GraphBuild { Graph* g; Binding* b; int cuda; const void* in; void* out; };
+  std::thread gbuilder;
+  std::mutex gb_m;
+  std::condition_variable gb_cv;
+  std::deque<GraphBuild> gb_q;
+  bool gb_stop = false;
 };
 
 namespace {
@@ -1914,6 +1923,55 @@ void driver_main(sf_runtime* rt, Job* Jp) {
   }
 }
 
+// Captures a request chain (direct launches with PDL, request I/O in place) into one graph per
+// (in, out) buffer pair, on its own stream and thread, and publishes it to the binding.
+void graph_builder_main(sf_runtime* rt) {
+  std::unique_lock<std::mutex> lk(rt->gb_m);
+  while (true) {
+    rt->gb_cv.wait(lk, [&] { return rt->gb_stop || !rt->gb_q.empty(); });
+    if (rt->gb_stop) break;
+    const sf_runtime::GraphBuild job = rt->gb_q.front();
+    rt->gb_q.pop_front();
+    lk.unlock();
+    cudaSetDevice(job.cuda);
+    Graph& g = *job.g;
+    Binding& B = *job.b;
+    cudaStream_t cap = nullptr;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    sfk::set_pdl(true);
+    cudaError_t ce = cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking);
+    if (ce == cudaSuccess) ce = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
+    bool ok = ce == cudaSuccess;
+    for (size_t k = 0; ok && k < B.versions.size(); ++k) {
+      Capture c{g, B, cap, false, &B.prepared};
+      c.redir_in = g.input_tid;
+      c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(job.in));
+      c.redir_out = g.output_tid;
+      c.out_ptr = static_cast<uint8_t*>(job.out);
+      ok = launch_subgraph_ops(c, static_cast<int>(k)) == SF_OK;
+    }
+    sfk::set_pdl(false);
+    if (cap) {
+      const cudaError_t ee = cudaStreamEndCapture(cap, &graph);
+      ok = ok && ee == cudaSuccess && graph;
+    }
+    size_t nk = 0;
+    if (ok && cudaGraphGetNodes(graph, nullptr, &nk) != cudaSuccess) ok = false;
+    sfk::count_launch(uint64_t(0) - nk);  // captured kernels: counted at each replay instead
+    if (ok && cudaGraphInstantiate(&exec, graph, 0) != cudaSuccess) ok = false;
+    if (!ok) cudaGetLastError();
+    if (graph) cudaGraphDestroy(graph);
+    if (cap) cudaStreamDestroy(cap);
+    {
+      std::lock_guard<std::mutex> gl(B.chain_m);
+      B.chain_pending.erase({job.in, job.out});
+      if (ok) B.chain_graphs[{job.in, job.out}] = {exec, static_cast<uint64_t>(nk)};
+    }
+    lk.lock();
+  }
+}
+
 void dispatcher_main(sf_runtime* rt, Slot* S) {
   cudaSetDevice(S->cuda);
   std::unique_lock<std::mutex> lk(rt->m);
@@ -2027,47 +2085,34 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
-    // one graph launch for the whole chain when it was captured for this buffer pair
+    // one graph launch for the whole chain once the builder thread captured it for this
+    // request-buffer pair (built off the critical path; until then: direct launches)
     static const bool use_graph = std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1';
     bool graphed = false;
     if (e == cudaSuccess && direct && in_place && use_graph && S->l2_setaside == 0) {
-      auto key = std::make_pair(r->in, r->out);
-      auto it = B->chain_graphs.find(key);
-      if (it == B->chain_graphs.end() && B->chain_graphs.size() < 64) {
-        // capture the chain (direct launches, PDL) on a private stream into one graph
-        cudaStream_t cap = nullptr;
-        cudaGraph_t graph = nullptr;
-        cudaGraphExec_t exec = nullptr;
-        const uint64_t l0 = sfk::launches();
-        cudaError_t ce = cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking);
-        if (ce == cudaSuccess) ce = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
-        bool ok = ce == cudaSuccess;
-        for (size_t k = 0; ok && k < B->versions.size(); ++k) {
-          Capture c{g, *B, cap, false, &B->prepared};
-          c.redir_in = g.input_tid;
-          c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(r->in));
-          c.redir_out = g.output_tid;
-          c.out_ptr = static_cast<uint8_t*>(r->out);
-          ok = launch_subgraph_ops(c, static_cast<int>(k)) == SF_OK;
+      const auto key = std::make_pair(r->in, r->out);
+      cudaGraphExec_t exec = nullptr;
+      uint64_t nk = 0;
+      bool enqueue = false;
+      {
+        std::lock_guard<std::mutex> gl(B->chain_m);
+        auto it = B->chain_graphs.find(key);
+        if (it != B->chain_graphs.end()) {
+          exec = it->second.first;
+          nk = it->second.second;
+        } else if (B->chain_graphs.size() + B->chain_pending.size() < 64 && !B->chain_pending.count(key)) {
+          B->chain_pending.insert(key);
+          enqueue = true;
         }
-        if (cap) {
-          const cudaError_t ee = cudaStreamEndCapture(cap, &graph);
-          ok = ok && ee == cudaSuccess && graph;
-        }
-        const uint64_t nk = sfk::launches() - l0;
-        sfk::count_launch(uint64_t(0) - nk);  // captured, not launched
-        if (ok && cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess) {
-          it = B->chain_graphs.emplace(key, std::make_pair(exec, nk)).first;
-        } else {
-          cudaGetLastError();
-        }
-        if (graph) cudaGraphDestroy(graph);
-        if (cap) cudaStreamDestroy(cap);
       }
-      if (it != B->chain_graphs.end()) {
-        e = cudaGraphLaunch(it->second.first, S->s_infer);
-        sfk::count_launch(it->second.second);
+      if (exec) {
+        e = cudaGraphLaunch(exec, S->s_infer);
+        sfk::count_launch(nk);
         graphed = true;
+      } else if (enqueue) {
+        std::lock_guard<std::mutex> ql(rt->gb_m);
+        rt->gb_q.push_back({&g, B, S->cuda, r->in, r->out});
+        rt->gb_cv.notify_one();
       }
     }
     for (size_t k = 0; !graphed && e == cudaSuccess && k < B->versions.size(); ++k) {
@@ -2200,6 +2245,8 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
   sf_runtime* p = rt.release();
   for (auto& S : p->slots)
     if (!S->remote) S->dispatcher = std::thread(dispatcher_main, p, S.get());
+  if (std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1')
+    p->gbuilder = std::thread(graph_builder_main, p);
   *out = p;
   return SF_OK;
 }
@@ -2224,6 +2271,12 @@ void sf_destroy(sf_runtime* rt) {
     if (J->driver.joinable()) J->driver.join();
   for (auto& S : rt->slots)
     if (S->dispatcher.joinable()) S->dispatcher.join();
+  {
+    std::lock_guard<std::mutex> gl(rt->gb_m);
+    rt->gb_stop = true;
+    rt->gb_cv.notify_all();
+  }
+  if (rt->gbuilder.joinable()) rt->gbuilder.join();
   for (auto& F : rt->feeds)
     if (F->stager.joinable()) F->stager.join();
   for (auto& F : rt->feeds) {
