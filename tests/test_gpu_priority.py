@@ -79,7 +79,9 @@ def test_training_preempts_training(P, tier, home, W):
     g_lo, g_hi = _graphs()
     # the low-priority job must still be running when the high-priority one arrives (a C1
     # iteration takes ~0.1 ms, so a short job can finish during a host hiccup) and outlive it
-    it_lo, it_hi = 400, 5
+    # the high-priority job runs long enough (~1 ms) for the migrated low-priority job to
+    # resume on the peer while it is still present (5 iterations proved too short once)
+    it_lo, it_hi = 400, 12
     base_lo = _solo(P, g_lo, it_lo, LO_SEED)
     base_hi = _solo(P, g_hi, it_hi, HI_SEED)
     slots = 2 if tier == "peer" else 1
@@ -104,7 +106,7 @@ def test_training_preempts_training(P, tier, home, W):
         assert got_lo[i].tobytes() == base_lo[i].tobytes(), g_lo.tensors[i].name
     for i in st_hi:
         assert got_hi[i].tobytes() == base_hi[i].tobytes(), g_hi.tensors[i].name
-    # oracle parity on the high-priority job (5 iterations); the 400-iteration low-priority
+    # oracle parity on the high-priority job (12 iterations); the 400-iteration low-priority
     # trajectory is checked bit for bit against its solo GPU run above (ReLU kinks make long
     # fp32 horizons unsuitable for a 1e-4 oracle bar, reading Q19)
     ref_hi = R.run(g_hi, it_hi, st_hi, D.datasets(g_hi), keep_stagings=False)
