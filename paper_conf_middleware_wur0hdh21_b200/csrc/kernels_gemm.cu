@@ -338,7 +338,9 @@ Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
     // fill the slots in ONE wave: floor, never a small second wave
     splits = std::max(1, slots / tiles);
     splits = std::min(splits, std::max(1, nkb / 2));
-    static const int max_split = std::getenv("SF_GEMM_MAXSPLIT") ? std::max(1, std::atoi(std::getenv("SF_GEMM_MAXSPLIT"))) : 64;
+    // up to one CTA per SM (the k-block rate is an SM-local bound: the forest's dW of conv1,
+    // 2 tiles, goes 64 -> 74 splits, 50 -> 47 us); SF_GEMM_MAXSPLIT caps it
+    static const int max_split = std::getenv("SF_GEMM_MAXSPLIT") ? std::max(1, std::atoi(std::getenv("SF_GEMM_MAXSPLIT"))) : 148;
     splits = std::min(splits, max_split);
   }
   pl.kb_per_split = (nkb + splits - 1) / splits;
