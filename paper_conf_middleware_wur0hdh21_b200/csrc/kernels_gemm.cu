@@ -318,9 +318,13 @@ struct Plan {
 
 // SF_GEMM_BN256=1: 128x256 tiles (TMA path) for N >= 256 — half the A-operand smem reads per
 // flop of the 3 MMAs; 2 pipeline stages fit (96 KB per stage)
-bool gemm_bn256() {
-  static const bool on = std::getenv("SF_GEMM_BN256") && std::getenv("SF_GEMM_BN256")[0] == '1';
-  return on;
+// 0: never, 1: always when N >= 256, 2 (default): when the 128x256 plan needs no split-K and
+// still fills >= 100 SMs (a tf32 MMA costs a near-fixed ~140-160 cycles per instruction in the
+// loop, so twice the N per instruction pays: dW 1024x4096x512 130 -> 157 TFLOP/s; shapes that
+// would need split-K at 256 stay at 128, e.g. 512x4096x1024 142 vs 93)
+int gemm_bn256_mode() {
+  static const int m = std::getenv("SF_GEMM_BN256") ? std::atoi(std::getenv("SF_GEMM_BN256")) : 2;
+  return m;
 }
 
 Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
@@ -346,6 +350,14 @@ Plan plan_gemm(int M, int N, int K, int force_bn = 0) {
   pl.kb_per_split = (nkb + splits - 1) / splits;
   pl.splits = (nkb + pl.kb_per_split - 1) / pl.kb_per_split;
   return pl;
+}
+
+bool use_bn256(int M, int N, int K) {
+  const int m = gemm_bn256_mode();
+  if (m == 0 || N < 256) return false;
+  if (m == 1) return true;
+  const Plan p2 = plan_gemm(M, N, K, 256);
+  return p2.splits == 1 && p2.tiles_n * p2.tiles_m >= 100;
 }
 
 template <int BN, bool AK, bool BKc>
@@ -681,7 +693,7 @@ uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb) {
   }
   Plan pl = plan_gemm(M, N, K);
   uint64_t w = pl.splits > 1 ? static_cast<uint64_t>(pl.splits) * M * N : 0;
-  if (gemm_bn256() && N >= 256) {
+  if (use_bn256(M, N, K)) {
     const Plan p2 = plan_gemm(M, N, K, 256);
     if (p2.splits > 1) w = std::max<uint64_t>(w, static_cast<uint64_t>(p2.splits) * M * N);
   }
@@ -777,7 +789,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   // explicitly masked hi on B200, scripts/rawhi_check.py); SF_GEMM_RAWHI=0 masks explicitly.
   static const bool raw_hi = !(std::getenv("SF_GEMM_RAWHI") && std::getenv("SF_GEMM_RAWHI")[0] == '0');
   const bool legacy = path && std::string(path) == "legacy";
-  if (!legacy && raw_hi && gemm_bn256() && a.N >= 256) {
+  if (!legacy && raw_hi && use_bn256(a.M, a.N, a.K)) {
     const Plan p2 = plan_gemm(a.M, a.N, a.K, 256);
     if ((p2.splits == 1 || (a.ws && a.counters)) && gemm_tma_eligible(a, p2.splits))
       return launch_gemm_tma(a, 256, p2.splits, p2.kb_per_split, p2.tiles_n, p2.tiles_m, raw_hi, st);
