@@ -424,7 +424,8 @@ int32_t sf_stage_u8_normalize(void* user, int64_t iter, void* const* dst, const 
 /* ---- inference (the preempter) --------------------------------------------------- */
 typedef struct sf_timing {
   uint64_t arrival_ns;   /* scheduled arrival (CLOCK_MONOTONIC) */
-  uint64_t start_ns;     /* inference launched on the device */
+  uint64_t start_ns;     /* the request chain's start on the device (GPU timeline mapped to
+                            CLOCK_MONOTONIC, Q37; host dispatch time if unmapped) */
   uint64_t end_ns;       /* completion observed */
   int32_t dev;
   int32_t preempted_job; /* job cut by this request, or -1 */
@@ -459,6 +460,11 @@ typedef struct sf_trace_event {
                                   (<= t0 when queued behind an in-flight predecessor) */
   /* inference: iter = -1, or the training job whose subgraphs dispatched before t0 this
      request was ordered after on the device (early_launch); t0 is then its dispatch time */
+  uint64_t d0_ns, d1_ns;       /* DEVICE execution interval on the CLOCK_MONOTONIC axis: timing
+                                  events recorded on the stream right before the subgraph's
+                                  graph (request chain) and right after it, mapped through a
+                                  %globaltimer anchor (reading Q37); a superset of
+                                  the kernels' execution; 0 = unavailable (train / infer only) */
 } sf_trace_event;
 sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* n_out);
 uint64_t sf_now_ns(void); /* CLOCK_MONOTONIC */
@@ -526,6 +532,17 @@ sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t
                      int64_t n, float lr, float beta1, float beta2, float eps, void* stream);
 /* Fill n bytes at dst (device) with byte value (0xFF = poison). */
 sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream);
+/* Diagnostics: the kernel path of the last GEMM the CALLING THREAD launched (sf_op_gemm,
+ * sf_op_gemm_bias_act, or a subgraph op launched directly on this thread).
+ * kind: 1 tcgen05 TMA tile GEMM (bn = tile width 64 / 128 / 256, splits = split-K factor),
+ *       2 tcgen05 GEMM with LDG producers (pitches TMA cannot map), 3 TMA cluster GEMV,
+ *       4 row-contiguous GEMV (TB), 5 register cluster GEMV, 6 split-K GEMV + reduce,
+ *       7 plain GEMV; 0 = none yet.
+ * a_mn / b_mn: operand stored MN-major (A as [K][M], i.e. TA; B as [K][N], i.e. not TB). */
+typedef struct sf_gemm_path {
+  int32_t kind, bn, splits, a_mn, b_mn, pad;
+} sf_gemm_path;
+sf_status sf_last_gemm_path(sf_gemm_path* out);
 /* Number of kernels this process launched through the library so far. */
 uint64_t sf_kernel_launches(void);
 

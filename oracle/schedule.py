@@ -14,7 +14,8 @@ trace or the GPU runtime's recorded one):
       waiting for the outstanding nodes of a preempted job to complete is on the
       critical path" (section 5.2.3).  Checked as
       start(infer) - max(arrival, end of the previous inference on that device)
-      <= max train-subgraph duration on that device + slack.
+      <= window x max train-subgraph duration on that device + slack, where ``window`` is
+      the number of subgraphs the runtime may have dispatched ahead of its boundary gate.
   I4  cut rule (reading Q13): a request arriving while S_k runs is served at the
       boundary after S_k — more precisely, no training subgraph is DISPATCHED after the
       arrival and before the inference starts (subgraphs already dispatched to the GPU are
@@ -24,14 +25,18 @@ trace or the GPU runtime's recorded one):
       immediately after submission"; "upon the arrival of a high
       priority model, the low priority one is preempted and migrated"): on a device, from a
       job's submission there until its last subgraph there ends, no training subgraph of a
-      lower-priority job is DISPATCHED there; and the high-priority job's first subgraph
+      lower-priority job is DISPATCHED there; at most ``window`` lower-priority subgraphs
+      execute on the device after the submission and before the high-priority job's first
+      subgraph (the outstanding subgraphs drain, nothing more); and that first subgraph
       starts within ``window`` x (longest lower-priority subgraph on the device) + slack of
-      its submission (the outstanding subgraphs drain, nothing more).
+      the submission.
 
 Event dicts: {"dev", "job", "kind": "train"|"infer", "iter", "k", "t0", "t1",
 "arrival" (infer only), "after" (infer only, optional: the training job it was ordered
-after on the device), "launch" (train only, optional: dispatch time)}; times in any
-consistent unit.
+after on the device), "launch" (train only, optional: dispatch time), "d0"/"d1"
+(optional: the DEVICE execution interval on the same clock, 0 if unknown)}; times in any
+consistent unit.  ``device_view`` turns a recorded trace into device intervals: every
+invariant is then checked on when the GPU executed the work, not on when the host saw it.
 
 Pins (tests/test_oracle_schedule.py): hand-built violating traces for I1..I4 are
 rejected; the discrete-event model's traces satisfy them; closed-form latencies of
@@ -59,6 +64,22 @@ def _device_ordered(a: dict, b: dict) -> bool:
                 and t.get("launch", t["t0"]) <= r["t0"]):
             return True
     return False
+
+
+def device_view(events: Sequence[dict]) -> List[dict]:
+    """Train / infer events on the DEVICE timeline: t0, t1 := d0, d1 (the GPU execution
+    interval); the host interval is kept as h0, h1 and the host-side "after" dependency is
+    dropped (device intervals of dependent work are disjoint by themselves).  Events that
+    carry no device interval (host stages, or d0 == 0) are returned unchanged."""
+    out = []
+    for e in events:
+        e = dict(e)
+        if e.get("kind") in ("train", "infer") and e.get("d0") and e.get("d1"):
+            e["h0"], e["h1"] = e["t0"], e["t1"]
+            e["t0"], e["t1"] = e["d0"], e["d1"]
+            e.pop("after", None)
+        out.append(e)
+    return out
 
 
 def check_no_corun(events: Sequence[dict]) -> None:
@@ -102,20 +123,44 @@ def check_job_order(events: Sequence[dict], n_sub: Dict[int, int],
                 it, k = it + 1, 0
 
 
-def check_preempt_latency(events: Sequence[dict], slack: float) -> None:
-    """I3: inference start - ready time <= longest training subgraph on that device + slack."""
+def preempt_latency_report(events: Sequence[dict], slack: float, window: int = 1) -> dict:
+    """I3 per request: wait = start - ready, ready = max(arrival, end of the previous
+    inference on the device); bound = window x (longest training subgraph on the device) +
+    slack (``window`` subgraphs may be dispatched ahead of the boundary gate).  A request over
+    the bound is a HOST outlier when its host dispatch decision ("h0", device_view) itself came
+    later than ready + bound — the dispatcher thread was late, which no device-side drain
+    explains — else a violation.  Returns {"n", "bound", "violations", "host_outliers",
+    "waits"}."""
     by_dev: Dict[int, List[dict]] = {}
     for e in events:
         by_dev.setdefault(e["dev"], []).append(e)
+    rep = {"n": 0, "bound": {}, "violations": [], "host_outliers": [], "waits": []}
     for d, evs in by_dev.items():
         longest = max([e["t1"] - e["t0"] for e in evs if e["kind"] == "train"], default=0.0)
+        bound = window * longest + slack
+        rep["bound"][d] = bound
         prev_end = float("-inf")
         for e in sorted([e for e in evs if e["kind"] == "infer"], key=lambda e: e["t0"]):
             ready = max(e["arrival"], prev_end)
-            if e["t0"] - ready > longest + slack:
-                raise InvariantError(f"dev {d}: inference waited {e['t0'] - ready} > "
-                                     f"{longest} + {slack}")
+            wait = e["t0"] - ready
+            rep["n"] += 1
+            rep["waits"].append(wait)
+            if wait > bound:
+                host_late = e.get("h0") is not None and e["h0"] - ready > bound
+                (rep["host_outliers"] if host_late else rep["violations"]).append((e, wait))
             prev_end = e["t1"]
+    return rep
+
+
+def check_preempt_latency(events: Sequence[dict], slack: float, window: int = 1) -> None:
+    """I3: inference start - ready time <= window x longest training subgraph on that
+    device + slack, for every request."""
+    r = preempt_latency_report(events, slack, window)
+    bad = r["violations"] + r["host_outliers"]
+    if bad:
+        e, w = bad[0]
+        raise InvariantError(f"dev {e['dev']}: inference waited {w} > {r['bound'][e['dev']]} "
+                             f"({len(bad)} of {r['n']} requests)")
 
 
 def check_cut_rule(events: Sequence[dict]) -> None:
@@ -151,6 +196,10 @@ def check_priority(events: Sequence[dict], prio: Dict[int, int],
                     f"dev {dev}: job {e['job']} (prio {prio[e['job']]}) dispatched "
                     f"({e['iter']},{e['k']}) at {e.get('launch', e['t0'])} while job {hj} "
                     f"(prio {prio[hj]}) was present [{ts},{end})")
+        drained = [e for e in lower if e["t1"] > ts and e["t0"] < mine[0]["t0"]]
+        if len(drained) > window:
+            raise InvariantError(f"dev {dev}: {len(drained)} lower-priority subgraphs ran after "
+                                 f"job {hj}'s submission at {ts} (window {window})")
         longest = max([e["t1"] - e["t0"] for e in lower], default=0.0)
         if mine[0]["t0"] - ts > window * longest + slack:
             raise InvariantError(f"dev {dev}: job {hj} started {mine[0]['t0'] - ts} after "

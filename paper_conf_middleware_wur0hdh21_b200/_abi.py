@@ -96,7 +96,7 @@ class sf_timing(C.Structure):
 class sf_trace_event(C.Structure):
     _fields_ = [("dev", C.c_int32), ("job", C.c_int32), ("kind", C.c_int32), ("k", C.c_int32),
                 ("iter", C.c_int64), ("t0_ns", C.c_uint64), ("t1_ns", C.c_uint64),
-                ("arrival_ns", C.c_uint64)]
+                ("arrival_ns", C.c_uint64), ("d0_ns", C.c_uint64), ("d1_ns", C.c_uint64)]
 
 
 class sf_cut_request(C.Structure):
@@ -118,6 +118,11 @@ class sf_u8_stage(C.Structure):
     _fields_ = [("images", C.c_void_p), ("labels", C.c_void_p), ("pool_rows", C.c_int64),
                 ("batch", C.c_int32), ("cols", C.c_int32), ("img_w", C.c_int32),
                 ("seed", C.c_uint32)]
+
+
+class sf_gemm_path(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("bn", C.c_int32), ("splits", C.c_int32), ("a_mn", C.c_int32),
+                ("b_mn", C.c_int32), ("pad", C.c_int32)]
 
 
 class sf_copy_desc(C.Structure):
@@ -180,6 +185,7 @@ PROTOTYPES = {
     "sf_op_adam": (_st, [_vp, _vp, _vp, _vp, _vp, C.c_int64, C.c_float, C.c_float, C.c_float,
                          C.c_float, _vp]),
     "sf_op_fill": (_st, [_vp, C.c_uint64, C.c_int32, _vp]),
+    "sf_last_gemm_path": (_st, [_P(sf_gemm_path)]),
     "sf_kernel_launches": (C.c_uint64, []),
 }
 

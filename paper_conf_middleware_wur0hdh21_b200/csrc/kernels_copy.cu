@@ -261,6 +261,20 @@ cudaError_t launch_feed(const void* pool, const int32_t* step, void* x, uint64_t
   return cudaGetLastError();
 }
 
+// Clock anchor (device trace, reading Q37): one thread writes %globaltimer (ns) to
+// `dst` (mapped pinned host memory) with a system-scope store, so the host reads it without a
+// CUDA call and ties the GPU timeline to CLOCK_MONOTONIC.
+__global__ void stamp_kernel(unsigned long long* dst) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  asm volatile("st.global.relaxed.sys.u64 [%0], %1;" ::"l"(dst), "l"(t) : "memory");
+}
+cudaError_t launch_stamp(unsigned long long* dst, cudaStream_t st) {
+  stamp_kernel<<<1, 1, 0, st>>>(dst);
+  count_launch();
+  return cudaGetLastError();
+}
+
 __global__ void step_inc_kernel(int32_t* step) { *step += 1; }
 cudaError_t launch_step_inc(int32_t* step, cudaStream_t st) {
   step_inc_kernel<<<1, 1, 0, st>>>(step);

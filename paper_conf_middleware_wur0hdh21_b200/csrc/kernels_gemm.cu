@@ -706,16 +706,34 @@ uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb) {
   return static_cast<uint64_t>(pl.tiles_m) * pl.tiles_n;
 }
 
+namespace {
+thread_local GemmPath g_last_path;
+}
+GemmPath last_gemm_path() { return g_last_path; }
+
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   if (a.M <= 0 || a.N <= 0) return cudaSuccess;
-  if (gemv_rows_eligible(a)) return launch_gemv_rows(a, st);
+  g_last_path = GemmPath{};
+  g_last_path.a_mn = a.ta;
+  g_last_path.b_mn = !a.tb;
+  g_last_path.splits = 1;
+  auto take = [](int kind, int bn = 0, int splits = 1) {
+    g_last_path.kind = kind;
+    g_last_path.bn = bn;
+    g_last_path.splits = splits;
+  };
+  if (gemv_rows_eligible(a)) { take(kGemvRows); return launch_gemv_rows(a, st); }
   if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)))
     return cudaErrorInvalidValue;  // fused epilogue only exists on the GEMV path
   // M <= 8 paths: SF_GEMV = tma (default: TMA-streamed cluster GEMV) | cluster (register-
   // streamed cluster GEMV) | split (split-K GEMV + separate reduce kernel)
   static const char gemv_path = std::getenv("SF_GEMV") ? std::getenv("SF_GEMV")[0] : 't';
-  if (gemv_path == 't' && use_gemv(a.M, a.ta, a.tb) && gemv_tma_eligible(a)) return launch_gemv_tma(a, st);
+  if (gemv_path == 't' && use_gemv(a.M, a.ta, a.tb) && gemv_tma_eligible(a)) {
+    take(kGemvTma);
+    return launch_gemv_tma(a, st);
+  }
   if (gemv_path != 's' && use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)) {
+    take(kGemvCluster);
     // widest column block that still gives >= 2 CTAs per SM (the stream needs the MLP)
     const int nq = a.N / 4;
     int QW = 4;
@@ -748,6 +766,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   }
   if (use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb) && a.ws) {
     Gemv4Plan g = plan_gemv4(a.N, a.K);
+    take(kGemvSplit, 0, g.splits);
     dim3 grid(g.col_blocks, g.splits);
 #define SF_GEMV4(MR) gemv4_kernel<MR><<<grid, 256, 0, st>>>(a.A, a.B, a.ws, a.M, a.N, a.K, a.lda, a.ldb, g.kper)
     if (a.M == 1) SF_GEMV4(1);
@@ -768,6 +787,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   if (use_gemv(a.M, a.ta, a.tb)) {
     GemvPlan g = plan_gemv(a.N, a.K);
     if (g.splits > 1 && (!a.ws || !a.counters)) return cudaErrorInvalidValue;
+    take(kGemvPlain, 0, g.splits);
     dim3 grid(g.cols_blocks, g.splits);
 #define SF_GEMV(MR)                                                                          \
   gemv_kernel<MR><<<grid, 256, 0, st>>>(a.A, a.B, a.C, a.M, a.N, a.K, a.lda, a.ldb, a.ldc,   \
@@ -791,11 +811,16 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
   const bool legacy = path && std::string(path) == "legacy";
   if (!legacy && raw_hi && use_bn256(a.M, a.N, a.K)) {
     const Plan p2 = plan_gemm(a.M, a.N, a.K, 256);
-    if ((p2.splits == 1 || (a.ws && a.counters)) && gemm_tma_eligible(a, p2.splits))
+    if ((p2.splits == 1 || (a.ws && a.counters)) && gemm_tma_eligible(a, p2.splits)) {
+      take(kGemmTma, 256, p2.splits);
       return launch_gemm_tma(a, 256, p2.splits, p2.kb_per_split, p2.tiles_n, p2.tiles_m, raw_hi, st);
+    }
   }
-  if (!legacy && gemm_tma_eligible(a, pl.splits))
+  if (!legacy && gemm_tma_eligible(a, pl.splits)) {
+    take(kGemmTma, pl.bn, pl.splits);
     return launch_gemm_tma(a, pl.bn, pl.splits, pl.kb_per_split, pl.tiles_n, pl.tiles_m, raw_hi, st);
+  }
+  take(kGemmLdg, pl.bn, pl.splits);
   Params p;
   p.A = a.A; p.B = a.B; p.C = a.C;
   p.M = a.M; p.N = a.N; p.K = a.K; p.lda = a.lda; p.ldb = a.ldb; p.ldc = a.ldc;

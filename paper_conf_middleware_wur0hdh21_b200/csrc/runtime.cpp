@@ -173,6 +173,22 @@ struct Slot {
   cudaEvent_t ev_infer = nullptr;
   cudaEvent_t ev_i0 = nullptr;  // timing: request chain start (ev_infer marks its end)
   unsigned long long* tstamp = nullptr;  // device {start, end} x 2 (pack/peer, unpack)
+  // Device clock anchors (reading Q37): a stamp kernel writes %globaltimer into mapped
+  // pinned memory and a timing event is recorded right behind it; any timing event of this
+  // device then maps to CLOCK_MONOTONIC as g + elapsed(anchor, event) + offset, where offset
+  // ties the GPU timer to the host clock (host read before launch / after the value landed).
+  struct Anchor {
+    cudaEvent_t ev;
+    uint64_t enq_ns;   // host time the anchor was enqueued
+    uint64_t g_ns;     // %globaltimer written by the stamp kernel
+    int64_t offset_ns; // host = device + offset (midpoint of the launch..observed window)
+    uint64_t unc_ns;   // half that window
+  };
+  cudaStream_t s_clk = nullptr;
+  unsigned long long* clk_host = nullptr;  // pinned, mapped
+  unsigned long long* clk_dev = nullptr;
+  std::mutex clk_m;
+  std::deque<Anchor> anchors;
   std::atomic<int> owner{-1};  // device token (atomic: the spinning dispatcher polls it)
   size_t l2_setaside = 0, l2_max_window = 0;  // persisting L2 for inference weights
   std::deque<Request*> q;
@@ -224,6 +240,7 @@ struct Job {
   std::thread driver;
   std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
   std::vector<cudaEvent_t> ev_ring;  // [slot * kMaxInflight + i]: in-flight subgraph ends
+  std::vector<cudaEvent_t> ev_start; // [slot * kMaxInflight + i]: their starts (device trace)
   std::vector<cudaEvent_t> ev_ck;    // [slot * kCkEvents + i]: host-tier copy chunks in flight
 };
 
@@ -271,6 +288,7 @@ struct sf_runtime {
   bool shutting_down = false;
   std::atomic<bool> stop_spin{false};
   std::vector<sf_trace_event> trace;
+  std::thread clk;  // refreshes every local slot's device clock anchor (Slot::Anchor)
   size_t trace_cap = 1 << 16;
   size_t trace_dropped = 0;
   // background builder of per-buffer-pair inference chain graphs (SF_INFER_GRAPH=1)
@@ -953,6 +971,7 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
   J.ev_r.assign(n, nullptr);
   J.ev_ring.assign(n * kMaxInflight, nullptr);
+  J.ev_start.assign(n * kMaxInflight, nullptr);
   J.ev_ck.assign(n * kCkEvents, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
@@ -960,9 +979,11 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
     if (rt->slots[s]->remote) continue;
     SF_CK(cudaSetDevice(rt->slots[s]->cuda));
     SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
-    SF_CK(cudaEventCreateWithFlags(&J.ev_r[s], cudaEventDisableTiming));
-    for (int i = 0; i < kMaxInflight; ++i)
-      SF_CK(cudaEventCreateWithFlags(&J.ev_ring[s * kMaxInflight + i], cudaEventDisableTiming));
+    SF_CK(cudaEventCreate(&J.ev_r[s]));  // timing: device resume point
+    for (int i = 0; i < kMaxInflight; ++i) {  // timing events: device intervals of subgraphs
+      SF_CK(cudaEventCreate(&J.ev_ring[s * kMaxInflight + i]));
+      SF_CK(cudaEventCreate(&J.ev_start[s * kMaxInflight + i]));
+    }
     for (int i = 0; i < kCkEvents; ++i)
       SF_CK(cudaEventCreateWithFlags(&J.ev_ck[s * kCkEvents + i], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_a[s]));
@@ -1007,6 +1028,63 @@ float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
   }
   return ms * 1000.f;
 }
+
+// ---- device clock (trace intervals on the GPU timeline, reading Q37) -------------
+// One anchor: 3 stamp rounds on the slot's high-priority clock stream; the round with the
+// tightest host window (launch .. value observed in pinned memory) becomes the anchor.
+cudaError_t refresh_anchor(Slot& S) {
+  cudaError_t e = cudaSetDevice(S.cuda);
+  if (e != cudaSuccess) return e;
+  Slot::Anchor best{nullptr, 0, 0, 0, ~0ull};
+  for (int round = 0; round < 3; ++round) {
+    volatile unsigned long long* h = S.clk_host;
+    *h = 0ull;
+    cudaEvent_t ev = nullptr;
+    if ((e = cudaEventCreate(&ev)) != cudaSuccess) return e;
+    const uint64_t h0 = now_ns();
+    e = sfk::launch_stamp(S.clk_dev, S.s_clk);
+    if (e == cudaSuccess) e = cudaEventRecord(ev, S.s_clk);
+    if (e != cudaSuccess) { cudaEventDestroy(ev); return e; }
+    unsigned long long g = 0;
+    while ((g = *h) == 0ull) {
+      if (now_ns() - h0 > 200000000ull) break;  // 200 ms: the device is saturated, skip
+      cpu_relax();
+    }
+    const uint64_t h1 = now_ns();
+    if ((e = cudaEventSynchronize(ev)) != cudaSuccess) { cudaEventDestroy(ev); return e; }
+    if (g == 0ull || (h1 - h0) / 2 >= best.unc_ns) { cudaEventDestroy(ev); continue; }
+    if (best.ev) cudaEventDestroy(best.ev);
+    best = Slot::Anchor{ev, h0, g, static_cast<int64_t>((h0 + h1) / 2) - static_cast<int64_t>(g),
+                        (h1 - h0) / 2};
+  }
+  if (!best.ev) return cudaSuccess;
+  std::lock_guard<std::mutex> lk(S.clk_m);
+  S.anchors.push_back(best);
+  while (S.anchors.size() > 64) {
+    cudaEventDestroy(S.anchors.front().ev);
+    S.anchors.pop_front();
+  }
+  return cudaSuccess;
+}
+
+// CLOCK_MONOTONIC ns of a completed timing event of slot S enqueued at host time enq_ns (by the
+// latest anchor enqueued at least 100 us earlier, so elapsed() is positive); 0 if unavailable.
+uint64_t event_host_ns(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
+  std::lock_guard<std::mutex> lk(S.clk_m);
+  const Slot::Anchor* a = nullptr;
+  for (auto it = S.anchors.rbegin(); it != S.anchors.rend(); ++it)
+    if (it->enq_ns + 100000 <= enq_ns) { a = &*it; break; }
+  if (!a) return 0;
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, a->ev, ev) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  const double dev_ns = static_cast<double>(a->g_ns) + static_cast<double>(ms) * 1e6;
+  return static_cast<uint64_t>(dev_ns + static_cast<double>(a->offset_ns));
+}
+
+void clock_main(sf_runtime* rt);
 
 bool slot_has_inference(sf_runtime* rt, int s) { return !slot_of(rt, s).q.empty(); }
 
@@ -1801,6 +1879,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
       // wait on the peer store) has executed when this event completes on the device
       cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
+      if (e == cudaSuccess) e = cudaEventRecord(J.ev_start[dev * kMaxInflight + ev], S.s_train);
       if (e == cudaSuccess && F) {  // this iteration's fed tensors into the arena, then S_0
         const uint8_t* src = (F->shared ? F->dbuf : F->host) + fslot * F->stride;
         uint8_t* arena = g.bind[dev]->arena;
@@ -1873,6 +1952,16 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     const uint64_t t1 = now_ns();
     if (f.stamp && !t_res) t_res = t1;
+    // device execution interval on the host clock (0 when no anchor covers it)
+    uint64_t d0 = 0, d1 = 0;
+    if (e == cudaSuccess) {
+      d0 = event_host_ns(S, J.ev_start[f.dev * kMaxInflight + f.ev], f.t0);
+      d1 = event_host_ns(S, J.ev_ring[f.dev * kMaxInflight + f.ev], f.t0);
+      if (f.stamp) {  // the resume point as the GPU saw it
+        const uint64_t r = event_host_ns(S, J.ev_r[f.dev], f.t0);
+        if (r) t_res = r;
+      }
+    }
     float unpack_us = -1.f, h2d_us = 0.f, peer_us = -1.f;
     if (e == cudaSuccess && f.stamp && J.adopted_pending) {
       J.adopted_pending = false;  // the copy was timed by the exporting process
@@ -1908,6 +1997,8 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     tev.iter = f.it;
     tev.t0_ns = std::max(f.t0, last_t1);  // queued behind its predecessor on the stream
     tev.t1_ns = t1;
+    tev.d0_ns = d0;
+    tev.d1_ns = d1;
     {
       const double d = (t1 - tev.t0_ns) * 1e-3;
       est_us[f.k] = est_us[f.k] > 0.0 ? 0.75 * est_us[f.k] + 0.25 * d : d;
@@ -1968,6 +2059,20 @@ void graph_builder_main(sf_runtime* rt) {
       B.chain_pending.erase({job.in, job.out});
       if (ok) B.chain_graphs[{job.in, job.out}] = {exec, static_cast<uint64_t>(nk)};
     }
+    lk.lock();
+  }
+}
+
+// Refreshes every local slot's clock anchor every 200 ms (float elapsed times stay exact to
+// well under 1 us; offset drift between the GPU timer and CLOCK_MONOTONIC is re-measured).
+void clock_main(sf_runtime* rt) {
+  std::unique_lock<std::mutex> lk(rt->m);
+  while (!rt->shutting_down) {
+    rt->cv.wait_for(lk, std::chrono::milliseconds(200), [&] { return rt->shutting_down; });
+    if (rt->shutting_down) break;
+    lk.unlock();
+    for (auto& S : rt->slots)
+      if (!S->remote && refresh_anchor(*S) != cudaSuccess) cudaGetLastError();
     lk.lock();
   }
 }
@@ -2148,10 +2253,16 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       dev_ms = -1.f;
       cudaGetLastError();
     }
+    uint64_t d0 = 0, d1 = 0;
+    if (e == cudaSuccess) {
+      d0 = event_host_ns(*S, S->ev_i0, tl0);
+      d1 = event_host_ns(*S, S->ev_infer, tl0);
+    }
     lk.lock();
-    // an early-launched chain starts on the device when the job's drain completes: its start
-    // is taken as completion - device time (never earlier than the true device start)
-    r->start = dep && dev_ms >= 0.f ? std::max(t0, t1 - static_cast<uint64_t>(dev_ms * 1e6f)) : t0;
+    // start = the request chain's start on the GPU (device clock); without an anchor: an
+    // early-launched chain starts when the job's drain completes, taken as completion - device
+    // time (never earlier than the true device start)
+    r->start = d0 ? d0 : dep && dev_ms >= 0.f ? std::max(t0, t1 - static_cast<uint64_t>(dev_ms * 1e6f)) : t0;
     r->end = t1;
     r->device_us = dev_ms >= 0.f ? dev_ms * 1e3f : -1.f;
     r->launch_us = static_cast<float>((tl1 - tl0) * 1e-3);
@@ -2163,6 +2274,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     sf_trace_event ev{};
     ev.dev = S->id; ev.job = static_cast<int32_t>(kInferOwner | (r->id & 0xFFFFF)); ev.kind = SF_EV_INFER;
     ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
+    ev.d0_ns = d0; ev.d1_ns = d1;
     ev.iter = dep ? static_cast<int64_t>(dep->id) : -1;  // device-ordered after that job's dispatched subgraphs
     push_trace(rt, ev);
     if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
@@ -2219,6 +2331,10 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
     SF_CK(cudaEventCreate(&S->ev_infer));
     SF_CK(cudaEventCreate(&S->ev_i0));
     SF_CK(cudaMalloc(&S->tstamp, 4 * sizeof(unsigned long long)));
+    SF_CK(cudaStreamCreateWithPriority(&S->s_clk, cudaStreamNonBlocking, hi));
+    SF_CK(cudaHostAlloc(reinterpret_cast<void**>(&S->clk_host), 64, cudaHostAllocMapped | cudaHostAllocPortable));
+    SF_CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S->clk_dev), S->clk_host, 0));
+    SF_CK(refresh_anchor(*S));
     if (cfg->infer_l2_persist_bytes > 0) {
       int mx = 0, mw = 0;
       SF_CK(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, c));
@@ -2245,6 +2361,7 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
   sf_runtime* p = rt.release();
   for (auto& S : p->slots)
     if (!S->remote) S->dispatcher = std::thread(dispatcher_main, p, S.get());
+  p->clk = std::thread(clock_main, p);
   if (std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1')
     p->gbuilder = std::thread(graph_builder_main, p);
   *out = p;
@@ -2271,6 +2388,7 @@ void sf_destroy(sf_runtime* rt) {
     if (J->driver.joinable()) J->driver.join();
   for (auto& S : rt->slots)
     if (S->dispatcher.joinable()) S->dispatcher.join();
+  if (rt->clk.joinable()) rt->clk.join();
   {
     std::lock_guard<std::mutex> gl(rt->gb_m);
     rt->gb_stop = true;
@@ -2317,7 +2435,10 @@ void sf_destroy(sf_runtime* rt) {
       cudaSetDevice(rt->slots[s]->cuda);
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_r[s]);
-      for (int i = 0; i < kMaxInflight; ++i) cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
+      for (int i = 0; i < kMaxInflight; ++i) {
+        cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
+        cudaEventDestroy(J->ev_start[s * kMaxInflight + i]);
+      }
       for (int i = 0; i < kCkEvents; ++i) cudaEventDestroy(J->ev_ck[s * kCkEvents + i]);
       cudaEventDestroy(J->ev_a[s]);
       cudaEventDestroy(J->ev_b[s]);
@@ -2332,6 +2453,9 @@ void sf_destroy(sf_runtime* rt) {
     cudaEventDestroy(S->ev_infer);
     cudaEventDestroy(S->ev_i0);
     cudaFree(S->tstamp);
+    for (auto& a : S->anchors) cudaEventDestroy(a.ev);
+    cudaStreamDestroy(S->s_clk);
+    cudaFreeHost(S->clk_host);
   }
   delete rt;
 }
@@ -3065,6 +3189,18 @@ static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, in
 sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
                      int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
   return op_gemm(A, B, C, M, N, K, lda, ldb, ldc, flags, nullptr, nullptr, nullptr, false, stream);
+}
+
+sf_status sf_last_gemm_path(sf_gemm_path* out) {
+  if (!out) return fail(SF_EINVAL, "null argument");
+  const sfk::GemmPath p = sfk::last_gemm_path();
+  out->kind = p.kind;
+  out->bn = p.bn;
+  out->splits = p.splits;
+  out->a_mn = p.a_mn;
+  out->b_mn = p.b_mn;
+  out->pad = 0;
+  return SF_OK;
 }
 
 sf_status sf_debug_chain_trace(void* dev_buf) {

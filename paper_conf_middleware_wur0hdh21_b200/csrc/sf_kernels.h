@@ -68,6 +68,11 @@ bool gemm_can_fuse_bias(int M, int N, int K, bool ta, bool tb, int ldb);
 uint64_t gemm_workspace_floats(int M, int N, int K, bool ta, bool tb);
 uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
+// The kernel path the calling thread's last launch_gemm took (diagnostics; sf_last_gemm_path).
+enum GemmPathKind { kGemmTma = 1, kGemmLdg = 2, kGemvTma = 3, kGemvRows = 4, kGemvCluster = 5,
+                    kGemvSplit = 6, kGemvPlain = 7 };
+struct GemmPath { int kind = 0, bn = 0, splits = 0, a_mn = 0, b_mn = 0; };
+GemmPath last_gemm_path();
 // TMA-fed variant (kernels_gemm_tma.cu): needs 16-B aligned pointers and row pitches.
 bool gemm_tma_eligible(const GemmArgs& a, int splits);
 // M <= 8 (inference): TMA-streamed cluster GEMV with fused reduction + bias/ReLU epilogue.
@@ -137,6 +142,8 @@ cudaError_t launch_adam(const AdamDesc* d, int n, uint64_t total, const int32_t*
 cudaError_t launch_feed(const void* pool, const int32_t* step, void* x, uint64_t x_bytes,
                         int64_t pool_period, cudaStream_t st);
 cudaError_t launch_step_inc(int32_t* step, cudaStream_t st);
+// Clock anchor: writes %globaltimer to dst (device-visible mapped pinned host memory).
+cudaError_t launch_stamp(unsigned long long* dst, cudaStream_t st);
 
 // Library-wide kernel launch counter (evidence of the native path).
 void count_launch(uint64_t n = 1);

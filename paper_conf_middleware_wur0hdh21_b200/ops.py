@@ -36,6 +36,18 @@ def gemm(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, flags: int = 0, st
                            flags, _s(stream)), "sf_op_gemm")
 
 
+GEMM_PATH_KINDS = {1: "tma", 2: "ldg", 3: "gemv_tma", 4: "gemv_rows", 5: "gemv_cluster",
+                   6: "gemv_split", 7: "gemv"}
+
+
+def last_gemm_path() -> dict:
+    """Kernel path of the last GEMM this thread launched (sf_last_gemm_path, diagnostics)."""
+    p = A.sf_gemm_path()
+    check(lib().sf_last_gemm_path(C.byref(p)), "sf_last_gemm_path")
+    return {"kind": GEMM_PATH_KINDS.get(p.kind, "none"), "bn": p.bn, "splits": p.splits,
+            "a_mn": bool(p.a_mn), "b_mn": bool(p.b_mn)}
+
+
 def gemm_bias_act(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, biases: Sequence[torch.Tensor],
                   relu: bool, flags: int = 0, stream=None) -> None:
     """C = act(op(A) op(B) (+C if ACC) + sum(biases)) — forward layer with fused epilogue."""

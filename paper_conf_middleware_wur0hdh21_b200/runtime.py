@@ -271,7 +271,7 @@ class Runtime:
             e = buf[i]
             kind = {A.EV_TRAIN: "train", A.EV_INFER: "infer", A.EV_HOST: "host"}.get(e.kind, "migrate")
             d = {"dev": e.dev, "job": e.job, "kind": kind, "iter": e.iter, "k": e.k,
-                 "t0": e.t0_ns, "t1": e.t1_ns}
+                 "t0": e.t0_ns, "t1": e.t1_ns, "d0": e.d0_ns, "d1": e.d1_ns}
             if kind == "infer":
                 d["arrival"] = e.arrival_ns
                 if e.iter >= 0:

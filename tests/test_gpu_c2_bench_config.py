@@ -1,0 +1,168 @@
+"""GPU parity at the configuration bench.py times (C4@1GPU, SURVEY.md 8(d) / DESIGN.md section 9).
+
+The bench's training job is the FULL ResNet-50-shaped forest: batch 8, spatial_div 1 (conv1's
+implicit-GEMM M = 100,352), 534 Keras variables + the data cursor = 535 live tensors at cut 0
+(204,881,220 B), partitioned MAX_OPS=1 with the SGD update in 8 byte-balanced chunks, run with
+an in-flight window of 2 under a 50 us time-aware budget, early launch of the preempter,
+deferred and full-duplex host round trips, a spinning dispatcher.  Bars (BASELINE.json
+north_star, "no work is lost"):
+  - migrated bytes bit-exact: the cut-0 staging equals the oracle's pack of the seeded state
+    byte for byte (header, 535 entries, payloads, zero padding);
+  - a mid-iteration cut after one full iteration: header / entries / padding bit-exact, payloads
+    within 1e-4 of the oracle (fp32) and exact (int32);
+  - seeded preemptions over 3 iterations to the host tier and to a peer slot (released arenas
+    poisoned) are bit-identical to the unpreempted GPU run, and within 1e-4 of the oracle;
+  - an open-loop stream of batch-1 requests (the bench's own preemption driver) over 20
+    iterations leaves the state bit-identical to the unpreempted run.
+"""
+import time
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import graph as OG, runner as R, schedule as SC, staging as S
+from sf_inputs import data as D, graphs as G
+from sf_inputs.ir import F32
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+HOST = -1
+BENCH = dict(max_inflight=2, inflight_budget_us=50, early_launch=True, host_duplex=True,
+             defer_migration=True, dispatch_spin_us=-1)
+
+
+def rel(a, b):
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-30))
+
+
+@pytest.fixture(scope="module")
+def W():
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_middleware_wur0hdh21_b200 import runtime as RT
+    g = G.resnet50_forest(batch=8, spatial_div=1)
+    parts = OG.partition(g, "max_ops", 1, update_chunks=8)
+    st, ds = D.init_state(g), D.datasets(g)
+    return RT, g, parts, st, ds
+
+
+def run(W, iters, schedule=(), slots=1, requests=0, **kw):
+    RT, g, parts, st, ds = W
+    cfg = dict(BENCH, poison=True)
+    cfg.update(kw)
+    rt = RT.Runtime([0] * slots, **cfg)
+    gh = rt.register(g)
+    gh.partition("max_ops", 1, update_chunks=8)
+    assert gh.n_subgraphs == len(parts)
+    for s in range(slots):
+        gh.bind(s, staging=True, host_staging=True)
+        gh.load(s, ds)
+    gh.load(0, st)
+    tms = []
+    if requests:
+        gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M")
+        ghi = rt.register(gi, priority=1)
+        ghi.partition()
+        ghi.bind(0, staging=False)
+        ghi.load(0, D.init_state(gi, seed=D.SEED_INFER))
+        x = torch.from_numpy(D.infer_inputs(gi, 1)[0]).cuda()
+        out = torch.empty(1, 1000, device="cuda")
+    job = rt.start_training(gh, 0, iters, HOST, schedule=schedule)
+    if requests:
+        rng = np.random.default_rng(7)
+        reqs = []
+        while rt.job_info(job)["state_name"] not in ("done", "failed") and len(reqs) < requests:
+            time.sleep(rng.exponential(1e-3))
+            reqs.append(rt.submit(ghi, 0, x.data_ptr(), out.data_ptr()))
+            if len(reqs) > 4:
+                tms.append(rt.wait(reqs[-5], 60))
+        tms += [rt.wait(r, 60) for r in reqs[len(tms):]]
+    rt.wait_job(job, 600)
+    info = rt.job_info(job)
+    dev = info["dev"]
+    state = {i: gh.read(dev, i) for i in st}
+    hs = gh.mem[0]["host_staging"].numpy().copy()
+    trace = rt.trace()
+    rt.close()
+    return state, info, hs, trace, tms
+
+
+def test_cut0_staging_equals_oracle_pack_all_535_entries(W):
+    RT, g, parts, st, ds = W
+    L = OG.live_set(g, parts, 0)
+    assert len(L) == 535 and OG.live_bytes(g, L) == 204_881_216 + 4
+    _, info, hs, _, _ = run(W, 1, schedule=[(0, 0, HOST)])
+    assert info["n_preemptions"] == 1
+    expect = S.pack(g, L, st, 0, 0)
+    hdr, ents = S.parse(expect)
+    assert len(ents) == 535
+    got = hs[:len(expect)].tobytes()
+    if got != expect:  # name the first differing entry
+        for (tid, dt, off, nb) in ents:
+            assert got[off:off + nb] == expect[off:off + nb], g.tensors[tid].name
+    assert got == expect
+
+
+@pytest.mark.parametrize("k_of", ["dlogits_layer20", "update_chunk"])
+def test_mid_iteration_cut_after_one_iteration(W, k_of):
+    RT, g, parts, st, ds = W
+    n = len(parts)
+    k = 20 * 5 + 3 if k_of == "dlogits_layer20" else n - 3
+    L = OG.live_set(g, parts, k)
+    if k_of == "dlogits_layer20":  # an in-flight activation crosses this cut
+        assert any(g.tensors[i].name.endswith("_dlogits") for i in L)
+    _, info, hs, _, _ = run(W, 2, schedule=[(1, k, HOST)])
+    assert info["n_preemptions"] == 1
+    ref = R.run(g, 2, st, ds, schedule=[(1, k, R.HOST)], parts=parts)
+    buf = ref.stagings[0][3]
+    hdr, ents = S.parse(buf)
+    assert [e[0] for e in ents] == L
+    ps = -(-(32 + 24 * len(ents)) // 256) * 256
+    gb = hs[:len(buf)].tobytes()
+    assert gb[:ps] == buf[:ps]  # header + entries + padding
+    for (tid, dt, off, nb) in ents:
+        a = np.frombuffer(gb[off:off + nb], np.float32 if dt == F32 else np.int32)
+        b = np.frombuffer(buf[off:off + nb], np.float32 if dt == F32 else np.int32)
+        if dt == F32:
+            assert rel(a, b) <= TOL, g.tensors[tid].name
+        else:
+            assert np.array_equal(a, b), g.tensors[tid].name
+        pad = -(-nb // 256) * 256
+        assert not any(gb[off + nb:off + pad]), g.tensors[tid].name
+
+
+def test_seeded_host_and_peer_preemptions_bitwise_and_vs_oracle(W):
+    RT, g, parts, st, ds = W
+    n = len(parts)
+    sched = D.preemption_schedule(3, n, 24, targets=[1, 0, HOST], seed=13)
+    base, _, _, _, _ = run(W, 3, slots=2)
+    got, info, _, trace, _ = run(W, 3, schedule=sched, slots=2)
+    assert info["n_preemptions"] >= 12, info
+    for i in base:
+        assert base[i].tobytes() == got[i].tobytes(), g.tensors[i].name
+    SC.check_job_order([e for e in trace if e["kind"] == "train"], {0: n}, start={0: (0, 0)})
+    ref = R.run(g, 3, st, ds, parts=parts, keep_stagings=False)
+    for i in ref.state:
+        if ref.state[i].dtype == np.float32:
+            assert rel(got[i], ref.state[i]) <= TOL, g.tensors[i].name
+        else:
+            assert np.array_equal(got[i], ref.state[i])
+
+
+def test_open_loop_requests_at_bench_config_bitwise(W):
+    """The bench's own preemption driver: requests of the 29.3M-parameter inference MLP
+    arrive open-loop (~1 per ms) while the job trains; every one that finds the job on the
+    GPU parks its live set in pinned memory (full duplex), poisoned arenas in between."""
+    RT, g, parts, st, ds = W
+    iters = 20
+    base, _, _, _, _ = run(W, iters)
+    got, info, _, trace, tms = run(W, iters, requests=400)
+    assert info["n_preemptions"] >= 5, info
+    for i in base:
+        assert base[i].tobytes() == got[i].tobytes(), g.tensors[i].name
+    evs = [e for e in trace if e["kind"] in ("train", "infer")]
+    SC.check_no_corun(evs)
+    SC.check_job_order([e for e in evs if e["kind"] == "train"], {0: len(parts)}, start={0: (0, 0)})

@@ -107,6 +107,60 @@ def test_gemm_vs_oracle(ops, M, N, K, flags):
     assert torch.equal(Ct, Ct2)
 
 
+# Shapes that take the default 128x256-tile path (use_bn256: N >= 256, no split-K at BN=256,
+# >= 100 tiles) in all four operand majorness instantiations gemm_tma_kernel<256, A_MN, B_MN>:
+# the C3 FFN / head weight gradients (TA: both operands MN-major), forward NN, the NT head,
+# TA|TB; ragged M / N / K tails; accumulate.  Each case asserts the path it took.
+GEMM_BN256 = [
+    (1024, 4096, 512, TA, True, True),        # C3 FFN dW (intermediate)
+    (4096, 1024, 512, TA, True, True),        # C3 FFN dW (output)
+    (30520, 1024, 512, TA, True, True),       # C3 head dW (word embedding, pitch-padded vocab)
+    (512, 30520, 1024, TB, False, False),     # C3 NT head: logits = h . word^T
+    (4096, 1024, 1024, 0, False, True),       # forward NN
+    (1024, 4096, 256, TA | TB, True, False),
+    (1100, 3000, 300, TA, True, True),        # ragged M, N, K
+    (1100, 3000, 300, 0, False, True),
+    (1024, 4096, 512, TA | ACC, True, True),  # accumulate
+    (1100, 3000, 300, TB | ACC, False, False),
+]
+
+
+@pytest.mark.parametrize("M,N,K,flags,a_mn,b_mn", GEMM_BN256)
+def test_gemm_bn256_tile_path_vs_oracle(ops, M, N, K, flags, a_mn, b_mn):
+    rng = np.random.default_rng(M + 5 * N + 11 * K + flags)
+    A = rng.standard_normal((K, M) if flags & TA else (M, K)).astype(np.float32)
+    B = rng.standard_normal((N, K) if flags & TB else (K, N)).astype(np.float32)
+    C0 = rng.standard_normal((M, N)).astype(np.float32)
+    ref = O.gemm(A, B, C0, flags)
+    Ct = cu(C0)
+    ops.gemm(cu(A), cu(B), Ct, flags)
+    path = ops.last_gemm_path()
+    assert path == {"kind": "tma", "bn": 256, "splits": 1, "a_mn": a_mn, "b_mn": b_mn}, path
+    got = Ct.cpu().numpy()
+    assert rel(got, ref) <= TOL, rel(got, ref)
+    Ct2 = cu(C0)
+    ops.gemm(cu(A), cu(B), Ct2, flags)
+    assert torch.equal(Ct, Ct2)
+
+
+def test_gemm_paths_of_existing_shapes(ops):
+    """The tile widths / split-K factors the planner picks for the C1 / C2 / C3 shapes of
+    GEMM_SHAPES (documents which instantiation each oracle case exercises)."""
+    seen = set()
+    for (M, N, K, flags) in GEMM_SHAPES:
+        A = torch.zeros((K, M) if flags & TA else (M, K), device="cuda")
+        B = torch.zeros((N, K) if flags & TB else (K, N), device="cuda")
+        C = torch.zeros((M, N), device="cuda")
+        ops.gemm(A, B, C, flags)
+        p = ops.last_gemm_path()
+        seen.add((p["kind"], p["bn"], p["a_mn"], p["b_mn"], p["splits"] > 1))
+    kinds = {s[0] for s in seen}
+    assert {"tma", "gemv_tma", "gemv_rows"} <= kinds, seen
+    # 128- and 64-wide tiles, with and without split-K
+    assert any(s[0] == "tma" and s[1] == 128 for s in seen) and any(s[0] == "tma" and s[1] == 64 for s in seen)
+    assert any(s[0] == "tma" and s[4] for s in seen) and any(s[0] == "tma" and not s[4] for s in seen)
+
+
 GEMM_EPI_SHAPES = [(1, 4096, 2048, 1, True), (1, 1000, 4096, 1, False), (8, 256, 784, 2, True),
                    (5, 516, 333, 3, True), (64, 256, 784, 1, True), (130, 96, 40, 2, False)]
 

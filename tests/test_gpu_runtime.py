@@ -360,7 +360,7 @@ def test_c3_full_size_mid_cut_peer_bitwise_and_sampled_oracle(P):
         rt.wait_job(job, 600)
         ji = rt.job_info(job)
         dev = ji["dev"]
-        out = {i: gh.read(dev, i) for i, t in enumerate(g.tensors) if t.kind in (0, 2)}
+        out = {i: gh.read(dev, i) for i, t in enumerate(g.tensors) if t.kind in (0, 1, 2)}
         logits = gh.read(dev, g.tid("logits"))
         loss = gh.read(dev, g.tid("loss"))
         live = gh.live_set(cut)[1]
@@ -378,7 +378,7 @@ def test_c3_full_size_mid_cut_peer_bitwise_and_sampled_oracle(P):
     # sampled oracle: the forward chain is row-independent, so logits rows can be recomputed
     # one token at a time with the oracle's ops (fp64 accumulate, fp32 outputs)
     from oracle import ops as O
-    from sf_inputs.ir import GEMM, BIAS_ACT, TB
+    from sf_inputs.ir import GEMM, BIAS_ACT, TA, TB
     rows = [0, 7, 255, 511]
     T = {i: a for i, a in st.items()}
     for r in rows:
@@ -394,6 +394,30 @@ def test_c3_full_size_mid_cut_peer_bitwise_and_sampled_oracle(P):
             elif op.type == BIAS_ACT:
                 h = O.bias_act(z, [T[b] for b in op.ins[1:]], True)
         assert rel(logits[r:r + 1], z) <= TOL, r
+    # sampled post-update state: the head's word-embedding rows (the 128x256-tile TA dW GEMM
+    # 30522x1024x512 through the padded-pitch path, then Adam at t = 1).  Its gradient
+    # dword = dlogits^T . h_pool depends on forward quantities only, which are continuous in
+    # rounding; gradients below a backward ReLU mask are not compared here, because a mask
+    # decided on a pre-activation within fp32 rounding of 0 legitimately flips (Q19).
+    ref_T = dict(st)
+    ref_T.update(ds)
+    shapes = {i: (t.rows, t.cols) for i, t in enumerate(g.tensors)}
+    from sf_inputs.ir import SOFTMAX_CE
+    for op in g.ops:
+        O.apply_op(op, ref_T, shapes)
+        if op.type == SOFTMAX_CE:
+            break
+    assert rel(loss, ref_T[g.tid("loss")]) <= TOL
+    word, wm, wv = g.tid("word_embeddings"), g.tid("word_embeddings_m"), g.tid("word_embeddings_v")
+    rng = np.random.default_rng(5)
+    vs = sorted(set([0, 1, 127, 128, 255, 256, 30519, 30520, 30521]) |
+                set(int(v) for v in rng.integers(0, 30522, 55)))
+    gword = O.gemm(ref_T[g.tid("dlogits")][:, vs], ref_T[g.tid("pool_h")], None, TA)
+    op_adam = next(op for op in g.ops if op.type == 8 and op.outs[0] == word)
+    w1, m1, v1 = O.adam(st[word][vs], st[wm][vs], st[wv][vs], gword, st[g.tid("step")], *op_adam.f[:4])
+    for name, got_t, ref_rows in (("w", base[word], w1), ("m", base[wm], m1), ("v", base[wv], v1)):
+        assert rel(got_t[vs], ref_rows) <= TOL, name
+    assert int(base[g.tid("step")][0, 0]) == 1
 
 
 @pytest.mark.parametrize("host_mode,defer", [(1, 0), (1, 1), (0, 1)])

@@ -124,6 +124,47 @@ def test_checker_rejects_long_wait_and_cut_rule():
         SC.check_cut_rule(evs)  # subgraph k=1 started at 10 after arrival 5
 
 
+def test_preempt_latency_window_and_host_outliers():
+    # two subgraphs of 10 in flight (window 2): a wait of 15 after the arrival is legal only
+    # with window >= 2
+    evs = [_ev(0, 0, "train", 0, 10), _ev(0, 0, "train", 10, 20, k=1),
+           _ev(0, 1, "infer", 20, 21, arrival=5)]
+    SC.check_preempt_latency(evs, 0, window=2)
+    with pytest.raises(SC.InvariantError):
+        SC.check_preempt_latency(evs, 0, window=1)
+    # a request whose host dispatch decision (h0) came after ready + bound is a host outlier,
+    # one dispatched in time but started late on the device is a violation
+    late_dev = dict(_ev(0, 1, "infer", 40, 41, arrival=5), h0=6)
+    late_host = dict(_ev(0, 1, "infer", 40, 41, arrival=5), h0=30)
+    r = SC.preempt_latency_report([evs[0], late_dev], 1, window=1)
+    assert len(r["violations"]) == 1 and not r["host_outliers"] and r["n"] == 1
+    r = SC.preempt_latency_report([evs[0], late_host], 1, window=1)
+    assert len(r["host_outliers"]) == 1 and not r["violations"]
+    assert r["bound"][0] == 11 and r["waits"] == [35]
+    # the ready time is the previous request's end when requests queue back to back
+    q = [_ev(0, 0, "train", 0, 10), _ev(0, 1, "infer", 10, 30, arrival=5),
+         _ev(0, 2, "infer", 30, 31, arrival=6)]
+    assert SC.preempt_latency_report(q, 0)["waits"] == [5, 0]
+
+
+def test_device_view_uses_device_intervals():
+    """Host intervals that overlap (a request observed before the subgraph's completion was
+    observed) are disjoint on the device; a device overlap is still caught."""
+    tr = dict(_ev(0, 0, "train", 0, 10), d0=2, d1=8)
+    r = dict(_ev(0, 1 << 20, "infer", 5, 30, arrival=4), d0=9, d1=20, after=0)
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun([tr, dict(r, after=None)])
+    dv = SC.device_view([tr, r])
+    assert (dv[0]["t0"], dv[0]["t1"], dv[0]["h0"]) == (2, 8, 0) and "after" not in dv[1]
+    SC.check_no_corun(dv)
+    with pytest.raises(SC.InvariantError):
+        SC.check_no_corun(SC.device_view([tr, dict(r, d0=7)]))
+    # events without a device interval pass through unchanged
+    host = {"dev": -1, "job": 5, "kind": "host", "iter": 0, "k": -1, "t0": 1, "t1": 2}
+    assert SC.device_view([host]) == [host]
+    assert SC.device_view([dict(tr, d0=0)])[0]["t0"] == 0
+
+
 def test_cut_rule_uses_dispatch_time():
     # S_1 dispatched (launch 9) before the arrival (10) but queued behind S_0 (t0 = 12):
     # allowed; a subgraph dispatched after the arrival is not
@@ -181,6 +222,14 @@ def test_priority_checker_rejects_lower_dispatch_and_late_start():
     with pytest.raises(SC.InvariantError):
         SC.check_priority(late, prio, {1: (0, 3)})
     SC.check_priority(late, prio, {1: (0, 3)}, window=3)
+    # two lower-priority subgraphs dispatched before the submission still drained after it:
+    # legal with an in-flight window of 2 only
+    two = [_ev(0, 0, "train", 0, 2), dict(_ev(0, 0, "train", 2, 4, k=1), launch=1),
+           dict(_ev(0, 0, "train", 4, 6, k=2), launch=2.5),
+           _ev(0, 1, "train", 6, 7), _ev(0, 1, "train", 7, 8, k=1)]
+    SC.check_priority(two, prio, {1: (0, 3)}, slack=10, window=2)
+    with pytest.raises(SC.InvariantError):
+        SC.check_priority(two, prio, {1: (0, 3)}, slack=10, window=1)
 
 
 def test_priority_model_closed_form():
