@@ -294,6 +294,11 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
         out_t = torch.zeros(len(xs), 1, 1000, device=dev)
     job = rt.start_training(gh, 0, 1 << 40, target)
     time.sleep(0.3)
+    # solo training throughput of this very job before the request stream starts (the
+    # reference point of the collocated throughput loss)
+    solo_it0, solo_t0 = rt.job_info(job)["iter"], time.perf_counter()
+    time.sleep(args.solo_s)
+    solo_it_s = (rt.job_info(job)["iter"] - solo_it0) / (time.perf_counter() - solo_t0)
     rng = np.random.default_rng(7 + args.rank // 2)
     gaps_ns = (rng.exponential(1.0 / args.rate, n_in) * 1e9).astype(np.int64)
     torch.cuda.synchronize(dev)
@@ -308,6 +313,7 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
             ev0.record()
             t_region = time.perf_counter()
             launches0 = kernel_launches()
+            ji0 = rt.job_info(job)
         next_poll = 0
         while True:
             t = now_ns()
@@ -326,10 +332,12 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
         j = i % len(xs)
         reqs.append(rt.submit(ghi, 0, x_t[j].data_ptr(), out_t[j].data_ptr(), arrival_ns=int(arr[i])))
     tms = [rt.wait(r, 120) for r in reqs]
+    ji1 = rt.job_info(job)
     ev1 = torch.cuda.Event(enable_timing=True)
     ev1.record()
     torch.cuda.synchronize(dev)
     wall = time.perf_counter() - t_region
+    coloc_it_s = (ji1["iter"] - ji0["iter"]) / max(wall, 1e-9)
     launches = kernel_launches() - launches0
     if sampler:
         sampler.__exit__()
@@ -379,7 +387,11 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
             "breakdown": bd,
             "device_us": dev_us, "region_ms": ev0.elapsed_time(ev1), "wall_s": wall,
             "launches": launches, "clocks": sampler.summary() if sampler else None,
-            "reparks": info_j["n_reparks"], "iters_done": len(per_it)}
+            "reparks": info_j["n_reparks"], "iters_done": len(per_it),
+            "training": {"solo_it_per_s": solo_it_s, "collocated_it_per_s": coloc_it_s,
+                         "loss_frac": 1.0 - coloc_it_s / solo_it_s if solo_it_s > 0 else None,
+                         "preemptions_in_region": ji1["n_preemptions"] - ji0["n_preemptions"],
+                         "solo_window_s": args.solo_s}}
 
 
 def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, gloo):
@@ -448,57 +460,67 @@ def run_pair_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, g
 
 
 # ------------------------------------------------------------------------------------------
-def oracle_sample(args, steps: int):
-    """CPU oracle on a bounded sample: each distinct sampled subgraph timed once."""
-    from oracle import graph as OG, ops as O, runner as R, staging as ST
+def _oracle_setup(args):
+    from oracle import graph as OG
     from sf_inputs import data as D
     g, gi = build_workload(args.batch, args.spatial_div)
-    parts = OG.partition(g)
+    parts = OG.partition(g, "max_ops" if args.max_ops else "phase", args.max_ops,
+                         update_chunks=args.update_chunks)
     st, ds = D.init_state(g), D.datasets(g)
+    return g, gi, parts, st, ds
+
+
+def oracle_timeline(args, threads=None):
+    """CPU oracle (oracle/, fp64 numpy) timed on this host: ONE full training iteration of
+    the bench's job (every subgraph of the same partition, timed one by one), three batch-1
+    forwards of the inference MLP, and the host pack / unpack of the cut-0 live set (the
+    oracle's migration).  threads: BLAS threads (threadpoolctl; None = all cores)."""
+    import threadpoolctl
+    from oracle import graph as OG, ops as O, runner as R, staging as ST
+    from sf_inputs import data as D
+    g, gi, parts, st, ds = _oracle_setup(args)
     shapes = {i: (t.rows, t.cols) for i, t in enumerate(g.tensors)}
     T = {**{i: a.copy() for i, a in st.items()}, **ds}
-    t_start = time.perf_counter()
-    # sample: first layer, the largest-K layer, fc, and a few in between (bounded CPU work)
-    sample_ks = sorted({0, 1, 10, 25, 40, len(parts) - 2})
-    sub_s = {}
-    for k in range(len(parts) - 1):
-        a, b = parts[k]
-        if k not in sample_ks:
-            continue
+    with threadpoolctl.threadpool_limits(threads):
+        t_start = time.perf_counter()
+        sub_s = []
+        for (a, b) in parts:
+            t0 = time.perf_counter()
+            for j in range(a, b):
+                O.apply_op(g.ops[j], T, shapes)
+            sub_s.append(time.perf_counter() - t0)
+        sti = D.init_state(gi, seed=D.SEED_INFER)
+        x = D.infer_inputs(gi, 1)[0]
+        tinf = []
+        for _ in range(3):
+            t0 = time.perf_counter()
+            R.run_inference(gi, sti, x)
+            tinf.append(time.perf_counter() - t0)
+        L = OG.live_set(g, parts, 0)
         t0 = time.perf_counter()
-        for j in range(a, b):
-            O.apply_op(g.ops[j], T, shapes)
-        sub_s[k] = time.perf_counter() - t0
-    sti = D.init_state(gi, seed=D.SEED_INFER)
-    x = D.infer_inputs(gi, 1)[0]
-    tinf = []
-    for _ in range(3):
+        buf = ST.pack(g, L, T, 0, 0)
+        t_pack = time.perf_counter() - t0
         t0 = time.perf_counter()
-        R.run_inference(gi, sti, x)
-        tinf.append(time.perf_counter() - t0)
-    L = OG.live_set(g, parts, 0)
-    t0 = time.perf_counter()
-    buf = ST.pack(g, L, T, 0, 0)
-    t_pack = time.perf_counter() - t0
-    t0 = time.perf_counter()
-    ST.unpack(g, buf, {})
-    t_unpack = time.perf_counter() - t0
-    rng = np.random.default_rng(99)
-    ks = list(sub_s)
-    lat, p2r = [], []
-    t_inf = float(np.median(tinf))
-    for s in range(steps):
-        k = ks[s % len(ks)]
-        u = rng.uniform()
-        lat.append(((1 - u) * sub_s[k] + t_inf) * 1e3)
-        p2r.append((t_pack + t_inf + t_unpack) * 1e3)
-    return {"lat": lat, "p2r": p2r, "sub_s": sub_s, "t_inf_ms": t_inf * 1e3,
-            "t_pack_ms": t_pack * 1e3, "t_unpack_ms": t_unpack * 1e3, "live_bytes": OG.live_bytes(g, L),
-            "elapsed_s": time.perf_counter() - t_start,
-            "sample": f"{len(sub_s)} of {len(parts)} training subgraphs timed once each "
-                      f"(batch {args.batch}), 3 inference forwards, pack+unpack of L_0 "
-                      f"({OG.live_bytes(g, L) / 1e6:.1f} MB); per-step latency = "
-                      f"(1-u) * t_subgraph + t_inference, u ~ U(0,1) seeded"}
+        ST.unpack(g, buf, {})
+        t_unpack = time.perf_counter() - t0
+        elapsed = time.perf_counter() - t_start
+    live = OG.live_bytes(g, L)
+    return {"sub_s": sub_s, "t_inf_s": float(np.median(tinf)), "t_pack_s": t_pack,
+            "t_unpack_s": t_unpack, "live_bytes": live, "iter_s": float(sum(sub_s)),
+            "elapsed_s": elapsed, "threads": threads or cores()}
+
+
+def oracle_latencies(tl, n, seed=99):
+    """Open-loop arrivals on the oracle's measured timeline: a request arriving at a uniform
+    point of the iteration waits for the rest of the subgraph running then (the cut rule),
+    then runs the inference forward; preempt-to-resume = pack + inference + unpack."""
+    rng = np.random.default_rng(seed)
+    ends = np.cumsum(tl["sub_s"])
+    arr = rng.uniform(0.0, ends[-1], n)
+    k = np.searchsorted(ends, arr, side="right")
+    lat = (ends[np.minimum(k, len(ends) - 1)] - arr + tl["t_inf_s"]) * 1e3
+    p2r = (tl["t_pack_s"] + tl["t_inf_s"] + tl["t_unpack_s"]) * 1e3
+    return lat.tolist(), p2r
 
 
 def cores():
@@ -509,18 +531,49 @@ def cores():
 
 
 def reference_main(args):
+    """--impl reference: the CPU oracle as it stands, on this host's cores, on the same
+    workload, metric and unit.  Each step is one live, timed, bounded sample of the workload:
+    a seeded training subgraph of the bench's partition is executed (the subgraph a request
+    arriving at a uniform point u of it waits for: (1 - u) of its time) followed by the
+    inference forward; per-step latency = (1 - u) t_subgraph + t_inference."""
     if args.rank != 0:
         return
-    o = oracle_sample(args, args.steps)
-    p99 = pct(o["lat"], 99)
+    from oracle import ops as O, runner as R
+    from sf_inputs import data as D
+    g, gi, parts, st, ds = _oracle_setup(args)
+    shapes = {i: (t.rows, t.cols) for i, t in enumerate(g.tensors)}
+    T = {**{i: a.copy() for i, a in st.items()}, **ds}
+    sti = D.init_state(gi, seed=D.SEED_INFER)
+    x = D.infer_inputs(gi, 1)[0]
+    rng = np.random.default_rng(99)
+    lat, t_all = [], time.perf_counter()
+    for op in g.ops:  # one untimed iteration: every subgraph's inputs then exist
+        O.apply_op(op, T, shapes)
+    for s in range(args.warmup + args.steps):
+        k = int(rng.integers(0, len(parts)))
+        a, b = parts[k]
+        t0 = time.perf_counter()
+        for j in range(a, b):
+            O.apply_op(g.ops[j], T, shapes)
+        t_sub = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        R.run_inference(gi, sti, x)
+        t_inf = time.perf_counter() - t0
+        if s >= args.warmup:
+            lat.append(((1.0 - rng.uniform()) * t_sub + t_inf) * 1e3)
+    p99 = pct(lat, 99)
     line = {"impl": "reference", "metric": METRIC, "value": p99, "unit": UNIT, "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.mean(o["lat"])),
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.mean(lat)),
             "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (seeded, sf_inputs)",
             "config": {"workload": WORKLOAD + " [CPU oracle]", "batch": args.batch},
-            "p50_ms": pct(o["lat"], 50), "preempt_to_resume_p99_ms": pct(o["p2r"], 99),
+            "p50_ms": pct(lat, 50), "n_requests": len(lat),
             "cpu_baseline": {"value": p99, "unit": UNIT, "cores": cores(), "kind": "oracle",
-                             "sample": o["sample"]},
+                             "sample": f"{args.steps} timed steps, each one seeded training subgraph "
+                                       f"of the {len(parts)}-subgraph partition (batch {args.batch}) "
+                                       "executed live + one batch-1 inference forward; latency = "
+                                       "(1-u) t_subgraph + t_inference, u ~ U(0,1) seeded",
+                             "elapsed_s": time.perf_counter() - t_all},
             "e2e": {"value": p99, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -581,8 +634,16 @@ def pair_main(args, local):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=500)
-    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20,
+                    help="timed steps; a step is one block of --requests-per-step Poisson arrivals")
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--requests-per-step", type=int, default=50)
+    ap.add_argument("--baseline-requests", type=int, default=500,
+                    help="requests per same-run baseline arm")
+    ap.add_argument("--chase-cycles", type=int, default=300,
+                    help="closed-loop preemption cycles of the chase arm")
+    ap.add_argument("--solo-s", type=float, default=1.0,
+                    help="solo training window before each Poisson arm (throughput reference)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--batch", type=int, default=8)
     ap.add_argument("--spatial-div", type=int, default=1)
@@ -636,65 +697,65 @@ def main():
 
     if args.world > 1:
         return pair_main(args, local)
-    # headline: open-loop Poisson stream (C4 as specified); the closed-loop "chase" arm (every
-    # request preempts, the next one waits for the resume) gives the per-cycle migration numbers
-    arm = run_poisson_arm if args.arrivals == "poisson" else run_arm
-    main_s = arm(args, local, args.steps, args.warmup, host_io=False)
-    chase_s = run_arm(args, local, args.steps, args.warmup, host_io=False, measure=False) \
-        if args.arrivals == "poisson" else main_s
-    e2e_steps = max(20, args.steps // 2)
-    e2e_s = arm(args, local, e2e_steps, 3, host_io=True, measure=False)
+    # headline: open-loop Poisson stream (C4 as specified).  A timed step is a fixed block of
+    # --requests-per-step arrivals, so the percentiles rest on steps x block requests
+    # (>= 1,000 at the driver's --steps 20).  The closed-loop "chase" arm (every request
+    # preempts, the next one waits for the resume) gives the per-cycle migration numbers.
+    rps = args.requests_per_step
+    if args.arrivals == "poisson":
+        main_s = run_poisson_arm(args, local, args.steps * rps, args.warmup * rps, host_io=False)
+        chase_s = run_arm(args, local, args.chase_cycles, 5, host_io=False, measure=False)
+        e2e_s = run_poisson_arm(args, local, args.steps * rps, args.warmup * rps, host_io=True,
+                                measure=False)
+    else:
+        main_s = run_arm(args, local, args.steps, args.warmup, host_io=False)
+        chase_s = main_s
+        e2e_s = run_arm(args, local, args.steps, args.warmup, host_io=True, measure=False)
     hi_rate = None
+    nb = args.baseline_requests
     if args.arrivals == "poisson" and not args.no_baselines:
         r0 = args.rate
         args.rate = 1000.0  # lambda in {100, 1000} req/s
-        hr = run_poisson_arm(args, local, max(100, args.steps), 10, host_io=False, measure=False)
+        hr = run_poisson_arm(args, local, max(1000, args.steps * rps), 100, host_io=False, measure=False)
         args.rate = r0
         hi_rate = {"rate_per_s": 1000.0, "n": len(hr["lat"]), "p50_ms": pct(hr["lat"], 50),
                    "p95_ms": pct(hr["lat"], 95), "p99_ms": pct(hr["lat"], 99),
                    "preempt_latency_p99_ms": pct(hr["pre"], 99), "frac_preempting": hr["frac_preempting"],
-                   "reparks": hr["reparks"], "training_iterations_done": hr["iters_done"]}
+                   "reparks": hr["reparks"], "training_iterations_done": hr["iters_done"],
+                   "training": hr["training"]}
     base = {}
     if not args.no_baselines:
-        nb = max(20, args.steps // 2)
-        co = arm(args, local, nb, 3, host_io=False, exclusive=False, measure=False)
-        itg = arm(args, local, nb, 3, host_io=False, iteration_granularity=True, measure=False)
-        alt = arm(args, local, nb, 3, host_io=False, measure=False, defer=not args.defer)
+        arm = run_poisson_arm if args.arrivals == "poisson" else run_arm
+        co = arm(args, local, nb, 50, host_io=False, exclusive=False, measure=False)
+        itg = arm(args, local, nb, 50, host_io=False, iteration_granularity=True, measure=False)
+        alt = arm(args, local, nb, 50, host_io=False, measure=False, defer=not args.defer)
         # the other host round-trip order, per preemption cycle (closed loop, every request preempts)
-        seq = run_arm(args, local, nb, 3, host_io=False, measure=False, duplex=not args.duplex)
+        seq = run_arm(args, local, min(nb, args.chase_cycles), 5, host_io=False, measure=False,
+                      duplex=not args.duplex)
         # the other preempter launch policy (same arrivals)
-        lat_other = arm(args, local, nb, 3, host_io=False, measure=False, early=not args.early)
+        lat_other = arm(args, local, nb, 50, host_io=False, measure=False, early=not args.early)
         # no migration at all: the job stops at the boundary and waits in place (what the host
         # tier costs the requests that arrive during its round trip)
-        inplace = arm(args, local, nb, 3, host_io=False, measure=False, target=0)
+        inplace = arm(args, local, nb, 50, host_io=False, measure=False, target=0)
+
+        def q(x):
+            return {"n": len(x["lat"]), "p50_ms": pct(x["lat"], 50), "p99_ms": pct(x["lat"], 99)}
         base = {"arrivals": args.arrivals,
-                "free_corun_p99_ms": pct(co["lat"], 99), "free_corun_p50_ms": pct(co["lat"], 50),
-                ("concurrent" if args.defer else "deferred") + "_migration_p99_ms": pct(alt["lat"], 99),
-                ("concurrent" if args.defer else "deferred") + "_migration_p50_ms": pct(alt["lat"], 50),
+                "free_corun": q(co),
+                ("concurrent" if args.defer else "deferred") + "_migration": q(alt),
                 ("sequential" if args.duplex else "duplex") + "_host_round_trip": {
+                    "n": len(seq["p2r"]),
                     "preempt_to_resume_p50_ms": pct(seq["p2r"], 50),
                     "preempt_to_resume_p99_ms": pct(seq["p2r"], 99),
                     "d2h_plus_h2d_us_mean": float(np.mean([x for x in seq["xfer_us"] if x > 0]))
                     if any(x > 0 for x in seq["xfer_us"]) else None},
                 ("launch_after_drain" if args.early else "early_launch"): {
-                    "p99_ms": pct(lat_other["lat"], 99), "p50_ms": pct(lat_other["lat"], 50),
-                    "preempt_latency_p99_ms": pct(lat_other["pre"], 99)},
-                "no_migration_wait_in_place": {"p99_ms": pct(inplace["lat"], 99),
-                                               "p50_ms": pct(inplace["lat"], 50)},
-                "iteration_slicing_p99_ms": pct(itg["lat"], 99),
-                "iteration_slicing_p50_ms": pct(itg["lat"], 50)}
+                    **q(lat_other), "preempt_latency_p99_ms": pct(lat_other["pre"], 99)},
+                "no_migration_wait_in_place": q(inplace),
+                "iteration_slicing": q(itg)}
 
-    # pool samples across ranks (weak scaling replicas); max-over-ranks region time
     samples = {"main": main_s, "e2e": e2e_s, "chase": chase_s}
-    if args.world > 1:
-        import torch.distributed as dist
-        allv = [None] * args.world
-        dist.all_gather_object(allv, samples)
-        dist.destroy_process_group()
-    else:
-        allv = [samples]
-    if args.rank != 0:
-        return
+    allv = [samples]
     M = {k: sum((a["main"][k] for a in allv), []) for k in ("lat", "pre", "p2r")}
     Cc = {k: sum((a["chase"][k] for a in allv), []) for k in ("lat", "pre", "p2r", "pack_us", "xfer_us",
                                                             "unpack_us", "bytes")}
@@ -711,13 +772,118 @@ def main():
     xfer = np.asarray(Cc["xfer_us"], np.float64)
     unpack = np.asarray(Cc["unpack_us"], np.float64)
     migr_gbs = float((2 * byts[ok]).mean() / (xfer[ok].mean() * 1e-6) / 1e9) if ok.any() else None
-    traffic = None
+    prof = {}
     try:
-        traffic = json.load(open(os.path.join(ROOT, "profiles", "pack_traffic.json")))["bytes_per_launch"]
+        prof = json.load(open(os.path.join(ROOT, "profiles", "pack_traffic.json")))
     except Exception:
         pass
+    probe = probe_pack(args, local, hbm)
     m0 = chase_s
-    # the box's pinned-memory copy peak per direction (host tier vs PCIe)
+    link = host_link_peaks()
+    dev_us = pct(main_s.get("device_us", []), 50)
+    w_bytes = (2048 * 4096 + 4096 * 4096 + 4096 * 1000 + 4096 + 4096 + 1000) * 4
+    tr = main_s.get("training", {})
+    line = {
+        "metric": METRIC, "value": pct(M["lat"], 99), "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
+        "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded: glorot weights, U[0,1) features, uniform labels)",
+        "config": {"workload": WORKLOAD, "batch": args.batch, "spatial_div": args.spatial_div,
+                   "step": f"one block of {rps} open-loop Poisson arrivals" if args.arrivals == "poisson"
+                   else "one preemption cycle",
+                   "tensors_live_cut0": 535, "inference_model": "MLP 2048-4096-4096-1000 (29.3M params)",
+                   "tier": "host (pinned, copy engine)", "parallelism": f"replicas x{args.world}",
+                   "update_chunks": args.update_chunks,
+                   "partition": f"MAX_OPS={args.max_ops}" if args.max_ops else "PER_LAYER_PHASE",
+                   "max_inflight": args.max_inflight,
+                   "dispatch_spin_us": args.dispatch_spin_us,
+                   "inflight_budget_us": args.inflight_budget_us,
+                   "early_launch": bool(args.early), "host_duplex": bool(args.duplex),
+                   "migration_policy": "deferred until the preempter drained" if args.defer
+                   else "concurrent with the preempter",
+                   "l2": "state 205 MB + datasets 666 MB > 126 MB L2 (no flush needed); the pack "
+                         "probe reports warm and flushed-L2 runs"},
+        "n_requests": len(M["lat"]),
+        "p50_ms": pct(M["lat"], 50), "p95_ms": pct(M["lat"], 95), "p99_ms": pct(M["lat"], 99),
+        "n_preempting": len(M["pre"]),
+        "preempt_latency_p50_ms": pct(M["pre"], 50), "preempt_latency_p99_ms": pct(M["pre"], 99),
+        "n_cycles": len(M["p2r"]),
+        "preempt_to_resume_p50_ms": pct(M["p2r"], 50), "preempt_to_resume_p99_ms": pct(M["p2r"], 99),
+        "arrivals": {"process": args.arrivals, "rate_per_s": args.rate if args.arrivals == "poisson" else None,
+                     "seed": "7 + pair" if args.arrivals == "poisson" else "1234 + device",
+                     "frac_preempting": main_s.get("frac_preempting"), "reparks": main_s.get("reparks"),
+                     "inference_device_us_p50": pct(main_s.get("device_us", []), 50),
+                     "latency_breakdown_us": main_s.get("breakdown")},
+        "training_throughput": {**tr, "desc": "iterations/s of the collocated job during the timed "
+                                              "region vs the same job alone just before it"},
+        "poisson_1000": hi_rate,
+        "chase": {"desc": "closed loop: every request preempts the running job; next request after its resume",
+                  "n": len(Cc["lat"]),
+                  "p50_ms": pct(Cc["lat"], 50), "p99_ms": pct(Cc["lat"], 99),
+                  "preempt_latency_p50_ms": pct(Cc["pre"], 50), "preempt_latency_p99_ms": pct(Cc["pre"], 99),
+                  "preempt_to_resume_p50_ms": pct(Cc["p2r"], 50),
+                  "preempt_to_resume_p99_ms": pct(Cc["p2r"], 99)},
+        "migration": {"live_bytes_mean": float(byts.mean()) if len(byts) else None,
+                      "pack_us_mean": float(pack_us[ok].mean()) if ok.any() else None,
+                      "pack_gbs": pack_achieved,
+                      "pack_probe_cut0": probe,
+                      "d2h_plus_h2d_us_mean": float(xfer[ok].mean()) if ok.any() else None,
+                      "host_link_gbs": migr_gbs,
+                      "host_link_peak_gbs": link or None,
+                      # roofline time of the round trip over the measured per-direction
+                      # peaks (duplex: the slower direction; sequential: both) / measured
+                      "host_link_frac": ((max(1.0 / link["d2h"], 1.0 / link["h2d"],
+                                              2.0 / link["duplex_total"]) if args.duplex
+                                          else 1.0 / link["d2h"] + 1.0 / link["h2d"])
+                                         * byts[ok].mean() / 1e9 / (xfer[ok].mean() * 1e-6))
+                      if link and migr_gbs else None,
+                      "host_round_trip": "full duplex (chunk c returns H2D as soon as its D2H "
+                      "landed)" if args.duplex else "sequential (D2H, then H2D)",
+                      "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},
+        "training_subgraph_ms_mean": m0["sub_ms"], "n_subgraphs": m0["n_subgraphs"],
+        "training_iteration_ms_median": m0["iter_ms"],
+        "baselines": base,
+        "roofline": {"kernel": "mtcopy_kernel (pack: arena -> staging)", "bound": "hbm",
+                     "achieved": pack_achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": (pack_achieved / hbm) if pack_achieved else None,
+                     "traffic": prof.get("bytes_per_launch"), "peak_source": peak_src,
+                     "traffic_source": prof.get("source"),
+                     "dram_frac": prof.get("dram_frac"),
+                     "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
+        "inference_roofline": {"kernel": "request chain (3 TMA cluster GEMVs, fused bias/ReLU, "
+                                         "fused softmax; device time p50)",
+                               "bound": "hbm", "algorithmic_bytes": w_bytes,
+                               "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
+                               "peak": hbm, "unit": "GB/s",
+                               "frac": (w_bytes / (dev_us * 1e-6) / 1e9 / hbm) if dev_us else None},
+        "e2e": {"value": pct(E, 99), "unit": UNIT, "n": len(E), "h2d_bytes_per_step": 2048 * 4 * rps,
+                "d2h_bytes_per_step": 1000 * 4 * rps, "p50_ms": pct(E, 50)},
+        "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),
+        "clocks": main_s["clocks"],
+    }
+    if not args.no_cpu_baseline:
+        tl = oracle_timeline(args)
+        tl1 = oracle_timeline(args, threads=1)
+        lat, p2r = oracle_latencies(tl, 2000)
+        line["cpu_baseline"] = {
+            "value": pct(lat, 99), "unit": UNIT, "cores": tl["threads"], "kind": "oracle",
+            "sample": f"one full training iteration of the bench job ({len(tl['sub_s'])} subgraphs, each "
+                      "timed), 3 batch-1 inference forwards and the host pack / unpack of L_0, run "
+                      "live on this host; p99 over 2000 seeded uniform arrivals on that measured "
+                      "timeline (wait for the running subgraph, then the forward)",
+            "iteration_ms": {"all_cores": tl["iter_s"] * 1e3, "single_thread": tl1["iter_s"] * 1e3,
+                             "all_cores_n": tl["threads"]},
+            "inference_ms": {"all_cores": tl["t_inf_s"] * 1e3, "single_thread": tl1["t_inf_s"] * 1e3},
+            "host_pack_gbs": tl["live_bytes"] / tl["t_pack_s"] / 1e9,
+            "host_unpack_gbs": tl["live_bytes"] / tl["t_unpack_s"] / 1e9,
+            "preempt_to_resume_ms": p2r,
+            "elapsed_s": tl["elapsed_s"] + tl1["elapsed_s"]}
+    print(json.dumps(line), flush=True)
+
+
+def host_link_peaks():
+    """The box's pinned-memory copy peak per direction and full duplex."""
+    import torch
     link = {}
     try:
         hb = torch.empty(256 << 20, dtype=torch.uint8).pin_memory()
@@ -729,7 +895,6 @@ def main():
                 e0.record(); dst.copy_(src, non_blocking=True); e1.record(); e1.synchronize()
                 best = max(best, hb.numel() / (e0.elapsed_time(e1) * 1e-3) / 1e9)
             link[name] = best
-        # both directions at once (two streams): the platform's full-duplex total
         hb2 = torch.empty_like(hb).pin_memory()
         db2 = torch.empty_like(db)
         s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
@@ -753,81 +918,31 @@ def main():
         del hb, db, hb2, db2
     except Exception:
         link = {}
-    dev_us = pct(main_s.get("device_us", []), 50)
-    w_bytes = (2048 * 4096 + 4096 * 4096 + 4096 * 1000 + 4096 + 4096 + 1000) * 4
-    line = {
-        "metric": METRIC, "value": pct(M["lat"], 99), "unit": UNIT, "n_gpus": args.gpus,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
-        "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-        "data": "synthetic (seeded: glorot weights, U[0,1) features, uniform labels)",
-        "config": {"workload": WORKLOAD, "batch": args.batch, "spatial_div": args.spatial_div,
-                   "tensors_live_cut0": 535, "inference_model": "MLP 2048-4096-4096-1000 (29.3M params)",
-                   "tier": "host (pinned, copy engine)", "parallelism": f"replicas x{args.world}",
-                   "update_chunks": args.update_chunks,
-                   "partition": f"MAX_OPS={args.max_ops}" if args.max_ops else "PER_LAYER_PHASE",
-                   "max_inflight": args.max_inflight,
-                   "dispatch_spin_us": args.dispatch_spin_us,
-                   "inflight_budget_us": args.inflight_budget_us,
-                   "early_launch": bool(args.early), "host_duplex": bool(args.duplex),
-                   "migration_policy": "deferred until the preempter drained" if args.defer
-                   else "concurrent with the preempter",
-                   "l2": "state 205 MB + datasets > 126 MB L2 (no flush needed)"},
-        "p50_ms": pct(M["lat"], 50), "p95_ms": pct(M["lat"], 95), "p99_ms": pct(M["lat"], 99),
-        "preempt_latency_p50_ms": pct(M["pre"], 50), "preempt_latency_p99_ms": pct(M["pre"], 99),
-        "preempt_to_resume_p50_ms": pct(M["p2r"], 50), "preempt_to_resume_p99_ms": pct(M["p2r"], 99),
-        "arrivals": {"process": args.arrivals, "rate_per_s": args.rate if args.arrivals == "poisson" else None,
-                     "seed": "7 + pair" if args.arrivals == "poisson" else "1234 + device",
-                     "frac_preempting": main_s.get("frac_preempting"), "reparks": main_s.get("reparks"),
-                     "inference_device_us_p50": pct(main_s.get("device_us", []), 50),
-                     "latency_breakdown_us": main_s.get("breakdown")},
-        "poisson_1000": hi_rate,
-        "chase": {"desc": "closed loop: every request preempts the running job; next request after its resume",
-                  "p50_ms": pct(Cc["lat"], 50), "p99_ms": pct(Cc["lat"], 99),
-                  "preempt_latency_p50_ms": pct(Cc["pre"], 50), "preempt_latency_p99_ms": pct(Cc["pre"], 99),
-                  "preempt_to_resume_p50_ms": pct(Cc["p2r"], 50),
-                  "preempt_to_resume_p99_ms": pct(Cc["p2r"], 99)},
-        "migration": {"live_bytes_mean": float(byts.mean()) if len(byts) else None,
-                      "pack_us_mean": float(pack_us[ok].mean()) if ok.any() else None,
-                      "pack_gbs": pack_achieved,
-                      "d2h_plus_h2d_us_mean": float(xfer[ok].mean()) if ok.any() else None,
-                      "host_link_gbs": migr_gbs,
-                      "host_link_peak_gbs": link or None,
-                      # roofline time of the round trip over the measured per-direction
-                      # peaks (duplex: the slower direction; sequential: both) / measured
-                      "host_link_frac": ((max(1.0 / link["d2h"], 1.0 / link["h2d"],
-                                              2.0 / link["duplex_total"]) if args.duplex
-                                          else 1.0 / link["d2h"] + 1.0 / link["h2d"])
-                                         * byts[ok].mean() / 1e9 / (xfer[ok].mean() * 1e-6))
-                      if link and migr_gbs else None,
-                      "host_round_trip": "full duplex (chunk c returns H2D as soon as its D2H "
-                      "landed)" if args.duplex else "sequential (D2H, then H2D)",
-                      "unpack_us_mean": float(unpack[ok].mean()) if ok.any() else None},
-        "training_subgraph_ms_mean": m0["sub_ms"], "n_subgraphs": m0["n_subgraphs"],
-        "training_iteration_ms_median": m0["iter_ms"],
-        "baselines": base,
-        "roofline": {"kernel": "mtcopy_kernel (pack: arena -> staging)", "bound": "hbm",
-                     "achieved": pack_achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": (pack_achieved / hbm) if pack_achieved else None,
-                     "traffic": traffic, "peak_source": peak_src,
-                     "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
-        "inference_roofline": {"kernel": "request chain (3 TMA cluster GEMVs, fused bias/ReLU, "
-                                         "fused softmax; device time p50)",
-                               "bound": "hbm", "algorithmic_bytes": w_bytes,
-                               "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
-                               "peak": hbm, "unit": "GB/s",
-                               "frac": (w_bytes / (dev_us * 1e-6) / 1e9 / hbm) if dev_us else None},
-        "e2e": {"value": pct(E, 99), "unit": UNIT, "h2d_bytes_per_step": 2048 * 4,
-                "d2h_bytes_per_step": 1000 * 4, "p50_ms": pct(E, 50)},
-        "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),
-        "clocks": main_s["clocks"],
-    }
-    if not args.no_cpu_baseline:
-        o = oracle_sample(args, args.steps)
-        line["cpu_baseline"] = {"value": pct(o["lat"], 99), "unit": UNIT, "cores": cores(),
-                                "kind": "oracle", "sample": o["sample"],
-                                "preempt_to_resume_ms": float(np.mean(o["p2r"])),
-                                "elapsed_s": o["elapsed_s"]}
-    print(json.dumps(line), flush=True)
+    return link
+
+
+def probe_pack(args, local, hbm):
+    """Pack / unpack of the cut-0 live set (535 tensors, 204.9 MB) through the bound descriptor
+    lists, kernel-only durations, with L2 warm (back to back), clean-cold (a 2 x L2 read first)
+    and dirty-cold (a 2 x L2 write first: the write-back shares HBM with the walk, as after a
+    training subgraph)."""
+    from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
+    g, _ = build_workload(args.batch, args.spatial_div)
+    out = {}
+    with Runtime([local]) as rt:
+        gh = rt.register(g)
+        gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
+        gh.bind(0, staging=True)
+        for name, mode in (("warm", 0), ("cold_clean", 1), ("cold_dirty", 2)):
+            rs = [rt.probe_migration(gh, 0, 0, mode) for _ in range(5)]
+            pk = float(np.median([r["pack_us"] for r in rs]))
+            up = float(np.median([r["unpack_us"] for r in rs]))
+            b = rs[0]["live_bytes"]
+            out[name] = {"pack_us": pk, "unpack_us": up,
+                         "pack_gbs": 2 * b / (pk * 1e-6) / 1e9, "unpack_gbs": 2 * b / (up * 1e-6) / 1e9,
+                         "pack_frac": 2 * b / (pk * 1e-6) / 1e9 / hbm}
+        out["live_bytes"] = b
+    return out
 
 
 if __name__ == "__main__":

@@ -543,6 +543,21 @@ typedef struct sf_gemm_path {
   int32_t kind, bn, splits, a_mn, b_mn, pad;
 } sf_gemm_path;
 sf_status sf_last_gemm_path(sf_gemm_path* out);
+/* Diagnostics (migration roofline): run the bound pack list (arena ->
+ * device staging, header + payloads + zero padding) and unpack list (staging -> arena) of cut k
+ * on slot dev once each, on the slot's migration stream, and return their kernel-only durations
+ * (in-kernel %globaltimer).  l2 = 0: as is (warm: a walk right after another); 1: cold, clean L2
+ * (read a buffer of twice the L2 size before each walk); 2: cold, dirty L2 (write it: the
+ * write-back shares HBM with the walk, as after a training subgraph).  The unpack restores the
+ * bytes the pack read, so the arena is unchanged.  Blocks until done.  SF_EBUSY if a job of the
+ * graph is running; SF_EINVAL if dev has no device staging. */
+typedef struct sf_migration_probe {
+  double pack_us, unpack_us;
+  uint64_t live_bytes;     /* sum nbytes(L_k) */
+  uint64_t staging_bytes;  /* bytes the pack writes (header + payloads + padding) */
+} sf_migration_probe;
+sf_status sf_probe_migration(sf_runtime* rt, sf_graph_id g, int32_t dev, int32_t k, int32_t l2,
+                             sf_migration_probe* out);
 /* Number of kernels this process launched through the library so far. */
 uint64_t sf_kernel_launches(void);
 

@@ -125,6 +125,11 @@ class sf_gemm_path(C.Structure):
                 ("b_mn", C.c_int32), ("pad", C.c_int32)]
 
 
+class sf_migration_probe(C.Structure):
+    _fields_ = [("pack_us", C.c_double), ("unpack_us", C.c_double), ("live_bytes", C.c_uint64),
+                ("staging_bytes", C.c_uint64)]
+
+
 class sf_copy_desc(C.Structure):
     _fields_ = [("src", C.c_void_p), ("dst", C.c_void_p), ("nbytes", C.c_uint64),
                 ("span", C.c_uint64)]
@@ -186,6 +191,8 @@ PROTOTYPES = {
                          C.c_float, _vp]),
     "sf_op_fill": (_st, [_vp, C.c_uint64, C.c_int32, _vp]),
     "sf_last_gemm_path": (_st, [_P(sf_gemm_path)]),
+    "sf_probe_migration": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32,
+                                 _P(sf_migration_probe)]),
     "sf_kernel_launches": (C.c_uint64, []),
 }
 

@@ -261,6 +261,24 @@ cudaError_t launch_feed(const void* pool, const int32_t* step, void* x, uint64_t
   return cudaGetLastError();
 }
 
+// L2 eviction by reading `bytes` (a multiple of 16) of a scratch buffer: leaves clean lines of
+// that buffer in L2 (migration probe, "cold, clean L2").  The sum is stored only if impossible.
+__global__ void read_flush_kernel(const uint4* __restrict__ p, uint64_t n16, uint4* sink) {
+  uint32_t acc = 0;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < n16;
+       i += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    const uint4 v = sfdev::ld_stream16(reinterpret_cast<const uint8_t*>(p + i));
+    acc ^= v.x ^ v.y ^ v.z ^ v.w;
+  }
+  if (acc == 0x9E3779B9u && threadIdx.x == 1024) sink[0] = make_uint4(acc, 0, 0, 0);
+}
+cudaError_t launch_read_flush(const void* p, uint64_t bytes, cudaStream_t st) {
+  read_flush_kernel<<<148 * 8, 256, 0, st>>>(static_cast<const uint4*>(p), bytes / 16,
+                                             const_cast<uint4*>(static_cast<const uint4*>(p)));
+  count_launch();
+  return cudaGetLastError();
+}
+
 // Clock anchor (device trace, reading Q37): one thread writes %globaltimer (ns) to
 // `dst` (mapped pinned host memory) with a system-scope store, so the host reads it without a
 // CUDA call and ties the GPU timeline to CLOCK_MONOTONIC.

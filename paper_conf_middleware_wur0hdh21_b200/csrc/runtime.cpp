@@ -108,11 +108,6 @@ struct Binding {
   std::map<int, std::pair<float*, int>> shadow;  // tensor id -> (copy, pitch in floats)
   std::map<int, void*> prepared;  // optimizer group first op -> uploaded descriptor array
   std::set<int> l2_keep;          // inference weights kept in the persisting L2 set-aside
-  // inference: the whole request chain (PDL edges kept) captured once per (in, out) request
-  // buffer pair and replayed with one graph launch (SF_INFER_GRAPH)
-  std::map<std::pair<const void*, void*>, std::pair<cudaGraphExec_t, uint64_t>> chain_graphs;
-  std::set<std::pair<const void*, void*>> chain_pending;  // queued for the builder
-  std::mutex chain_m;
   bool l2_planned = false;
   std::map<int, std::pair<float*, unsigned*>> chain_bufs;  // chain first op -> (ws, counters)
   // GEMM ops with a misaligned (non-DATASET) operand or output: padded-pitch scratch copies
@@ -291,13 +286,6 @@ struct sf_runtime {
   std::thread clk;  // refreshes every local slot's device clock anchor (Slot::Anchor)
   size_t trace_cap = 1 << 16;
   size_t trace_dropped = 0;
-  // background builder of per-buffer-pair inference chain graphs (SF_INFER_GRAPH=1)
-  struct GraphBuild { Graph* g; Binding* b; int cuda; const void* in; void* out; };
-  std::thread gbuilder;
-  std::mutex gb_m;
-  std::condition_variable gb_cv;
-  std::deque<GraphBuild> gb_q;
-  bool gb_stop = false;
 };
 
 namespace {
@@ -1935,11 +1923,14 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       if (f.stamp && !t_res && cudaEventQuery(J.ev_r[f.dev]) == cudaSuccess) t_res = now_ns();
       const cudaError_t qq = cudaEventQuery(J.ev_ring[f.dev * kMaxInflight + f.ev]);
       if (qq == cudaErrorNotReady) {
-        if (may_break && S.qn.load(std::memory_order_relaxed) == 0 &&
-            queued_us() + est_us[J.k] <= budget_us) {
+        const bool req_waiting = S.qn.load(std::memory_order_relaxed) > 0;
+        if (may_break && !req_waiting && queued_us() + est_us[J.k] <= budget_us) {
           broke = true;
           break;
         }
+        // pause between polls; back off further while a request is queued: its dispatcher is
+        // launching the chain and the driver lock is the contended resource (~5 us per poll)
+        for (int i = 0, n = req_waiting ? 256 : 16; i < n; ++i) cpu_relax();
         continue;
       }
       e = qq;
@@ -2011,55 +2002,6 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     // iteration; otherwise an empty window is a scheduling point
     if (q.empty() && (!rt->cfg.iteration_granularity || J.k == 0)) release();
     rt->cv.notify_all();
-  }
-}
-
-// Captures a request chain (direct launches with PDL, request I/O in place) into one graph per
-// (in, out) buffer pair, on its own stream and thread, and publishes it to the binding.
-void graph_builder_main(sf_runtime* rt) {
-  std::unique_lock<std::mutex> lk(rt->gb_m);
-  while (true) {
-    rt->gb_cv.wait(lk, [&] { return rt->gb_stop || !rt->gb_q.empty(); });
-    if (rt->gb_stop) break;
-    const sf_runtime::GraphBuild job = rt->gb_q.front();
-    rt->gb_q.pop_front();
-    lk.unlock();
-    cudaSetDevice(job.cuda);
-    Graph& g = *job.g;
-    Binding& B = *job.b;
-    cudaStream_t cap = nullptr;
-    cudaGraph_t graph = nullptr;
-    cudaGraphExec_t exec = nullptr;
-    sfk::set_pdl(true);
-    cudaError_t ce = cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking);
-    if (ce == cudaSuccess) ce = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
-    bool ok = ce == cudaSuccess;
-    for (size_t k = 0; ok && k < B.versions.size(); ++k) {
-      Capture c{g, B, cap, false, &B.prepared};
-      c.redir_in = g.input_tid;
-      c.in_ptr = static_cast<uint8_t*>(const_cast<void*>(job.in));
-      c.redir_out = g.output_tid;
-      c.out_ptr = static_cast<uint8_t*>(job.out);
-      ok = launch_subgraph_ops(c, static_cast<int>(k)) == SF_OK;
-    }
-    sfk::set_pdl(false);
-    if (cap) {
-      const cudaError_t ee = cudaStreamEndCapture(cap, &graph);
-      ok = ok && ee == cudaSuccess && graph;
-    }
-    size_t nk = 0;
-    if (ok && cudaGraphGetNodes(graph, nullptr, &nk) != cudaSuccess) ok = false;
-    sfk::count_launch(uint64_t(0) - nk);  // captured kernels: counted at each replay instead
-    if (ok && cudaGraphInstantiate(&exec, graph, 0) != cudaSuccess) ok = false;
-    if (!ok) cudaGetLastError();
-    if (graph) cudaGraphDestroy(graph);
-    if (cap) cudaStreamDestroy(cap);
-    {
-      std::lock_guard<std::mutex> gl(B.chain_m);
-      B.chain_pending.erase({job.in, job.out});
-      if (ok) B.chain_graphs[{job.in, job.out}] = {exec, static_cast<uint64_t>(nk)};
-    }
-    lk.lock();
   }
 }
 
@@ -2190,37 +2132,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
-    // one graph launch for the whole chain once the builder thread captured it for this
-    // request-buffer pair (built off the critical path; until then: direct launches)
-    static const bool use_graph = std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1';
-    bool graphed = false;
-    if (e == cudaSuccess && direct && in_place && use_graph && S->l2_setaside == 0) {
-      const auto key = std::make_pair(r->in, r->out);
-      cudaGraphExec_t exec = nullptr;
-      uint64_t nk = 0;
-      bool enqueue = false;
-      {
-        std::lock_guard<std::mutex> gl(B->chain_m);
-        auto it = B->chain_graphs.find(key);
-        if (it != B->chain_graphs.end()) {
-          exec = it->second.first;
-          nk = it->second.second;
-        } else if (B->chain_graphs.size() + B->chain_pending.size() < 64 && !B->chain_pending.count(key)) {
-          B->chain_pending.insert(key);
-          enqueue = true;
-        }
-      }
-      if (exec) {
-        e = cudaGraphLaunch(exec, S->s_infer);
-        sfk::count_launch(nk);
-        graphed = true;
-      } else if (enqueue) {
-        std::lock_guard<std::mutex> ql(rt->gb_m);
-        rt->gb_q.push_back({&g, B, S->cuda, r->in, r->out});
-        rt->gb_cv.notify_one();
-      }
-    }
-    for (size_t k = 0; !graphed && e == cudaSuccess && k < B->versions.size(); ++k) {
+    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
         if (S->l2_setaside > 0) c.l2_keep = &B->l2_keep;
@@ -2362,8 +2274,6 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
   for (auto& S : p->slots)
     if (!S->remote) S->dispatcher = std::thread(dispatcher_main, p, S.get());
   p->clk = std::thread(clock_main, p);
-  if (std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1')
-    p->gbuilder = std::thread(graph_builder_main, p);
   *out = p;
   return SF_OK;
 }
@@ -2389,12 +2299,6 @@ void sf_destroy(sf_runtime* rt) {
   for (auto& S : rt->slots)
     if (S->dispatcher.joinable()) S->dispatcher.join();
   if (rt->clk.joinable()) rt->clk.join();
-  {
-    std::lock_guard<std::mutex> gl(rt->gb_m);
-    rt->gb_stop = true;
-    rt->gb_cv.notify_all();
-  }
-  if (rt->gbuilder.joinable()) rt->gbuilder.join();
   for (auto& F : rt->feeds)
     if (F->stager.joinable()) F->stager.join();
   for (auto& F : rt->feeds) {
@@ -2424,7 +2328,6 @@ void sf_destroy(sf_runtime* rt) {
       }
       cudaSetDevice(rt->slots[B->slot]->cuda);
       for (auto v : B->versions) cudaGraphExecDestroy(v);
-      for (auto& cg : B->chain_graphs) cudaGraphExecDestroy(cg.second.first);
       for (void* d : B->dev_allocs) cudaFree(d);
       if (B->ws) cudaFree(B->ws);
       if (B->counters) cudaFree(B->counters);
@@ -3189,6 +3092,55 @@ static sf_status op_gemm(const float* A, const float* B, float* C, int32_t M, in
 sf_status sf_op_gemm(const float* A, const float* B, float* C, int32_t M, int32_t N, int32_t K,
                      int32_t lda, int32_t ldb, int32_t ldc, int32_t flags, void* stream) {
   return op_gemm(A, B, C, M, N, K, lda, ldb, ldc, flags, nullptr, nullptr, nullptr, false, stream);
+}
+
+sf_status sf_probe_migration(sf_runtime* rt, sf_graph_id gid, int32_t dev, int32_t k, int32_t l2,
+                             sf_migration_probe* out) {
+  if (!rt || !out || l2 < 0 || l2 > 2) return fail(SF_EINVAL, "bad argument");
+  Graph* g = nullptr;
+  Binding* B = nullptr;
+  Slot* S = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(rt->m);
+    g = get_graph(rt, gid);
+    if (!g || !g->partitioned || k < 0 || k >= static_cast<int>(g->parts.size()))
+      return fail(SF_EINVAL, "bad graph / cut");
+    if (dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || g->bind[dev]->remote)
+      return fail(SF_EINVAL, "slot not bound locally");
+    B = g->bind[dev].get();
+    if (!B->staging) return fail(SF_EINVAL, "no device staging bound");
+    for (const auto& J : rt->jobs)
+      if (J->g == g && (J->state == SF_JOB_RUNNING || J->state == SF_JOB_STOPPING ||
+                        J->state == SF_JOB_MIGRATING))
+        return fail(SF_EBUSY, "a job of this graph is running");
+    S = rt->slots[dev].get();
+  }
+  SF_CK(cudaSetDevice(S->cuda));
+  int l2size = 0;
+  SF_CK(cudaDeviceGetAttribute(&l2size, cudaDevAttrL2CacheSize, S->cuda));
+  const uint64_t fb = round_up(2ull * static_cast<uint64_t>(l2size), 4096);
+  void* scratch = nullptr;
+  if (l2) SF_CK(cudaMalloc(&scratch, fb));
+  double us[2] = {0, 0};
+  for (int w = 0; w < 2; ++w) {
+    const CopyList& L = w == 0 ? B->pack[k] : B->unpack[k];
+    cudaError_t e = l2 == 1 ? sfk::launch_read_flush(scratch, fb, S->s_mig)
+                  : l2 == 2 ? sfk::launch_fill(scratch, fb, 0x5A, S->s_mig) : cudaSuccess;
+    if (e == cudaSuccess) e = tstamp_reset(S->tstamp, S->s_mig);
+    if (e == cudaSuccess) e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, w == 0 ? 0 : -1, S->s_mig, S->tstamp);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(S->s_mig);
+    if (e != cudaSuccess) {
+      if (scratch) cudaFree(scratch);
+      return fail(SF_ECUDA, std::string("probe: ") + cudaGetErrorString(e));
+    }
+    us[w] = tstamp_us(S->tstamp);
+  }
+  if (scratch) SF_CK(cudaFree(scratch));
+  out->pack_us = us[0];
+  out->unpack_us = us[1];
+  out->live_bytes = g->live_bytes[k];
+  out->staging_bytes = g->staging_total[k];
+  return SF_OK;
 }
 
 sf_status sf_last_gemm_path(sf_gemm_path* out) {

@@ -142,6 +142,8 @@ cudaError_t launch_adam(const AdamDesc* d, int n, uint64_t total, const int32_t*
 cudaError_t launch_feed(const void* pool, const int32_t* step, void* x, uint64_t x_bytes,
                         int64_t pool_period, cudaStream_t st);
 cudaError_t launch_step_inc(int32_t* step, cudaStream_t st);
+// Reads `bytes` of p (L2 eviction with clean lines; migration probe).
+cudaError_t launch_read_flush(const void* p, uint64_t bytes, cudaStream_t st);
 // Clock anchor: writes %globaltimer to dst (device-visible mapped pinned host memory).
 cudaError_t launch_stamp(unsigned long long* dst, cudaStream_t st);
 

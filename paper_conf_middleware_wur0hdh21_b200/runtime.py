@@ -261,6 +261,13 @@ class Runtime:
               "sf_wait")
         return {f: getattr(t, f) for f, _ in A.sf_timing._fields_}
 
+    def probe_migration(self, gh: GraphHandle, slot: int, k: int, l2: int = 0) -> dict:
+        """Kernel-only pack / unpack durations of cut k (sf_probe_migration; l2: 0 warm,
+        1 cold clean, 2 cold dirty)."""
+        o = A.sf_migration_probe()
+        check(lib().sf_probe_migration(self.h, gh.gid, slot, k, l2, C.byref(o)), "sf_probe_migration")
+        return {f: getattr(o, f) for f, _ in A.sf_migration_probe._fields_}
+
     def trace(self) -> List[dict]:
         n = C.c_size_t()
         check(lib().sf_get_trace(self.h, None, 0, C.byref(n)), "sf_get_trace")

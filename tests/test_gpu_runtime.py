@@ -223,7 +223,7 @@ def test_inference_vs_oracle_and_auto_preemption_invariants(P, W, early):
     RT, A = P
     g = G.mlp_train()
     gi = G.mlp_infer()
-    rt, gh, st, ds = setup(P, g, slots=1, max_inflight=W, early_launch=early)
+    rt, gh, st, ds = setup(P, g, slots=1, max_inflight=W, early_launch=early, dispatch_spin_us=-1)
     ghi = rt.register(gi, priority=1)
     ghi.partition()
     ghi.bind(0, staging=False)
@@ -252,12 +252,30 @@ def test_inference_vs_oracle_and_auto_preemption_invariants(P, W, early):
     evs = [dict(e, job=(1 if e["kind"] == "infer" else 0)) for e in trace]
     if early:
         assert sum("after" in e for e in evs) >= 10  # the early path was taken
-    SC.check_no_corun(evs)
-    SC.check_job_order([e for e in evs if e["kind"] == "train"], {0: n}, start={0: (0, 0)})
-    SC.check_cut_rule(evs)
-    # ns: host-observed boundaries + gate; the slack absorbs OS scheduling outliers of the
-    # driver / dispatcher threads (typical waits are tens of us)
-    SC.check_preempt_latency(evs, slack=5e6)
+    SC.check_no_corun(evs)  # host intervals (supersets) with the recorded device dependency
+    # device intervals (GPU timeline, reading Q37): every train / infer event carries one
+    dv = SC.device_view(evs)
+    assert all(e["d0"] and e["d1"] >= e["d0"] for e in dv if e["kind"] in ("train", "infer"))
+    SC.check_no_corun(dv)  # no "after" needed: the GPU never ran them together
+    SC.check_job_order([e for e in dv if e["kind"] == "train"], {0: n}, start={0: (0, 0)})
+    SC.check_cut_rule(dv)
+    check_i3_device(dv, W, early)
+
+
+def check_i3_device(dv, W, early):
+    """I3 on device intervals: wait <= W x longest subgraph + slack.  Slack: 20 us when the
+    chain is enqueued behind the drain on the device (early launch: the GPU starts it the
+    moment the dispatched subgraphs end); 50 us when the host launches it after observing the
+    drain (event poll + token hand-off + first launch, Q32).  A request whose host
+    dispatch decision itself came after ready + bound (the spinning dispatcher thread was
+    descheduled) is a host outlier: at most max(1, 2%) of them, and never a device-side
+    violation."""
+    r = SC.preempt_latency_report(dv, slack=20e3 if early else 50e3, window=W)
+    print("I3 bound us", {d: b / 1e3 for d, b in r["bound"].items()},
+          "p50/max wait us", np.median(r["waits"]) / 1e3, max(r["waits"]) / 1e3,
+          "host outliers", len(r["host_outliers"]))
+    assert not r["violations"], [(e["arrival"], w) for e, w in r["violations"]]
+    assert len(r["host_outliers"]) <= max(1, int(0.02 * r["n"]))
 
 
 def test_error_paths(P):
@@ -610,6 +628,7 @@ def test_open_loop_requests_during_swap_in_are_bitwise(P, defer, duplex, early):
     trace = [e for e in rt.trace() if e["kind"] in ("train", "infer")]
     rt.close()
     SC.check_no_corun(trace)
+    SC.check_no_corun(SC.device_view(trace))
     assert info["n_preemptions"] >= (3 if early else 5), info
     print("preemptions", info["n_preemptions"], "re-parks", info["n_reparks"])
     assert_bitwise(base, got)
@@ -735,3 +754,4 @@ def test_requests_chase_peer_migrations_bitwise(P, early):
     for r in range(len(tims)):
         assert rel(out[r].cpu().numpy(), R.run_inference(gi, sti, xs[r])) <= TOL
     SC.check_no_corun(trace)
+    SC.check_no_corun(SC.device_view(trace))
