@@ -203,7 +203,17 @@ typedef struct sf_config {
                                     requests carry the job in `iter` (invariant 1 through the
                                     device dependency); ignored with iteration_granularity;
                                     0: launch after the drain was observed on the host */
-  int32_t pad1;
+  int32_t drain_gate;            /* 1 (with early_launch and max_inflight >= 2): a training
+                                    subgraph queued behind an in-flight one is enqueued behind a
+                                    stream wait on a host gate word; a request that preempts the
+                                    job holds that gate, so the GPU runs the request right after
+                                    the RUNNING subgraph and the queued one after the request
+                                    (it was dispatched before the arrival and still runs before
+                                    the cut): the preemption latency is the
+                                    running subgraph's residual only.  Dekker-style handshake
+                                    over PCIe (reading Q38); when the GPU may already
+                                    have passed the gate the request waits for both, as without
+                                    the gate.  0: off */
 } sf_config;
 
 /* Create a runtime: enables peer access between distinct CUDA devices of the slots,
@@ -459,7 +469,8 @@ typedef struct sf_trace_event {
   uint64_t arrival_ns;         /* inference: scheduled arrival; train: host dispatch time
                                   (<= t0 when queued behind an in-flight predecessor) */
   /* inference: iter = -1, or the training job whose subgraphs dispatched before t0 this
-     request was ordered after on the device (early_launch); t0 is then its dispatch time */
+     request was ordered after on the device (early_launch); t0 is then its dispatch time;
+     k = 1 when the drain gate held the job's queued subgraphs behind this request */
   uint64_t d0_ns, d1_ns;       /* DEVICE execution interval on the CLOCK_MONOTONIC axis: timing
                                   events recorded on the stream right before the subgraph's
                                   graph (request chain) and right after it, mapped through a
@@ -558,6 +569,17 @@ typedef struct sf_migration_probe {
 } sf_migration_probe;
 sf_status sf_probe_migration(sf_runtime* rt, sf_graph_id g, int32_t dev, int32_t k, int32_t l2,
                              sf_migration_probe* out);
+/* Diagnostics (C5 migration sweep): move the live set of cut k from local slot
+ * src into slot dst's arena (a local slot of another device, or a REMOTE slot mapped with
+ * sf_import_arena) once, on src's migration stream, and return the duration.  engine:
+ *   0 the peer-store descriptor walk (the product path; kernel-only %globaltimer time),
+ *   1 copy engines, one cudaMemcpyBatchAsync per ~2 MB of tensors,
+ *   2 copy engines, one cudaMemcpyAsync per tensor (per-tensor cudaMemcpyPeerAsync),
+ *   3 copy engines, ONE cudaMemcpyAsync of the arena span the live tensors cover;
+ * CE times are CUDA events around the copies.  Blocks until done.  *bytes_moved = live bytes
+ * (engine 3: the span).  SF_EBUSY if a job of the graph is running. */
+sf_status sf_probe_peer(sf_runtime* rt, sf_graph_id g, int32_t src, int32_t dst, int32_t k,
+                        int32_t engine, double* us, uint64_t* bytes_moved);
 /* Number of kernels this process launched through the library so far. */
 uint64_t sf_kernel_launches(void);
 

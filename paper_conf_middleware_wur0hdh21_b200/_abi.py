@@ -58,7 +58,7 @@ class sf_config(C.Structure):
                 ("inflight_budget_us", C.c_int32), ("migrate_home", C.c_int32),
                 ("migration_engine", C.c_int32), ("host_stage_inline", C.c_int32),
                 ("host_duplex", C.c_int32), ("infer_l2_persist_bytes", C.c_uint64),
-                ("early_launch", C.c_int32), ("pad1", C.c_int32)]
+                ("early_launch", C.c_int32), ("drain_gate", C.c_int32)]
 
 
 class sf_partition_opts(C.Structure):
@@ -191,6 +191,8 @@ PROTOTYPES = {
                          C.c_float, _vp]),
     "sf_op_fill": (_st, [_vp, C.c_uint64, C.c_int32, _vp]),
     "sf_last_gemm_path": (_st, [_P(sf_gemm_path)]),
+    "sf_probe_peer": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
+                            _P(C.c_double), _P(C.c_uint64)]),
     "sf_probe_migration": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32,
                                  _P(sf_migration_probe)]),
     "sf_kernel_launches": (C.c_uint64, []),

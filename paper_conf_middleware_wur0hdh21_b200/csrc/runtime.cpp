@@ -184,6 +184,13 @@ struct Slot {
   unsigned long long* clk_dev = nullptr;
   std::mutex clk_m;
   std::deque<Anchor> anchors;
+  // drain gate (cfg.drain_gate, reading Q38): pinned mapped words, own cache lines.
+  // gate[0] = G: a queued subgraph with ticket t runs once (int32)(G - t) >= 0; the host holds
+  // tickets >= t with G = t - 1.  gate[16] = A: the GPU writes t right before its wait on G.
+  volatile uint32_t* gate = nullptr;
+  CUdeviceptr gate_G = 0, gate_A = 0;
+  uint32_t next_ticket = 1;  // per-slot launch tickets (rt->m)
+  bool gate_held = false;
   std::atomic<int> owner{-1};  // device token (atomic: the spinning dispatcher polls it)
   size_t l2_setaside = 0, l2_max_window = 0;  // persisting L2 for inference weights
   std::deque<Request*> q;
@@ -217,6 +224,13 @@ struct Job {
   bool launching = false;
   cudaEvent_t last_ev = nullptr;
   int n_inflight = 0;
+  struct Infl { uint32_t ticket; bool gated; cudaEvent_t end; };
+  std::deque<Infl> infl;  // in-flight subgraphs, oldest first (drain gate; rt->m)
+  // drain gate: a request held this job's queued subgraphs and ran first; the job still
+  // migrates to its auto_target at its next boundary (the preemption the request triggered),
+  // even when the request already finished by then
+  bool gate_cut_pending = false;
+  uint64_t gate_t_req = 0;
   sf_cut_info cut{};
   bool resume_req = false;
   int resume_dev = -1;
@@ -635,8 +649,9 @@ sf_status upload(Binding& b, const void* host, size_t bytes, void** out) {
 // [-> BIAS_ACT] ... [-> SOFTMAX] inside [j, e), each GEMM reading the previous layer's output.
 // Returns the number of ops covered (0 = no chain of >= 2 layers starts at j).
 int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
-  // opt-in (SF_CHAIN=1): parity-tested, but on the C4 model the per-layer GEMV kernels under
-  // programmatic dependent launch are faster (inference path)
+  // opt-in (SF_CHAIN=1): the persistent streaming chain is parity-green, but on the C4 model
+  // the per-layer GEMV kernels under programmatic dependent launch measure faster (DESIGN.md
+  // reading Q39: grid-barrier and imbalance cost per layer boundary)
   static const bool enabled = std::getenv("SF_CHAIN") && std::getenv("SF_CHAIN")[0] == '1';
   if (!enabled) return 0;
   Graph& g = c.g;
@@ -1017,6 +1032,31 @@ float elapsed_us(cudaEvent_t a, cudaEvent_t b) {
   return ms * 1000.f;
 }
 
+// ---- stream memory operations (drain gate): driver entry points resolved at run time ----------
+using StreamValueFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+StreamValueFn stream_mem_fn(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return reinterpret_cast<StreamValueFn>(fn);
+}
+StreamValueFn wait_value32() {
+  static StreamValueFn f = stream_mem_fn("cuStreamWaitValue32");
+  return f;
+}
+StreamValueFn write_value32() {
+  static StreamValueFn f = stream_mem_fn("cuStreamWriteValue32");
+  return f;
+}
+constexpr uint32_t kGateOpenAhead = 0x40000000u;  // G = next ticket + this: every ticket passes
+void gate_open(Slot& S) {  // rt->m held
+  S.gate[0] = S.next_ticket + kGateOpenAhead;
+  std::atomic_thread_fence(std::memory_order_seq_cst);
+  S.gate_held = false;
+}
+
 // ---- device clock (trace intervals on the GPU timeline, reading Q37) -------------
 // One anchor: 3 stamp rounds on the slot's high-priority clock stream; the round with the
 // tightest host window (launch .. value observed in pinned memory) becomes the anchor.
@@ -1068,8 +1108,17 @@ uint64_t event_host_ns(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
     cudaGetLastError();
     return 0;
   }
+  // the host offset: from the anchor with the tightest launch..observed window within 2 s of
+  // this one (a stamp delayed behind busy SMs gives a loose window; drift over 2 s is ~us)
+  int64_t off = a->offset_ns;
+  uint64_t unc = a->unc_ns;
+  for (const auto& b : S.anchors)
+    if (b.unc_ns < unc && (b.enq_ns > a->enq_ns ? b.enq_ns - a->enq_ns : a->enq_ns - b.enq_ns) < 2000000000ull) {
+      off = b.offset_ns;
+      unc = b.unc_ns;
+    }
   const double dev_ns = static_cast<double>(a->g_ns) + static_cast<double>(ms) * 1e6;
-  return static_cast<uint64_t>(dev_ns + static_cast<double>(a->offset_ns));
+  return static_cast<uint64_t>(dev_ns + static_cast<double>(off));
 }
 
 void clock_main(sf_runtime* rt);
@@ -1752,8 +1801,9 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       const bool req_inf = slot_has_inference(rt, J.dev);
       const Job* hp = req_inf ? nullptr : higher_training(rt, J, J.dev);
       const bool has_inf = req_inf || hp != nullptr;
-      const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu && has_inf &&
-                             J.auto_target != J.dev;
+      if (J.gate_cut_pending && J.auto_target == J.dev) J.gate_cut_pending = false;  // waits in place
+      const bool auto_want = rt->cfg.auto_preempt && rt->cfg.exclusive_gpu &&
+                             (has_inf || J.gate_cut_pending) && J.auto_target != J.dev;
       // migrate_home: back to the start slot once it is free (no inference queued there, no
       // present job of priority >= ours); a peer move like any other
       const bool home_want = rt->cfg.migrate_home && !has_inf && J.dev != J.home &&
@@ -1771,9 +1821,11 @@ void driver_main(sf_runtime* rt, Job* Jp) {
           if (!J.preempt_req) {
             J.preempt_park = false;
             J.preempt_target = home_want ? J.home : J.auto_target;
-            J.t_req = req_inf ? slot_of(rt, J.dev).q.front()->arrival
-                              : hp ? hp->t_submit : now_ns();
+            J.t_req = J.gate_cut_pending ? J.gate_t_req
+                      : req_inf ? slot_of(rt, J.dev).q.front()->arrival
+                      : hp ? hp->t_submit : now_ns();
           }
+          J.gate_cut_pending = false;
           const int src = J.dev;
           const bool peer = J.preempt_target != SF_TARGET_HOST;
           if (do_preempt(rt, J, lk) != SF_OK) break;
@@ -1859,6 +1911,11 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       }
       const bool stamp = J.stamp_resume;
       J.stamp_resume = false;
+      // drain gate: a subgraph queued behind an in-flight one waits on the slot's gate word, so
+      // a request arriving meanwhile can run before it (reading Q38)
+      const bool gated = rt->cfg.drain_gate && S.gate && !q.empty();
+      const uint32_t ticket = S.next_ticket++;
+      if (rt->cfg.drain_gate && S.gate && !S.gate_held && (ticket & 0xFFFFF) == 0) gate_open(S);
       const int ev = ev_next;
       ev_next = (ev_next + 1) % W;
       const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
@@ -1867,6 +1924,14 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       // resume point: everything stream-ordered before it (H2D + unpack, or the cross-slot
       // wait on the peer store) has executed when this event completes on the device
       cudaError_t e = stamp ? cudaEventRecord(J.ev_r[dev], S.s_train) : cudaSuccess;
+      if (e == cudaSuccess && gated) {
+        // A = t (posted write), then wait until (int32)(G - t) >= 0: the GPU's read of G cannot
+        // pass its write of A on PCIe, which the dispatcher's hold handshake relies on
+        if (write_value32()(reinterpret_cast<CUstream>(S.s_train), S.gate_A, ticket, 0) != CUDA_SUCCESS ||
+            wait_value32()(reinterpret_cast<CUstream>(S.s_train), S.gate_G, ticket, CU_STREAM_WAIT_VALUE_GEQ) !=
+                CUDA_SUCCESS)
+          e = cudaErrorLaunchFailure;
+      }
       if (e == cudaSuccess) e = cudaEventRecord(J.ev_start[dev * kMaxInflight + ev], S.s_train);
       if (e == cudaSuccess && F) {  // this iteration's fed tensors into the arena, then S_0
         const uint8_t* src = (F->shared ? F->dbuf : F->host) + fslot * F->stride;
@@ -1889,6 +1954,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       }
       if (q.empty()) front_start = t0;
       q.push_back({it, k, dev, ev, t0, stamp});
+      J.infl.push_back({ticket, gated, J.ev_ring[dev * kMaxInflight + ev]});
       J.last_ev = J.ev_ring[dev * kMaxInflight + ev];
       J.n_inflight = static_cast<int>(q.size());
       if (S.qn.load(std::memory_order_acquire) > 0) rt->cv.notify_all();  // a waiting dispatcher
@@ -1969,6 +2035,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     }
     lk.lock();
     q.pop_front();
+    if (!J.infl.empty()) J.infl.pop_front();
     J.n_inflight = static_cast<int>(q.size());
     if (f.k == 0 && g.feed) feed_consumed(*g.feed, f.it, g.feed_member);
     if (f.stamp) {
@@ -2065,8 +2132,30 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     Request* r = S->q.front();
     Job* dep = free_for_inference() ? nullptr : steal_from();
     cudaEvent_t dep_ev = nullptr;
+    bool held_now = false;
     if (dep) {
       dep_ev = dep->n_inflight > 0 ? dep->last_ev : nullptr;
+      // drain gate: hold the queued subgraphs (tickets >= the second in flight) so the chain
+      // runs right after the RUNNING one.  Dekker handshake: store G = t - 1, full fence, load
+      // A.  A still < t: the GPU's read of G (which cannot pass its write of A) comes after our
+      // store, so it sees the hold.  Otherwise it may have passed: release, wait for all.
+      if (S->gate && dep->infl.size() >= 2 && dep->infl[1].gated && !S->gate_held) {
+        const uint32_t t = dep->infl[1].ticket;
+        S->gate[0] = t - 1u;
+        std::atomic_thread_fence(std::memory_order_seq_cst);
+        const uint32_t a = S->gate[16];
+        if (static_cast<int32_t>(a - t) < 0) {
+          S->gate_held = true;
+          held_now = true;
+          dep_ev = dep->infl[0].end;
+          if (!dep->gate_cut_pending) {
+            dep->gate_cut_pending = true;
+            dep->gate_t_req = r->arrival;
+          }
+        } else {
+          gate_open(*S);
+        }
+      }
       dep->holds_token = false;  // the job re-acquires the token before its next launch
       if (r->preempted_job < 0) {
         r->preempted_job = static_cast<int>(dep->id);
@@ -2188,8 +2277,10 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
     ev.d0_ns = d0; ev.d1_ns = d1;
     ev.iter = dep ? static_cast<int64_t>(dep->id) : -1;  // device-ordered after that job's dispatched subgraphs
+    ev.k = held_now ? 1 : 0;  // drain gate: the job's queued subgraphs were held behind this request
     push_trace(rt, ev);
     if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
+    if (S->gate_held && S->q.empty()) gate_open(*S);  // the held subgraphs run now
     rt->cv.notify_all();
   }
 }
@@ -2247,6 +2338,18 @@ sf_status sf_create(const sf_config* cfg, sf_runtime** out) {
     SF_CK(cudaHostAlloc(reinterpret_cast<void**>(&S->clk_host), 64, cudaHostAllocMapped | cudaHostAllocPortable));
     SF_CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&S->clk_dev), S->clk_host, 0));
     SF_CK(refresh_anchor(*S));
+    if (cfg->drain_gate) {
+      if (!wait_value32() || !write_value32()) return fail(SF_EUNSUPPORTED, "stream memory operations unavailable");
+      void* gp = nullptr;
+      SF_CK(cudaHostAlloc(&gp, 128, cudaHostAllocMapped | cudaHostAllocPortable));
+      std::memset(gp, 0, 128);
+      S->gate = static_cast<volatile uint32_t*>(gp);
+      void* dp = nullptr;
+      SF_CK(cudaHostGetDevicePointer(&dp, gp, 0));
+      S->gate_G = reinterpret_cast<CUdeviceptr>(dp);
+      S->gate_A = reinterpret_cast<CUdeviceptr>(dp) + 64;
+      gate_open(*S);
+    }
     if (cfg->infer_l2_persist_bytes > 0) {
       int mx = 0, mw = 0;
       SF_CK(cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, c));
@@ -2359,6 +2462,7 @@ void sf_destroy(sf_runtime* rt) {
     for (auto& a : S->anchors) cudaEventDestroy(a.ev);
     cudaStreamDestroy(S->s_clk);
     cudaFreeHost(S->clk_host);
+    if (S->gate) cudaFreeHost(const_cast<uint32_t*>(S->gate));
   }
   delete rt;
 }
@@ -3140,6 +3244,72 @@ sf_status sf_probe_migration(sf_runtime* rt, sf_graph_id gid, int32_t dev, int32
   out->unpack_us = us[1];
   out->live_bytes = g->live_bytes[k];
   out->staging_bytes = g->staging_total[k];
+  return SF_OK;
+}
+
+sf_status sf_probe_peer(sf_runtime* rt, sf_graph_id gid, int32_t src, int32_t dst, int32_t k,
+                        int32_t engine, double* us, uint64_t* bytes_moved) {
+  if (!rt || !us || engine < 0 || engine > 3) return fail(SF_EINVAL, "bad argument");
+  Graph* g = nullptr;
+  Binding *B = nullptr, *D = nullptr;
+  Slot* S = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(rt->m);
+    g = get_graph(rt, gid);
+    if (!g || !g->partitioned || k < 0 || k >= static_cast<int>(g->parts.size()))
+      return fail(SF_EINVAL, "bad graph / cut");
+    const int ns = static_cast<int>(rt->slots.size());
+    if (src < 0 || src >= ns || dst < 0 || dst >= ns || src == dst || !g->bind[src] || g->bind[src]->remote ||
+        !g->bind[dst])
+      return fail(SF_EINVAL, "bad slots");
+    B = g->bind[src].get();
+    D = g->bind[dst].get();
+    if (!B->peer.count(dst)) return fail(SF_EINVAL, "no peer list to dst");
+    for (const auto& J : rt->jobs)
+      if (J->g == g && (J->state == SF_JOB_RUNNING || J->state == SF_JOB_STOPPING ||
+                        J->state == SF_JOB_MIGRATING))
+        return fail(SF_EBUSY, "a job of this graph is running");
+    S = rt->slots[src].get();
+  }
+  SF_CK(cudaSetDevice(S->cuda));
+  cudaEvent_t e0, e1;
+  SF_CK(cudaEventCreate(&e0));
+  SF_CK(cudaEventCreate(&e1));
+  uint64_t moved = g->live_bytes[k];
+  cudaError_t e = tstamp_reset(S->tstamp, S->s_mig);
+  if (e == cudaSuccess) e = cudaEventRecord(e0, S->s_mig);
+  if (e == cudaSuccess) {
+    if (engine == 0) {
+      const CopyList& L = B->peer[dst][k];
+      e = sfk::launch_mtcopy(L.d, L.n, L.total_chunks, -1, S->s_mig, S->tstamp);
+    } else if (engine == 1) {
+      Job none;
+      e = ce_segments(none, *S, src, cut_segments(*g, k, B->arena, D->arena, 2), S->s_mig, false);
+    } else if (engine == 2) {
+      for (const Seg& sg : cut_segments(*g, k, B->arena, D->arena, 2))
+        if ((e = cudaMemcpyAsync(sg.dst, sg.src, sg.n, cudaMemcpyDefault, S->s_mig)) != cudaSuccess) break;
+    } else {
+      uint64_t lo = ~0ull, hi = 0;
+      for (uint32_t t : g->live[k]) {
+        lo = std::min(lo, g->T[t].offset);
+        hi = std::max(hi, g->T[t].offset + g->T[t].nbytes);
+      }
+      moved = hi > lo ? hi - lo : 0;
+      if (moved) e = cudaMemcpyAsync(D->arena + lo, B->arena + lo, moved, cudaMemcpyDefault, S->s_mig);
+    }
+  }
+  if (e == cudaSuccess) e = cudaEventRecord(e1, S->s_mig);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(S->s_mig);
+  double t = -1.0;
+  if (e == cudaSuccess) {
+    t = engine == 0 ? tstamp_us(S->tstamp) : -1.0;
+    if (t < 0) t = elapsed_us(e0, e1);
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (e != cudaSuccess) return fail(SF_ECUDA, std::string("probe peer: ") + cudaGetErrorString(e));
+  *us = t;
+  if (bytes_moved) *bytes_moved = moved;
   return SF_OK;
 }
 

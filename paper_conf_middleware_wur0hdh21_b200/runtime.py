@@ -140,7 +140,7 @@ class Runtime:
                  dispatch_spin_us: int = 0, inflight_budget_us: int = 0,
                  migrate_home: bool = False, migration_engine: int = 0,
                  host_stage_inline: bool = False, infer_l2_persist_bytes: int = 0,
-                 host_duplex: bool = False, early_launch: bool = False):
+                 host_duplex: bool = False, early_launch: bool = False, drain_gate: bool = False):
         self.ordinals = list(ordinals)
         arr = (C.c_int32 * len(self.ordinals))(*self.ordinals)
         cfg = A.sf_config(len(self.ordinals), arr, int(exclusive), int(auto_preempt),
@@ -148,7 +148,7 @@ class Runtime:
                           max_inflight, int(defer_migration), budget_bytes, dispatch_spin_us,
                           inflight_budget_us, int(migrate_home), migration_engine,
                           int(host_stage_inline), int(host_duplex), infer_l2_persist_bytes,
-                          int(early_launch), 0)
+                          int(early_launch), int(drain_gate))
         h = C.c_void_p()
         check(lib().sf_create(C.byref(cfg), C.byref(h)), "sf_create")
         self.h = h
@@ -267,6 +267,13 @@ class Runtime:
         o = A.sf_migration_probe()
         check(lib().sf_probe_migration(self.h, gh.gid, slot, k, l2, C.byref(o)), "sf_probe_migration")
         return {f: getattr(o, f) for f, _ in A.sf_migration_probe._fields_}
+
+    def probe_peer(self, gh: GraphHandle, src: int, dst: int, k: int = 0, engine: int = 0):
+        """Move cut k's live set src -> dst once (sf_probe_peer); returns (us, bytes)."""
+        us, nb = C.c_double(), C.c_uint64()
+        check(lib().sf_probe_peer(self.h, gh.gid, src, dst, k, engine, C.byref(us), C.byref(nb)),
+              "sf_probe_peer")
+        return us.value, nb.value
 
     def trace(self) -> List[dict]:
         n = C.c_size_t()

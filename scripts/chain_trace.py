@@ -25,11 +25,13 @@ for it in range(12):
     torch.cuda.synchronize()
     res.append(e0.elapsed_time(e1) * 1e3)
 lib().sf_debug_chain_trace(None)
-t = tr.view(160, 8, 8)[:, :n, :].cpu().numpy().astype(np.float64)
+t = tr.view(160, 8, 8)[:, :n + 1, :].cpu().numpy().astype(np.float64)
 t0 = t[t > 0].min()
 print("event-timed us (cold L2):", np.round(res[2:], 1))
-names = ["start", "x", "-", "box0", "units", "xchg", "out", "done"]
-for l in range(n):
+# mlp_stream_kernel events: 0 layer start, 1 my rows streamed, 2 partials of all CTAs published
+# (grid barrier), 3 reduced (next layer's x slice / the output slice); done at [n][7]
+names = ["start", "streamed", "barrier", "reduced", "-", "-", "-", "done"]
+for l in range(n + 1):
     row = []
     for e in range(8):
         v = t[:, l, e]

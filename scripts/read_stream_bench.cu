@@ -1,0 +1,158 @@
+// Micro-benchmark: pure HBM READ streaming rate on B200 for the inference chain's weight
+// stream (117 MB for the C4 model), cold L2 (a 512 MB write flush before each run), kernel
+// time from in-kernel %globaltimer (first CTA start .. last CTA end).
+//   mode 0: cp.async.bulk 1-D copies into an smem ring (one producer thread per CTA), consumer
+//           warps read the slot and release it (the mlp_stream_kernel pattern)
+//   mode 1: LDG.128 (ld.global.nc.L1::no_allocate) grid-stride, U loads in flight per thread
+// Build+run: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/rsb scripts/read_stream_bench.cu && /tmp/rsb
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include <cstdio>
+#include <cstdlib>
+#include <algorithm>
+#include <vector>
+
+#define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("%s: %s\n", #x, cudaGetErrorString(e)); return 1; } } while (0)
+
+__device__ unsigned long long g_t0 = ~0ull, g_t1 = 0;
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+
+__global__ void bulk_kernel(const float4* __restrict__ src, long long n4, int slot_f4, int slots, float* sink) {
+  extern __shared__ __align__(1024) unsigned char sm[];
+  float4* ring = reinterpret_cast<float4*>(sm);
+  uint64_t* full = reinterpret_cast<uint64_t*>(ring + size_t(slots) * slot_f4);
+  uint64_t* empty = full + slots;
+  const int tid = threadIdx.x, nc = blockDim.x - 32;
+  if (tid == 0) {
+    atomicMin(&g_t0, gtime());
+    for (int s = 0; s < slots; ++s) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(&full[s])));
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(su32(&empty[s])), "r"(nc / 32));
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const long long per = (n4 + gridDim.x - 1) / gridDim.x;
+  const long long a0 = blockIdx.x * per, a1 = min(n4, a0 + per);
+  const int nch = a1 > a0 ? static_cast<int>((a1 - a0 + slot_f4 - 1) / slot_f4) : 0;
+  if (tid >= nc) {
+    if (tid == nc) {
+      for (int j = 0; j < nch; ++j) {
+        const int s = j % slots;
+        if (j >= slots) {
+          const uint32_t par = ((j / slots) - 1) & 1;
+          asm volatile("{\n\t.reg .pred p;\n\tW1:\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W1;\n\t}"
+                       :: "r"(su32(&empty[s])), "r"(par) : "memory");
+        }
+        const long long b = a0 + static_cast<long long>(j) * slot_f4;
+        const int n = static_cast<int>(min(static_cast<long long>(slot_f4), a1 - b));
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(su32(&full[s])), "r"(n * 16) : "memory");
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     :: "r"(su32(ring + size_t(s) * slot_f4)), "l"(src + b), "r"(n * 16), "r"(su32(&full[s])) : "memory");
+      }
+    }
+  } else {
+    float acc = 0.f;
+    for (int j = 0; j < nch; ++j) {
+      const int s = j % slots;
+      const uint32_t par = (j / slots) & 1;
+      asm volatile("{\n\t.reg .pred p;\n\tW2:\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W2;\n\t}"
+                   :: "r"(su32(&full[s])), "r"(par) : "memory");
+      const float4* t = ring + size_t(s) * slot_f4;
+      for (int i = tid; i < slot_f4; i += nc) acc += t[i].x;
+      __syncwarp();
+      if ((tid & 31) == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(su32(&empty[s])) : "memory");
+    }
+    if (acc == 1234.5f) sink[0] = acc;
+  }
+  __syncthreads();
+  if (tid == 0) atomicMax(&g_t1, gtime());
+}
+
+template <int U>
+__global__ void ldg_kernel(const float4* __restrict__ src, long long n4, float* sink) {
+  if (threadIdx.x == 0) atomicMin(&g_t0, gtime());
+  float acc = 0.f;
+  const long long stride = static_cast<long long>(gridDim.x) * blockDim.x;
+  long long i = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x;
+  for (; i + (U - 1) * stride < n4; i += U * stride) {
+    float4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                   : "=f"(v[u].x), "=f"(v[u].y), "=f"(v[u].z), "=f"(v[u].w) : "l"(src + i + u * stride));
+#pragma unroll
+    for (int u = 0; u < U; ++u) acc += v[u].x + v[u].w;
+  }
+  for (; i < n4; i += stride) acc += src[i].x;
+  if (acc == 1234.5f) sink[0] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) atomicMax(&g_t1, gtime());
+}
+
+int main(int argc, char** argv) {
+  const long long bytes = argc > 1 ? atoll(argv[1]) : 117084064ll;
+  const long long n4 = bytes / 16;
+  float4* W;
+  float* sink;
+  uint8_t* flush;
+  CK(cudaMalloc(&W, n4 * 16));
+  CK(cudaMemset(W, 0, n4 * 16));
+  CK(cudaMalloc(&sink, 64));
+  CK(cudaMalloc(&flush, 512 << 20));
+  int sms = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
+  auto run = [&](auto launch, const char* name) -> int {
+    std::vector<double> us;
+    for (int it = 0; it < 7; ++it) {
+      CK(cudaMemset(flush, it, 512 << 20));
+      unsigned long long i0 = ~0ull, i1 = 0;
+      CK(cudaMemcpyToSymbol(g_t0, &i0, 8));
+      CK(cudaMemcpyToSymbol(g_t1, &i1, 8));
+      CK(cudaDeviceSynchronize());
+      launch();
+      CK(cudaGetLastError());
+      CK(cudaDeviceSynchronize());
+      unsigned long long t0, t1;
+      CK(cudaMemcpyFromSymbol(&t0, g_t0, 8));
+      CK(cudaMemcpyFromSymbol(&t1, g_t1, 8));
+      if (it) us.push_back((t1 - t0) * 1e-3);
+    }
+    double best = 1e9, med;
+    for (double u : us) best = u < best ? u : best;
+    std::vector<double> s = us;
+    std::sort(s.begin(), s.end());
+    med = s[s.size() / 2];
+    printf("%-44s best %7.2f us (%6.0f GB/s)  median %7.2f us (%6.0f GB/s)\n", name, best, bytes / (best * 1e-6) / 1e9,
+           med, bytes / (med * 1e-6) / 1e9);
+    return 0;
+  };
+  char nm[128];
+  for (int cpsm : {1, 2}) {
+    for (int slot_kb : {16, 32}) {
+      for (int ring_kb : {96, 192}) {
+        if (cpsm == 2 && ring_kb > 96) continue;
+        const int slot_f4 = slot_kb * 64, slots = ring_kb / slot_kb;
+        const size_t smem = size_t(slots) * slot_f4 * 16 + 2 * slots * 8;
+        CK(cudaFuncSetAttribute(bulk_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        for (int nc : {128, 512}) {
+          snprintf(nm, sizeof nm, "bulk %d CTA/SM slot %2d KB ring %3d KB cons %d", cpsm, slot_kb, ring_kb, nc);
+          run([&] { bulk_kernel<<<sms * cpsm, nc + 32, smem>>>(W, n4, slot_f4, slots, sink); }, nm);
+        }
+      }
+    }
+  }
+  for (int cpsm : {2, 4, 8}) {
+    snprintf(nm, sizeof nm, "ldg U=8 %d CTA/SM x 256 thr", cpsm);
+    run([&] { ldg_kernel<8><<<sms * cpsm, 256>>>(W, n4, sink); }, nm);
+    snprintf(nm, sizeof nm, "ldg U=16 %d CTA/SM x 256 thr", cpsm);
+    run([&] { ldg_kernel<16><<<sms * cpsm, 256>>>(W, n4, sink); }, nm);
+  }
+  return 0;
+}

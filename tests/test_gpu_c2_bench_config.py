@@ -152,14 +152,15 @@ def test_seeded_host_and_peer_preemptions_bitwise_and_vs_oracle(W):
             assert np.array_equal(got[i], ref.state[i])
 
 
-def test_open_loop_requests_at_bench_config_bitwise(W):
+@pytest.mark.parametrize("gate", [False, True])
+def test_open_loop_requests_at_bench_config_bitwise(W, gate):
     """The bench's own preemption driver: requests of the 29.3M-parameter inference MLP
     arrive open-loop (~1 per ms) while the job trains; every one that finds the job on the
     GPU parks its live set in pinned memory (full duplex), poisoned arenas in between."""
     RT, g, parts, st, ds = W
     iters = 20
     base, _, _, _, _ = run(W, iters)
-    got, info, _, trace, tms = run(W, iters, requests=400)
+    got, info, _, trace, tms = run(W, iters, requests=400, drain_gate=gate)
     assert info["n_preemptions"] >= 5, info
     for i in base:
         assert base[i].tobytes() == got[i].tobytes(), g.tensors[i].name
@@ -172,7 +173,12 @@ def test_open_loop_requests_at_bench_config_bitwise(W):
     SC.check_no_corun(dv)
     SC.check_job_order([e for e in dv if e["kind"] == "train"], {0: len(parts)}, start={0: (0, 0)})
     SC.check_cut_rule(dv)
-    r = SC.preempt_latency_report(dv, slack=20e3, window=2)
+    held = sum(e["kind"] == "infer" and e["k"] == 1 for e in evs)
+    print("drain gate held", held, "of", sum(e["kind"] == "infer" for e in evs))
+    if gate:
+        assert held >= 1
+    # with the drain gate only the running subgraph drains (window 1)
+    r = SC.preempt_latency_report(dv, slack=20e3, window=1 if gate else 2)
     print("I3 bound us", r["bound"][0] / 1e3, "max wait us", max(r["waits"]) / 1e3,
           "n", r["n"], "host outliers", len(r["host_outliers"]))
     assert not r["violations"], [(e["arrival"], w) for e, w in r["violations"]]
