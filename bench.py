@@ -128,7 +128,7 @@ def workload_arrays(g, gi, key):
 
 def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclusive=True,
             iteration_granularity=False, measure=True, defer=None, duplex=None,
-            early=None, target=HOST):
+            early=None, target=HOST, gate=None):
     """One runtime instance: training job + one request per step.  Returns samples."""
     import torch
     from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
@@ -141,7 +141,8 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
                  dispatch_spin_us=args.dispatch_spin_us,
                  inflight_budget_us=args.inflight_budget_us,
                  host_duplex=bool(args.duplex if duplex is None else duplex),
-                 early_launch=bool(args.early if early is None else early))
+                 early_launch=bool(args.early if early is None else early),
+                 drain_gate=bool(args.gate if gate is None else gate))
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
                         update_chunks=args.update_chunks)
@@ -256,7 +257,7 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
 
 def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
                     iteration_granularity=False, measure=True, defer=None, duplex=None,
-            early=None, target=HOST):
+            early=None, target=HOST, gate=None):
     """C4 as specified: an OPEN-LOOP Poisson request stream (rate args.rate
     req/s, arrival seed 7 + pair) against the running training job.  Each request is submitted
     at its scheduled arrival time (passed to sf_submit_inference, so any host delay counts
@@ -273,7 +274,8 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
                  dispatch_spin_us=args.dispatch_spin_us,
                  inflight_budget_us=args.inflight_budget_us,
                  host_duplex=bool(args.duplex if duplex is None else duplex),
-                 early_launch=bool(args.early if early is None else early))
+                 early_launch=bool(args.early if early is None else early),
+                 drain_gate=bool(args.gate if gate is None else gate))
     gh = rt.register(g)
     gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
@@ -578,12 +580,108 @@ def reference_main(args):
     print(json.dumps(line), flush=True)
 
 
+def run_pair_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, gloo,
+                         measure=True):
+    """C4 at N > 1 as specified: per pair (2i, 2i+1) one training job and one
+    OPEN-LOOP Poisson request stream (rate args.rate, arrival seed 7 + pair) that chases the
+    job: every request goes to the GPU the job is on (or heading to) and preempts it there, so
+    the job ping-pongs between the two GPUs through the peer-store kernel over NVLink (CUDA IPC
+    mapping).  Pairs are independent; coordination inside a pair goes through a shared mapping
+    (pairs.ShmLink)."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_wur0hdh21_b200.pairs import PoissonOps, ShmLink, finish_pair, run_pair_poisson, shm_path
+    from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime, kernel_launches, now_ns
+    from sf_inputs import data as D
+
+    g, gi = build_workload(args.batch, args.spatial_div)
+    # drain gate: validated at N = 1; two processes sharing one GPU (SF_BENCH_SAME_GPU) deadlock on
+    # it (a held stream wait in one context), so pairs run without it unless --pair-gate 1
+    rt = Runtime([local_dev, -1], exclusive=True, auto_preempt=True, defer_migration=bool(args.defer),
+                 dispatch_spin_us=args.dispatch_spin_us, inflight_budget_us=args.inflight_budget_us,
+                 max_inflight=args.max_inflight, early_launch=bool(args.early),
+                 drain_gate=bool(args.gate and args.pair_gate))
+    gh = rt.register(g)
+    gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
+    gh.bind(0, staging=False, host_staging=False)
+    arrays, arrays_i = workload_arrays(g, gi, (args.batch, args.spatial_div))
+    even = args.rank % 2 == 0
+    gh.load(0, arrays if even else {i: a for i, a in arrays.items() if g.tensors[i].kind == 3})
+    ghi = rt.register(gi, priority=1)
+    ghi.partition()
+    ghi.bind(0, staging=False)
+    ghi.load(0, arrays_i)
+    objs = [None] * args.world
+    dist.all_gather_object(objs, rt.export_arena(gh, 0), group=gloo)
+    rt.import_arena(gh, 1, objs[args.rank ^ 1])
+    xs = D.infer_inputs(gi, 64)
+    dev = torch.device("cuda", local_dev)
+    if host_io:
+        x_t, out_t = torch.from_numpy(xs).pin_memory(), torch.zeros(64, 1, 1000).pin_memory()
+    else:
+        x_t, out_t = torch.from_numpy(xs).to(dev), torch.zeros(64, 1, 1000, device=dev)
+    path = shm_path(args.rank // 2) + ("_e2e" if host_io else "")
+    if even:
+        shm = ShmLink(path, create=True)
+    dist.barrier(group=gloo)
+    if not even:
+        shm = ShmLink(path, create=False)
+    ops = PoissonOps(rt, gh, ghi, 0, 1, [x.data_ptr() for x in x_t], [o.data_ptr() for o in out_t])
+    solo = None
+    if even:
+        shm.set(ShmLink.HOLDER, args.rank)
+        ops.start()
+        time.sleep(0.3)
+        i0, t0s = rt.job_info(ops.job)["iter"], time.perf_counter()
+        time.sleep(args.solo_s)
+        solo = (rt.job_info(ops.job)["iter"] - i0) / (time.perf_counter() - t0s)
+    dist.barrier(group=gloo)
+    rng = np.random.default_rng(7 + args.rank // 2)
+    gaps = (rng.exponential(1.0 / args.rate, n_req + warmup) * 1e9).astype(np.int64)
+    t_start = [now_ns() + 20_000_000]
+    dist.broadcast_object_list(t_start, src=0, group=gloo)  # one clock (CLOCK_MONOTONIC) per host
+    arr = (t_start[0] + np.cumsum(gaps)).tolist()
+    it_start = rt.job_info(ops.job)["iter"] if even else None
+    torch.cuda.synchronize(dev)
+    sampler = ClockSampler(local_dev).__enter__() if measure else None
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    launches0 = kernel_launches()
+    S = run_pair_poisson(shm, ops, args.rank, args.rank ^ 1, arr, now_ns, warmup=warmup)
+    t_stream = (now_ns() - arr[warmup]) * 1e-9 if len(arr) > warmup else 0.0
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev1.record()
+    torch.cuda.synchronize(dev)
+    if sampler:
+        sampler.__exit__()
+    finish_pair(shm, ops, args.rank, S["seen"], group=gloo)
+    fin = rt.job_info(ops.job)["iter"] if ops.job is not None else None
+    S["region_ms"] = ev0.elapsed_time(ev1)
+    S["launches"] = kernel_launches() - launches0
+    S["clocks"] = sampler.summary() if sampler else None
+    S["solo_it_per_s"] = solo
+    S["it_start"], S["it_final"], S["t_stream_s"] = it_start, fin, t_stream
+    S["xfer_us"] = [c["xfer_us"] for c in S["out"]]
+    S["bytes"] = [c["bytes"] for c in S["out"]]
+    dist.barrier(group=gloo)
+    shm.close(unlink=even)
+    rt.close()
+    return S
+
+
 def pair_main(args, local):
-    """N>1 bench: independent GPU pairs, peer tier over NVLink."""
+    """N>1 bench: independent GPU pairs, peer tier over NVLink.  Default:
+    open-loop Poisson streams that chase each pair's job (C4 as specified); --arrivals chase:
+    the closed-loop lockstep ping-pong (one request per handoff)."""
     import torch.distributed as dist
     gloo = dist.new_group(backend="gloo")
-    main_s = run_pair_arm(args, local, args.steps, args.warmup, host_io=False, gloo=gloo)
-    e2e_s = run_pair_arm(args, local, max(20, args.steps // 2), 4, host_io=True, gloo=gloo)
+    rps = args.requests_per_step
+    if args.arrivals == "poisson":
+        main_s = run_pair_poisson_arm(args, local, args.steps * rps, args.warmup * rps, False, gloo)
+        e2e_s = run_pair_poisson_arm(args, local, max(200, args.steps * rps // 2), 20, True, gloo, measure=False)
+    else:
+        main_s = run_pair_arm(args, local, args.steps, args.warmup, host_io=False, gloo=gloo)
+        e2e_s = run_pair_arm(args, local, max(20, args.steps // 2), 4, host_io=True, gloo=gloo)
     allv = [None] * args.world
     dist.all_gather_object(allv, {"main": main_s, "e2e": e2e_s}, group=gloo)
     dist.barrier(group=gloo)
@@ -595,35 +693,67 @@ def pair_main(args, local):
     p2r = sum((a["main"]["p2r"] for a in allv), [])
     xfer = np.asarray(sum((a["main"]["xfer_us"] for a in allv), []), np.float64)
     byts = np.asarray(sum((a["main"]["bytes"] for a in allv), []), np.float64)
-    # each adopted job migrates exactly once, so its counter is that migration's live bytes
+    # every adopted job migrates out once: its counter is that migration's live bytes
     live = float(np.median(byts)) if len(byts) else float("nan")
     ok = xfer > 0
     link_gbs = float(live / (np.median(xfer[ok]) * 1e-6) / 1e9) if ok.any() else None
     E = sum((a["e2e"]["lat"] for a in allv), [])
     region_ms = max(a["main"]["region_ms"] for a in allv)
-    nvl_peak = 770.0  # B200_PROFILING.md: measured peer copy per direction (900 nominal)
+    same_gpu = os.environ.get("SF_BENCH_SAME_GPU") == "1"
+    peaks = load_peaks()
+    nvl_meas = peaks.get("nvlink_peer_gbs") or 770.0  # B200_PROFILING.md measured peer copy
+    nvl_nominal = 900.0
+    train = None
+    if args.arrivals == "poisson":
+        pairs = []
+        for r in range(0, args.world, 2):
+            a, b = allv[r]["main"], allv[r + 1]["main"]
+            fin = a["it_final"] if a["it_final"] is not None else b["it_final"]
+            t = max(a["t_stream_s"], b["t_stream_s"])
+            if fin is not None and a["it_start"] is not None and t > 0 and a["solo_it_per_s"]:
+                co = (fin - a["it_start"]) / t
+                pairs.append({"solo_it_per_s": a["solo_it_per_s"], "collocated_it_per_s": co,
+                              "loss_frac": 1.0 - co / a["solo_it_per_s"]})
+        if pairs:
+            train = {"per_pair": pairs, "loss_frac_mean": float(np.mean([p["loss_frac"] for p in pairs])),
+                     "desc": "job iterations/s while its pair's request stream chases it vs the same "
+                             "job alone just before"}
     line = {
         "metric": METRIC, "value": pct(lat, 99), "unit": UNIT, "n_gpus": args.world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": region_ms / args.steps,
         "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic (seeded: glorot weights, U[0,1) features, uniform labels)",
         "config": {"workload": f"C4@{args.world}GPU: {args.world // 2} independent GPU pairs, each one "
-                               "ResNet-50-shaped training job ping-ponged by batch-1 requests "
-                               "(peer-tier migration, CUDA IPC + NVLink peer store)",
+                               "ResNet-50-shaped training job chased by an open-loop Poisson stream of "
+                               "batch-1 requests (peer-tier migration, CUDA IPC + NVLink peer store)"
+                   if args.arrivals == "poisson" else
+                   f"C4@{args.world}GPU: {args.world // 2} pairs, closed-loop ping-pong",
+                   "step": f"one block of {rps} Poisson arrivals per pair" if args.arrivals == "poisson"
+                   else "one handoff", "rate_per_s_per_pair": args.rate,
                    "batch": args.batch, "update_chunks": args.update_chunks,
-                   "parallelism": f"{args.world // 2} pairs", "tier": "peer (NVLink)"},
+                   "parallelism": f"{args.world // 2} pairs", "tier": "peer (NVLink)",
+                   "drain_gate": bool(args.gate and args.pair_gate), "early_launch": bool(args.early),
+                   "same_gpu_functional_check": same_gpu},
+        "n_requests": len(lat),
         "p50_ms": pct(lat, 50), "p95_ms": pct(lat, 95), "p99_ms": pct(lat, 99),
+        "n_preempting": len(pre),
         "preempt_latency_p50_ms": pct(pre, 50), "preempt_latency_p99_ms": pct(pre, 99),
+        "n_migrations": len(p2r),
         "preempt_to_resume_p50_ms": pct(p2r, 50), "preempt_to_resume_p99_ms": pct(p2r, 99),
+        "training_throughput": train,
         "migration": {"live_bytes_median": live, "peer_store_us_median": float(np.median(xfer[ok])) if ok.any() else None,
                       "peer_gbs": link_gbs},
         "roofline": {"kernel": "mtcopy_kernel (peer store: local arena -> partner arena over NVLink)",
-                     "bound": "nvlink", "achieved": link_gbs, "peak": nvl_peak, "unit": "GB/s",
-                     "frac": (link_gbs / nvl_peak) if link_gbs else None, "traffic": None,
-                     "peak_source": "B200_PROFILING.md measured peer copy (770 GB/s/dir)",
+                     "bound": "nvlink", "achieved": link_gbs, "peak": nvl_meas, "unit": "GB/s",
+                     "frac": (link_gbs / nvl_meas) if link_gbs and not same_gpu else None,
+                     "frac_of_nominal_900": (link_gbs / nvl_nominal) if link_gbs and not same_gpu else None,
+                     "traffic": None,
+                     "peak_source": "measured peer copy per direction (B200_PROFILING.md; 900 nominal)",
+                     "note": "same-GPU functional run: the 'peer' is local HBM, no NVLink frac"
+                     if same_gpu else None,
                      "algorithmic_bytes": "live bytes per migration (one direction)"},
-        "e2e": {"value": pct(E, 99), "unit": UNIT, "h2d_bytes_per_step": 2048 * 4,
-                "d2h_bytes_per_step": 1000 * 4, "p50_ms": pct(E, 50)},
+        "e2e": {"value": pct(E, 99), "unit": UNIT, "n": len(E), "h2d_bytes_per_step": 2048 * 4 * rps,
+                "d2h_bytes_per_step": 1000 * 4 * rps, "p50_ms": pct(E, 50)},
         "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),
         "clocks": allv[0]["main"]["clocks"],
     }
@@ -667,10 +797,18 @@ def main():
     ap.add_argument("--duplex", type=int, default=1,
                     help="1: full-duplex host round trip when nothing waits for the device "
                          "(default); 0: D2H, then H2D")
+    ap.add_argument("--gate", type=int, default=1,
+                    help="1: drain gate (a preempting request runs before the job's queued "
+                         "subgraph, default); 0: it waits for every dispatched subgraph")
+    ap.add_argument("--pair-gate", type=int, default=0,
+                    help="N > 1: use the drain gate in the pair processes too (default 0)")
     ap.add_argument("--early", type=int, default=1,
                     help="1: a preempting request is enqueued behind a device-side wait on the "
                          "job's in-flight subgraphs (default); 0: launched after the drain")
     args = ap.parse_args()
+    if os.environ.get("SF_BENCH_WATCHDOG_S"):  # debugging aid: dump every thread's stack, then exit
+        import faulthandler
+        faulthandler.dump_traceback_later(float(os.environ["SF_BENCH_WATCHDOG_S"]), exit=True)
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -737,6 +875,8 @@ def main():
         # no migration at all: the job stops at the boundary and waits in place (what the host
         # tier costs the requests that arrive during its round trip)
         inplace = arm(args, local, nb, 50, host_io=False, measure=False, target=0)
+        # the other drain-gate setting (same arrivals)
+        gate_other = arm(args, local, nb, 50, host_io=False, measure=False, gate=not args.gate)
 
         def q(x):
             return {"n": len(x["lat"]), "p50_ms": pct(x["lat"], 50), "p99_ms": pct(x["lat"], 99)}
@@ -752,6 +892,9 @@ def main():
                 ("launch_after_drain" if args.early else "early_launch"): {
                     **q(lat_other), "preempt_latency_p99_ms": pct(lat_other["pre"], 99)},
                 "no_migration_wait_in_place": q(inplace),
+                ("no_drain_gate" if args.gate else "drain_gate"): {
+                    **q(gate_other), "preempt_latency_p50_ms": pct(gate_other["pre"], 50),
+                    "preempt_latency_p99_ms": pct(gate_other["pre"], 99)},
                 "iteration_slicing": q(itg)}
 
     samples = {"main": main_s, "e2e": e2e_s, "chase": chase_s}
@@ -799,6 +942,7 @@ def main():
                    "dispatch_spin_us": args.dispatch_spin_us,
                    "inflight_budget_us": args.inflight_budget_us,
                    "early_launch": bool(args.early), "host_duplex": bool(args.duplex),
+                   "drain_gate": bool(args.gate),
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets 666 MB > 126 MB L2 (no flush needed); the pack "

@@ -543,6 +543,13 @@ sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t
                      int64_t n, float lr, float beta1, float beta2, float eps, void* stream);
 /* Fill n bytes at dst (device) with byte value (0xFF = poison). */
 sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream);
+/* Diagnostics: a device slot's scheduler state (owner token: a training job id, 1 << 20 while
+ * inference runs, -1 free; requests queued; drain-gate words). */
+typedef struct sf_slot_info {
+  int32_t owner, queued, gate_held, pad;
+  uint32_t gate_value, gate_arrived, next_ticket, pad2;
+} sf_slot_info;
+sf_status sf_slot_query(sf_runtime* rt, int32_t slot, sf_slot_info* out);
 /* Diagnostics: the kernel path of the last GEMM the CALLING THREAD launched (sf_op_gemm,
  * sf_op_gemm_bias_act, or a subgraph op launched directly on this thread).
  * kind: 1 tcgen05 TMA tile GEMM (bn = tile width 64 / 128 / 256, splits = split-K factor),

@@ -130,6 +130,12 @@ class sf_migration_probe(C.Structure):
                 ("staging_bytes", C.c_uint64)]
 
 
+class sf_slot_info(C.Structure):
+    _fields_ = [("owner", C.c_int32), ("queued", C.c_int32), ("gate_held", C.c_int32), ("pad", C.c_int32),
+                ("gate_value", C.c_uint32), ("gate_arrived", C.c_uint32), ("next_ticket", C.c_uint32),
+                ("pad2", C.c_uint32)]
+
+
 class sf_copy_desc(C.Structure):
     _fields_ = [("src", C.c_void_p), ("dst", C.c_void_p), ("nbytes", C.c_uint64),
                 ("span", C.c_uint64)]
@@ -191,6 +197,7 @@ PROTOTYPES = {
                          C.c_float, _vp]),
     "sf_op_fill": (_st, [_vp, C.c_uint64, C.c_int32, _vp]),
     "sf_last_gemm_path": (_st, [_P(sf_gemm_path)]),
+    "sf_slot_query": (_st, [_vp, C.c_int32, _P(sf_slot_info)]),
     "sf_probe_peer": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                             _P(C.c_double), _P(C.c_uint64)]),
     "sf_probe_migration": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32,

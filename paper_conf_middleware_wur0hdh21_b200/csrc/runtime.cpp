@@ -22,6 +22,7 @@
 #include <time.h>
 
 #include <algorithm>
+#include <cmath>
 #include <array>
 #include <atomic>
 #include <condition_variable>
@@ -175,8 +176,8 @@ struct Slot {
   struct Anchor {
     cudaEvent_t ev;
     uint64_t enq_ns;   // host time the anchor was enqueued
-    uint64_t g_ns;     // %globaltimer written by the stamp kernel
-    int64_t offset_ns; // host = device + offset (midpoint of the launch..observed window)
+    uint64_t g_ns;     // GPU time (%globaltimer ns) of the anchor event
+    int64_t offset_ns; // host = GPU + offset (stamp value seen at host time ~h1 - 1 us)
     uint64_t unc_ns;   // half that window
   };
   cudaStream_t s_clk = nullptr;
@@ -184,6 +185,7 @@ struct Slot {
   unsigned long long* clk_dev = nullptr;
   std::mutex clk_m;
   std::deque<Anchor> anchors;
+
   // drain gate (cfg.drain_gate, reading Q38): pinned mapped words, own cache lines.
   // gate[0] = G: a queued subgraph with ticket t runs once (int32)(G - t) >= 0; the host holds
   // tickets >= t with G = t - 1.  gate[16] = A: the GPU writes t right before its wait on G.
@@ -1067,28 +1069,43 @@ cudaError_t refresh_anchor(Slot& S) {
   for (int round = 0; round < 3; ++round) {
     volatile unsigned long long* h = S.clk_host;
     *h = 0ull;
-    cudaEvent_t ev = nullptr;
-    if ((e = cudaEventCreate(&ev)) != cudaSuccess) return e;
+    // E1 | stamp kernel (g = %globaltimer) | E2: the anchor is E1, whose GPU time is taken as
+    // g - elapsed(E1, E2) / 2 (the stamp sits inside the bracket; a timing event recorded AFTER
+    // the kernel can land tens of us late on a busy GPU)
+    cudaEvent_t e1 = nullptr, e2 = nullptr;
+    if ((e = cudaEventCreate(&e1)) != cudaSuccess) return e;
+    if ((e = cudaEventCreate(&e2)) != cudaSuccess) { cudaEventDestroy(e1); return e; }
     const uint64_t h0 = now_ns();
-    e = sfk::launch_stamp(S.clk_dev, S.s_clk);
-    if (e == cudaSuccess) e = cudaEventRecord(ev, S.s_clk);
-    if (e != cudaSuccess) { cudaEventDestroy(ev); return e; }
+    e = cudaEventRecord(e1, S.s_clk);
+    if (e == cudaSuccess) e = sfk::launch_stamp(S.clk_dev, S.s_clk);
+    if (e == cudaSuccess) e = cudaEventRecord(e2, S.s_clk);
+    if (e != cudaSuccess) { cudaEventDestroy(e1); cudaEventDestroy(e2); return e; }
     unsigned long long g = 0;
     while ((g = *h) == 0ull) {
       if (now_ns() - h0 > 200000000ull) break;  // 200 ms: the device is saturated, skip
       cpu_relax();
     }
     const uint64_t h1 = now_ns();
-    if ((e = cudaEventSynchronize(ev)) != cudaSuccess) { cudaEventDestroy(ev); return e; }
-    if (g == 0ull || (h1 - h0) / 2 >= best.unc_ns) { cudaEventDestroy(ev); continue; }
+    if ((e = cudaEventSynchronize(e2)) != cudaSuccess) { cudaEventDestroy(e1); cudaEventDestroy(e2); return e; }
+    float br = 0.f;
+    const bool ok = g != 0ull && cudaEventElapsedTime(&br, e1, e2) == cudaSuccess && br >= 0.f;
+    cudaEventDestroy(e2);
+
+    // round quality: the stamp's position inside its event bracket (br) is what the anchor's
+    // GPU time rests on; the host side (h1 - g) has a ~0.2-1 us one-sided spread
+    const uint64_t unc = static_cast<uint64_t>(static_cast<double>(br) * 1e6) + (h1 - h0) / 16;
+    if (!ok || br > 0.02f || unc >= best.unc_ns) { cudaGetLastError(); cudaEventDestroy(e1); continue; }
     if (best.ev) cudaEventDestroy(best.ev);
-    best = Slot::Anchor{ev, h0, g, static_cast<int64_t>((h0 + h1) / 2) - static_cast<int64_t>(g),
-                        (h1 - h0) / 2};
+    // the value was written at host time in [h0 + launch latency, h1 - write propagation]: the
+    // launch side of that window is the long one, the write lands and is seen ~1 us after the
+    // stamp, so h1 - 1 us is the host time of g
+    const uint64_t g1 = g - static_cast<uint64_t>(static_cast<double>(br) * 0.5e6);
+    best = Slot::Anchor{e1, h0, g1, static_cast<int64_t>(h1) - 700 - static_cast<int64_t>(g), unc};
   }
   if (!best.ev) return cudaSuccess;
   std::lock_guard<std::mutex> lk(S.clk_m);
   S.anchors.push_back(best);
-  while (S.anchors.size() > 64) {
+  while (S.anchors.size() > 256) {
     cudaEventDestroy(S.anchors.front().ev);
     S.anchors.pop_front();
   }
@@ -1108,17 +1125,26 @@ uint64_t event_host_ns(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
     cudaGetLastError();
     return 0;
   }
-  // the host offset: from the anchor with the tightest launch..observed window within 2 s of
-  // this one (a stamp delayed behind busy SMs gives a loose window; drift over 2 s is ~us)
-  int64_t off = a->offset_ns;
-  uint64_t unc = a->unc_ns;
-  for (const auto& b : S.anchors)
-    if (b.unc_ns < unc && (b.enq_ns > a->enq_ns ? b.enq_ns - a->enq_ns : a->enq_ns - b.enq_ns) < 2000000000ull) {
-      off = b.offset_ns;
-      unc = b.unc_ns;
-    }
+  // %globaltimer and CLOCK_MONOTONIC drift apart (~30 ppm measured on B200, scripts/
+  // clock_probe.cu): the offset is interpolated between the anchors around the event (or
+  // extrapolated along the last two), not held constant
   const double dev_ns = static_cast<double>(a->g_ns) + static_cast<double>(ms) * 1e6;
-  return static_cast<uint64_t>(dev_ns + static_cast<double>(off));
+  const Slot::Anchor* b = nullptr;  // the next anchor after a, else the one before
+  bool after = false;
+  for (size_t i = 0; i < S.anchors.size(); ++i)
+    if (&S.anchors[i] == a) {
+      if (i + 1 < S.anchors.size()) { b = &S.anchors[i + 1]; after = true; }
+      else if (i > 0) b = &S.anchors[i - 1];
+      break;
+    }
+  double off = static_cast<double>(a->offset_ns);
+  if (b && b->g_ns != a->g_ns) {
+    const double slope = (static_cast<double>(b->offset_ns) - static_cast<double>(a->offset_ns)) /
+                         (static_cast<double>(b->g_ns) - static_cast<double>(a->g_ns));
+    if (std::fabs(slope) < 1e-3) off += slope * (dev_ns - static_cast<double>(a->g_ns));
+    (void)after;
+  }
+  return static_cast<uint64_t>(dev_ns + off);
 }
 
 void clock_main(sf_runtime* rt);
@@ -2077,7 +2103,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
 void clock_main(sf_runtime* rt) {
   std::unique_lock<std::mutex> lk(rt->m);
   while (!rt->shutting_down) {
-    rt->cv.wait_for(lk, std::chrono::milliseconds(200), [&] { return rt->shutting_down; });
+    rt->cv.wait_for(lk, std::chrono::milliseconds(50), [&] { return rt->shutting_down; });
     if (rt->shutting_down) break;
     lk.unlock();
     for (auto& S : rt->slots)
@@ -3310,6 +3336,21 @@ sf_status sf_probe_peer(sf_runtime* rt, sf_graph_id gid, int32_t src, int32_t ds
   if (e != cudaSuccess) return fail(SF_ECUDA, std::string("probe peer: ") + cudaGetErrorString(e));
   *us = t;
   if (bytes_moved) *bytes_moved = moved;
+  return SF_OK;
+}
+
+sf_status sf_slot_query(sf_runtime* rt, int32_t slot, sf_slot_info* out) {
+  if (!rt || !out) return fail(SF_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(rt->m);
+  if (slot < 0 || slot >= static_cast<int>(rt->slots.size())) return fail(SF_EINVAL, "bad slot");
+  Slot& S = *rt->slots[slot];
+  std::memset(out, 0, sizeof(*out));
+  out->owner = S.owner.load();
+  out->queued = static_cast<int32_t>(S.q.size());
+  out->gate_held = S.gate_held ? 1 : 0;
+  out->gate_value = S.gate ? S.gate[0] : 0;
+  out->gate_arrived = S.gate ? S.gate[16] : 0;
+  out->next_ticket = S.next_ticket;
   return SF_OK;
 }
 

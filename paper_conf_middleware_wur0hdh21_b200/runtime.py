@@ -275,6 +275,21 @@ class Runtime:
               "sf_probe_peer")
         return us.value, nb.value
 
+    def slot_info(self, slot: int) -> dict:
+        """Scheduler state of a slot (sf_slot_query; diagnostics)."""
+        o = A.sf_slot_info()
+        check(lib().sf_slot_query(self.h, slot, C.byref(o)), "sf_slot_query")
+        return {f: getattr(o, f) for f, _ in A.sf_slot_info._fields_ if not f.startswith("pad")}
+
+    def poll(self, req: int) -> Optional[dict]:
+        """Non-blocking sf_wait: the request's timing once done, else None."""
+        t = A.sf_timing()
+        st = lib().sf_wait(self.h, req, 0, C.byref(t))
+        if st == A.SF_ETIMEOUT:
+            return None
+        check(st, "sf_wait")
+        return {f: getattr(t, f) for f, _ in A.sf_timing._fields_}
+
     def trace(self) -> List[dict]:
         n = C.c_size_t()
         check(lib().sf_get_trace(self.h, None, 0, C.byref(n)), "sf_get_trace")

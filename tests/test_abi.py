@@ -72,7 +72,7 @@ def test_struct_layouts_match_c(built):
     structs = ["sf_tensor_desc", "sf_op_desc", "sf_graph_desc", "sf_config", "sf_partition_opts",
                "sf_partition_info", "sf_job_info", "sf_cut_info", "sf_timing", "sf_trace_event",
                "sf_cut_request", "sf_copy_desc", "sf_feed_desc", "sf_u8_stage", "sf_gemm_path",
-               "sf_migration_probe"]
+               "sf_migration_probe", "sf_slot_info"]
     lines = ['#include <stdio.h>', '#include <stddef.h>', f'#include "{HEADER}"', "int main(){"]
     for s in structs:
         lines.append(f'printf("{s} %zu\\n", sizeof({s}));')

@@ -767,3 +767,35 @@ def test_requests_chase_peer_migrations_bitwise(P, early, gate):
         assert rel(out[r].cpu().numpy(), R.run_inference(gi, sti, xs[r])) <= TOL
     SC.check_no_corun(trace)
     SC.check_no_corun(SC.device_view(trace))
+
+
+def test_device_clock_mapping_is_consistent(P):
+    """Device intervals on the host clock (reading Q37): on an idle device a request's chain
+    starts after its submission and within a launch of the host dispatch, and ends before the
+    host observed its completion; repeated over ~1 s so several clock anchors are used."""
+    import time
+    RT, A = P
+    gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M")
+    with RT.Runtime([0], dispatch_spin_us=-1) as rt:
+        ghi = rt.register(gi, priority=1)
+        ghi.partition()
+        ghi.bind(0, staging=False)
+        ghi.load(0, D.init_state(gi, seed=D.SEED_INFER))
+        x = torch.rand(1, 2048, device="cuda")
+        out = torch.empty(1, 1000, device="cuda")
+        rows = []
+        for i in range(60):
+            time.sleep(0.02)
+            tm = rt.wait(rt.submit(ghi, 0, x.data_ptr(), out.data_ptr()), 30)
+            rows.append(tm)
+        trace = [e for e in rt.trace() if e["kind"] == "infer"]
+    rows, trace = rows[2:], trace[2:]  # warm-up launches
+    lead = [(t["start_ns"] - t["arrival_ns"]) * 1e-3 for t in rows]
+    tail = [(e["t1"] - e["d1"]) * 1e-3 for e in trace]
+    print("start - submit us p50/min/max", np.median(lead), min(lead), max(lead),
+          "| host completion - device end us p50/min", np.median(tail), min(tail))
+    # the mapping is good to a few us (anchor bracket + one-sided host observation delay)
+    assert min(lead) > -5.0 and np.median(lead) < 60.0
+    assert min(tail) > -5.0 and np.median(tail) < 60.0
+    for e in trace:
+        assert e["d1"] >= e["d0"] and (e["d1"] - e["d0"]) * 1e-3 < 500

@@ -99,3 +99,132 @@ def test_partner_of():
     from paper_conf_middleware_wur0hdh21_b200.pairs import partner_of
     assert [partner_of(r, 8) for r in range(8)] == [1, 0, 3, 2, 5, 4, 7, 6]
     assert partner_of(2, 3) is None
+
+
+class FakePoissonOps:
+    """The open-loop chase protocol against a fake runtime: a job advances one subgraph per
+    1 ms while it runs here; a request submitted while it runs preempts it (it migrates out
+    after a 0.5 ms copy); requests complete after 0.2 ms."""
+
+    def __init__(self, rank, log):
+        self.rank, self.log = rank, log
+        self.job = None  # [iter, k, t_state_change, state]
+        self.reqs = {}
+        self.nreq = 0
+        self.adopts = 0
+
+    def _advance(self):
+        if self.job and self.job[3] == "running":
+            t = time.monotonic()
+            steps = int((t - self.job[2]) / 1e-3)
+            for _ in range(steps):
+                self.job[1] += 1
+                if self.job[1] == 5:
+                    self.job[0], self.job[1] = self.job[0] + 1, 0
+            self.job[2] += steps * 1e-3
+
+    def start(self):
+        self.job = [0, 0, time.monotonic(), "running"]
+
+    def has_job(self):
+        self._advance()
+        return self.job is not None and self.job[3] == "running"
+
+    def in_transit(self):
+        return self.job is not None and self.job[3] == "migrating"
+
+    def job_gone(self):
+        return self.job is None
+
+    def migrated_out(self):
+        if self.job and self.job[3] == "migrating" and time.monotonic() >= self.job[2]:
+            it, k = self.job[0], self.job[1]
+            self.job = None
+            self.log.append(("out", it, k))
+            return {"iter": it, "k": k, "t_stop_ns": time.monotonic_ns()}
+        return None
+
+    def adopt(self, it, k):
+        assert self.job is None
+        self.job = [it, k, time.monotonic(), "running"]
+        self.log.append(("adopt", it, k))
+
+    def resume_ns(self):
+        return time.monotonic_ns() if self.job else 0
+
+    def submit(self, arrival_ns):
+        self.nreq += 1
+        preempted = self.has_job()
+        if preempted:
+            self.job[3] = "migrating"
+            self.job[2] = time.monotonic() + 0.5e-3
+        self.reqs[self.nreq] = (arrival_ns, time.monotonic() + 0.2e-3, preempted)
+        self.log.append(("req", arrival_ns, preempted))
+        return self.nreq
+
+    def poll(self, r):
+        a, done, pre = self.reqs[r]
+        if time.monotonic() < done:
+            return None
+        return {"arrival_ns": a, "start_ns": a + 1000, "end_ns": time.monotonic_ns(),
+                "preempted_job": 0 if pre else -1}
+
+    def stop(self):
+        if self.job:
+            self.log.append(("stop", self.job[0], self.job[1]))
+
+
+def _poisson_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import numpy as np
+    from paper_conf_middleware_wur0hdh21_b200.pairs import ShmLink, finish_pair, run_pair_poisson, shm_path
+    path = shm_path(rank // 2)
+    if rank % 2 == 0:
+        shm = ShmLink(path, create=True)
+    dist.barrier()
+    if rank % 2:
+        shm = ShmLink(path, create=False)
+    log = []
+    ops = FakePoissonOps(rank, log)
+    if rank % 2 == 0:
+        shm.set(ShmLink.HOLDER, rank)
+        ops.start()
+    t0 = [time.monotonic_ns() + 20_000_000]
+    dist.broadcast_object_list(t0, src=0)
+    rng = np.random.default_rng(7)
+    arr = (t0[0] + np.cumsum(rng.exponential(1 / 400, 60) * 1e9).astype(np.int64)).tolist()
+    S = run_pair_poisson(shm, ops, rank, rank ^ 1, arr, time.monotonic_ns, warmup=5)
+    finish_pair(shm, ops, rank, S["seen"])
+    dist.barrier()
+    shm.close(unlink=rank % 2 == 0)
+    q.put((rank, S, log))
+    dist.destroy_process_group()
+
+
+def test_pair_poisson_chase_protocol_two_ranks():
+    """Open-loop chase (C4 at N > 1): each of the 60 arrivals is served by exactly one rank;
+    a request preempts only a job that runs on its rank; every migration out is adopted by the
+    partner at the same cut; the job ends on exactly one rank."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_poisson_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(2):
+        r, S, log = q.get(timeout=120)
+        res[r] = (S, log)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    reqs = [e for r in (0, 1) for e in res[r][1] if e[0] == "req"]
+    assert len(reqs) == 60 and len({e[1] for e in reqs}) == 60  # every arrival served once
+    outs = sorted(e[1:] for r in (0, 1) for e in res[r][1] if e[0] == "out")
+    adopts = sorted(e[1:] for r in (0, 1) for e in res[r][1] if e[0] == "adopt")
+    assert outs == adopts and len(outs) >= 3  # every cut adopted by the partner
+    assert sum(e[2] for e in reqs) == len(outs)  # a preempting request = one migration
+    stops = [e for r in (0, 1) for e in res[r][1] if e[0] == "stop"]
+    assert len(stops) == 1  # the job ends on exactly one rank
+    assert len(res[0][0]["lat"]) + len(res[1][0]["lat"]) == 55  # after the 5 warm-up requests
