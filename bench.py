@@ -994,8 +994,8 @@ def main():
                      "traffic_source": prof.get("source"),
                      "dram_frac": prof.get("dram_frac"),
                      "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
-        "inference_roofline": {"kernel": "request chain (3 TMA cluster GEMVs, fused bias/ReLU, "
-                                         "fused softmax; device time p50)",
+        "inference_roofline": {"kernel": "request chain (3 LDG-streamed cluster GEMVs over blocked weights "
+                                         "under PDL, fused bias/ReLU, fused softmax; device time p50)",
                                "bound": "hbm", "algorithmic_bytes": w_bytes,
                                "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
                                "peak": hbm, "unit": "GB/s",

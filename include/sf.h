@@ -543,6 +543,11 @@ sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t
                      int64_t n, float lr, float beta1, float beta2, float eps, void* stream);
 /* Fill n bytes at dst (device) with byte value (0xFF = poison). */
 sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream);
+/* Inference weights are read into a blocked copy (contiguous per-CTA blocks for the
+ * LDG-streamed GEMV, reading Q39) at the binding's first request.  Call this after
+ * rewriting an inference graph's weights in the arena of slot dev: the copy is rebuilt at the
+ * next request (stream-ordered on the request stream). */
+sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id g, int32_t dev);
 /* Diagnostics: a device slot's scheduler state (owner token: a training job id, 1 << 20 while
  * inference runs, -1 free; requests queued; drain-gate words). */
 typedef struct sf_slot_info {
@@ -555,7 +560,7 @@ sf_status sf_slot_query(sf_runtime* rt, int32_t slot, sf_slot_info* out);
  * kind: 1 tcgen05 TMA tile GEMM (bn = tile width 64 / 128 / 256, splits = split-K factor),
  *       2 tcgen05 GEMM with LDG producers (pitches TMA cannot map), 3 TMA cluster GEMV,
  *       4 row-contiguous GEMV (TB), 5 register cluster GEMV, 6 split-K GEMV + reduce,
- *       7 plain GEMV; 0 = none yet.
+ *       7 plain GEMV, 8 LDG GEMV over blocked constant weights; 0 = none yet.
  * a_mn / b_mn: operand stored MN-major (A as [K][M], i.e. TA; B as [K][N], i.e. not TB). */
 typedef struct sf_gemm_path {
   int32_t kind, bn, splits, a_mn, b_mn, pad;

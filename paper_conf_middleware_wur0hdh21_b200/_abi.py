@@ -198,6 +198,7 @@ PROTOTYPES = {
     "sf_op_fill": (_st, [_vp, C.c_uint64, C.c_int32, _vp]),
     "sf_last_gemm_path": (_st, [_P(sf_gemm_path)]),
     "sf_slot_query": (_st, [_vp, C.c_int32, _P(sf_slot_info)]),
+    "sf_refresh_constants": (_st, [_vp, C.c_uint32, C.c_int32]),
     "sf_probe_peer": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                             _P(C.c_double), _P(C.c_uint64)]),
     "sf_probe_migration": (_st, [_vp, C.c_uint32, C.c_int32, C.c_int32, C.c_int32,

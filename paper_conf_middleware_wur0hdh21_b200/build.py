@@ -20,8 +20,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC,
          "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
-SOURCES = ["kernels_copy.cu", "kernels_gemm.cu", "kernels_gemm_tma.cu", "kernels_elem.cu", "kernels_chain.cu",
-           "runtime.cpp"]
+SOURCES = ["kernels_copy.cu", "kernels_gemm.cu", "kernels_gemm_tma.cu", "kernels_gemv.cu", "kernels_elem.cu",
+           "kernels_chain.cu", "runtime.cpp"]
 
 
 def _compile(src: str) -> str:

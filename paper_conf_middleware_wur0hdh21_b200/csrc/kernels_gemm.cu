@@ -722,6 +722,7 @@ cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st) {
     g_last_path.bn = bn;
     g_last_path.splits = splits;
   };
+  if (gemv_blk_eligible(a)) { take(kGemvBlocked); return launch_gemv_blk(a, st); }
   if (gemv_rows_eligible(a)) { take(kGemvRows); return launch_gemv_rows(a, st); }
   if ((a.bias[0] || a.relu) && !(use_gemv(a.M, a.ta, a.tb) && gemv4_ok(a.A, a.B, a.C, a.N, a.ldb)))
     return cudaErrorInvalidValue;  // fused epilogue only exists on the GEMV path

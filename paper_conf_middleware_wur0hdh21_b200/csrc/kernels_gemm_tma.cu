@@ -587,7 +587,8 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
                 float* __restrict__ Y, int M, int N, int K, int ldx, int ldy, int kper, int acc,
                 const float* __restrict__ b1, const float* __restrict__ b2,
                 const float* __restrict__ b3, int relu, int b_const, int l2_hint,
-                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
+                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter,
+                const char* __restrict__ pf, unsigned long long pf_bytes) {
   using Cfg = GvCfg<MR, BC>;
   constexpr int QW = Cfg::QW, RL = Cfg::RL, S = Cfg::S;
   extern __shared__ __align__(1024) unsigned char gv_smem[];
@@ -642,6 +643,18 @@ gemv_tma_kernel(const __grid_constant__ CUtensorMap tmW, const float* __restrict
         else
           tma_load_2d(sfdev::smem_u32(ring) + slot * Cfg::BOX, &tmW, sfdev::smem_u32(&full[slot]), c0,
                       k0 + i * kGvRows);
+      }
+      // the NEXT layer's weights (constant) to L2 once this CTA's own stream is issued: HBM
+      // keeps streaming through this layer's reduction, the next launch and its ramp (DESIGN.md
+      // reading Q39); this CTA's share of [pf, pf + pf_bytes) in 64 KB bulk prefetches
+      if (pf != nullptr && pf_bytes > 0) {
+        const unsigned long long G = gridDim.x;
+        const unsigned long long lo = (pf_bytes * blockIdx.x / G) & ~15ull;
+        const unsigned long long hi = blockIdx.x + 1 == G ? pf_bytes : (pf_bytes * (blockIdx.x + 1) / G) & ~15ull;
+        for (unsigned long long o = lo; o < hi; o += 65536) {
+          const unsigned n = static_cast<unsigned>(hi - o < 65536 ? hi - o : 65536);
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(pf + o), "r"(n) : "memory");
+        }
       }
     }
     __syncwarp();
@@ -1134,7 +1147,7 @@ cudaError_t launch_gemv_t(const CUtensorMap& w, const GemmArgs& a, int kper, cud
   return launch_k(kern, dim3(grid), dim3(288), smem, st, w, a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc,
                   kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
                   a.b_const ? 1 : 0, a.l2_hint | (gemv_prefetch() ? kGvPrefetch : 0), a.sm_out, a.sm_ldo,
-                  a.sm_counter);
+                  a.sm_counter, static_cast<const char*>(a.pf_next), a.pf_next ? a.pf_bytes : 0ull);
 }
 
 template <int BC>

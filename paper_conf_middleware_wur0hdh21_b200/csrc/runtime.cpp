@@ -115,6 +115,10 @@ struct Binding {
   // refreshed inside the version graph (copy2d before / after the GEMM)
   struct PadBuf { float* p = nullptr; int pitch = 0; };
   std::map<int, std::array<PadBuf, 3>> gemm_pad;  // op index -> {A, B, C}
+  // inference: constant GEMV weights re-laid out in contiguous blocks (kernels_gemv.cu), built at
+  // the binding's first request (sf_refresh_constants rebuilds them after the weights change)
+  std::map<int, std::pair<void*, sfk::GemvBlockPlan>> blocked;  // tensor id -> (copy, plan)
+  bool blocked_ready = false;
   std::vector<void*> dev_allocs;
 };
 
@@ -811,6 +815,14 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
         ga.ws = c.b.ws; ga.counters = c.b.counters;
         ga.b_const = !g.op_written[o.in[1]];
         if (c.l2_keep) ga.l2_hint = c.l2_keep->count(o.in[1]) ? 1 : 2;
+        {
+          auto bk = c.b.blocked.find(o.in[1]);
+          if (bk != c.b.blocked.end() && bk->second.second.ok && ga.M <= 8) {
+            ga.Bblk = bk->second.first;
+            ga.blk_qw = bk->second.second.qw;
+            ga.blk_kper = bk->second.second.kper;
+          }
+        }
         auto sa = c.b.shadow.find(o.in[0]);
         if (sa != c.b.shadow.end()) { ga.A = sa->second.first; ga.lda = sa->second.second; }
         auto sb = c.b.shadow.find(o.in[1]);
@@ -864,6 +876,17 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
               ga.sm_ldo = g.T[g.ops[j + 2].out[0]].cols;
               ga.sm_counter = c.b.counters + (g.counter_slots - 1);
               used = 3;
+            }
+            // the next GEMM of the chain streams constant weights: prefetch them to L2 from this
+            // one (SF_GEMV_NEXT_PF=0 disables)
+            static const bool next_pf = !(std::getenv("SF_GEMV_NEXT_PF") && std::getenv("SF_GEMV_NEXT_PF")[0] == '0');
+            if (next_pf && !ga.Bblk && j + used < e && g.ops[j + used].type == SF_OP_GEMM) {
+              const sf_op_desc& nx = g.ops[j + used];
+              const Tensor& NB = g.T[nx.in[1]];
+              if (!g.op_written[nx.in[1]] && !(nx.flags & (SF_GEMM_TA | SF_GEMM_TB)) && !c.b.shadow.count(nx.in[1])) {
+                ga.pf_next = c.f(nx.in[1]);
+                ga.pf_bytes = NB.nbytes;
+              }
             }
             err = sfk::launch_gemm(ga, c.st);
             if (err != cudaSuccess) return fail(SF_ECUDA, "op " + std::to_string(j) + ": " + cudaGetErrorString(err));
@@ -2236,6 +2259,32 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       return a.type == cudaMemoryTypeDevice;
     };
     const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
+    // blocked copies of the constant GEMV weights (first request of the binding; reading Q39)
+    static const bool blocked_on = !(std::getenv("SF_GEMV_BLOCKED") && std::getenv("SF_GEMV_BLOCKED")[0] == '0');
+    if (direct && blocked_on && !B->blocked_ready) {
+      for (const auto& o : g.ops) {
+        if (o.type != SF_OP_GEMM || (o.flags & (SF_GEMM_TA | SF_GEMM_TB | SF_GEMM_ACC)) || g.op_written[o.in[1]])
+          continue;
+        const Tensor &Bt = g.T[o.in[1]], &Ct = g.T[o.out[0]];
+        if (Ct.rows > 8 || B->shadow.count(o.in[1])) continue;
+        const sfk::GemvBlockPlan pl = sfk::plan_gemv_block(Ct.rows, Bt.cols, Bt.rows);
+        if (!pl.ok) continue;
+        auto& slot = B->blocked[o.in[1]];
+        if (!slot.first || slot.second.bytes != pl.bytes) {
+          void* d = nullptr;
+          if (cudaMalloc(&d, pl.bytes) != cudaSuccess) { cudaGetLastError(); B->blocked.erase(o.in[1]); continue; }
+          B->dev_allocs.push_back(d);
+          slot.first = d;
+        }
+        slot.second = pl;
+        if (sfk::launch_gemv_block_layout(reinterpret_cast<const float*>(B->arena + Bt.offset), slot.first, Bt.rows,
+                                          Bt.cols, Bt.cols, pl, S->s_infer) != cudaSuccess) {
+          cudaGetLastError();
+          slot.second.ok = false;
+        }
+      }
+      B->blocked_ready = true;
+    }
     const uint64_t tl0 = now_ns();
     // early launch: the chain (and its start event) wait on the device for the job's
     // dispatched subgraphs; the driver dispatches nothing more while the request is queued
@@ -3336,6 +3385,16 @@ sf_status sf_probe_peer(sf_runtime* rt, sf_graph_id gid, int32_t src, int32_t ds
   if (e != cudaSuccess) return fail(SF_ECUDA, std::string("probe peer: ") + cudaGetErrorString(e));
   *us = t;
   if (bytes_moved) *bytes_moved = moved;
+  return SF_OK;
+}
+
+sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id gid, int32_t dev) {
+  if (!rt) return fail(SF_EINVAL, "null runtime");
+  std::lock_guard<std::mutex> lk(rt->m);
+  Graph* g = get_graph(rt, gid);
+  if (!g || dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || g->bind[dev]->remote)
+    return fail(SF_EINVAL, "slot not bound locally");
+  g->bind[dev]->blocked_ready = false;
   return SF_OK;
 }
 

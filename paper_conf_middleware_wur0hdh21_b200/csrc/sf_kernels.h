@@ -52,7 +52,25 @@ struct GemmArgs {
   // L2 policy of the GEMV weight stream: 0 default, 1 keep (evict_last: held in the persisting
   // L2 set-aside across requests), 2 stream (evict_first: do not displace kept weights)
   int l2_hint = 0;
+  // TMA GEMV: constant weights of the NEXT layer (contiguous bytes) prefetched to L2 by this
+  // kernel's CTAs once their own stream is issued (inference chains; nullptr = none)
+  const void* pf_next = nullptr;
+  uint64_t pf_bytes = 0;
+  // constant B re-laid out in contiguous blocks (kernels_gemv.cu): the LDG-streamed GEMV
+  const void* Bblk = nullptr;
+  int blk_qw = 0, blk_kper = 0;
 };
+// Blocked layout of a constant GEMV weight (kernels_gemv.cu)
+struct GemvBlockPlan {
+  bool ok = false;
+  int qw = 0, kper = 0, n_cb = 0;
+  uint64_t bytes = 0;
+};
+GemvBlockPlan plan_gemv_block(int M, int N, int K);
+cudaError_t launch_gemv_block_layout(const float* W, void* Wb, int K, int N, int ldw, const GemvBlockPlan& p,
+                                     cudaStream_t st);
+bool gemv_blk_eligible(const GemmArgs& a);
+cudaError_t launch_gemv_blk(const GemmArgs& a, cudaStream_t st);
 bool gemv_softmax_fusable(const GemmArgs& a);
 // M <= 8 with B stored [N][K] (TB, the inference weight layout): row-contiguous streaming GEMV
 // with the same fused epilogue / softmax (kernels_gemm_tma.cu).
@@ -70,7 +88,7 @@ uint64_t gemm_counter_slots(int M, int N, int K, bool ta, bool tb);
 cudaError_t launch_gemm(const GemmArgs& a, cudaStream_t st);
 // The kernel path the calling thread's last launch_gemm took (diagnostics; sf_last_gemm_path).
 enum GemmPathKind { kGemmTma = 1, kGemmLdg = 2, kGemvTma = 3, kGemvRows = 4, kGemvCluster = 5,
-                    kGemvSplit = 6, kGemvPlain = 7 };
+                    kGemvSplit = 6, kGemvPlain = 7, kGemvBlocked = 8 };
 struct GemmPath { int kind = 0, bn = 0, splits = 0, a_mn = 0, b_mn = 0; };
 GemmPath last_gemm_path();
 // TMA-fed variant (kernels_gemm_tma.cu): needs 16-B aligned pointers and row pitches.

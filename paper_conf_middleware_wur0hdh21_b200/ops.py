@@ -37,7 +37,7 @@ def gemm(A_: torch.Tensor, B: torch.Tensor, C_: torch.Tensor, flags: int = 0, st
 
 
 GEMM_PATH_KINDS = {1: "tma", 2: "ldg", 3: "gemv_tma", 4: "gemv_rows", 5: "gemv_cluster",
-                   6: "gemv_split", 7: "gemv"}
+                   6: "gemv_split", 7: "gemv", 8: "gemv_blocked"}
 
 
 def last_gemm_path() -> dict:

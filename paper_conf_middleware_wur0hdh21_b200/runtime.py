@@ -124,6 +124,10 @@ class GraphHandle:
     def arena_bytes(self, slot: int) -> torch.Tensor:
         return self.mem[slot]["arena"]
 
+    def refresh_constants(self, slot: int) -> None:
+        """Rebuild the blocked inference-weight copies at the next request (sf_refresh_constants)."""
+        check(lib().sf_refresh_constants(self.rt.h, self.gid, slot), "sf_refresh_constants")
+
     def attach_feed(self, feed: int, tensor_ids: Sequence[int]) -> None:
         """Feed these INPUT / LABEL tensors from host feed ``feed`` (sf_attach_feed)."""
         arr = (C.c_uint32 * len(tensor_ids))(*tensor_ids)

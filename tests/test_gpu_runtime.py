@@ -575,13 +575,14 @@ np.save(sys.argv[1], out.cpu().numpy())
 """
 
 
-@pytest.mark.parametrize("env,spin", [({}, -1), ({"SF_CHAIN": "1"}, -1), ({"SF_CHAIN": "1", "SF_PDL": "0"}, 0),
+@pytest.mark.parametrize("env,spin", [({}, -1), ({"SF_GEMV_BLOCKED": "0"}, -1), ({"SF_CHAIN": "1"}, -1),
+                                      ({"SF_CHAIN": "1", "SF_PDL": "0"}, 0),
                                       ({"SF_INFER_DIRECT": "0"}, 0), ({"SF_GEMV": "split"}, 2000),
                                       ({"SF_GEMV": "cluster", "SF_INFER_DIRECT": "0"}, -1),
                                       ({"WT": "1"}, -1), ({"WT": "1", "SF_INFER_DIRECT": "0"}, 0),
                                       ({"WT": "1", "SF_FUSE_SOFTMAX": "0", "SF_INFER_REDIRECT": "0",
                                         "SF_PDL": "0"}, 0)],
-                         ids=["default", "chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv",
+                         ids=["default", "tma-gemv", "chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv",
                               "rows", "rows-graphs", "rows-unfused"])
 def test_inference_paths_vs_oracle(env, spin, tmp_path):
     """Every inference launch path (fused chain, PDL direct launches, captured graphs, the
