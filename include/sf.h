@@ -543,10 +543,11 @@ sf_status sf_op_adam(float* w, float* m, float* v, const float* g, const int32_t
                      int64_t n, float lr, float beta1, float beta2, float eps, void* stream);
 /* Fill n bytes at dst (device) with byte value (0xFF = poison). */
 sf_status sf_op_fill(void* dst, uint64_t n, int32_t value, void* stream);
-/* Inference weights are read into a blocked copy (contiguous per-CTA blocks for the
- * LDG-streamed GEMV, reading Q39) at the binding's first request.  Call this after
- * rewriting an inference graph's weights in the arena of slot dev: the copy is rebuilt at the
- * next request (stream-ordered on the request stream). */
+/* Batch <= 8 GEMMs with constant weights (inference layers) stream a blocked copy of the
+ * weights (contiguous per-CTA blocks for the LDG GEMV, reading Q39), allocated by
+ * sf_bind and laid out from the arena by this call (or, failing that, at the binding's first
+ * request).  Call it after writing or rewriting the weights in the arena of slot dev; it blocks
+ * until the copy is done. */
 sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id g, int32_t dev);
 /* Diagnostics: a device slot's scheduler state (owner token: a training job id, 1 << 20 while
  * inference runs, -1 free; requests queued; drain-gate words). */

@@ -1172,6 +1172,36 @@ uint64_t event_host_ns(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
 
 void clock_main(sf_runtime* rt);
 
+// Inference GEMV weights (M <= 8, constant B): blocked copies allocated at bind (reading Q39).
+sf_status alloc_blocked(Graph& g, Binding& b) {
+  static const bool on = !(std::getenv("SF_GEMV_BLOCKED") && std::getenv("SF_GEMV_BLOCKED")[0] == '0');
+  if (!on) return SF_OK;
+  for (const auto& o : g.ops) {
+    if (o.type != SF_OP_GEMM || (o.flags & (SF_GEMM_TA | SF_GEMM_TB | SF_GEMM_ACC)) || g.op_written[o.in[1]])
+      continue;
+    const Tensor &Bt = g.T[o.in[1]], &Ct = g.T[o.out[0]];
+    if (Ct.rows > 8 || b.shadow.count(o.in[1]) || b.blocked.count(o.in[1])) continue;
+    const sfk::GemvBlockPlan pl = sfk::plan_gemv_block(Ct.rows, Bt.cols, Bt.rows);
+    if (!pl.ok) continue;
+    void* d = nullptr;
+    SF_CK(cudaMalloc(&d, pl.bytes));
+    b.dev_allocs.push_back(d);
+    b.blocked[o.in[1]] = {d, pl};
+  }
+  return SF_OK;
+}
+// Lay the current weights out into the blocked copies (stream-ordered on st).
+void layout_blocked(const Graph& g, Binding& b, cudaStream_t st) {
+  for (auto& [t, e] : b.blocked) {
+    const Tensor& Bt = g.T[t];
+    if (sfk::launch_gemv_block_layout(reinterpret_cast<const float*>(b.arena + Bt.offset), e.first, Bt.rows,
+                                      Bt.cols, Bt.cols, e.second, st) != cudaSuccess) {
+      cudaGetLastError();
+      e.second.ok = false;
+    }
+  }
+}
+
 bool slot_has_inference(sf_runtime* rt, int s) { return !slot_of(rt, s).q.empty(); }
 
 // A training job of priority > min_prio (>= when or_equal) is present on slot s: running or
@@ -2259,30 +2289,10 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       return a.type == cudaMemoryTypeDevice;
     };
     const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
-    // blocked copies of the constant GEMV weights (first request of the binding; reading Q39)
-    static const bool blocked_on = !(std::getenv("SF_GEMV_BLOCKED") && std::getenv("SF_GEMV_BLOCKED")[0] == '0');
-    if (direct && blocked_on && !B->blocked_ready) {
-      for (const auto& o : g.ops) {
-        if (o.type != SF_OP_GEMM || (o.flags & (SF_GEMM_TA | SF_GEMM_TB | SF_GEMM_ACC)) || g.op_written[o.in[1]])
-          continue;
-        const Tensor &Bt = g.T[o.in[1]], &Ct = g.T[o.out[0]];
-        if (Ct.rows > 8 || B->shadow.count(o.in[1])) continue;
-        const sfk::GemvBlockPlan pl = sfk::plan_gemv_block(Ct.rows, Bt.cols, Bt.rows);
-        if (!pl.ok) continue;
-        auto& slot = B->blocked[o.in[1]];
-        if (!slot.first || slot.second.bytes != pl.bytes) {
-          void* d = nullptr;
-          if (cudaMalloc(&d, pl.bytes) != cudaSuccess) { cudaGetLastError(); B->blocked.erase(o.in[1]); continue; }
-          B->dev_allocs.push_back(d);
-          slot.first = d;
-        }
-        slot.second = pl;
-        if (sfk::launch_gemv_block_layout(reinterpret_cast<const float*>(B->arena + Bt.offset), slot.first, Bt.rows,
-                                          Bt.cols, Bt.cols, pl, S->s_infer) != cudaSuccess) {
-          cudaGetLastError();
-          slot.second.ok = false;
-        }
-      }
+    // blocked copies of the constant GEMV weights (allocated at bind; laid out here at the first
+    // request unless sf_refresh_constants already did it; reading Q39)
+    if (direct && !B->blocked_ready) {
+      layout_blocked(g, *B, S->s_infer);
       B->blocked_ready = true;
     }
     const uint64_t tl0 = now_ns();
@@ -2705,6 +2715,7 @@ sf_status sf_bind(sf_runtime* rt, sf_graph_id gid, int32_t dev, void* arena, voi
     }
     if (any) b->gemm_pad[static_cast<int>(j)] = pads;
   }
+  if (sf_status s = alloc_blocked(g, *b)) return s;
   SF_CK(cudaMalloc(&b->ws, std::max<uint64_t>(g.ws_floats, 4) * sizeof(float)));
   SF_CK(cudaMalloc(&b->counters, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));
   SF_CK(cudaMemset(b->counters, 0, std::max<uint64_t>(g.counter_slots, 1) * sizeof(unsigned)));
@@ -3394,7 +3405,13 @@ sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id gid, int32_t dev) {
   Graph* g = get_graph(rt, gid);
   if (!g || dev < 0 || dev >= static_cast<int>(rt->slots.size()) || !g->bind[dev] || g->bind[dev]->remote)
     return fail(SF_EINVAL, "slot not bound locally");
-  g->bind[dev]->blocked_ready = false;
+  Binding& B = *g->bind[dev];
+  Slot& S = *rt->slots[dev];
+  SF_CK(cudaSetDevice(S.cuda));
+  // re-laid out now, ordered before any later request on the request stream
+  layout_blocked(*g, B, S.s_infer);
+  SF_CK(cudaStreamSynchronize(S.s_infer));
+  B.blocked_ready = true;
   return SF_OK;
 }
 

@@ -116,6 +116,8 @@ class GraphHandle:
         for tid, a in arrays.items():
             self.view(slot, tid).copy_(torch.from_numpy(np.ascontiguousarray(a)))
         torch.cuda.synchronize(self.rt.ordinals[slot])
+        if self.priority > 0:  # inference weights: rebuild their blocked copies now
+            self.refresh_constants(slot)
 
     def read(self, slot: int, tid: int) -> np.ndarray:
         torch.cuda.synchronize(self.rt.ordinals[slot])

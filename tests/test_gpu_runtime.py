@@ -256,7 +256,8 @@ def test_inference_vs_oracle_and_auto_preemption_invariants(P, W, early, gate):
     evs = [dict(e, job=(1 if e["kind"] == "infer" else 0)) for e in trace]
     if early:
         assert sum("after" in e for e in evs) >= 10  # the early path was taken
-    SC.check_no_corun(evs)  # host intervals (supersets) with the recorded device dependency
+    if not gate:  # host intervals (supersets) with the recorded device dependency; a subgraph
+        SC.check_no_corun(evs)  # held by the drain gate spans later requests' host intervals
     # device intervals (GPU timeline, reading Q37): every train / infer event carries one
     dv = SC.device_view(evs)
     assert all(e["d0"] and e["d1"] >= e["d0"] for e in dv if e["kind"] in ("train", "infer"))
@@ -640,7 +641,8 @@ def test_open_loop_requests_during_swap_in_are_bitwise(P, defer, duplex, early, 
     got = {i: gh.read(0, i) for i in st}
     trace = [e for e in rt.trace() if e["kind"] in ("train", "infer")]
     rt.close()
-    SC.check_no_corun(trace)
+    if not gate:
+        SC.check_no_corun(trace)
     SC.check_no_corun(SC.device_view(trace))
     assert info["n_preemptions"] >= (3 if early else 5), info
     print("preemptions", info["n_preemptions"], "re-parks", info["n_reparks"])
@@ -766,7 +768,8 @@ def test_requests_chase_peer_migrations_bitwise(P, early, gate):
     assert len(tims) >= 3
     for r in range(len(tims)):
         assert rel(out[r].cpu().numpy(), R.run_inference(gi, sti, xs[r])) <= TOL
-    SC.check_no_corun(trace)
+    if not gate:
+        SC.check_no_corun(trace)
     SC.check_no_corun(SC.device_view(trace))
 
 
