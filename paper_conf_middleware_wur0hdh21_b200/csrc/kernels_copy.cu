@@ -68,11 +68,12 @@ struct SDesc {
 };
 
 __global__ void __launch_bounds__(kCopyThreads)
-mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t total, uint64_t per_block,
+mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t total, uint64_t per_block,
               int64_t patch_iter, unsigned long long* tstamp) {
   // optional device-side duration: [0] = earliest CTA start, [1] = latest CTA end (ns)
   if (tstamp && threadIdx.x == 0) atomicMin(&tstamp[0], sfdev::globaltimer());
-  const uint64_t c0 = static_cast<uint64_t>(blockIdx.x) * per_block;
+  // this launch covers chunks [base, total) of the flat chunk space
+  const uint64_t c0 = base + static_cast<uint64_t>(blockIdx.x) * per_block;
   const uint64_t c1 = min(c0 + per_block, total);
   __shared__ SDesc sd[kBatch + 1];
   __shared__ int s_first, s_last;
@@ -160,12 +161,24 @@ cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
   const int waves = waves_arg > 0 ? waves_arg : waves_env;
   blocks = std::min<uint64_t>(blocks, 148ull * bps * waves);
   blocks = std::max<uint64_t>(blocks, 1);
-  const uint64_t per_block = (total_chunks + blocks - 1) / blocks;
-  blocks = (total_chunks + per_block - 1) / per_block;
-  mtcopy_kernel<<<static_cast<unsigned>(blocks), kCopyThreads, 0, st>>>(d_descs, n, total_chunks,
-                                                                        per_block, patch_iter, tstamp);
-  count_launch();
-  return cudaGetLastError();
+  // Live sets above 3 GB go in 2 GB windows, one launch each: with ~1200 CTAs each walking its
+  // own multi-MB slice, the concurrent streams of a >4 GB walk spread over more 2 MB pages than
+  // the GPU's TLBs cover and the walk drops from 6.1 to 4.6 TB/s (scripts/cliff_probe.py, the
+  // round-1 "C5 cliff"); windows keep every slice's pages within reach
+  const uint64_t win = total_chunks * 16 > (3ull << 30) ? (2ull << 30) / 16 : total_chunks;
+  for (uint64_t w0 = 0; w0 < total_chunks; w0 += win) {
+    const uint64_t w1 = std::min(total_chunks, w0 + win), cnt = w1 - w0;
+    uint64_t nb = std::min<uint64_t>(blocks, (cnt + min_chunks - 1) / min_chunks);
+    nb = std::max<uint64_t>(nb, 1);
+    const uint64_t per_block = (cnt + nb - 1) / nb;
+    nb = (cnt + per_block - 1) / per_block;
+    mtcopy_kernel<<<static_cast<unsigned>(nb), kCopyThreads, 0, st>>>(d_descs, n, w0, w1, per_block,
+                                                                      patch_iter, tstamp);
+    count_launch();
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 __global__ void fill_kernel(uint8_t* dst, uint64_t n, uint32_t word) {

@@ -59,6 +59,30 @@ def test_mtcopy_adversarial_sizes_bit_exact(ops):
     assert np.array_equal(dst.cpu().numpy(), expect)
 
 
+def test_mtcopy_windowed_walk_above_3gb_bit_exact(ops):
+    """Live sets above 3 GB are walked in 2 GB windows (one launch each):
+    3 descriptors straddling the window boundaries, ragged tails and zero padding, bit-exact."""
+    sizes = [1_300_000_004, 1_400_000_000, 1_000_012]
+    spans = [-(-s // 256) * 256 for s in sizes]
+    total = sum(spans)
+    g = torch.Generator(device="cuda").manual_seed(3)
+    src = torch.randint(0, 256, (total,), dtype=torch.uint8, device="cuda", generator=g)
+    dst = torch.full((total,), 0xAB, dtype=torch.uint8, device="cuda")
+    descs, o = [], 0
+    for s_, sp in zip(sizes, spans):
+        descs.append((src.data_ptr() + o, dst.data_ptr() + o, s_, sp))
+        o += sp
+    ops.mtcopy(descs)
+    torch.cuda.synchronize()
+    o = 0
+    for s_, sp in zip(sizes, spans):
+        assert torch.equal(dst[o:o + s_], src[o:o + s_])
+        assert not bool(dst[o + s_:o + sp].any())  # zero padding
+        o += sp
+    del src, dst
+    torch.cuda.empty_cache()
+
+
 def test_mtcopy_patch_iter(ops):
     src = cu(np.arange(64, dtype=np.uint8))
     dst = torch.zeros(64, dtype=torch.uint8, device="cuda")
