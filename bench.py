@@ -991,6 +991,7 @@ def main():
                      "achieved": pack_achieved, "peak": hbm, "unit": "GB/s",
                      "frac": (pack_achieved / hbm) if pack_achieved else None,
                      "traffic": prof.get("bytes_per_launch"), "peak_source": peak_src,
+                     "traffic_algorithmic_bytes": prof.get("algorithmic_bytes_per_launch"),
                      "traffic_source": prof.get("source"),
                      "dram_frac": prof.get("dram_frac"),
                      "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
