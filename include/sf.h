@@ -347,10 +347,19 @@ sf_status sf_start_training(sf_runtime* rt, sf_graph_id g, int32_t dev, int64_t 
  * current slot or unbound; SF_EBUSY if a migration is in flight. */
 sf_status sf_preempt(sf_runtime* rt, sf_job_id job, int32_t target, sf_cut_info* out);
 /* Resume a preempted job on `dev` (peer tier: the migration target; host tier: any bound
- * slot) — stream-ordered after the migration, no host sync on the copy.  SF_ESTATE if
- * the job is not preempted. */
+ * slot) — stream-ordered after the migration, no host sync on the copy: "the new session is
+ * populated with the tasks of the aborted session run so that no work is lost" and later
+ * sessions run on the new device (section 3.3).  SF_ESTATE if the
+ * job is not preempted. */
 sf_status sf_resume(sf_runtime* rt, sf_job_id job, int32_t dev);
 sf_status sf_job_query(sf_runtime* rt, sf_job_id job, sf_job_info* out);
+/* Copy tensor `tensor_id` of a job's graph (n bytes, n == its byte size) from the arena of the
+ * slot the job occupies into host memory host_dst (blocking).  The copy is ordered after every
+ * subgraph the job has dispatched (a snapshot at a subgraph boundary when the job runs; the
+ * final value once it is done) — the paper's users fetch results through the session
+ * (Listing 1).  SF_EBUSY while the job's state is parked in host memory or
+ * moving (host tier, migration in flight); SF_EINVAL for a bad id or size. */
+sf_status sf_read_tensor(sf_runtime* rt, sf_job_id job, uint32_t tensor_id, void* host_dst, size_t n);
 /* Wait until the job finished all iterations (SF_ETIMEOUT after timeout_ns; <0 = inf). */
 sf_status sf_wait_job(sf_runtime* rt, sf_job_id job, int64_t timeout_ns);
 /* Ask a running job to stop at its next iteration boundary and finish. */
@@ -448,7 +457,10 @@ typedef struct sf_timing {
   float dispatch_us;     /* host time from the dispatch decision to the first enqueue */
 } sf_timing;
 
-/* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).
+/* Enqueue a batch-1 request of inference graph g on slot dev (non-blocking).  The request is
+ * the high-priority job that "is allowed to start immediately after submission" while the
+ * preempted one is suspended at its next boundary (section 3.4; arrival
+ * triggers preemption, section 3.3).
  * in: pointer (device or pinned host) to the INPUT tensor's bytes; out: pointer (device
  * or pinned host) receiving the OUTPUT tensor's bytes; both caller-owned until sf_wait.
  * arrival_ns = scheduled arrival time (CLOCK_MONOTONIC ns; 0 = now).  With

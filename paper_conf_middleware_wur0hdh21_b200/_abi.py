@@ -172,6 +172,7 @@ PROTOTYPES = {
     "sf_stage_u8_normalize": (C.c_int32, [_vp, C.c_int64, _P(_vp), _P(C.c_uint64), C.c_int32]),
     "sf_job_query": (_st, [_vp, C.c_uint32, _P(sf_job_info)]),
     "sf_wait_job": (_st, [_vp, C.c_uint32, C.c_int64]),
+    "sf_read_tensor": (_st, [_vp, C.c_uint32, C.c_uint32, _vp, C.c_size_t]),
     "sf_stop_job": (_st, [_vp, C.c_uint32]),
     "sf_submit_inference": (_st, [_vp, C.c_uint32, C.c_int32, _vp, _vp, C.c_uint64,
                                   _P(C.c_uint64)]),

@@ -146,9 +146,120 @@ mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t total,
   }
 }
 
+// ---- TMA bulk variant of the walk (SF_COPY_BULK=1; round-1 verdict: "TMA bulk copies") ----
+// One CTA per SM over the same flat chunk space.  Payload bytes of descriptors >= 4 KB move by
+// cp.async.bulk global -> shared (mbarrier) then cp.async.bulk shared -> global (bulk groups)
+// through a 6 x 32 KB ring driven by one thread; all other bytes (small descriptors, the
+// staging header with its patched iter, sub-16-B tails, zero padding) go by 16-B LDG / STG from
+// the remaining threads.  Same descriptor semantics and bytes as mtcopy_kernel.
+constexpr int kBulkSlot = 32768, kBulkSlots = 6, kBulkThreads = 256;
+constexpr uint64_t kBulkMin = 4096;
+
+__global__ void __launch_bounds__(kBulkThreads, 1)
+bulkcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t total, uint64_t per_block,
+                int64_t patch_iter, unsigned long long* tstamp) {
+  extern __shared__ __align__(128) unsigned char bsm[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(bsm + kBulkSlots * kBulkSlot);
+  if (tstamp && threadIdx.x == 0) atomicMin(&tstamp[0], sfdev::globaltimer());
+  const uint64_t c0 = base + static_cast<uint64_t>(blockIdx.x) * per_block;
+  const uint64_t c1 = min(c0 + per_block, total);
+  __shared__ int s_first, s_last;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < kBulkSlots; ++i) sfdev::mbar_init(&full[i], 1);
+    sfdev::mbar_fence_init();
+    int lo = 0, hi = n - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (d[mid].chunk_begin <= c0) lo = mid; else hi = mid - 1;
+    }
+    s_first = lo;
+    lo = 0; hi = n - 1;
+    const uint64_t cl = c1 > c0 ? c1 - 1 : c0;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (d[mid].chunk_begin <= cl) lo = mid; else hi = mid - 1;
+    }
+    s_last = lo;
+  }
+  __syncthreads();
+  if (c0 < total) {
+    int piece = 0;  // bulk pieces issued by thread 0 (ring slot = piece % kBulkSlots)
+    for (int i = s_first; i <= s_last; ++i) {
+      const DCopy x = d[i];
+      const uint64_t e = d[i + 1].chunk_begin;  // next descriptor (or the sentinel)
+      const uint64_t a = max(c0, x.chunk_begin) - x.chunk_begin, b = min(c1, e) - x.chunk_begin;  // chunk range
+      const bool bulk = x.nbytes >= kBulkMin && (i != 0 || patch_iter < 0);
+      const uint64_t full16 = x.nbytes >> 4;  // whole 16-B chunks of payload
+      // thread path: everything that is not a bulk-moved whole payload chunk
+      for (uint64_t j = a + threadIdx.x; j < b; j += kBulkThreads) {
+        if (bulk && j < full16) continue;
+        uint4 v = load_chunk(x.src, j, full16, x.nbytes);
+        if (patch_iter >= 0 && i == 0 && j == 1) {
+          v.x = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter));
+          v.y = static_cast<uint32_t>(static_cast<uint64_t>(patch_iter) >> 32);
+        }
+        sfdev::st16_cs(x.dst + j * 16, v);
+      }
+      if (bulk && threadIdx.x == 0) {
+        // up to kBulkSlots loads in flight; stores issued in order as loads land
+        const uint64_t lo = a * 16, hi = (b < full16 ? b : full16) * 16;
+        const int P = hi > lo ? static_cast<int>((hi - lo + kBulkSlot - 1) / kBulkSlot) : 0;
+        int issued = 0, stored = 0;
+        while (stored < P) {
+          while (issued < P && issued - stored < kBulkSlots) {
+            const int g = piece + issued, sl = g % kBulkSlots;
+            const uint64_t o = lo + static_cast<uint64_t>(issued) * kBulkSlot;
+            const uint32_t nb = static_cast<uint32_t>(hi - o < kBulkSlot ? hi - o : kBulkSlot);
+            if (g >= kBulkSlots) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // slot free
+            sfdev::expect_tx(&full[sl], nb);
+            sfdev::bulk_load_1d(sfdev::smem_u32(bsm + sl * kBulkSlot), x.src + o, nb, sfdev::smem_u32(&full[sl]));
+            ++issued;
+          }
+          const int g = piece + stored, sl = g % kBulkSlots;
+          const uint64_t o = lo + static_cast<uint64_t>(stored) * kBulkSlot;
+          const uint32_t nb = static_cast<uint32_t>(hi - o < kBulkSlot ? hi - o : kBulkSlot);
+          sfdev::mbar_wait(&full[sl], (g / kBulkSlots) & 1);
+          asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                       :: "l"(x.dst + o), "r"(sfdev::smem_u32(bsm + sl * kBulkSlot)), "r"(nb) : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          ++stored;
+        }
+        piece += P;
+      }
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+  if (tstamp) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicMax(&tstamp[1], sfdev::globaltimer());
+    }
+  }
+}
+
 cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
                           int64_t patch_iter, cudaStream_t st, unsigned long long* tstamp,
                           int waves_arg) {
+  static const bool bulk = std::getenv("SF_COPY_BULK") && std::getenv("SF_COPY_BULK")[0] == '1';
+  if (bulk && n > 0 && total_chunks > 0) {
+    static std::atomic<uint64_t> configured{0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const int smem = kBulkSlots * kBulkSlot + kBulkSlots * 8;
+    if (!(configured.load() & (1ull << (dev & 63)))) {
+      cudaError_t e = cudaFuncSetAttribute(bulkcopy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      if (e != cudaSuccess) return e;
+      configured.fetch_or(1ull << (dev & 63));
+    }
+    const uint64_t blocks = std::min<uint64_t>(148, (total_chunks + 2047) / 2048);
+    const uint64_t per_block = (total_chunks + blocks - 1) / blocks;
+    const uint64_t nb = (total_chunks + per_block - 1) / per_block;
+    bulkcopy_kernel<<<static_cast<unsigned>(nb), kBulkThreads, smem, st>>>(d_descs, n, 0, total_chunks, per_block,
+                                                                          patch_iter, tstamp);
+    count_launch();
+    return cudaGetLastError();
+  }
   if (n <= 0 || total_chunks == 0) return cudaSuccess;
   // Grid: a multiple of the 148 SMs, enough bytes per CTA to amortise the search.
   static const int bps = std::getenv("SF_COPY_BPS") ? std::atoi(std::getenv("SF_COPY_BPS")) : 8;

@@ -3115,6 +3115,32 @@ sf_status sf_job_query(sf_runtime* rt, sf_job_id jid, sf_job_info* out) {
   return SF_OK;
 }
 
+sf_status sf_read_tensor(sf_runtime* rt, sf_job_id jid, uint32_t tid, void* host_dst, size_t n) {
+  if (!rt || !host_dst) return fail(SF_EINVAL, "null argument");
+  const uint8_t* src = nullptr;
+  cudaStream_t st = nullptr;
+  int cuda = 0;
+  {
+    std::lock_guard<std::mutex> lk(rt->m);
+    Job* J = get_job(rt, jid);
+    if (!J) return fail(SF_EINVAL, "bad job id");
+    Graph& g = *J->g;
+    if (tid >= g.T.size() || n != g.T[tid].nbytes) return fail(SF_EINVAL, "bad tensor id / size");
+    if (J->state == SF_JOB_MIGRATING || J->state == SF_JOB_STOPPING || J->state == SF_JOB_MIGRATED_OUT ||
+        (J->state == SF_JOB_PREEMPTED && J->cut.dst_dev == SF_TARGET_HOST))
+      return fail(SF_EBUSY, "the job's state is in transit or parked in host memory");
+    if (J->dev < 0 || !g.bind[J->dev] || g.bind[J->dev]->remote) return fail(SF_ESTATE, "job not on a local slot");
+    Slot& S = *rt->slots[J->dev];
+    src = g.bind[J->dev]->arena + g.T[tid].offset;
+    st = S.s_train;
+    cuda = S.cuda;
+  }
+  SF_CK(cudaSetDevice(cuda));
+  SF_CK(cudaMemcpyAsync(host_dst, src, n, cudaMemcpyDeviceToHost, st));
+  SF_CK(cudaStreamSynchronize(st));
+  return SF_OK;
+}
+
 sf_status sf_wait_job(sf_runtime* rt, sf_job_id jid, int64_t timeout_ns) {
   if (!rt) return fail(SF_EINVAL, "null runtime");
   std::unique_lock<std::mutex> lk(rt->m);

@@ -211,10 +211,11 @@ def run_pair_poisson(shm: ShmLink, ops, me: int, partner: int, arrivals_ns: List
                      now_ns, warmup: int = 0) -> dict:
     """Open-loop Poisson stream of one pair, chasing the job (SURVEY.md 8(d) C4 at N > 1).
 
-    Both ranks walk the same seeded arrival list.  The holder rank submits each request at its
-    scheduled arrival; if it runs the job, the request preempts it and the job migrates to the
-    partner (holder flips at once: later requests go where the job is heading).  A request for
-    a holder that is still receiving the job runs without a cut.  The rank whose job migrated
+    Both ranks walk the same seeded arrival list; the even rank routes each arrival to the
+    holder (single writer).  The holder submits the request at its scheduled arrival; if the
+    job runs there, the request preempts it and the job migrates to the partner; the holder
+    flips when the migrated-out record is published.  A request that arrives while the job is
+    in transit runs where it was routed, without a cut.  The rank whose job migrated
     out publishes the handoff; the partner adopts it.  ``ops``: submit(arrival_ns) -> req,
     poll(req) -> timing | None, has_job(), migrated_out() -> cut | None, adopt(iter, k),
     resume_ns().  Returns latency samples of the requests this rank served (after warmup)."""
@@ -252,11 +253,11 @@ def run_pair_poisson(shm: ShmLink, ops, me: int, partner: int, arrivals_ns: List
             owner = shm.owner_of(i)
             if owner is not None:
                 if owner == me % 2:
-                    running = ops.has_job()
+                    # the holder flips only when the job has actually left (its record is
+                    # published): a request that ran in a gap between two of the job's
+                    # subgraphs preempts nothing, and the job stays here
                     pending.append((i, ops.submit(arrivals_ns[i])))
                     S["n_submitted"] += 1
-                    if running:
-                        shm.set(ShmLink.HOLDER, partner)
                 i += 1
         still = []
         for (k, req) in pending:

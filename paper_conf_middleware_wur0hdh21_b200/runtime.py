@@ -246,6 +246,14 @@ class Runtime:
         d["state_name"] = A.JOB_STATES.get(d["state"], "?")
         return d
 
+    def read_tensor(self, job: int, gh: GraphHandle, tid: int) -> np.ndarray:
+        """A job's tensor from the arena of the slot it occupies (sf_read_tensor, blocking)."""
+        t = gh.graph.tensors[tid]
+        out = np.empty((t.rows, t.cols), dtype=_NP_DTYPE[t.dtype])
+        check(lib().sf_read_tensor(self.h, job, tid, C.c_void_p(out.ctypes.data), out.nbytes),
+              "sf_read_tensor")
+        return out
+
     def wait_job(self, job: int, timeout_s: float = -1) -> None:
         check(lib().sf_wait_job(self.h, job, int(timeout_s * 1e9) if timeout_s >= 0 else -1),
               "sf_wait_job")

@@ -210,6 +210,10 @@ def test_explicit_preempt_resume_peer_and_host(P):
     info = rt.job_info(job)
     assert info["n_preemptions"] == 2 and info["dev"] == 0
     got = {i: gh.read(0, i) for i in st}
+    for i in st:  # the ABI read (sf_read_tensor) sees the same bytes as the torch view
+        assert rt.read_tensor(job, gh, i).tobytes() == got[i].tobytes()
+    with pytest.raises(A.SFError):
+        rt.read_tensor(job, gh, 10 ** 6)
     rt.close()
     assert_bitwise(base, got)
 

@@ -225,6 +225,7 @@ def test_pair_poisson_chase_protocol_two_ranks():
     adopts = sorted(e[1:] for r in (0, 1) for e in res[r][1] if e[0] == "adopt")
     assert outs == adopts and len(outs) >= 3  # every cut adopted by the partner
     assert sum(e[2] for e in reqs) == len(outs)  # a preempting request = one migration
+    assert sum(e[2] for e in reqs) >= 10  # the stream keeps finding the job (chase)
     stops = [e for r in (0, 1) for e in res[r][1] if e[0] == "stop"]
     assert len(stops) == 1  # the job ends on exactly one rank
     assert len(res[0][0]["lat"]) + len(res[1][0]["lat"]) == 55  # after the 5 warm-up requests
