@@ -641,14 +641,19 @@ def run_pair_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io:
     t_start = [now_ns() + 20_000_000]
     dist.broadcast_object_list(t_start, src=0, group=gloo)  # one clock (CLOCK_MONOTONIC) per host
     arr = (t_start[0] + np.cumsum(gaps)).tolist()
-    it_start = rt.job_info(ops.job)["iter"] if even else None
+    it_start = None
+    if even:  # the job's iteration at the first arrival
+        while now_ns() < arr[0]:
+            pass
+        it_start = rt.job_info(ops.job)["iter"]
     torch.cuda.synchronize(dev)
     sampler = ClockSampler(local_dev).__enter__() if measure else None
     ev0 = torch.cuda.Event(enable_timing=True)
     ev0.record()
     launches0 = kernel_launches()
     S = run_pair_poisson(shm, ops, args.rank, args.rank ^ 1, arr, now_ns, warmup=warmup)
-    t_stream = (now_ns() - arr[warmup]) * 1e-9 if len(arr) > warmup else 0.0
+    # the job's progress is counted from the stream's first arrival (it_start) to its end
+    t_stream = (now_ns() - arr[0]) * 1e-9
     ev1 = torch.cuda.Event(enable_timing=True)
     ev1.record()
     torch.cuda.synchronize(dev)
