@@ -149,10 +149,10 @@ mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t total,
 // ---- TMA bulk variant of the walk (SF_COPY_BULK=1; round-1 verdict: "TMA bulk copies") ----
 // One CTA per SM over the same flat chunk space.  Payload bytes of descriptors >= 4 KB move by
 // cp.async.bulk global -> shared (mbarrier) then cp.async.bulk shared -> global (bulk groups)
-// through a 6 x 32 KB ring driven by one thread; all other bytes (small descriptors, the
+// through a 7 x 32 KB ring driven by one thread (5 loads ahead); all other bytes (small descriptors, the
 // staging header with its patched iter, sub-16-B tails, zero padding) go by 16-B LDG / STG from
 // the remaining threads.  Same descriptor semantics and bytes as mtcopy_kernel.
-constexpr int kBulkSlot = 32768, kBulkSlots = 6, kBulkThreads = 256;
+constexpr int kBulkSlot = 32768, kBulkSlots = 7, kBulkAhead = 5, kBulkThreads = 256;
 constexpr uint64_t kBulkMin = 4096;
 
 __global__ void __launch_bounds__(kBulkThreads, 1)
@@ -201,28 +201,30 @@ bulkcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t tota
         sfdev::st16_cs(x.dst + j * 16, v);
       }
       if (bulk && threadIdx.x == 0) {
-        // up to kBulkSlots loads in flight; stores issued in order as loads land
+        // software pipeline over this descriptor's pieces: kBulkAhead loads in flight, the
+        // store of piece p issued as soon as its load lands; a load may reuse the slot of the
+        // store kBulkSlots pieces back once at most kBulkSlots - kBulkAhead newer stores
+        // are still reading shared memory (a constant wait_group count, counted globally)
         const uint64_t lo = a * 16, hi = (b < full16 ? b : full16) * 16;
         const int P = hi > lo ? static_cast<int>((hi - lo + kBulkSlot - 1) / kBulkSlot) : 0;
-        int issued = 0, stored = 0;
-        while (stored < P) {
-          while (issued < P && issued - stored < kBulkSlots) {
-            const int g = piece + issued, sl = g % kBulkSlots;
-            const uint64_t o = lo + static_cast<uint64_t>(issued) * kBulkSlot;
-            const uint32_t nb = static_cast<uint32_t>(hi - o < kBulkSlot ? hi - o : kBulkSlot);
-            if (g >= kBulkSlots) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // slot free
-            sfdev::expect_tx(&full[sl], nb);
-            sfdev::bulk_load_1d(sfdev::smem_u32(bsm + sl * kBulkSlot), x.src + o, nb, sfdev::smem_u32(&full[sl]));
-            ++issued;
-          }
-          const int g = piece + stored, sl = g % kBulkSlots;
-          const uint64_t o = lo + static_cast<uint64_t>(stored) * kBulkSlot;
+        auto issue = [&](int k) {
+          const int g = piece + k, sl = g % kBulkSlots;
+          const uint64_t o = lo + static_cast<uint64_t>(k) * kBulkSlot;
+          const uint32_t nb = static_cast<uint32_t>(hi - o < kBulkSlot ? hi - o : kBulkSlot);
+          if (g >= kBulkSlots) asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(kBulkSlots - kBulkAhead) : "memory");
+          sfdev::expect_tx(&full[sl], nb);
+          sfdev::bulk_load_1d(sfdev::smem_u32(bsm + sl * kBulkSlot), x.src + o, nb, sfdev::smem_u32(&full[sl]));
+        };
+        for (int k = 0; k < P && k < kBulkAhead; ++k) issue(k);
+        for (int k = 0; k < P; ++k) {
+          const int g = piece + k, sl = g % kBulkSlots;
+          const uint64_t o = lo + static_cast<uint64_t>(k) * kBulkSlot;
           const uint32_t nb = static_cast<uint32_t>(hi - o < kBulkSlot ? hi - o : kBulkSlot);
           sfdev::mbar_wait(&full[sl], (g / kBulkSlots) & 1);
           asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
                        :: "l"(x.dst + o), "r"(sfdev::smem_u32(bsm + sl * kBulkSlot)), "r"(nb) : "memory");
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-          ++stored;
+          if (k + kBulkAhead < P) issue(k + kBulkAhead);
         }
         piece += P;
       }

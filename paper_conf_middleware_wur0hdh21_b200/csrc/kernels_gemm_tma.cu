@@ -39,11 +39,13 @@ constexpr int kConvWarps = 8;
 constexpr int kMmaWarp = 9;
 constexpr int kThreads = 10 * 32;
 
-template <int BN>
+// BKT = 16 (128x256 tiles): half-depth stages, twice as many in the same shared memory, K-major
+// operands in SWIZZLE_64B (64-B rows) and MN-major blocks of 32 x 16 (2 KiB)
+template <int BN, int BKT = BK>
 struct TCfg {
-  static constexpr int STAGES = BN == 64 ? 4 : BN == 128 ? 3 : 2;
-  static constexpr int A_BYTES = BM * BK * 4;
-  static constexpr int B_BYTES = BN * BK * 4;
+  static constexpr int STAGES = BKT == 16 ? 4 : BN == 64 ? 4 : BN == 128 ? 3 : 2;
+  static constexpr int A_BYTES = BM * BKT * 4;
+  static constexpr int B_BYTES = BN * BKT * 4;
   static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
   static constexpr uint32_t TMEM_COLS = BN;
@@ -52,21 +54,30 @@ struct TCfg {
 struct TParams {
   int M, N, K, ldc;
   int splits, kb_per_split, acc, dbg, stages;
+  int cluster_reduce;  // 1: the splits of a tile form one cluster (1, 1, splits) and reduce over DSMEM
   float* C;
   float* ws;
   unsigned* counters;
 };
 
-__device__ __forceinline__ uint64_t desc_k(uint32_t saddr) {  // K-major SW128
+template <int BKT = BK>
+__device__ __forceinline__ uint64_t desc_k(uint32_t saddr) {
+  // K-major: BKT = 32 -> SWIZZLE_128B (layout 2, 8-row groups 1024 B apart); BKT = 16 ->
+  // SWIZZLE_64B (layout 4, 8-row groups 512 B apart)
+  if constexpr (BKT == 16)
+    return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (1ull << 16) | (32ull << 32) | (1ull << 46) |
+           (4ull << 61);
   return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (1ull << 16) | (64ull << 32) | (1ull << 46) |
          (2ull << 61);
 }
+template <int BKT = BK>
 __device__ __forceinline__ uint64_t desc_mn(uint32_t saddr) {
   // MN-major 32-bit operands use SWIZZLE_128B_BASE32B (layout type 1; 32-B swizzle atoms,
   // CUTLASS Layout_MN_SW128_32B_Atom): 4-row K groups 512 B apart (SBO), 32-element MN
   // blocks 4096 B apart (LBO).  TMA writes it with CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B.
-  return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (256ull << 16) | (32ull << 32) |
-         (1ull << 46) | (1ull << 61);
+  // (BKT = 16: the MN blocks are 2048 B apart)
+  return static_cast<uint64_t>((saddr & 0x3FFFFu) >> 4) | (static_cast<uint64_t>(BKT * 8) << 16) |
+         (32ull << 32) | (1ull << 46) | (1ull << 61);
 }
 
 using sfdev::tma_load_2d;
@@ -118,11 +129,12 @@ __device__ __forceinline__ void split_tile(float4* __restrict__ x, float4* __res
   }
 }
 
-template <int BN, bool A_MN, bool B_MN, bool RAW_HI>
+template <int BN, bool A_MN, bool B_MN, bool RAW_HI, int BKT = BK>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, TParams p) {
-  using C = TCfg<BN>;
+  using C = TCfg<BN, BKT>;
+  constexpr int BK = BKT;  // k-block depth of this instantiation
   const int NS = p.stages;  // ring depth (<= C::STAGES; 2 for short K: two CTAs per SM)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -168,14 +180,14 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         const int k0 = (kb_begin + i) * BK;
         if constexpr (A_MN) {
 #pragma unroll
-          for (int b = 0; b < BM / 32; ++b) tma_load_2d(st + b * 4096, &tmA, bar, m0 + 32 * b, k0);
+          for (int b = 0; b < BM / 32; ++b) tma_load_2d(st + b * (BK * 128), &tmA, bar, m0 + 32 * b, k0);
         } else {
           tma_load_2d(st, &tmA, bar, k0, m0);
         }
         const uint32_t sb = st + 2 * C::A_BYTES;
         if constexpr (B_MN) {
 #pragma unroll
-          for (int b = 0; b < BN / 32; ++b) tma_load_2d(sb + b * 4096, &tmB, bar, n0 + 32 * b, k0);
+          for (int b = 0; b < BN / 32; ++b) tma_load_2d(sb + b * (BK * 128), &tmB, bar, n0 + 32 * b, k0);
         } else {
           tma_load_2d(sb, &tmB, bar, k0, n0);
         }
@@ -216,8 +228,8 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         for (int kk = 0; kk < BK / 8; ++kk) {
           const uint32_t ao = A_MN ? kk * 1024 : kk * 32;
           const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
-          auto da = [&](uint32_t x) { return A_MN ? desc_mn(x + ao) : desc_k(x + ao); };
-          auto db = [&](uint32_t x) { return B_MN ? desc_mn(x + bo) : desc_k(x + bo); };
+          auto da = [&](uint32_t x) { return A_MN ? desc_mn<BK>(x + ao) : desc_k<BK>(x + ao); };
+          auto db = [&](uint32_t x) { return B_MN ? desc_mn<BK>(x + bo) : desc_k<BK>(x + bo); };
           if (!(p.dbg & 4)) {  // dbg bit 2 (probe only, wrong results): hi.hi MMA alone
             sfdev::mma_tf32(tmem, da(a_lo), db(b_hi), idesc, (i | kk) != 0);
             sfdev::mma_tf32(tmem, da(a_hi), db(b_lo), idesc, 1u);
@@ -255,6 +267,15 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
             if (n0 + c0 + j < p.N)
               r[j] = __float_as_uint(__uint_as_float(r[j]) + p.C[static_cast<size_t>(row) * p.ldc + n0 + c0 + j]);
       }
+      if (p.cluster_reduce) {  // this split's partial -> own smem, 32x32 blocks (col block, quarter)
+        uint8_t* blk = smem + ((c0 >> 5) * 4 + q) * 4096;
+#pragma unroll
+        for (int ch = 0; ch < 8; ++ch) {
+          const uint32_t off = lane * 128 + ((ch ^ (lane & 7)) << 4);
+          *reinterpret_cast<uint4*>(blk + off) = make_uint4(r[4 * ch], r[4 * ch + 1], r[4 * ch + 2], r[4 * ch + 3]);
+        }
+        continue;
+      }
       if (p.dbg & 1) {  // debug: plain global stores of the accumulator
         const int row = m0 + row0 + lane;
         if (row < p.M && p.splits == 1)
@@ -285,6 +306,41 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA writes before generic ops
     }
     __syncwarp();
+  }
+  if (p.cluster_reduce) {
+    // split-K without a workspace: the tile's S splits are one cluster; after every partial
+    // sits in its CTA's smem, CTA z sums its 1/S share of the tile's 16-B chunks over the
+    // cluster's smem in the fixed order z' = 0..S-1 (then + C when accumulating) and stores it
+    __syncwarp();
+    cooperative_groups::cluster_group cl = cooperative_groups::this_cluster();
+    cl.sync();
+    const int S = p.splits;
+    constexpr int CPR = BN / 4;  // 16-B chunks per tile row
+    constexpr int TOT = BM * CPR;
+    const int per = (TOT + S - 1) / S;
+    const int c_beg = z * per, c_end = min(TOT, c_beg + per);
+    for (int c = c_beg + static_cast<int>(threadIdx.x); c < c_end; c += kThreads) {
+      const int row = c / CPR, col4 = c % CPR;
+      const int gr = m0 + row, gc = n0 + col4 * 4;
+      if (gr >= p.M || gc >= p.N) continue;
+      const int ln = row & 31, ch = col4 & 7;
+      const uint32_t off = (((col4 >> 3) * 4 + (row >> 5)) * 4096) + ln * 128 + ((ch ^ (ln & 7)) << 4);
+      float4 v[8];
+#pragma unroll
+      for (int zz = 0; zz < 8; ++zz)
+        if (zz < S) v[zz] = *reinterpret_cast<const float4*>(cl.map_shared_rank(smem + off, zz));
+      float4 t = v[0];
+#pragma unroll
+      for (int zz = 1; zz < 8; ++zz)
+        if (zz < S) { t.x += v[zz].x; t.y += v[zz].y; t.z += v[zz].z; t.w += v[zz].w; }
+      float4* o = reinterpret_cast<float4*>(p.C + static_cast<size_t>(gr) * p.ldc + gc);
+      if (p.acc) {
+        const float4 c0v = *o;
+        t.x = c0v.x + t.x; t.y = c0v.y + t.y; t.z = c0v.z + t.z; t.w = c0v.w + t.w;
+      }
+      *o = t;
+    }
+    cl.sync();  // no CTA leaves (freeing its smem) while a peer still reads it
   }
   sfdev::tc_fence_before();
   __syncthreads();
@@ -1064,20 +1120,38 @@ bool map3d_ws(CUtensorMap* m, const void* base, uint64_t N, uint64_t M, uint64_t
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int BN, bool AM, bool BMn, bool RAW>
+template <int BN, bool AM, bool BMn, bool RAW, int BKT = BK>
 cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
                          const TParams& p, dim3 grid, cudaStream_t st) {
-  auto kern = gemm_tma_kernel<BN, AM, BMn, RAW>;
+  auto kern = gemm_tma_kernel<BN, AM, BMn, RAW, BKT>;
+  using TC = TCfg<BN, BKT>;
   static std::atomic<uint64_t> configured{0};
   int dev = 0;
   cudaGetDevice(&dev);
   const uint64_t bit = 1ull << (dev & 63);
   if (!(configured.load() & bit)) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, TCfg<BN>::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, TC::SMEM);
     if (e != cudaSuccess) return e;
     configured.fetch_or(bit);
   }
-  const int smem = p.stages * TCfg<BN>::STAGE_BYTES + 1024 + 256;
+  const int smem = p.stages * TC::STAGE_BYTES + 1024 + 256;
+  if (p.cluster_reduce) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 1;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = p.splits;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, a, b, c, p);
+    count_launch();
+    return e;
+  }
   kern<<<grid, kThreads, smem, st>>>(a, b, c, p);
   count_launch();
   return cudaGetLastError();
@@ -1111,13 +1185,13 @@ cudaError_t dispatch_persistent(bool a_mn, bool b_mn, const CUtensorMap& a, cons
   return launch_persistent_t<BN, false, false>(a, b, c, p, st);
 }
 
-template <int BN, bool RAW>
+template <int BN, bool RAW, int BKT = BK>
 cudaError_t dispatch_major(bool a_mn, bool b_mn, const CUtensorMap& a, const CUtensorMap& b,
                            const CUtensorMap& c, const TParams& p, dim3 grid, cudaStream_t st) {
-  if (a_mn && b_mn) return launch_tma_t<BN, true, true, RAW>(a, b, c, p, grid, st);
-  if (a_mn) return launch_tma_t<BN, true, false, RAW>(a, b, c, p, grid, st);
-  if (b_mn) return launch_tma_t<BN, false, true, RAW>(a, b, c, p, grid, st);
-  return launch_tma_t<BN, false, false, RAW>(a, b, c, p, grid, st);
+  if (a_mn && b_mn) return launch_tma_t<BN, true, true, RAW, BKT>(a, b, c, p, grid, st);
+  if (a_mn) return launch_tma_t<BN, true, false, RAW, BKT>(a, b, c, p, grid, st);
+  if (b_mn) return launch_tma_t<BN, false, true, RAW, BKT>(a, b, c, p, grid, st);
+  return launch_tma_t<BN, false, false, RAW, BKT>(a, b, c, p, grid, st);
 }
 
 
@@ -1297,11 +1371,16 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   CUtensorMap ma, mb, mc;
   // A: op(A) is M x K.  Stored [M][K] (K-major) or [K][M] (MN-major).
   constexpr CUtensorMapSwizzle kMN = CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
-  bool ok = a_mn ? map2d(&ma, a.A, a.M, a.K, static_cast<uint64_t>(a.lda) * 4, 32, 32, kMN)
-                 : map2d(&ma, a.A, a.K, a.M, static_cast<uint64_t>(a.lda) * 4, 32, BM);
+  // 128x256 tiles stage K in 16-deep blocks (4 stages instead of 2 in the same shared memory:
+  // the 2-stage ring left the MMAs waiting on TMA latency); SF_GEMM_BK256=32 restores 32
+  static const int bk256 = std::getenv("SF_GEMM_BK256") ? std::atoi(std::getenv("SF_GEMM_BK256")) : 16;
+  const int bk = bn == 256 && bk256 == 16 && splits == 1 ? 16 : 32;
+  const CUtensorMapSwizzle kK = bk == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B;
+  bool ok = a_mn ? map2d(&ma, a.A, a.M, a.K, static_cast<uint64_t>(a.lda) * 4, 32, bk, kMN)
+                 : map2d(&ma, a.A, a.K, a.M, static_cast<uint64_t>(a.lda) * 4, bk, BM, kK);
   // B: op(B) is K x N.  Stored [K][N] (MN-major) or [N][K] (TB, K-major).
-  ok = ok && (b_mn ? map2d(&mb, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, 32, 32, kMN)
-                   : map2d(&mb, a.B, a.K, a.N, static_cast<uint64_t>(a.ldb) * 4, 32, bn));
+  ok = ok && (b_mn ? map2d(&mb, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, 32, bk, kMN)
+                   : map2d(&mb, a.B, a.K, a.N, static_cast<uint64_t>(a.ldb) * 4, bk, bn, kK));
   ok = ok && (splits == 1 ? map2d(&mc, a.C, a.N, a.M, static_cast<uint64_t>(a.ldc) * 4, 32, 32)
                           : map3d_ws(&mc, a.ws, a.N, a.M, splits));
   if (!ok) return cudaErrorInvalidValue;
@@ -1312,10 +1391,16 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   // split-K shapes keep the deep ring).  SF_GEMM_STAGES overrides.
   static const int stages_env = std::getenv("SF_GEMM_STAGES") ? std::atoi(std::getenv("SF_GEMM_STAGES")) : -1;
   const int max_stages = bn == 64 ? TCfg<64>::STAGES : bn == 128 ? TCfg<128>::STAGES : TCfg<256>::STAGES;
-  int stages = max_stages;
-  if (stages_env > 0) stages = std::min(stages_env, max_stages);
+  int stages = bk == 16 ? TCfg<256, 16>::STAGES : max_stages;
+  if (stages_env > 0) stages = std::min(stages_env, bk == 16 ? TCfg<256, 16>::STAGES : max_stages);
   else if (bn == 64 && (splits == 1 ? tiles_n * tiles_m > 148 : gemm_dual64())) stages = 2;  // 2 x 97 KB fit an SM
-  TParams p{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, dbg, stages, a.C, a.ws, a.counters};
+  // split-K over 2..8 splits reduces inside the kernel (cluster of the tile's splits, DSMEM):
+  // no workspace round trip, no reduce launch; SF_GEMM_CLUSTER_RED=0 keeps the workspace path
+  static const bool cl_env = !(std::getenv("SF_GEMM_CLUSTER_RED") && std::getenv("SF_GEMM_CLUSTER_RED")[0] == '0');
+  const bool cl_red = cl_env && splits >= 2 && splits <= 8 && a.ldc % 4 == 0 &&
+                      reinterpret_cast<uintptr_t>(a.C) % 16 == 0;
+  TParams p{a.M, a.N, a.K, a.ldc, splits, bk == 16 ? (a.K + 15) / 16 : kb_per_split, a.acc ? 1 : 0, dbg, stages,
+            cl_red ? 1 : 0, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;
   // persistent CTAs (double-buffered TMEM) measured equal to per-tile CTAs on the forest
@@ -1330,11 +1415,12 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
     e = raw_hi ? dispatch_major<64, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<64, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
   else if (bn == 256)
-    e = dispatch_major<256, true>(a_mn, b_mn, ma, mb, mc, p, grid, st);
+    e = bk == 16 ? dispatch_major<256, true, 16>(a_mn, b_mn, ma, mb, mc, p, grid, st)
+                 : dispatch_major<256, true>(a_mn, b_mn, ma, mb, mc, p, grid, st);
   else
     e = raw_hi ? dispatch_major<128, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<128, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
-  if (e != cudaSuccess || splits == 1) return e;
+  if (e != cudaSuccess || splits == 1 || cl_red) return e;
   if (a.ldc % 4 || reinterpret_cast<uintptr_t>(a.C) % 16) return cudaErrorInvalidValue;
   const uint64_t total4 = static_cast<uint64_t>(a.M) * a.N / 4;
   splitk_reduce_kernel<<<static_cast<unsigned>((total4 + 31) / 32), 256, 0, st>>>(

@@ -23,4 +23,4 @@ for name, M, N, Kd, fl in shapes:
     e1.record(); e1.synchronize()
     us = e0.elapsed_time(e1) * 1e3 / n
     print(json.dumps({"name": name, "M": M, "N": N, "K": Kd, "us": round(us, 1),
-                      "tflops_alg": round(2 * M * N * Kd / us / 1e6, 1)}), flush=True)
+                      "tflops_alg": round(2 * M * N * Kd / us / 1e6, 1), "path": K.last_gemm_path()}), flush=True)
