@@ -20,6 +20,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <atomic>
 #include <map>
@@ -41,12 +42,19 @@ constexpr int kThreads = 10 * 32;
 
 // BKT = 16 (128x256 tiles): half-depth stages, twice as many in the same shared memory, K-major
 // operands in SWIZZLE_64B (64-B rows) and MN-major blocks of 32 x 16 (2 KiB)
-template <int BN, int BKT = BK>
+//
+// ATM (A in TMEM): the converters read the raw A tile once from shared memory and write its tf32
+// hi / lo split straight into TMEM columns (tcgen05.st); the MMAs take A from TMEM and only B
+// from shared memory.  Shared-memory traffic per k-block is what bounds this loop (TMA writes +
+// converter reads / writes + MMA operand reads at ~128 B/clk: 192 KB -> 1500 cycles per 128x128
+// k-block with A in smem, 128 KB with A in TMEM); the stage then holds A raw + B raw + B lo.
+template <int BN, int BKT = BK, bool ATM = false>
 struct TCfg {
-  static constexpr int STAGES = BKT == 16 ? 4 : BN == 64 ? 4 : BN == 128 ? 3 : 2;
   static constexpr int A_BYTES = BM * BKT * 4;
   static constexpr int B_BYTES = BN * BKT * 4;
-  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int STAGE_BYTES = ATM ? A_BYTES + 2 * B_BYTES : 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int STAGES = ATM ? (BN == 64 ? 6 : BN == 128 ? 4 : BKT == 16 ? 5 : 2)
+                                    : BKT == 16 ? 4 : BN == 64 ? 4 : BN == 128 ? 3 : 2;
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
   static constexpr uint32_t TMEM_COLS = BN;
 };
@@ -129,11 +137,102 @@ __device__ __forceinline__ void split_tile(float4* __restrict__ x, float4* __res
   }
 }
 
-template <int BN, bool A_MN, bool B_MN, bool RAW_HI, int BKT = BK>
+__device__ __forceinline__ float lds32(uint32_t a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+  return v;
+}
+template <int NR>
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const float (&v)[NR]) {  // 32x32b.xNR
+  static_assert(NR == 8 || NR == 16, "tmem_st: 8 or 16 columns");
+  if constexpr (NR == 16)
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};"
+                 :: "r"(taddr), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]),
+                    "f"(v[7]), "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]),
+                    "f"(v[15]) : "memory");
+  else
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+                 :: "r"(taddr), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]),
+                    "f"(v[7]) : "memory");
+}
+__device__ __forceinline__ void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                            uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}"
+      :: "r"(d_tmem), "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate));
+}
+
+// Split-K reduction of one tile over its cluster (S CTAs, rank = split index z): CTA z sums its
+// 1/S share of the tile's 16-B chunks over the S partials (32x32 swizzled blocks in each CTA's
+// smem) in the fixed order 0..S-1, then + C when accumulating.  Loads go out in batches of
+// about 16 remote 16-B reads per thread before any is consumed (one DSMEM round trip per batch).
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t cluster_map(uint32_t saddr, int rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+
+// Split-K reduction of one tile inside its cluster (S CTAs, rank = split z).  Every CTA holds
+// its fp32 partial in smem [0, T) as 32x32 swizzled blocks (block = col block * 4 + quarter).
+// Owner z reduces the 16-B chunks [z PER, (z+1) PER): each other CTA pushes that range of its
+// partial into the owner's receive slot with ONE bulk DSMEM copy (completion on the owner's
+// mbarrier), then the owner sums its own and the S-1 received ranges from local smem in the
+// fixed order z' = 0..S-1 (+ C when accumulating) and stores the chunks to C.
+template <int BN>
+__device__ __forceinline__ void cluster_push_reduce(uint8_t* smem, uint64_t* red_bar, const TParams& p, int m0,
+                                                    int n0, int z) {
+  constexpr int T = BM * BN * 4, TOT = T / 16;
+  const int S = p.splits;
+  const int PER = (TOT + S - 1) / S;
+  auto len = [&](int o) { return max(0, min(TOT, (o + 1) * PER) - o * PER); };
+  const uint32_t sbase = sfdev::smem_u32(smem), bar = sfdev::smem_u32(red_bar);
+  if (threadIdx.x == 0) {
+    const int mine = len(z);
+    if (mine > 0) expect_tx(red_bar, static_cast<uint32_t>((S - 1) * mine * 16));
+    else sfdev::mbar_arrive(red_bar);
+    for (int o = 0; o < S; ++o) {
+      if (o == z || len(o) == 0) continue;
+      const int slot = z < o ? z : z - 1;
+      const uint32_t dst = cluster_map(sbase + T + slot * PER * 16, o);
+      asm volatile("cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                   :: "r"(dst), "r"(sbase + o * PER * 16), "r"(len(o) * 16), "r"(cluster_map(bar, o)) : "memory");
+    }
+  }
+  sfdev::mbar_wait(red_bar, 0);
+  const int c_beg = z * PER, c_end = c_beg + len(z);
+  for (int c = c_beg + static_cast<int>(threadIdx.x); c < c_end; c += kThreads) {
+    const int off = c * 16;
+    const int block = off >> 12, within = off & 4095;
+    const int ln = within >> 7, ch = ((within >> 4) & 7) ^ (ln & 7);
+    const int row = (block & 3) * 32 + ln, col4 = (block >> 2) * 8 + ch;
+    const int gr = m0 + row, gc = n0 + col4 * 4;
+    float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int zz = 0; zz < S; ++zz) {
+      const uint32_t a = zz == z ? sbase + off : sbase + T + (zz < z ? zz : zz - 1) * PER * 16 + (c - c_beg) * 16;
+      const float4 v = lds128(a);
+      if (zz == 0) t = v;
+      else { t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w; }
+    }
+    if (gr >= p.M || gc >= p.N) continue;
+    float4* o = reinterpret_cast<float4*>(p.C + static_cast<size_t>(gr) * p.ldc + gc);
+    if (p.acc) {
+      const float4 cv = *o;
+      t.x = cv.x + t.x; t.y = cv.y + t.y; t.z = cv.z + t.z; t.w = cv.w + t.w;
+    }
+    *o = t;
+  }
+}
+
+template <int BN, bool A_MN, bool B_MN, bool RAW_HI, int BKT = BK, bool ATM = false>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, TParams p) {
-  using C = TCfg<BN, BKT>;
+  using C = TCfg<BN, BKT, ATM>;
   constexpr int BK = BKT;  // k-block depth of this instantiation
   const int NS = p.stages;  // ring depth (<= C::STAGES; 2 for short K: two CTAs per SM)
   extern __shared__ uint8_t smem_raw[];
@@ -144,30 +243,41 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   uint64_t* empty = conv_full + NS;
   uint64_t* done = empty + NS;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(done + 1);
+  uint64_t* red_bar = done + 2;  // split-K cluster reduction (receive slots complete here)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM, z = blockIdx.z;
+  __shared__ long long tsd[8];  // phase probe (SF_GEMM_DEBUG bit 3: clock64 stamps, printf of 3 CTAs)
+  if ((p.dbg & 8) && threadIdx.x == 0) tsd[0] = clock64();
   const int nkb_total = (p.K + BK - 1) / BK;
   const int kb_begin = z * p.kb_per_split;
   const int nkb = max(0, min(nkb_total, kb_begin + p.kb_per_split) - kb_begin);
-
   if (threadIdx.x == 0) {
     for (int s = 0; s < NS; ++s) {
       sfdev::mbar_init(&tma_full[s], 1);
       sfdev::mbar_init(&conv_full[s], kConvWarps);
       sfdev::mbar_init(&empty[s], 1);
     }
+    sfdev::mbar_init(red_bar, 1);
     sfdev::mbar_init(done, 1);
     sfdev::mbar_fence_init();
     asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
     asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
   }
-  if (warp == kMmaWarp) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
+  // ATM: accumulator in columns [0, BN), stage s's A hi / lo at BN + 2 s BK (+ BK); a 2-stage
+  // ring (two CTAs per SM) fits 256 columns, deeper rings take all 512
+  const bool tm_small = !ATM || BN + NS * 2 * BK <= 256;
+  if (warp == kMmaWarp) {
+    if (!ATM) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
+    else if (tm_small) sfdev::tmem_alloc<256>(tmem_slot);
+    else sfdev::tmem_alloc<512>(tmem_slot);
+  }
   sfdev::tc_fence_before();
   __syncthreads();
   sfdev::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if ((p.dbg & 8) && threadIdx.x == 0) tsd[1] = clock64();
 
   if (warp == 0) {
     if (lane == 0) {
@@ -184,7 +294,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         } else {
           tma_load_2d(st, &tmA, bar, k0, m0);
         }
-        const uint32_t sb = st + 2 * C::A_BYTES;
+        const uint32_t sb = st + (ATM ? 1 : 2) * C::A_BYTES;
         if constexpr (B_MN) {
 #pragma unroll
           for (int b = 0; b < BN / 32; ++b) tma_load_2d(sb + b * (BK * 128), &tmB, bar, n0 + 32 * b, k0);
@@ -193,11 +303,69 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         }
       }
     }
+  } else if (ATM && warp <= kConvWarps) {
+    // B: lo split in shared memory (all 256 threads).  A: warp w owns TMEM lane quarter w % 4
+    // (rows 32 q + lane) and K half h; its thread reads its row's BK / 2 raw values, writes
+    // hi = raw (the MMA reads only the tf32 bits) and lo = tf32(x - tf32(x)) into TMEM.
+    const int t = threadIdx.x - 32;
+    const int q = warp & 3, h = (warp - 1) >> 2;
+    constexpr int KH = BK / 2;
+    const int r = 32 * q + lane;
+    const uint32_t lane_base = static_cast<uint32_t>(32 * q) << 16;
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % NS;
+      sfdev::mbar_wait(&tma_full[s], (i / NS) & 1);
+      if ((p.dbg & 8) && i == 0 && threadIdx.x == 32) tsd[2] = clock64();
+      uint8_t* st = smem + s * C::STAGE_BYTES;
+      const uint32_t sa = sfdev::smem_u32(st);
+      float x[KH];
+      if constexpr (A_MN) {  // SWIZZLE_128B rows of 32 M (one block per quarter), BK rows of K
+        const uint32_t base = sa + q * (BK * 128) + (lane & 3) * 4;
+#pragma unroll
+        for (int j = 0; j < KH; ++j) {
+          const int k = h * KH + j;
+          x[j] = lds32(base + k * 128 + ((((lane >> 2) ^ (k & 7))) << 4));
+        }
+      } else if constexpr (BK == 32) {  // K-major SWIZZLE_128B: 128-B rows
+#pragma unroll
+        for (int cc = 0; cc < KH / 4; ++cc) {
+          const int c = h * (KH / 4) + cc;
+          const float4 v = lds128(sa + r * 128 + ((c ^ (r & 7)) << 4));
+          x[4 * cc] = v.x; x[4 * cc + 1] = v.y; x[4 * cc + 2] = v.z; x[4 * cc + 3] = v.w;
+        }
+      } else {  // K-major SWIZZLE_64B: 64-B rows
+#pragma unroll
+        for (int cc = 0; cc < KH / 4; ++cc) {
+          const int c = h * (KH / 4) + cc;
+          const float4 v = lds128(sa + r * 64 + ((c ^ ((r >> 1) & 3)) << 4));
+          x[4 * cc] = v.x; x[4 * cc + 1] = v.y; x[4 * cc + 2] = v.z; x[4 * cc + 3] = v.w;
+        }
+      }
+      if (!(p.dbg & 2)) {
+        float lo[KH];
+#pragma unroll
+        for (int j = 0; j < KH; ++j) lo[j] = tf32_trunc(x[j] - tf32_trunc(x[j]));
+        const uint32_t col = static_cast<uint32_t>(BN + s * 2 * BK + h * KH);
+        tmem_st<KH>(tmem + lane_base + col, x);
+        tmem_st<KH>(tmem + lane_base + col + BK, lo);
+        float4* b = reinterpret_cast<float4*>(st + C::A_BYTES);
+        float4* blo = reinterpret_cast<float4*>(st + C::A_BYTES + C::B_BYTES);
+        split_tile<C::B_BYTES / 16 / 256, true>(b, blo, t);
+      } else {
+        tmem_st<KH>(tmem + lane_base + static_cast<uint32_t>(BN + s * 2 * BK + h * KH), x);
+      }
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      sfdev::fence_proxy_async_smem();
+      sfdev::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) sfdev::mbar_arrive(&conv_full[s]);
+    }
   } else if (warp <= kConvWarps) {
     const int t = threadIdx.x - 32;  // 0..255
     for (int i = 0; i < nkb; ++i) {
       const int s = i % NS;
       sfdev::mbar_wait(&tma_full[s], (i / NS) & 1);
+      if ((p.dbg & 8) && i == 0 && threadIdx.x == 32) tsd[2] = clock64();
       uint8_t* st = smem + s * C::STAGE_BYTES;
       float4* a = reinterpret_cast<float4*>(st);
       float4* alo = reinterpret_cast<float4*>(st + C::A_BYTES);
@@ -213,14 +381,28 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     }
   } else {
     // MMA issuer
-    constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((A_MN ? 1u : 0u) << 15) |
+    constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((A_MN && !ATM ? 1u : 0u) << 15) |
                                ((B_MN ? 1u : 0u) << 16) | (uint32_t(BN >> 3) << 17) |
                                (uint32_t(BM >> 4) << 24);
     for (int i = 0; i < nkb; ++i) {
       const int s = i % NS;
       sfdev::mbar_wait(&conv_full[s], (i / NS) & 1);
       sfdev::tc_fence_after();
-      if (lane == 0) {
+      if (ATM && lane == 0) {
+        const uint32_t b_hi = sfdev::smem_u32(smem + s * C::STAGE_BYTES) + C::A_BYTES, b_lo = b_hi + C::B_BYTES;
+        const uint32_t a_hi = tmem + static_cast<uint32_t>(BN + s * 2 * BK), a_lo = a_hi + BK;
+#pragma unroll
+        for (int kk = 0; kk < BK / 8; ++kk) {
+          const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
+          auto db = [&](uint32_t x) { return B_MN ? desc_mn<BK>(x + bo) : desc_k<BK>(x + bo); };
+          if (!(p.dbg & 4)) {
+            mma_tf32_ts(tmem, a_lo + kk * 8, db(b_hi), idesc, (i | kk) != 0);
+            mma_tf32_ts(tmem, a_hi + kk * 8, db(b_lo), idesc, 1u);
+          }
+          mma_tf32_ts(tmem, a_hi + kk * 8, db(b_hi), idesc, (p.dbg & 4) ? ((i | kk) != 0) : 1u);
+        }
+        sfdev::mma_commit(&empty[s]);
+      } else if (!ATM && lane == 0) {
         const uint32_t base = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
         const uint32_t a_hi = base, a_lo = base + C::A_BYTES;
         const uint32_t b_hi = base + 2 * C::A_BYTES, b_lo = b_hi + C::B_BYTES;
@@ -240,6 +422,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       }
       __syncwarp();
     }
+    if ((p.dbg & 8) && lane == 0) tsd[3] = clock64();
     if (lane == 0) sfdev::mma_commit(done);
     __syncwarp();
   }
@@ -247,6 +430,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   if (warp >= 1 && warp <= 4) {
     sfdev::mbar_wait(done, 0);
     sfdev::tc_fence_after();
+    if ((p.dbg & 8) && threadIdx.x == 32) tsd[4] = clock64();
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     const int row0 = q * 32;
     uint8_t* ebuf = smem + q * 2 * 4096;  // stage memory is free once `done` fired
@@ -274,6 +458,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
           const uint32_t off = lane * 128 + ((ch ^ (lane & 7)) << 4);
           *reinterpret_cast<uint4*>(blk + off) = make_uint4(r[4 * ch], r[4 * ch + 1], r[4 * ch + 2], r[4 * ch + 3]);
         }
+        sfdev::fence_proxy_async_smem();  // the partial leaves by bulk copy (async proxy)
         continue;
       }
       if (p.dbg & 1) {  // debug: plain global stores of the accumulator
@@ -307,268 +492,34 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     }
     __syncwarp();
   }
+  if ((p.dbg & 8) && threadIdx.x == 32) tsd[5] = clock64();
   if (p.cluster_reduce) {
-    // split-K without a workspace: the tile's S splits are one cluster; after every partial
-    // sits in its CTA's smem, CTA z sums its 1/S share of the tile's 16-B chunks over the
-    // cluster's smem in the fixed order z' = 0..S-1 (then + C when accumulating) and stores it
+    // split-K without a workspace: the tile's S splits are one cluster (cluster_push_reduce)
     __syncwarp();
-    cooperative_groups::cluster_group cl = cooperative_groups::this_cluster();
-    cl.sync();
-    const int S = p.splits;
-    constexpr int CPR = BN / 4;  // 16-B chunks per tile row
-    constexpr int TOT = BM * CPR;
-    const int per = (TOT + S - 1) / S;
-    const int c_beg = z * per, c_end = min(TOT, c_beg + per);
-    for (int c = c_beg + static_cast<int>(threadIdx.x); c < c_end; c += kThreads) {
-      const int row = c / CPR, col4 = c % CPR;
-      const int gr = m0 + row, gc = n0 + col4 * 4;
-      if (gr >= p.M || gc >= p.N) continue;
-      const int ln = row & 31, ch = col4 & 7;
-      const uint32_t off = (((col4 >> 3) * 4 + (row >> 5)) * 4096) + ln * 128 + ((ch ^ (ln & 7)) << 4);
-      float4 v[8];
-#pragma unroll
-      for (int zz = 0; zz < 8; ++zz)
-        if (zz < S) v[zz] = *reinterpret_cast<const float4*>(cl.map_shared_rank(smem + off, zz));
-      float4 t = v[0];
-#pragma unroll
-      for (int zz = 1; zz < 8; ++zz)
-        if (zz < S) { t.x += v[zz].x; t.y += v[zz].y; t.z += v[zz].z; t.w += v[zz].w; }
-      float4* o = reinterpret_cast<float4*>(p.C + static_cast<size_t>(gr) * p.ldc + gc);
-      if (p.acc) {
-        const float4 c0v = *o;
-        t.x = c0v.x + t.x; t.y = c0v.y + t.y; t.z = c0v.z + t.z; t.w = c0v.w + t.w;
-      }
-      *o = t;
-    }
-    cl.sync();  // no CTA leaves (freeing its smem) while a peer still reads it
+    cluster_sync_all();  // every partial in smem (made visible to the async proxy by its writers)
+    if ((p.dbg & 8) && threadIdx.x == 0) tsd[6] = clock64();
+    cluster_push_reduce<BN>(smem, red_bar, p, m0, n0, z);
+    __syncwarp();
+    cluster_sync_all();  // no CTA leaves (freeing its smem) while a peer still copies from it
   }
   sfdev::tc_fence_before();
   __syncthreads();
   sfdev::tc_fence_after();
-  if (warp == kMmaWarp) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
+  if ((p.dbg & 8) && threadIdx.x == 0) {
+    tsd[7] = clock64();
+    const unsigned bid = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+    if (bid == 0 || bid == gridDim.x * gridDim.y * gridDim.z - 1 || bid == 37)
+      printf("PHASE bid %u nkb %d setup %lld firstTMA %lld mma_end %lld epi_start %lld epi_end %lld cl1 %lld end %lld\n",
+             bid, nkb, tsd[1] - tsd[0], tsd[2] - tsd[0], tsd[3] - tsd[0], tsd[4] - tsd[0], tsd[5] - tsd[0],
+             p.cluster_reduce ? tsd[6] - tsd[0] : -1ll, tsd[7] - tsd[0]);
+  }
+  if (warp == kMmaWarp) {
+    if (!ATM) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
+    else if (tm_small) sfdev::tmem_dealloc<256>(tmem);
+    else sfdev::tmem_dealloc<512>(tmem);
+  }
 }
 
-// ---- persistent variant -----------------------------------------------------------------
-// One CTA per SM loops over work units u = blockIdx.x + i * gridDim.x (tile_n fastest, then
-// tile_m, then split z).  TMEM holds two accumulators: the MMA warp fills unit i+1 while the
-// epilogue warps (10-13, one per TMEM lane quarter) drain unit i, so epilogue, prologue and
-// TMA latency overlap the tensor work.  Same per-tile arithmetic as gemm_tma_kernel.
-constexpr int kPThreads = 14 * 32;  // 0 TMA, 1-8 convert, 9 MMA, 10-13 epilogue
-
-template <int BN>
-struct PCfg {
-  static constexpr int STAGES = BN == 64 ? 4 : 3;
-  static constexpr int A_BYTES = BM * BK * 4;
-  static constexpr int B_BYTES = BN * BK * 4;
-  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int EPI_BYTES = 4 * 2 * 4096;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_BYTES + 1024 + 256;
-  static constexpr uint32_t TMEM_COLS = 2 * BN;
-};
-
-struct PParams {
-  int M, N, K, ldc;
-  int splits, kb_per_split, acc;
-  int tiles_n, tiles_m, units;
-  float* C;
-};
-
-template <int BN, bool A_MN, bool B_MN>
-__global__ void __launch_bounds__(kPThreads, 1)
-gemm_tma_persistent_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                           const __grid_constant__ CUtensorMap tmC, PParams p) {
-  using C = PCfg<BN>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                             ~static_cast<uintptr_t>(1023));
-  uint8_t* epi = smem + C::STAGES * C::STAGE_BYTES;
-  uint64_t* tma_full = reinterpret_cast<uint64_t*>(epi + C::EPI_BYTES);
-  uint64_t* conv_full = tma_full + C::STAGES;
-  uint64_t* empty = conv_full + C::STAGES;
-  uint64_t* acc_full = empty + C::STAGES;   // [2]
-  uint64_t* acc_empty = acc_full + 2;       // [2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nkb_total = (p.K + BK - 1) / BK;
-
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < C::STAGES; ++s) {
-      sfdev::mbar_init(&tma_full[s], 1);
-      sfdev::mbar_init(&conv_full[s], kConvWarps);
-      sfdev::mbar_init(&empty[s], 1);
-    }
-    for (int a = 0; a < 2; ++a) {
-      sfdev::mbar_init(&acc_full[a], 1);
-      sfdev::mbar_init(&acc_empty[a], 4);
-    }
-    sfdev::mbar_fence_init();
-    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
-    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
-    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
-  }
-  if (warp == kMmaWarp) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
-  sfdev::tc_fence_before();
-  __syncthreads();
-  sfdev::tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-
-  auto unit_coords = [&](int u, int& n0, int& m0, int& z, int& kb_begin, int& nkb) {
-    const int tn = u % p.tiles_n;
-    const int rest = u / p.tiles_n;
-    const int tm = rest % p.tiles_m;
-    z = rest / p.tiles_m;
-    n0 = tn * BN;
-    m0 = tm * BM;
-    kb_begin = z * p.kb_per_split;
-    nkb = max(0, min(nkb_total, kb_begin + p.kb_per_split) - kb_begin);
-  };
-
-  if (warp == 0) {
-    if (lane == 0) {
-      int it = 0;  // global stage counter across units
-      for (int u = blockIdx.x; u < p.units; u += gridDim.x) {
-        int n0, m0, z, kb_begin, nkb;
-        unit_coords(u, n0, m0, z, kb_begin, nkb);
-        for (int i = 0; i < nkb; ++i, ++it) {
-          const int s = it % C::STAGES, round = it / C::STAGES;
-          if (round > 0) sfdev::mbar_wait(&empty[s], (round - 1) & 1);
-          const uint32_t st = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
-          const uint32_t bar = sfdev::smem_u32(&tma_full[s]);
-          expect_tx(&tma_full[s], C::A_BYTES + C::B_BYTES);
-          const int k0 = (kb_begin + i) * BK;
-          if constexpr (A_MN) {
-#pragma unroll
-            for (int b = 0; b < BM / 32; ++b) tma_load_2d(st + b * 4096, &tmA, bar, m0 + 32 * b, k0);
-          } else {
-            tma_load_2d(st, &tmA, bar, k0, m0);
-          }
-          const uint32_t sb = st + 2 * C::A_BYTES;
-          if constexpr (B_MN) {
-#pragma unroll
-            for (int b = 0; b < BN / 32; ++b) tma_load_2d(sb + b * 4096, &tmB, bar, n0 + 32 * b, k0);
-          } else {
-            tma_load_2d(sb, &tmB, bar, k0, n0);
-          }
-        }
-      }
-    }
-  } else if (warp <= kConvWarps) {
-    const int t = threadIdx.x - 32;
-    int it = 0;
-    for (int u = blockIdx.x; u < p.units; u += gridDim.x) {
-      int n0, m0, z, kb_begin, nkb;
-      unit_coords(u, n0, m0, z, kb_begin, nkb);
-      for (int i = 0; i < nkb; ++i, ++it) {
-        const int s = it % C::STAGES;
-        sfdev::mbar_wait(&tma_full[s], (it / C::STAGES) & 1);
-        uint8_t* st = smem + s * C::STAGE_BYTES;
-        split_tile<C::A_BYTES / 16 / 256, true>(reinterpret_cast<float4*>(st),
-                                                reinterpret_cast<float4*>(st + C::A_BYTES), t);
-        split_tile<C::B_BYTES / 16 / 256, true>(reinterpret_cast<float4*>(st + 2 * C::A_BYTES),
-                                                reinterpret_cast<float4*>(st + 2 * C::A_BYTES + C::B_BYTES), t);
-        sfdev::fence_proxy_async_smem();
-        __syncwarp();
-        if (lane == 0) sfdev::mbar_arrive(&conv_full[s]);
-      }
-    }
-  } else if (warp == kMmaWarp) {
-    constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((A_MN ? 1u : 0u) << 15) |
-                               ((B_MN ? 1u : 0u) << 16) | (uint32_t(BN >> 3) << 17) |
-                               (uint32_t(BM >> 4) << 24);
-    int it = 0, t_local = 0;
-    for (int u = blockIdx.x; u < p.units; u += gridDim.x, ++t_local) {
-      int n0, m0, z, kb_begin, nkb;
-      unit_coords(u, n0, m0, z, kb_begin, nkb);
-      const int a = t_local & 1;
-      sfdev::mbar_wait(&acc_empty[a], ((t_local >> 1) & 1) ^ 1);  // epilogue freed it
-      sfdev::tc_fence_after();
-      const uint32_t d = tmem + a * BN;
-      for (int i = 0; i < nkb; ++i, ++it) {
-        const int s = it % C::STAGES;
-        sfdev::mbar_wait(&conv_full[s], (it / C::STAGES) & 1);
-        sfdev::tc_fence_after();
-        if (lane == 0) {
-          const uint32_t base = sfdev::smem_u32(smem + s * C::STAGE_BYTES);
-          const uint32_t a_hi = base, a_lo = base + C::A_BYTES;
-          const uint32_t b_hi = base + 2 * C::A_BYTES, b_lo = b_hi + C::B_BYTES;
-#pragma unroll
-          for (int kk = 0; kk < BK / 8; ++kk) {
-            const uint32_t ao = A_MN ? kk * 1024 : kk * 32;
-            const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
-            auto da = [&](uint32_t x) { return A_MN ? desc_mn(x + ao) : desc_k(x + ao); };
-            auto db = [&](uint32_t x) { return B_MN ? desc_mn(x + bo) : desc_k(x + bo); };
-            sfdev::mma_tf32(d, da(a_lo), db(b_hi), idesc, (i | kk) != 0);
-            sfdev::mma_tf32(d, da(a_hi), db(b_lo), idesc, 1u);
-            sfdev::mma_tf32(d, da(a_hi), db(b_hi), idesc, 1u);
-          }
-          sfdev::mma_commit(&empty[s]);
-        }
-        __syncwarp();
-      }
-      if (lane == 0) sfdev::mma_commit(&acc_full[a]);
-      __syncwarp();
-    }
-  } else {
-    // epilogue warps 10-13: TMEM lane quarter (warp % 4)
-    const int q = warp & 3;
-    const int row0 = q * 32;
-    uint8_t* ebuf = epi + q * 2 * 4096;
-    int t_local = 0, nstore = 0;
-    for (int u = blockIdx.x; u < p.units; u += gridDim.x, ++t_local) {
-      int n0, m0, z, kb_begin, nkb;
-      unit_coords(u, n0, m0, z, kb_begin, nkb);
-      const int a = t_local & 1;
-      sfdev::mbar_wait(&acc_full[a], (t_local >> 1) & 1);
-      sfdev::tc_fence_after();
-#pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 32, ++nstore) {
-        uint32_t r[32];
-        sfdev::tmem_ld32(tmem + a * BN + (static_cast<uint32_t>(row0) << 16) + c0, r);
-        sfdev::tmem_ld_wait();
-        if (c0 + 32 >= BN) {  // all of this accumulator read: hand it back to the MMA warp
-          sfdev::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) sfdev::mbar_arrive(&acc_empty[a]);
-        }
-        if (p.splits == 1 && p.acc) {
-          const int row = m0 + row0 + lane;
-          if (row < p.M)
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-              if (n0 + c0 + j < p.N)
-                r[j] = __float_as_uint(__uint_as_float(r[j]) + p.C[static_cast<size_t>(row) * p.ldc + n0 + c0 + j]);
-        }
-        uint8_t* buf = ebuf + (nstore & 1) * 4096;
-        if (nstore >= 2) {
-          if (lane == 0) bulk_wait_read1();
-          __syncwarp();
-        }
-#pragma unroll
-        for (int ch = 0; ch < 8; ++ch) {
-          const uint32_t off = lane * 128 + ((ch ^ (lane & 7)) << 4);
-          *reinterpret_cast<uint4*>(buf + off) = make_uint4(r[4 * ch], r[4 * ch + 1], r[4 * ch + 2], r[4 * ch + 3]);
-        }
-        sfdev::fence_proxy_async_smem();
-        __syncwarp();
-        if (lane == 0) {
-          if (p.splits == 1) tma_store_2d(&tmC, sfdev::smem_u32(buf), n0 + c0, m0 + row0);
-          else tma_store_3d(&tmC, sfdev::smem_u32(buf), n0 + c0, m0 + row0, z);
-          bulk_commit();
-        }
-      }
-    }
-    if (lane == 0) {
-      bulk_wait_all();
-      asm volatile("fence.proxy.async.global;" ::: "memory");
-    }
-    __syncwarp();
-  }
-  sfdev::tc_fence_before();
-  __syncthreads();
-  sfdev::tc_fence_after();
-  if (warp == kMmaWarp) sfdev::tmem_dealloc<C::TMEM_COLS>(tmem);
-}
 
 // Deterministic split-K reduction: C[m][n] (+)= sum_{z} ws[z][m][n].  Block = 32 float4
 // output groups x 8 split lanes; lane zl sums z = zl, zl+8, ... (two accumulators), the 8
@@ -1120,11 +1071,13 @@ bool map3d_ws(CUtensorMap* m, const void* base, uint64_t N, uint64_t M, uint64_t
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int BN, bool AM, bool BMn, bool RAW, int BKT = BK>
+thread_local bool g_cluster_used = false;  // the last launch_tma_t reduced its split-K in-kernel
+
+template <int BN, bool AM, bool BMn, bool RAW, int BKT = BK, bool ATM = false>
 cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
                          const TParams& p, dim3 grid, cudaStream_t st) {
-  auto kern = gemm_tma_kernel<BN, AM, BMn, RAW, BKT>;
-  using TC = TCfg<BN, BKT>;
+  auto kern = gemm_tma_kernel<BN, AM, BMn, RAW, BKT, ATM>;
+  using TC = TCfg<BN, BKT, ATM>;
   static std::atomic<uint64_t> configured{0};
   int dev = 0;
   cudaGetDevice(&dev);
@@ -1135,7 +1088,49 @@ cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUten
     configured.fetch_or(bit);
   }
   const int smem = p.stages * TC::STAGE_BYTES + 1024 + 256;
+  g_cluster_used = false;
   if (p.cluster_reduce) {
+    // all tiles' clusters must be co-resident in one wave (clusters of S one-CTA-per-SM CTAs
+    // leave GPC remainders idle: 36 clusters of 4 need a second wave on 148 SMs); otherwise
+    // the workspace + reduce-kernel path runs instead
+    static std::mutex mu;
+    static std::map<std::tuple<int, int, int>, int> cap;  // (device, S, smem) -> max active clusters
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int ncl = 0;
+    {
+      std::lock_guard<std::mutex> lk(mu);
+      auto key = std::make_tuple(dev, p.splits, smem);
+      auto it = cap.find(key);
+      if (it == cap.end()) {
+        cudaLaunchConfig_t oc = {};
+        oc.gridDim = grid;
+        oc.blockDim = dim3(kThreads);
+        oc.dynamicSmemBytes = smem;
+        cudaLaunchAttribute oa[1];
+        oa[0].id = cudaLaunchAttributeClusterDimension;
+        oa[0].val.clusterDim.x = 1;
+        oa[0].val.clusterDim.y = 1;
+        oa[0].val.clusterDim.z = p.splits;
+        oc.attrs = oa;
+        oc.numAttrs = 1;
+        if (cudaOccupancyMaxActiveClusters(&ncl, kern, &oc) != cudaSuccess) {
+          cudaGetLastError();
+          ncl = 0;
+        }
+        cap[key] = ncl;
+      } else {
+        ncl = it->second;
+      }
+    }
+    if (static_cast<long>(grid.x) * grid.y > ncl) {
+      TParams q = p;
+      q.cluster_reduce = 0;
+      kern<<<grid, kThreads, smem, st>>>(a, b, c, q);
+      count_launch();
+      return cudaGetLastError();
+    }
+    g_cluster_used = true;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = grid;
     cfg.blockDim = dim3(kThreads);
@@ -1157,41 +1152,14 @@ cudaError_t launch_tma_t(const CUtensorMap& a, const CUtensorMap& b, const CUten
   return cudaGetLastError();
 }
 
-template <int BN, bool AM, bool BMn>
-cudaError_t launch_persistent_t(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c,
-                                const PParams& p, cudaStream_t st) {
-  auto kern = gemm_tma_persistent_kernel<BN, AM, BMn>;
-  static std::atomic<uint64_t> configured{0};
-  int dev = 0;
-  cudaGetDevice(&dev);
-  const uint64_t bit = 1ull << (dev & 63);
-  if (!(configured.load() & bit)) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<BN>::SMEM);
-    if (e != cudaSuccess) return e;
-    configured.fetch_or(bit);
-  }
-  const int grid = std::min(p.units, 148);
-  kern<<<grid, kPThreads, PCfg<BN>::SMEM, st>>>(a, b, c, p);
-  count_launch();
-  return cudaGetLastError();
-}
 
-template <int BN>
-cudaError_t dispatch_persistent(bool a_mn, bool b_mn, const CUtensorMap& a, const CUtensorMap& b,
-                                const CUtensorMap& c, const PParams& p, cudaStream_t st) {
-  if (a_mn && b_mn) return launch_persistent_t<BN, true, true>(a, b, c, p, st);
-  if (a_mn) return launch_persistent_t<BN, true, false>(a, b, c, p, st);
-  if (b_mn) return launch_persistent_t<BN, false, true>(a, b, c, p, st);
-  return launch_persistent_t<BN, false, false>(a, b, c, p, st);
-}
-
-template <int BN, bool RAW, int BKT = BK>
+template <int BN, bool RAW, int BKT = BK, bool ATM = false>
 cudaError_t dispatch_major(bool a_mn, bool b_mn, const CUtensorMap& a, const CUtensorMap& b,
                            const CUtensorMap& c, const TParams& p, dim3 grid, cudaStream_t st) {
-  if (a_mn && b_mn) return launch_tma_t<BN, true, true, RAW, BKT>(a, b, c, p, grid, st);
-  if (a_mn) return launch_tma_t<BN, true, false, RAW, BKT>(a, b, c, p, grid, st);
-  if (b_mn) return launch_tma_t<BN, false, true, RAW, BKT>(a, b, c, p, grid, st);
-  return launch_tma_t<BN, false, false, RAW, BKT>(a, b, c, p, grid, st);
+  if (a_mn && b_mn) return launch_tma_t<BN, true, true, RAW, BKT, ATM>(a, b, c, p, grid, st);
+  if (a_mn) return launch_tma_t<BN, true, false, RAW, BKT, ATM>(a, b, c, p, grid, st);
+  if (b_mn) return launch_tma_t<BN, false, true, RAW, BKT, ATM>(a, b, c, p, grid, st);
+  return launch_tma_t<BN, false, false, RAW, BKT, ATM>(a, b, c, p, grid, st);
 }
 
 
@@ -1376,7 +1344,17 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   static const int bk256 = std::getenv("SF_GEMM_BK256") ? std::atoi(std::getenv("SF_GEMM_BK256")) : 16;
   const int bk = bn == 256 && bk256 == 16 && splits == 1 ? 16 : 32;
   const CUtensorMapSwizzle kK = bk == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B;
-  bool ok = a_mn ? map2d(&ma, a.A, a.M, a.K, static_cast<uint64_t>(a.lda) * 4, 32, bk, kMN)
+  // A in TMEM (the default for the raw-hi kernels; SF_GEMM_ATM=0 keeps A in shared memory): an
+  // MN-major A tile is then only read by the converters, so it lands as plain SWIZZLE_128B rows
+  static const bool atm_env = !(std::getenv("SF_GEMM_ATM") && std::getenv("SF_GEMM_ATM")[0] == '0');
+  const bool atm = atm_env && raw_hi;
+  // split-K over 2..8 splits reduces inside the kernel (cluster of the tile's splits, DSMEM):
+  // no workspace round trip, no reduce launch; SF_GEMM_CLUSTER_RED=0 keeps the workspace path
+  static const bool cl_env = !(std::getenv("SF_GEMM_CLUSTER_RED") && std::getenv("SF_GEMM_CLUSTER_RED")[0] == '0');
+  const bool cl_red = cl_env && splits >= 2 && splits <= 8 && bn <= 128 && a.ldc % 4 == 0 &&
+                      reinterpret_cast<uintptr_t>(a.C) % 16 == 0;
+  bool ok = a_mn ? map2d(&ma, a.A, a.M, a.K, static_cast<uint64_t>(a.lda) * 4, 32, bk,
+                         atm ? CU_TENSOR_MAP_SWIZZLE_128B : kMN)
                  : map2d(&ma, a.A, a.K, a.M, static_cast<uint64_t>(a.lda) * 4, bk, BM, kK);
   // B: op(B) is K x N.  Stored [K][N] (MN-major) or [N][K] (TB, K-major).
   ok = ok && (b_mn ? map2d(&mb, a.B, a.N, a.K, static_cast<uint64_t>(a.ldb) * 4, 32, bk, kMN)
@@ -1390,27 +1368,25 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   // loads (tall forest GEMMs: 100352x64x148 41.9 -> 29.7 us, 25088x64x576 33.7 -> 27.6 us;
   // split-K shapes keep the deep ring).  SF_GEMM_STAGES overrides.
   static const int stages_env = std::getenv("SF_GEMM_STAGES") ? std::atoi(std::getenv("SF_GEMM_STAGES")) : -1;
-  const int max_stages = bn == 64 ? TCfg<64>::STAGES : bn == 128 ? TCfg<128>::STAGES : TCfg<256>::STAGES;
-  int stages = bk == 16 ? TCfg<256, 16>::STAGES : max_stages;
-  if (stages_env > 0) stages = std::min(stages_env, bk == 16 ? TCfg<256, 16>::STAGES : max_stages);
+  const int max_stages =
+      atm ? (bn == 64 ? TCfg<64, 32, true>::STAGES : bn == 128 ? TCfg<128, 32, true>::STAGES
+                                                                : bk == 16 ? TCfg<256, 16, true>::STAGES
+                                                                           : TCfg<256, 32, true>::STAGES)
+          : (bn == 64 ? TCfg<64>::STAGES : bn == 128 ? TCfg<128>::STAGES
+                                                     : bk == 16 ? TCfg<256, 16>::STAGES : TCfg<256>::STAGES);
+  int stages = max_stages;
+  if (stages_env > 0) stages = std::min(stages_env, max_stages);
   else if (bn == 64 && (splits == 1 ? tiles_n * tiles_m > 148 : gemm_dual64())) stages = 2;  // 2 x 97 KB fit an SM
-  // split-K over 2..8 splits reduces inside the kernel (cluster of the tile's splits, DSMEM):
-  // no workspace round trip, no reduce launch; SF_GEMM_CLUSTER_RED=0 keeps the workspace path
-  static const bool cl_env = !(std::getenv("SF_GEMM_CLUSTER_RED") && std::getenv("SF_GEMM_CLUSTER_RED")[0] == '0');
-  const bool cl_red = cl_env && splits >= 2 && splits <= 8 && a.ldc % 4 == 0 &&
-                      reinterpret_cast<uintptr_t>(a.C) % 16 == 0;
   TParams p{a.M, a.N, a.K, a.ldc, splits, bk == 16 ? (a.K + 15) / 16 : kb_per_split, a.acc ? 1 : 0, dbg, stages,
             cl_red ? 1 : 0, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;
-  // persistent CTAs (double-buffered TMEM) measured equal to per-tile CTAs on the forest
-  // shapes (profiles/r01_ncu_summary.md); opt in with SF_GEMM_PERSISTENT=1
-  static const bool persistent = std::getenv("SF_GEMM_PERSISTENT") && std::getenv("SF_GEMM_PERSISTENT")[0] == '1';
-  if (persistent && raw_hi && bn != 256) {
-    PParams pp{a.M, a.N, a.K, a.ldc, splits, kb_per_split, a.acc ? 1 : 0, tiles_n, tiles_m,
-               tiles_n * tiles_m * splits, a.C};
-    e = bn == 64 ? dispatch_persistent<64>(a_mn, b_mn, ma, mb, mc, pp, st)
-                 : dispatch_persistent<128>(a_mn, b_mn, ma, mb, mc, pp, st);
+  g_cluster_used = false;
+  if (atm) {
+    e = bn == 64    ? dispatch_major<64, true, 32, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
+        : bn == 128 ? dispatch_major<128, true, 32, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
+        : bk == 16  ? dispatch_major<256, true, 16, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
+                    : dispatch_major<256, true, 32, true>(a_mn, b_mn, ma, mb, mc, p, grid, st);
   } else if (bn == 64)
     e = raw_hi ? dispatch_major<64, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<64, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
@@ -1420,7 +1396,7 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   else
     e = raw_hi ? dispatch_major<128, true>(a_mn, b_mn, ma, mb, mc, p, grid, st)
                : dispatch_major<128, false>(a_mn, b_mn, ma, mb, mc, p, grid, st);
-  if (e != cudaSuccess || splits == 1 || cl_red) return e;
+  if (e != cudaSuccess || splits == 1 || (cl_red && g_cluster_used)) return e;
   if (a.ldc % 4 || reinterpret_cast<uintptr_t>(a.C) % 16) return cudaErrorInvalidValue;
   const uint64_t total4 = static_cast<uint64_t>(a.M) * a.N / 4;
   splitk_reduce_kernel<<<static_cast<unsigned>((total4 + 31) / 32), 256, 0, st>>>(

@@ -2212,6 +2212,20 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     Job* dep = free_for_inference() ? nullptr : steal_from();
     cudaEvent_t dep_ev = nullptr;
     bool held_now = false;
+    // a device that looks free may still run a job's subgraphs that a drain-gate hold released
+    // when the previous chain ended (the job gave the token up with them in flight): the chain
+    // is device-ordered after them as well (invariant 1)
+    Job* drain = nullptr;
+    if (!dep && excl) {
+      for (auto& jp : rt->jobs) {
+        Job* Jx = jp.get();
+        if (Jx && Jx->dev == S->id && Jx->n_inflight > 0 && Jx->last_ev) {
+          drain = Jx;
+          dep_ev = Jx->last_ev;
+          break;
+        }
+      }
+    }
     if (dep) {
       dep_ev = dep->n_inflight > 0 ? dep->last_ev : nullptr;
       // drain gate: hold the queued subgraphs (tickets >= the second in flight) so the chain
@@ -2361,7 +2375,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     ev.dev = S->id; ev.job = static_cast<int32_t>(kInferOwner | (r->id & 0xFFFFF)); ev.kind = SF_EV_INFER;
     ev.t0_ns = t0; ev.t1_ns = t1; ev.arrival_ns = r->arrival;
     ev.d0_ns = d0; ev.d1_ns = d1;
-    ev.iter = dep ? static_cast<int64_t>(dep->id) : -1;  // device-ordered after that job's dispatched subgraphs
+    ev.iter = dep ? static_cast<int64_t>(dep->id) : drain ? static_cast<int64_t>(drain->id) : -1;  // device-ordered after that job's dispatched subgraphs
     ev.k = held_now ? 1 : 0;  // drain gate: the job's queued subgraphs were held behind this request
     push_trace(rt, ev);
     if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
