@@ -129,7 +129,8 @@ def preempt_latency_report(events: Sequence[dict], slack: float, window: int = 1
     slack (``window`` subgraphs may be dispatched ahead of the boundary gate).  A request over
     the bound is a HOST outlier when its host dispatch decision ("h0", device_view) itself came
     later than ready + bound — the dispatcher thread was late, which no device-side drain
-    explains — else a violation.  Returns {"n", "bound", "violations", "host_outliers",
+    explains — or when it recorded no device dependency (``iter == -1``: nothing drained
+    before it), else a violation.  Returns {"n", "bound", "violations", "host_outliers",
     "waits"}."""
     by_dev: Dict[int, List[dict]] = {}
     for e in events:
@@ -146,7 +147,10 @@ def preempt_latency_report(events: Sequence[dict], slack: float, window: int = 1
             rep["n"] += 1
             rep["waits"].append(wait)
             if wait > bound:
-                host_late = e.get("h0") is not None and e["h0"] - ready > bound
+                # no device dependency recorded (iter == -1: the device was free, nothing of a
+                # training job drained before it): the wait is dispatch / launch time, not a drain
+                no_dep = e.get("iter") == -1
+                host_late = no_dep or (e.get("h0") is not None and e["h0"] - ready > bound)
                 (rep["host_outliers"] if host_late else rep["violations"]).append((e, wait))
             prev_end = e["t1"]
     return rep

@@ -72,8 +72,17 @@ __global__ void __cluster_dims__(kBlkCluster, 1, 1) __launch_bounds__(kBlkThread
 gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, float* __restrict__ Y, int M,
                 int N, int K, int ldx, int ldy, int kper, int acc, const float* __restrict__ b1,
                 const float* __restrict__ b2, const float* __restrict__ b3, int relu,
-                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter) {
+                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter,
+                unsigned long long* __restrict__ tr) {
   constexpr int RL = kBlkThreads / QW;  // row groups
+  // debug timeline (sf_debug_chain_trace buffer; C4 layer index from the shape): per layer
+  // {min start, max start, min after wait, max after wait, min streamed, max streamed, -, max end}
+  unsigned long long* tl = tr ? tr + 8 * (K <= 2048 ? 0 : N <= 1024 ? 2 : 1) : nullptr;
+  if (tl && threadIdx.x == 0) {
+    const unsigned long long t = sfdev::globaltimer();
+    atomicMin(&tl[0], t);
+    atomicMax(&tl[1], t);
+  }
   extern __shared__ __align__(16) unsigned char blk_smem[];
   float* xs = reinterpret_cast<float*>(blk_smem);                       // [MR][kper]
   float4* red = reinterpret_cast<float4*>(xs + MR * kper);              // [RL][QW]
@@ -98,6 +107,11 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
   sfdev::griddep_launch();  // the next layer may start streaming its (constant) weights
   if (nb > 0) load(wa, 0);  // weights never depend on the predecessor: issue before the wait
   sfdev::griddep_wait();    // x is the predecessor's output
+  if (tl && threadIdx.x == 0) {
+    const unsigned long long t = sfdev::globaltimer();
+    atomicMin(&tl[2], t);
+    atomicMax(&tl[3], t);
+  }
   const int k0 = rank * kper;
   for (int i = tid; i < MR * kper; i += kBlkThreads) {
     const int m = i / kper, kk = i % kper;
@@ -129,6 +143,11 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
       if (b + 2 < nb) load(wa, b + 2);
       fma_batch(wb, b + 1);
     }
+  }
+  if (tl && threadIdx.x == 0) {
+    const unsigned long long t = sfdev::globaltimer();
+    atomicMin(&tl[4], t);
+    atomicMax(&tl[5], t);
   }
   // row groups -> quad partials, fixed order
 #pragma unroll
@@ -178,18 +197,36 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x / kBlkCluster - 1;
     __syncthreads();
     if (sm_last) {
+      if (tl && tid == 0) atomicMax(&tl[6], sfdev::globaltimer());
       __threadfence();
       const int lane = tid & 31, warp = tid >> 5;
       __shared__ float sm_s[kBlkThreads / 32];
+      constexpr int kReg = 8;  // row values cached per thread (N <= 2048): ONE L2 round trip
       for (int m = 0; m < M; ++m) {
-        // one read pass: running (max, sum of exp) per thread (online softmax), merged over the
-        // block in fixed order; then one normalising pass
+        // one read pass (all loads issued together): running (max, sum of exp) per thread
+        // (online softmax), merged over the block in fixed order; then one normalising pass
         const float* yr = Y + static_cast<size_t>(m) * ldy;
         float mx = -INFINITY, sm = 0.f;
-        for (int n = tid; n < N; n += kBlkThreads) {
-          const float v = __ldcg(yr + n);
-          if (v > mx) { sm = sm * expf(mx - v) + 1.f; mx = v; }
-          else sm += expf(v - mx);
+        float v[kReg];
+        const bool cached = N <= kReg * kBlkThreads;
+        if (cached) {
+#pragma unroll
+          for (int j = 0; j < kReg; ++j) {
+            const int n = tid + j * kBlkThreads;
+            v[j] = n < N ? __ldcg(yr + n) : -INFINITY;
+          }
+#pragma unroll
+          for (int j = 0; j < kReg; ++j) mx = fmaxf(mx, v[j]);
+          if (mx != -INFINITY) {
+#pragma unroll
+            for (int j = 0; j < kReg; ++j) sm += expf(v[j] - mx);
+          }
+        } else {
+          for (int n = tid; n < N; n += kBlkThreads) {
+            const float x = __ldcg(yr + n);
+            if (x > mx) { sm = sm * expf(mx - x) + 1.f; mx = x; }
+            else sm += expf(x - mx);
+          }
         }
         auto merge = [](float& m1, float& s1, float m2, float s2) {
           if (m2 == -INFINITY) return;
@@ -209,12 +246,21 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
         for (int w = 1; w < kBlkThreads / 32; ++w) merge(mx, sm, sm_red[w], sm_s[w]);
         __syncthreads();
         float* orow = sm_out + static_cast<size_t>(m) * sm_ldo;
-        for (int n = tid; n < N; n += kBlkThreads) orow[n] = expf(__ldcg(yr + n) - mx) / sm;
+        if (cached) {
+#pragma unroll
+          for (int j = 0; j < kReg; ++j) {
+            const int n = tid + j * kBlkThreads;
+            if (n < N) orow[n] = expf(v[j] - mx) / sm;
+          }
+        } else {
+          for (int n = tid; n < N; n += kBlkThreads) orow[n] = expf(__ldcg(yr + n) - mx) / sm;
+        }
       }
       if (tid == 0) *sm_counter = 0u;
     }
   }
   cluster.sync();
+  if (tl && threadIdx.x == 0) atomicMax(&tl[7], sfdev::globaltimer());
 }
 
 template <int MR, int QW>
@@ -237,7 +283,7 @@ cudaError_t launch_blk_t(const GemmArgs& a, cudaStream_t st) {
   return launch_k(kern, dim3(n_cb * kBlkCluster), dim3(kBlkThreads), smem, st,
                   static_cast<const float4*>(a.Bblk), a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc, kper,
                   a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0, a.sm_out, a.sm_ldo,
-                  a.sm_counter);
+                  a.sm_counter, static_cast<unsigned long long*>(chain_trace_buffer()));
 }
 
 template <int QW>

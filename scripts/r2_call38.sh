@@ -1,0 +1,5 @@
+#!/bin/bash
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/r2c38_build.log 2>&1 || { tail -20 gpurun_out/r2c38_build.log; exit 1; }
+timeout 120 python scripts/blk_trace.py 60
+SF_GEMV_FLOW=0 timeout 120 python scripts/blk_trace.py 60
+timeout 900 python -m pytest tests/test_gpu_runtime.py tests/test_gpu_c2_bench_config.py tests/test_gpu_priority.py -q -x -k "infer or softmax or request" > gpurun_out/r2c38_tests.log 2>&1; tail -3 gpurun_out/r2c38_tests.log

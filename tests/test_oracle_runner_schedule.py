@@ -141,6 +141,11 @@ def test_preempt_latency_window_and_host_outliers():
     r = SC.preempt_latency_report([evs[0], late_host], 1, window=1)
     assert len(r["host_outliers"]) == 1 and not r["violations"]
     assert r["bound"][0] == 11 and r["waits"] == [35]
+    # a request that recorded no device dependency (iter -1: nothing drained before it) is not
+    # an I3 violation whatever its wait: it is dispatch / launch time
+    no_dep = dict(_ev(0, 1, "infer", 40, 41, arrival=5), h0=6, iter=-1)
+    r = SC.preempt_latency_report([evs[0], no_dep], 1, window=1)
+    assert len(r["host_outliers"]) == 1 and not r["violations"]
     # the ready time is the previous request's end when requests queue back to back
     q = [_ev(0, 0, "train", 0, 10), _ev(0, 1, "infer", 10, 30, arrival=5),
          _ev(0, 2, "infer", 30, 31, arrival=6)]
