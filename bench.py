@@ -255,6 +255,25 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
     return S
 
 
+def wait_or_dump(rt, req, job, timeout_s):
+    """rt.wait with a diagnostic dump (slot / job state, trace tail) to stderr when a request
+    does not complete in time; then the process ends without running destructors."""
+    try:
+        return rt.wait(req, timeout_s)
+    except Exception as ex:  # noqa: BLE001 (diagnostics, then exit)
+        import traceback
+        print(f"request {req} did not complete: {ex}", file=sys.stderr)
+        try:
+            print("slot 0", rt.slot_info(0), file=sys.stderr)
+            print("job", rt.job_info(job), file=sys.stderr)
+            for e in rt.trace()[-12:]:
+                print("trace", e, file=sys.stderr)
+        except Exception:  # noqa: BLE001
+            traceback.print_exc()
+        sys.stderr.flush()
+        os._exit(3)
+
+
 def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool, exclusive=True,
                     iteration_granularity=False, measure=True, defer=None, duplex=None,
             early=None, target=HOST, gate=None):
@@ -333,7 +352,7 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
                     last = key
         j = i % len(xs)
         reqs.append(rt.submit(ghi, 0, x_t[j].data_ptr(), out_t[j].data_ptr(), arrival_ns=int(arr[i])))
-    tms = [rt.wait(r, 120) for r in reqs]
+    tms = [wait_or_dump(rt, r, job, 120) for r in reqs]
     ji1 = rt.job_info(job)
     ev1 = torch.cuda.Event(enable_timing=True)
     ev1.record()
@@ -813,6 +832,7 @@ def main():
     args = ap.parse_args()
     if os.environ.get("SF_BENCH_WATCHDOG_S"):  # debugging aid: dump every thread's stack, then exit
         import faulthandler
+        faulthandler.enable()  # a fatal signal also dumps every thread's Python stack
         faulthandler.dump_traceback_later(float(os.environ["SF_BENCH_WATCHDOG_S"]), exit=True)
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))

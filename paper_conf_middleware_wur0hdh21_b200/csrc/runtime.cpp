@@ -183,6 +183,10 @@ struct Slot {
     uint64_t g_ns;     // GPU time (%globaltimer ns) of the anchor event
     int64_t offset_ns; // host = GPU + offset (stamp value seen at host time ~h1 - 1 us)
     uint64_t unc_ns;   // half that window
+    // position on the slot's DEVICE timeline: chained exactly through the event timer,
+    // D_i = D_{i-1} + elapsed(anchor_{i-1}, anchor_i) (D_0 = g_0), so device times taken
+    // against different anchors are mutually consistent (their order is the GPU's order)
+    double D = 0.0;
   };
   cudaStream_t s_clk = nullptr;
   unsigned long long* clk_host = nullptr;  // pinned, mapped
@@ -303,6 +307,7 @@ struct sf_runtime {
   bool shutting_down = false;
   std::atomic<bool> stop_spin{false};
   std::vector<sf_trace_event> trace;
+  std::vector<std::pair<double, double>> trace_D;  // per trace event: device-timeline d0, d1 (NaN: none)
   std::thread clk;  // refreshes every local slot's device clock anchor (Slot::Anchor)
   size_t trace_cap = 1 << 16;
   size_t trace_dropped = 0;
@@ -310,9 +315,14 @@ struct sf_runtime {
 
 namespace {
 
-void push_trace(sf_runtime* rt, const sf_trace_event& e) {  // rt->m held
-  if (rt->trace.size() < rt->trace_cap) rt->trace.push_back(e);
-  else ++rt->trace_dropped;
+void push_trace(sf_runtime* rt, const sf_trace_event& e, double D0 = std::nan(""),
+                double D1 = std::nan("")) {  // rt->m held
+  if (rt->trace.size() < rt->trace_cap) {
+    rt->trace.push_back(e);
+    rt->trace_D.emplace_back(D0, D1);
+  } else {
+    ++rt->trace_dropped;
+  }
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1127,6 +1137,14 @@ cudaError_t refresh_anchor(Slot& S) {
   }
   if (!best.ev) return cudaSuccess;
   std::lock_guard<std::mutex> lk(S.clk_m);
+  best.D = static_cast<double>(best.g_ns);
+  if (!S.anchors.empty()) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, S.anchors.back().ev, best.ev) == cudaSuccess && ms >= 0.f)
+      best.D = S.anchors.back().D + static_cast<double>(ms) * 1e6;
+    else
+      cudaGetLastError();
+  }
   S.anchors.push_back(best);
   while (S.anchors.size() > 256) {
     cudaEventDestroy(S.anchors.front().ev);
@@ -1168,6 +1186,46 @@ uint64_t event_host_ns(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
     (void)after;
   }
   return static_cast<uint64_t>(dev_ns + off);
+}
+
+// Device-timeline position D of a completed timing event (see Slot::Anchor::D), by the latest
+// anchor enqueued at least 100 us before it; NaN if unavailable.
+double event_dev_D(Slot& S, cudaEvent_t ev, uint64_t enq_ns) {
+  std::lock_guard<std::mutex> lk(S.clk_m);
+  const Slot::Anchor* a = nullptr;
+  for (auto it = S.anchors.rbegin(); it != S.anchors.rend(); ++it)
+    if (it->enq_ns + 100000 <= enq_ns) { a = &*it; break; }
+  if (!a) return std::nan("");
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, a->ev, ev) != cudaSuccess) {
+    cudaGetLastError();
+    return std::nan("");
+  }
+  return a->D + static_cast<double>(ms) * 1e6;
+}
+
+// CLOCK_MONOTONIC ns of device-timeline position D with the slot's CURRENT anchors: the
+// offset host - D, known at every anchor, is interpolated linearly in D between the anchors
+// around it (held at the ends).  One mapping for all trace events read together, so it is
+// monotone in D: the device order of events survives into the trace.
+uint64_t dev_D_to_host(Slot& S, double D) {
+  std::lock_guard<std::mutex> lk(S.clk_m);
+  if (S.anchors.empty() || std::isnan(D)) return 0;
+  auto off = [](const Slot::Anchor& a) {
+    return static_cast<double>(a.g_ns) + static_cast<double>(a.offset_ns) - a.D;
+  };
+  const auto& A = S.anchors;
+  size_t hi = 0;
+  while (hi < A.size() && A[hi].D <= D) ++hi;
+  double o;
+  if (hi == 0) o = off(A.front());
+  else if (hi == A.size()) o = off(A.back());
+  else {
+    const Slot::Anchor &a = A[hi - 1], &b = A[hi];
+    const double w = b.D > a.D ? (D - a.D) / (b.D - a.D) : 0.0;
+    o = off(a) + w * (off(b) - off(a));
+  }
+  return static_cast<uint64_t>(D + o);
 }
 
 void clock_main(sf_runtime* rt);
@@ -2090,9 +2148,12 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     if (f.stamp && !t_res) t_res = t1;
     // device execution interval on the host clock (0 when no anchor covers it)
     uint64_t d0 = 0, d1 = 0;
+    double D0 = std::nan(""), D1 = std::nan("");
     if (e == cudaSuccess) {
       d0 = event_host_ns(S, J.ev_start[f.dev * kMaxInflight + f.ev], f.t0);
       d1 = event_host_ns(S, J.ev_ring[f.dev * kMaxInflight + f.ev], f.t0);
+      D0 = event_dev_D(S, J.ev_start[f.dev * kMaxInflight + f.ev], f.t0);
+      D1 = event_dev_D(S, J.ev_ring[f.dev * kMaxInflight + f.ev], f.t0);
       if (f.stamp) {  // the resume point as the GPU saw it
         const uint64_t r = event_host_ns(S, J.ev_r[f.dev], f.t0);
         if (r) t_res = r;
@@ -2143,7 +2204,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     tev.arrival_ns = f.t0;  // train events: host dispatch (launch) time
     last_t1 = t1;
     front_start = q.empty() ? 0 : std::max(q.front().t0, t1);
-    push_trace(rt, tev);
+    push_trace(rt, tev, D0, D1);
     // iteration-granularity (session time slicing baseline) keeps the device for the whole
     // iteration; otherwise an empty window is a scheduling point
     if (q.empty() && (!rt->cfg.iteration_granularity || J.k == 0)) release();
@@ -2214,9 +2275,12 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     bool held_now = false;
     // a device that looks free may still run a job's subgraphs that a drain-gate hold released
     // when the previous chain ended (the job gave the token up with them in flight): the chain
-    // is device-ordered after them as well (invariant 1)
+    // is device-ordered after them as well (invariant 1).  While the gate still holds them
+    // (requests queued back to back) they cannot start before it opens after this queue drains,
+    // and the running one was waited for by the request that took the hold: no wait (waiting
+    // on a held subgraph would deadlock the queue)
     Job* drain = nullptr;
-    if (!dep && excl) {
+    if (!dep && excl && !S->gate_held) {
       for (auto& jp : rt->jobs) {
         Job* Jx = jp.get();
         if (Jx && Jx->dev == S->id && Jx->n_inflight > 0 && Jx->last_ev) {
@@ -2354,9 +2418,12 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       cudaGetLastError();
     }
     uint64_t d0 = 0, d1 = 0;
+    double iD0 = std::nan(""), iD1 = std::nan("");
     if (e == cudaSuccess) {
       d0 = event_host_ns(*S, S->ev_i0, tl0);
       d1 = event_host_ns(*S, S->ev_infer, tl0);
+      iD0 = event_dev_D(*S, S->ev_i0, tl0);
+      iD1 = event_dev_D(*S, S->ev_infer, tl0);
     }
     lk.lock();
     // start = the request chain's start on the GPU (device clock); without an anchor: an
@@ -2377,7 +2444,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     ev.d0_ns = d0; ev.d1_ns = d1;
     ev.iter = dep ? static_cast<int64_t>(dep->id) : drain ? static_cast<int64_t>(drain->id) : -1;  // device-ordered after that job's dispatched subgraphs
     ev.k = held_now ? 1 : 0;  // drain gate: the job's queued subgraphs were held behind this request
-    push_trace(rt, ev);
+    push_trace(rt, ev, iD0, iD1);
     if (rt->cfg.exclusive_gpu && S->q.empty()) S->owner = -1;
     if (S->gate_held && S->q.empty()) gate_open(*S);  // the held subgraphs run now
     rt->cv.notify_all();
@@ -3237,7 +3304,22 @@ sf_status sf_get_trace(sf_runtime* rt, sf_trace_event* buf, size_t cap, size_t* 
   if (!rt) return fail(SF_EINVAL, "null runtime");
   std::lock_guard<std::mutex> lk(rt->m);
   const size_t n = std::min(cap, rt->trace.size());
-  if (buf) std::copy(rt->trace.begin(), rt->trace.begin() + n, buf);
+  if (buf) {
+    std::copy(rt->trace.begin(), rt->trace.begin() + n, buf);
+    // device intervals through ONE mapping (the slot's anchors as of now) for every event read
+    // together: their order is the GPU's order (reading Q37); events without a device-timeline
+    // position keep the value mapped at completion
+    for (size_t i = 0; i < n && i < rt->trace_D.size(); ++i) {
+      sf_trace_event& e = buf[i];
+      if (e.kind != SF_EV_TRAIN && e.kind != SF_EV_INFER) continue;
+      if (e.dev < 0 || static_cast<size_t>(e.dev) >= rt->slots.size() || !rt->slots[e.dev]) continue;
+      Slot& S = *rt->slots[e.dev];
+      const auto [D0, D1] = rt->trace_D[i];
+      if (std::isnan(D0) || std::isnan(D1)) continue;
+      const uint64_t m0 = dev_D_to_host(S, D0), m1 = dev_D_to_host(S, D1);
+      if (m0 && m1) { e.d0_ns = m0; e.d1_ns = m1; }
+    }
+  }
   if (n_out) *n_out = buf ? n : rt->trace.size();
   return SF_OK;
 }
