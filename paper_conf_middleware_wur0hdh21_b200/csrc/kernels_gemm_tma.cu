@@ -63,6 +63,7 @@ struct TParams {
   int M, N, K, ldc;
   int splits, kb_per_split, acc, dbg, stages;
   int cluster_reduce;  // 1: the splits of a tile form one cluster (1, 1, splits) and reduce over DSMEM
+  int merge;           // 128x64 tiles with A in TMEM: merged A_hi.[B_hi | B_lo] MMA (see MERGE)
   float* C;
   float* ws;
   unsigned* counters;
@@ -228,12 +229,20 @@ __device__ __forceinline__ void cluster_push_reduce(uint8_t* smem, uint64_t* red
   }
 }
 
+// 128x64 tiles run two CTAs per SM when the grid has more tiles than SMs (2-stage ring): the
+// register budget must leave room for both (<= 96 per thread at 320 threads)
 template <int BN, bool A_MN, bool B_MN, bool RAW_HI, int BKT = BK, bool ATM = false>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreads, BN == 64 ? 2 : 1)
 gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, TParams p) {
   using C = TCfg<BN, BKT, ATM>;
   constexpr int BK = BKT;  // k-block depth of this instantiation
+  // MERGE (128x64 tiles, A in TMEM): A_hi.B_hi and A_hi.B_lo in ONE N=128 MMA over the adjacent
+  // B_hi | B_lo stage buffers into two 64-column accumulators (+ A_lo.B_hi into the first),
+  // summed in the epilogue: 2 MMAs per K step instead of 3 (an N=64 tf32 MMA costs nearly
+  // as much as an N=128 one in this loop)
+  const bool MERGE = ATM && BN == 64 && p.merge;
+  const int ACC = MERGE ? 2 * BN : BN;  // accumulator TMEM columns
   const int NS = p.stages;  // ring depth (<= C::STAGES; 2 for short K: two CTAs per SM)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -267,7 +276,7 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   }
   // ATM: accumulator in columns [0, BN), stage s's A hi / lo at BN + 2 s BK (+ BK); a 2-stage
   // ring (two CTAs per SM) fits 256 columns, deeper rings take all 512
-  const bool tm_small = !ATM || BN + NS * 2 * BK <= 256;
+  const bool tm_small = !ATM || ACC + NS * 2 * BK <= 256;
   if (warp == kMmaWarp) {
     if (!ATM) sfdev::tmem_alloc<C::TMEM_COLS>(tmem_slot);
     else if (tm_small) sfdev::tmem_alloc<256>(tmem_slot);
@@ -345,14 +354,14 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         float lo[KH];
 #pragma unroll
         for (int j = 0; j < KH; ++j) lo[j] = tf32_trunc(x[j] - tf32_trunc(x[j]));
-        const uint32_t col = static_cast<uint32_t>(BN + s * 2 * BK + h * KH);
+        const uint32_t col = static_cast<uint32_t>(ACC + s * 2 * BK + h * KH);
         tmem_st<KH>(tmem + lane_base + col, x);
         tmem_st<KH>(tmem + lane_base + col + BK, lo);
         float4* b = reinterpret_cast<float4*>(st + C::A_BYTES);
         float4* blo = reinterpret_cast<float4*>(st + C::A_BYTES + C::B_BYTES);
         split_tile<C::B_BYTES / 16 / 256, true>(b, blo, t);
       } else {
-        tmem_st<KH>(tmem + lane_base + static_cast<uint32_t>(BN + s * 2 * BK + h * KH), x);
+        tmem_st<KH>(tmem + lane_base + static_cast<uint32_t>(ACC + s * 2 * BK + h * KH), x);
       }
       asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
       sfdev::fence_proxy_async_smem();
@@ -390,11 +399,17 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       sfdev::tc_fence_after();
       if (ATM && lane == 0) {
         const uint32_t b_hi = sfdev::smem_u32(smem + s * C::STAGE_BYTES) + C::A_BYTES, b_lo = b_hi + C::B_BYTES;
-        const uint32_t a_hi = tmem + static_cast<uint32_t>(BN + s * 2 * BK), a_lo = a_hi + BK;
+        const uint32_t a_hi = tmem + static_cast<uint32_t>(ACC + s * 2 * BK), a_lo = a_hi + BK;
 #pragma unroll
         for (int kk = 0; kk < BK / 8; ++kk) {
           const uint32_t bo = B_MN ? kk * 1024 : kk * 32;
           auto db = [&](uint32_t x) { return B_MN ? desc_mn<BK>(x + bo) : desc_k<BK>(x + bo); };
+          if (MERGE) {
+            constexpr uint32_t idesc2 = (idesc & ~(0x3Fu << 17)) | (uint32_t((2 * BN) >> 3) << 17);
+            mma_tf32_ts(tmem, a_hi + kk * 8, db(b_hi), idesc2, (i | kk) != 0);  // [B_hi | B_lo]
+            mma_tf32_ts(tmem, a_lo + kk * 8, db(b_hi), idesc, 1u);
+            continue;
+          }
           if (!(p.dbg & 4)) {
             mma_tf32_ts(tmem, a_lo + kk * 8, db(b_hi), idesc, (i | kk) != 0);
             mma_tf32_ts(tmem, a_hi + kk * 8, db(b_lo), idesc, 1u);
@@ -439,6 +454,13 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       uint32_t r[32];
       sfdev::tmem_ld32(tmem + (static_cast<uint32_t>(row0) << 16) + c0, r);
       sfdev::tmem_ld_wait();
+      if (MERGE) {  // + the A_hi.B_lo half
+        uint32_t r2[32];
+        sfdev::tmem_ld32(tmem + (static_cast<uint32_t>(row0) << 16) + BN + c0, r2);
+        sfdev::tmem_ld_wait();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) r[j] = __float_as_uint(__uint_as_float(r[j]) + __uint_as_float(r2[j]));
+      }
       if (nkb == 0) {
 #pragma unroll
         for (int j = 0; j < 32; ++j) r[j] = 0u;
@@ -1377,8 +1399,12 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   int stages = max_stages;
   if (stages_env > 0) stages = std::min(stages_env, max_stages);
   else if (bn == 64 && (splits == 1 ? tiles_n * tiles_m > 148 : gemm_dual64())) stages = 2;  // 2 x 97 KB fit an SM
+  // merged MMAs for 128x64 tiles (SF_GEMM_MERGE=0 disables): forest dW 576x64x25088 33.1 ->
+  // 26.9 us (one CTA per SM), forward 25088x64x576 24.9 -> 22.9 us (two per SM)
+  static const bool merge_env = !(std::getenv("SF_GEMM_MERGE") && std::getenv("SF_GEMM_MERGE")[0] == '0');
+  const bool merge = atm && bn == 64 && merge_env;
   TParams p{a.M, a.N, a.K, a.ldc, splits, bk == 16 ? (a.K + 15) / 16 : kb_per_split, a.acc ? 1 : 0, dbg, stages,
-            cl_red ? 1 : 0, a.C, a.ws, a.counters};
+            cl_red ? 1 : 0, merge ? 1 : 0, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);
   cudaError_t e;
   g_cluster_used = false;

@@ -20,7 +20,8 @@ with Runtime([0], max_inflight=1) as rt:
     ranges = [gh.subgraph_range(k) for k in range(gh.n_subgraphs)]
 d = {}
 for e in tr:
-    d.setdefault(e["k"], []).append((e["t1"] - e["t0"]) * 1e-3)
+    t0, t1 = (e["d0"], e["d1"]) if e.get("d0") and e.get("d1") else (e["t0"], e["t1"])  # device interval
+    d.setdefault(e["k"], []).append((t1 - t0) * 1e-3)
 rows = sorted(((float(np.median(v)), k) for k, v in d.items()), reverse=True)
 tot = sum(m for m, _ in rows)
 print(json.dumps({"n_subgraphs": len(rows), "iteration_us_sum_of_medians": round(tot, 1),
