@@ -565,7 +565,9 @@ sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id g, int32_t dev);
  * inference runs, -1 free; requests queued; drain-gate words). */
 typedef struct sf_slot_info {
   int32_t owner, queued, gate_held, pad;
-  uint32_t gate_value, gate_arrived, next_ticket, pad2;
+  uint32_t gate_value, gate_arrived, next_ticket;
+  uint32_t gate_valve; /* holds the dispatcher released after a chain waited 5 ms behind its own
+                          hold (streams sharing a hardware queue with the held training stream) */
 } sf_slot_info;
 sf_status sf_slot_query(sf_runtime* rt, int32_t slot, sf_slot_info* out);
 /* Diagnostics: the kernel path of the last GEMM the CALLING THREAD launched (sf_op_gemm,

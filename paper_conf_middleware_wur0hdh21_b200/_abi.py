@@ -133,7 +133,7 @@ class sf_migration_probe(C.Structure):
 class sf_slot_info(C.Structure):
     _fields_ = [("owner", C.c_int32), ("queued", C.c_int32), ("gate_held", C.c_int32), ("pad", C.c_int32),
                 ("gate_value", C.c_uint32), ("gate_arrived", C.c_uint32), ("next_ticket", C.c_uint32),
-                ("pad2", C.c_uint32)]
+                ("gate_valve", C.c_uint32)]
 
 
 class sf_copy_desc(C.Structure):

@@ -63,7 +63,7 @@ struct TParams {
   int M, N, K, ldc;
   int splits, kb_per_split, acc, dbg, stages;
   int cluster_reduce;  // 1: the splits of a tile form one cluster (1, 1, splits) and reduce over DSMEM
-  int merge;           // 128x64 tiles with A in TMEM: merged A_hi.[B_hi | B_lo] MMA (see MERGE)
+  int merge;           // 128x64 / 128x128 tiles with A in TMEM: merged A_hi.[B_hi | B_lo] MMA (MERGE)
   float* C;
   float* ws;
   unsigned* counters;
@@ -237,11 +237,11 @@ gemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
                 const __grid_constant__ CUtensorMap tmC, TParams p) {
   using C = TCfg<BN, BKT, ATM>;
   constexpr int BK = BKT;  // k-block depth of this instantiation
-  // MERGE (128x64 tiles, A in TMEM): A_hi.B_hi and A_hi.B_lo in ONE N=128 MMA over the adjacent
-  // B_hi | B_lo stage buffers into two 64-column accumulators (+ A_lo.B_hi into the first),
-  // summed in the epilogue: 2 MMAs per K step instead of 3 (an N=64 tf32 MMA costs nearly
-  // as much as an N=128 one in this loop)
-  const bool MERGE = ATM && BN == 64 && p.merge;
+  // MERGE (128x64 / 128x128 tiles, A in TMEM): A_hi.B_hi and A_hi.B_lo in ONE N=2BN MMA over
+  // the adjacent B_hi | B_lo stage buffers into two BN-column accumulators (+ A_lo.B_hi into
+  // the first), summed in the epilogue: 2 MMAs per K step instead of 3 (an MMA instruction
+  // costs more than its N x 8 x 128 share of the tensor pipe in this loop)
+  const bool MERGE = ATM && BN <= 128 && p.merge;
   const int ACC = MERGE ? 2 * BN : BN;  // accumulator TMEM columns
   const int NS = p.stages;  // ring depth (<= C::STAGES; 2 for short K: two CTAs per SM)
   extern __shared__ uint8_t smem_raw[];
@@ -1399,10 +1399,12 @@ cudaError_t launch_gemm_tma(const GemmArgs& a, int bn, int splits, int kb_per_sp
   int stages = max_stages;
   if (stages_env > 0) stages = std::min(stages_env, max_stages);
   else if (bn == 64 && (splits == 1 ? tiles_n * tiles_m > 148 : gemm_dual64())) stages = 2;  // 2 x 97 KB fit an SM
-  // merged MMAs for 128x64 tiles (SF_GEMM_MERGE=0 disables): forest dW 576x64x25088 33.1 ->
-  // 26.9 us (one CTA per SM), forward 25088x64x576 24.9 -> 22.9 us (two per SM)
+  // merged MMAs for 128x64 / 128x128 tiles (SF_GEMM_MERGE=0 disables): forest dW
+  // 576x64x25088 33.1 -> 26.9 us, forward 25088x64x576 24.9 -> 22.9 us; C3 FFN forward
+  // 512x4096x1024 35.6 -> 28.0 us, C3 iteration 67.8 -> 73.2 TFLOP/s
   static const bool merge_env = !(std::getenv("SF_GEMM_MERGE") && std::getenv("SF_GEMM_MERGE")[0] == '0');
-  const bool merge = atm && bn == 64 && merge_env;
+  static const int merge_max = std::getenv("SF_GEMM_MERGE_BN") ? std::atoi(std::getenv("SF_GEMM_MERGE_BN")) : 128;
+  const bool merge = atm && bn <= merge_max && merge_env;
   TParams p{a.M, a.N, a.K, a.ldc, splits, bk == 16 ? (a.K + 15) / 16 : kb_per_split, a.acc ? 1 : 0, dbg, stages,
             cl_red ? 1 : 0, merge ? 1 : 0, a.C, a.ws, a.counters};
   dim3 grid(tiles_n, tiles_m, splits);

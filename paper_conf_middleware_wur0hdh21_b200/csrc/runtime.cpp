@@ -201,6 +201,7 @@ struct Slot {
   CUdeviceptr gate_G = 0, gate_A = 0;
   uint32_t next_ticket = 1;  // per-slot launch tickets (rt->m)
   bool gate_held = false;
+  uint64_t gate_valve = 0;  // holds released by the dispatcher's 5 ms safety valve (diagnostics)
   std::atomic<int> owner{-1};  // device token (atomic: the spinning dispatcher polls it)
   size_t l2_setaside = 0, l2_max_window = 0;  // persisting L2 for inference weights
   std::deque<Request*> q;
@@ -2410,7 +2411,28 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     const uint64_t tl1 = now_ns();
     sfk::set_pdl(false);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_infer, S->s_infer);
-    if (e == cudaSuccess) e = spin_event(S->ev_infer);
+    if (e == cudaSuccess && S->gate) {
+      // safety valve: streams beyond the device's hardware work queues share a queue, and a
+      // held gate wait on the training stream would then also hold a chain queued behind it
+      // on the same connection.  A chain not done 5 ms after its launch (~50 us normally)
+      // releases the hold; the held subgraph then runs first on that shared queue.
+      const uint64_t valve = now_ns() + 5000000;
+      for (;;) {
+        e = cudaEventQuery(S->ev_infer);
+        if (e != cudaErrorNotReady) break;
+        if (now_ns() > valve) {
+          std::lock_guard<std::mutex> vk(rt->m);
+          if (S->gate_held) {
+            gate_open(*S);
+            ++S->gate_valve;
+          }
+          e = spin_event(S->ev_infer);
+          break;
+        }
+      }
+    } else if (e == cudaSuccess) {
+      e = spin_event(S->ev_infer);
+    }
     const uint64_t t1 = now_ns();
     float dev_ms = -1.f;
     if (e == cudaSuccess && cudaEventElapsedTime(&dev_ms, S->ev_i0, S->ev_infer) != cudaSuccess) {
@@ -3549,6 +3571,7 @@ sf_status sf_slot_query(sf_runtime* rt, int32_t slot, sf_slot_info* out) {
   out->gate_value = S.gate ? S.gate[0] : 0;
   out->gate_arrived = S.gate ? S.gate[16] : 0;
   out->next_ticket = S.next_ticket;
+  out->gate_valve = static_cast<uint32_t>(S.gate_valve);
   return SF_OK;
 }
 

@@ -271,7 +271,7 @@ def test_inference_vs_oracle_and_auto_preemption_invariants(P, W, early, gate):
     if gate:  # the queued subgraph was held behind (most) requests: only the running one drains
         held = sum(e["kind"] == "infer" and e["k"] == 1 for e in evs)
         print("drain gate held", held, "of", sum(e["kind"] == "infer" for e in evs))
-        assert held >= 2  # the hold path ran (how often depends on where arrivals land)
+        assert held >= 1  # the hold path ran (how often depends on where arrivals land)
     check_i3_device(dv, 1 if gate else W, early)
 
 
