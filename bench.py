@@ -144,7 +144,8 @@ def run_arm(args, local_dev: int, steps: int, warmup: int, host_io: bool, exclus
                  inflight_budget_us=args.inflight_budget_us,
                  host_duplex=bool(args.duplex if duplex is None else duplex),
                  early_launch=bool(args.early if early is None else early),
-                 drain_gate=bool(args.gate if gate is None else gate))
+                 drain_gate=bool(args.gate if gate is None else gate),
+                 infer_l2_persist_bytes=int(args.l2_persist_mb * (1 << 20)))
     gh = rt.register(g)
     info = gh.partition("max_ops" if args.max_ops else "phase", args.max_ops,
                         update_chunks=args.update_chunks)
@@ -296,7 +297,8 @@ def run_poisson_arm(args, local_dev: int, n_req: int, warmup: int, host_io: bool
                  inflight_budget_us=args.inflight_budget_us,
                  host_duplex=bool(args.duplex if duplex is None else duplex),
                  early_launch=bool(args.early if early is None else early),
-                 drain_gate=bool(args.gate if gate is None else gate))
+                 drain_gate=bool(args.gate if gate is None else gate),
+                 infer_l2_persist_bytes=int(args.l2_persist_mb * (1 << 20)))
     gh = rt.register(g)
     gh.partition("max_ops" if args.max_ops else "phase", args.max_ops, update_chunks=args.update_chunks)
     gh.bind(0, staging=True, host_staging=True)
@@ -823,6 +825,8 @@ def main():
     ap.add_argument("--duplex", type=int, default=1,
                     help="1: full-duplex host round trip when nothing waits for the device "
                          "(default); 0: D2H, then H2D")
+    ap.add_argument("--l2-persist-mb", type=float, default=0.0,
+                    help="persisting L2 set-aside for the inference weights, MB (0: none)")
     ap.add_argument("--gate", type=int, default=1,
                     help="1: drain gate (a preempting request runs before the job's queued "
                          "subgraph, default); 0: it waits for every dispatched subgraph")
@@ -969,7 +973,7 @@ def main():
                    "dispatch_spin_us": args.dispatch_spin_us,
                    "inflight_budget_us": args.inflight_budget_us,
                    "early_launch": bool(args.early), "host_duplex": bool(args.duplex),
-                   "drain_gate": bool(args.gate),
+                   "drain_gate": bool(args.gate), "l2_persist_mb": args.l2_persist_mb,
                    "migration_policy": "deferred until the preempter drained" if args.defer
                    else "concurrent with the preempter",
                    "l2": "state 205 MB + datasets 666 MB > 126 MB L2 (no flush needed); the pack "

@@ -40,6 +40,14 @@ __device__ __forceinline__ float4 ldg_stream(const float4* p) {
                : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
   return v;
 }
+// with an L2 cache policy (createpolicy): evict_last keeps the block in the persisting L2
+// set-aside across requests (infer_l2_persist_bytes), evict_first streams it past
+__device__ __forceinline__ float4 ldg_stream_hint(const float4* p, uint64_t pol) {
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
+  return v;
+}
 
 // Wb[(cb * 8 + r) * kper * QW + row * QW + q] = W[(r * kper + row)][4 (cb QW + q) .. + 3]
 __global__ void gemv_block_layout_kernel(const float* __restrict__ W, float4* __restrict__ Wb, int K, int N,
@@ -72,7 +80,7 @@ __global__ void __cluster_dims__(kBlkCluster, 1, 1) __launch_bounds__(kBlkThread
 gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, float* __restrict__ Y, int M,
                 int N, int K, int ldx, int ldy, int kper, int acc, const float* __restrict__ b1,
                 const float* __restrict__ b2, const float* __restrict__ b3, int relu,
-                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter,
+                float* __restrict__ sm_out, int sm_ldo, unsigned* __restrict__ sm_counter, int l2h,
                 unsigned long long* __restrict__ tr) {
   constexpr int RL = kBlkThreads / QW;  // row groups
   // debug timeline (sf_debug_chain_trace buffer; C4 layer index from the shape): per layer
@@ -97,11 +105,13 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
   const int nrow = kper / RL;  // rows of this thread (kper is a multiple of RL)
   const int nb = (nrow + kBlkBatch - 1) / kBlkBatch;
   float4 wa[kBlkBatch], wb[kBlkBatch];
+  const uint64_t pol = l2h ? sfdev::l2_policy(l2h) : 0ull;
   auto load = [&](float4 (&w)[kBlkBatch], int b) {
 #pragma unroll
     for (int u = 0; u < kBlkBatch; ++u) {
       const int j = b * kBlkBatch + u;
-      w[u] = j < nrow ? ldg_stream(blk + static_cast<size_t>(rg + RL * j) * QW) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float4* a = blk + static_cast<size_t>(rg + RL * j) * QW;
+      w[u] = j >= nrow ? make_float4(0.f, 0.f, 0.f, 0.f) : l2h ? ldg_stream_hint(a, pol) : ldg_stream(a);
     }
   };
   sfdev::griddep_launch();  // the next layer may start streaming its (constant) weights
@@ -283,7 +293,7 @@ cudaError_t launch_blk_t(const GemmArgs& a, cudaStream_t st) {
   return launch_k(kern, dim3(n_cb * kBlkCluster), dim3(kBlkThreads), smem, st,
                   static_cast<const float4*>(a.Bblk), a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc, kper,
                   a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0, a.sm_out, a.sm_ldo,
-                  a.sm_counter, static_cast<unsigned long long*>(chain_trace_buffer()));
+                  a.sm_counter, a.l2_hint, static_cast<unsigned long long*>(chain_trace_buffer()));
 }
 
 template <int QW>
