@@ -134,8 +134,8 @@ typedef uint64_t sf_req_id;
 
 /* Migration engine. */
 #define SF_MIG_SM 0 /* descriptor-walk kernels: pack / unpack / fused peer store (default) */
-#define SF_MIG_CE 1 /* copy engines only, zero SM work: one cudaMemcpyBatchAsync per ~2 MB of
-                       live tensors, arena -> pinned staging payloads (the CPU writes header and
+#define SF_MIG_CE 1 /* copy engines only, zero SM work: cudaMemcpyAsync per segment in ~2 MB
+                       groups (large tensors split), arena -> pinned staging payloads (the CPU writes header and
                        zero padding: same staging bytes as a pack), staging -> arena, or
                        arena -> peer arena; host_mode is ignored */
 
@@ -600,7 +600,7 @@ sf_status sf_probe_migration(sf_runtime* rt, sf_graph_id g, int32_t dev, int32_t
  * src into slot dst's arena (a local slot of another device, or a REMOTE slot mapped with
  * sf_import_arena) once, on src's migration stream, and return the duration.  engine:
  *   0 the peer-store descriptor walk (the product path; kernel-only %globaltimer time),
- *   1 copy engines, one cudaMemcpyBatchAsync per ~2 MB of tensors,
+ *   1 copy engines, cudaMemcpyAsync per segment in ~2 MB groups (large tensors split),
  *   2 copy engines, one cudaMemcpyAsync per tensor (per-tensor cudaMemcpyPeerAsync),
  *   3 copy engines, ONE cudaMemcpyAsync of the arena span the live tensors cover;
  * CE times are CUDA events around the copies.  Blocks until done.  *bytes_moved = live bytes

@@ -1310,8 +1310,8 @@ cudaError_t poison(Binding& b, cudaStream_t st) {
 
 
 // Copy-engine transfers.  A segment list is issued in ~2 MB batches (large segments split),
-// one cudaMemcpyBatchAsync per batch (per-segment cudaMemcpyAsync where the batch API is
-// unavailable), so no SM runs for the copy.  With `yield`, at most two batches are in flight
+// one cudaMemcpyAsync per segment (the batched copy API is closed on this GPU pool: it raised
+// Xid faults), so no SM runs for the copy.  With `yield`, at most two batches are in flight
 // and none is issued while a request is queued or running on the slot: copy-engine traffic
 // over PCIe slows a concurrent batch-1 forward by ~45% on B200 (scripts/infer_bench.py
 // COPY=d2h: 50 -> 74 us; reading Q22).  Returns once every batch has been issued and (yield)
@@ -1324,18 +1324,6 @@ struct Seg {
 
 cudaError_t issue_batch(std::vector<void*>& d, std::vector<void*>& s, std::vector<size_t>& n,
                         cudaStream_t st) {
-  static std::atomic<bool> batch_ok{!(std::getenv("SF_CE_NOBATCH") && std::getenv("SF_CE_NOBATCH")[0] == '1')};
-  if (d.size() > 1 && batch_ok.load(std::memory_order_relaxed)) {
-    cudaMemcpyAttributes attr{};
-    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-    size_t idx = 0, fail_idx = 0;
-    const cudaError_t e =
-        cudaMemcpyBatchAsync(d.data(), s.data(), n.data(), d.size(), &attr, &idx, 1, &fail_idx, st);
-    if (e == cudaSuccess) return e;
-    if (e != cudaErrorNotSupported && e != cudaErrorInvalidValue) return e;
-    cudaGetLastError();
-    batch_ok = false;  // fall back to one copy per segment from now on
-  }
   for (size_t i = 0; i < d.size(); ++i) {
     const cudaError_t e = cudaMemcpyAsync(d[i], s[i], n[i], cudaMemcpyDefault, st);
     if (e != cudaSuccess) return e;

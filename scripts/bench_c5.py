@@ -13,8 +13,8 @@ per-rank durations; GB/s per pair and aggregate, against 900 GB/s per direction 
   direction  uni  : even ranks send, odd ranks receive (4 concurrent one-way migrations)
              swap : both ranks of every pair send at once (bidirectional swap)
   engine     sm   : the peer-store descriptor walk (product path)
-             ce_batch / ce_tensor / ce_single : copy-engine baselines (cudaMemcpyBatchAsync per
-             2 MB, cudaMemcpyAsync per tensor = cudaMemcpyPeerAsync, one copy of the span)
+             ce_batch / ce_tensor / ce_single : copy-engine baselines (cudaMemcpyAsync per segment in
+             2 MB groups, cudaMemcpyAsync per tensor = cudaMemcpyPeerAsync, one copy of the span)
              nccl : torch.distributed NCCL send / recv of one contiguous buffer of the same size
 NVLink byte counters: run ONE rank's process under ncu (never a multi-rank command), e.g.
   ncu --metrics gpu__time_duration.sum,nvltx__bytes.sum,nvlrx__bytes.sum -k regex:mtcopy ...

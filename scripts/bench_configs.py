@@ -91,7 +91,7 @@ def c5(reps=4, engine=0, totals=None, mixes=None):
 
 
 def c5ce():
-    """Copy-engine-only peer migration (cudaMemcpyBatchAsync, no SM work) vs the SM
+    """Copy-engine-only peer migration (per-segment cudaMemcpyAsync in 2 MB groups, no SM work) vs the SM
     descriptor walk on the same live sets (same GPU: HBM -> HBM)."""
     totals = [1 << 20, 16 << 20, 256 << 20, 1 << 30]
     mixes = ("single", "resnet_hist", "all_4KB")
