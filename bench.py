@@ -31,13 +31,26 @@ import argparse
 import json
 import os
 
-os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")  # before any CUDA context (see the package)
 import subprocess
 import sys
 import threading
 import time
 
 import numpy as np
+
+
+def _gate_requested(argv) -> bool:
+    """--gate 1 / --gate=1 on the command line (read before any CUDA context exists)."""
+    for i, a in enumerate(argv):
+        if a == "--gate" and i + 1 < len(argv):
+            return argv[i + 1] == "1"
+        if a.startswith("--gate="):
+            return a.split("=", 1)[1] == "1"
+    return False
+
+
+if _gate_requested(sys.argv):  # the drain gate parks a stream: 32 hardware queues (see the package)
+    os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
@@ -827,9 +840,10 @@ def main():
                          "(default); 0: D2H, then H2D")
     ap.add_argument("--l2-persist-mb", type=float, default=0.0,
                     help="persisting L2 set-aside for the inference weights, MB (0: none)")
-    ap.add_argument("--gate", type=int, default=1,
+    ap.add_argument("--gate", type=int, default=0,
                     help="1: drain gate (a preempting request runs before the job's queued "
-                         "subgraph, default); 0: it waits for every dispatched subgraph")
+                         "subgraph); 0 (default, measured faster: DESIGN.md Q38): it waits for "
+                         "every dispatched subgraph")
     ap.add_argument("--pair-gate", type=int, default=0,
                     help="N > 1: use the drain gate in the pair processes too (default 0)")
     ap.add_argument("--early", type=int, default=1,
@@ -1026,8 +1040,12 @@ def main():
                      "traffic_source": prof.get("source"),
                      "dram_frac": prof.get("dram_frac"),
                      "algorithmic_bytes": "2 x live bytes per launch (read + write)"},
-        "inference_roofline": {"kernel": "request chain (3 LDG-streamed cluster GEMVs over blocked weights "
-                                         "under PDL, fused bias/ReLU, fused softmax; device time p50)",
+        "inference_roofline": {"kernel": ("request chain (mlp_fold_kernel: the whole MLP + softmax in one "
+                                          "cooperative kernel, column-split layer 0 over W0^T, row-split "
+                                          "layers after, one grid barrier; device time p50)")
+                               if os.environ.get("SF_CHAIN", "0") == "1" else
+                               "request chain (3 LDG-streamed cluster GEMVs over blocked weights "
+                               "under PDL, fused bias/ReLU, fused softmax; device time p50)",
                                "bound": "hbm", "algorithmic_bytes": w_bytes,
                                "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
                                "peak": hbm, "unit": "GB/s",

@@ -3,14 +3,12 @@
 The product path is libswitchflow_b200.so (CUDA kernels + C++ runtime, include/sf.h);
 this package only binds it.  See DESIGN.md.
 """
-import os as _os
-
-# The runtime keeps several streams per device (training, request, migration, clock) and the
-# drain gate parks the training stream on a memory wait; with the default 8 hardware work
-# queues, streams beyond that share a queue and a parked one can hold up its queue-mate.
-# Effective only if set before the process creates its CUDA context (bench.py and the tests
-# import this package first).
-_os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+# With the drain gate (sf_config.drain_gate, off by default) the training stream parks on a
+# memory wait; with the default 8 hardware work queues, streams beyond that share a queue and a
+# parked one can hold up its queue-mate (the runtime's 5 ms valve then releases it).  Callers
+# that turn the gate on should set CUDA_DEVICE_MAX_CONNECTIONS=32 before their CUDA context
+# exists (bench.py --gate 1 and the tests do); without the gate the default 8 queues measured
+# faster (bench: solo training 187 vs 142 iterations/s, DESIGN.md reading Q38).
 
 from ._abi import LIB_PATH, SFError, lib  # noqa: E402,F401
 

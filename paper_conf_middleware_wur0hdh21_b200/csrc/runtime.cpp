@@ -118,6 +118,8 @@ struct Binding {
   // inference: constant GEMV weights re-laid out in contiguous blocks (kernels_gemv.cu), built at
   // the binding's first request (sf_refresh_constants rebuilds them after the weights change)
   std::map<int, std::pair<void*, sfk::GemvBlockPlan>> blocked;  // tensor id -> (copy, plan)
+  // fused inference chain: layer-0 weights transposed (W_0^T, kernels_chain.cu), same lifetime
+  std::map<int, float*> folded;  // tensor id -> W_0^T
   bool blocked_ready = false;
   std::vector<void*> dev_allocs;
 };
@@ -147,6 +149,9 @@ struct Graph {
 
 constexpr int kInferOwner = 1 << 20;
 constexpr int kMaxInflight = 4;
+// timing-event ring per slot: twice the largest window, so a retired subgraph's events stay
+// valid until its device interval is mapped (deferred off the dispatch path)
+constexpr int kEvRing = 2 * kMaxInflight;
 constexpr int kCkEvents = 8;  // per slot: [0, 4) D2H chunk ring, [4, 8) H2D chunk ring
 
 struct Request {
@@ -259,8 +264,8 @@ struct Job {
   std::string error;
   std::thread driver;
   std::vector<cudaEvent_t> ev_sub, ev_a, ev_b, ev_c, ev_r;  // per slot; ev_r: resume point
-  std::vector<cudaEvent_t> ev_ring;  // [slot * kMaxInflight + i]: in-flight subgraph ends
-  std::vector<cudaEvent_t> ev_start; // [slot * kMaxInflight + i]: their starts (device trace)
+  std::vector<cudaEvent_t> ev_ring;  // [slot * kEvRing + i]: in-flight subgraph ends
+  std::vector<cudaEvent_t> ev_start; // [slot * kEvRing + i]: their starts (device trace)
   std::vector<cudaEvent_t> ev_ck;    // [slot * kCkEvents + i]: host-tier copy chunks in flight
 };
 
@@ -666,14 +671,14 @@ sf_status upload(Binding& b, const void* host, size_t bytes, void** out) {
 // [-> BIAS_ACT] ... [-> SOFTMAX] inside [j, e), each GEMM reading the previous layer's output.
 // Returns the number of ops covered (0 = no chain of >= 2 layers starts at j).
 int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
-  // opt-in (SF_CHAIN=1): the persistent streaming chain is parity-green, but on the C4 model
-  // the per-layer GEMV kernels under programmatic dependent launch measure faster (DESIGN.md
-  // reading Q39: grid-barrier and imbalance cost per layer boundary)
+  // opt-in (SF_CHAIN=1): the fused chain is parity-green, but on the C4 model the per-layer
+  // GEMV kernels under programmatic dependent launch measure faster (reading Q42:
+  // its two global reductions + softmax add a ~12 us serial tail after the weight stream)
   static const bool enabled = std::getenv("SF_CHAIN") && std::getenv("SF_CHAIN")[0] == '1';
   if (!enabled) return 0;
   Graph& g = c.g;
   sfk::ChainArgs a;
-  int i = j, prev_y = -1;
+  int i = j, prev_y = -1, w0 = -1;
   auto readers = [&](int t) {
     int n = 0;
     for (const auto& q : g.ops)
@@ -688,6 +693,7 @@ int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
     if (a.n_layers > 0 && (o.in[0] != prev_y || C.rows != a.M)) break;
     sfk::ChainLayerArgs& L = a.layer[a.n_layers];
     L = sfk::ChainLayerArgs{};
+    if (a.n_layers == 0) w0 = o.in[1];
     L.W = c.f(o.in[1]); L.ldw = B.cols;
     L.x = c.f(o.in[0]); L.ldx = A.cols;
     L.K = A.cols; L.N = C.cols;
@@ -717,6 +723,20 @@ int match_chain(Capture& c, int j, int e, sfk::ChainArgs* out) {
     ++i;
   }
   if (!sfk::chain_eligible(a)) return 0;
+  auto fw = c.b.folded.find(w0);
+  if (fw == c.b.folded.end()) {  // W_0^T: allocated in the prepare pass, laid out by layout_blocked
+    if (!c.dry) return 0;
+    void* d = nullptr;
+    const Tensor& W0 = g.T[w0];
+    if (cudaMalloc(&d, sfk::chain_w0t_floats(W0.rows, W0.cols) * sizeof(float)) != cudaSuccess) {
+      cudaGetLastError();
+      return 0;
+    }
+    c.b.dev_allocs.push_back(d);
+    fw = c.b.folded.emplace(w0, static_cast<float*>(d)).first;
+    c.b.blocked_ready = false;
+  }
+  a.w0t = fw->second;
   *out = a;
   return i - j;
 }
@@ -1009,8 +1029,8 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
   const size_t n = rt->slots.size();
   J.ev_sub.assign(n, nullptr); J.ev_a.assign(n, nullptr); J.ev_b.assign(n, nullptr); J.ev_c.assign(n, nullptr);
   J.ev_r.assign(n, nullptr);
-  J.ev_ring.assign(n * kMaxInflight, nullptr);
-  J.ev_start.assign(n * kMaxInflight, nullptr);
+  J.ev_ring.assign(n * kEvRing, nullptr);
+  J.ev_start.assign(n * kEvRing, nullptr);
   J.ev_ck.assign(n * kCkEvents, nullptr);
   int cur = 0;
   cudaGetDevice(&cur);
@@ -1019,9 +1039,9 @@ sf_status ensure_events(sf_runtime* rt, Job& J) {
     SF_CK(cudaSetDevice(rt->slots[s]->cuda));
     SF_CK(cudaEventCreateWithFlags(&J.ev_sub[s], cudaEventDisableTiming));
     SF_CK(cudaEventCreate(&J.ev_r[s]));  // timing: device resume point
-    for (int i = 0; i < kMaxInflight; ++i) {  // timing events: device intervals of subgraphs
-      SF_CK(cudaEventCreate(&J.ev_ring[s * kMaxInflight + i]));
-      SF_CK(cudaEventCreate(&J.ev_start[s * kMaxInflight + i]));
+    for (int i = 0; i < kEvRing; ++i) {  // timing events: device intervals of subgraphs
+      SF_CK(cudaEventCreate(&J.ev_ring[s * kEvRing + i]));
+      SF_CK(cudaEventCreate(&J.ev_start[s * kEvRing + i]));
     }
     for (int i = 0; i < kCkEvents; ++i)
       SF_CK(cudaEventCreateWithFlags(&J.ev_ck[s * kCkEvents + i], cudaEventDisableTiming));
@@ -1251,6 +1271,12 @@ sf_status alloc_blocked(Graph& g, Binding& b) {
 }
 // Lay the current weights out into the blocked copies (stream-ordered on st).
 void layout_blocked(const Graph& g, Binding& b, cudaStream_t st) {
+  for (auto& [t, d] : b.folded) {
+    const Tensor& Wt = g.T[t];
+    if (sfk::launch_chain_w0t_layout(reinterpret_cast<const float*>(b.arena + Wt.offset), Wt.cols, Wt.rows,
+                                     Wt.cols, d, st) != cudaSuccess)
+      cudaGetLastError();
+  }
   for (auto& [t, e] : b.blocked) {
     const Tensor& Bt = g.T[t];
     if (sfk::launch_gemv_block_layout(reinterpret_cast<const float*>(b.arena + Bt.offset), e.first, Bt.rows,
@@ -1878,6 +1904,35 @@ void driver_main(sf_runtime* rt, Job* Jp) {
   };
   int ev_next = 0;
   uint64_t last_t1 = 0;
+  // Retired subgraphs whose device interval is mapped later: the timing-event reads (anchor
+  // lookups + cudaEventElapsedTime, several us) run while the GPU executes the next subgraph
+  // instead of between the completion and the next launch.  Flushed, in retire order, at the
+  // start of the next retire wait and when the job ends.
+  struct PendTrace {
+    int dev, ev;
+    uint64_t t0;
+    sf_trace_event tev;
+    double D0, D1;
+  };
+  std::vector<PendTrace> pend;
+  auto map_pend = [&] {  // rt->m NOT held
+    for (auto& p : pend) {
+      Slot& PS = slot_of(rt, p.dev);
+      p.tev.d0_ns = event_host_ns(PS, J.ev_start[p.dev * kEvRing + p.ev], p.t0);
+      p.tev.d1_ns = event_host_ns(PS, J.ev_ring[p.dev * kEvRing + p.ev], p.t0);
+      p.D0 = event_dev_D(PS, J.ev_start[p.dev * kEvRing + p.ev], p.t0);
+      p.D1 = event_dev_D(PS, J.ev_ring[p.dev * kEvRing + p.ev], p.t0);
+    }
+  };
+  auto push_pend = [&] {  // rt->m held
+    for (auto& p : pend) push_trace(rt, p.tev, p.D0, p.D1);
+    pend.clear();
+  };
+  auto flush_pend_locked = [&] {  // off the dispatch path (cut, idle waits): rt->m held
+    if (pend.empty()) return;
+    map_pend();
+    push_pend();
+  };
   int64_t broke_for = -1;  // front (it * n + k) whose wait was left early once
   std::unique_lock<std::mutex> lk(rt->m);
   bool pending_peer_stats = false;
@@ -1896,6 +1951,12 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     const bool finished = J.it >= J.iters || (J.stop_req && J.k == 0) || rt->shutting_down;
     if (finished) {
       if (q.empty()) {
+        if (!pend.empty()) {
+          lk.unlock();
+          map_pend();
+          lk.lock();
+          push_pend();
+        }
         release();
         J.state = SF_JOB_DONE;
         if (g.feed) {
@@ -1954,6 +2015,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
           J.gate_cut_pending = false;
           const int src = J.dev;
           const bool peer = J.preempt_target != SF_TARGET_HOST;
+          flush_pend_locked();
           if (do_preempt(rt, J, lk) != SF_OK) break;
           if (J.state == SF_JOB_DONE || J.state == SF_JOB_MIGRATED_OUT) break;
           if (peer) { pending_peer_stats = true; stats_slot = src; }
@@ -1962,6 +2024,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       } else if (yield_to_inf) {
         if (q.empty()) {
           release();
+          flush_pend_locked();
           rt->cv.wait(lk);
           continue;
         }
@@ -1987,6 +2050,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
         if (!feed_ok) {
           if (q.empty()) {
             release();
+            flush_pend_locked();
             rt->cv.wait(lk);
             continue;
           }
@@ -1994,6 +2058,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
           // invariant 1: no other model's subgraph on this device
           if (S.owner != -1) {
             if (q.empty()) {
+              flush_pend_locked();
               rt->cv.wait(lk);
               continue;
             }
@@ -2043,7 +2108,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       const uint32_t ticket = S.next_ticket++;
       if (rt->cfg.drain_gate && S.gate && !S.gate_held && (ticket & 0xFFFFF) == 0) gate_open(S);
       const int ev = ev_next;
-      ev_next = (ev_next + 1) % W;
+      ev_next = (ev_next + 1) % (2 * W);
       const uint64_t t0 = now_ns();  // decision time, under the lock (trace superset interval)
       lk.unlock();
       cudaSetDevice(S.cuda);
@@ -2058,7 +2123,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
                 CUDA_SUCCESS)
           e = cudaErrorLaunchFailure;
       }
-      if (e == cudaSuccess) e = cudaEventRecord(J.ev_start[dev * kMaxInflight + ev], S.s_train);
+      if (e == cudaSuccess) e = cudaEventRecord(J.ev_start[dev * kEvRing + ev], S.s_train);
       if (e == cudaSuccess && F) {  // this iteration's fed tensors into the arena, then S_0
         const uint8_t* src = (F->shared ? F->dbuf : F->host) + fslot * F->stride;
         uint8_t* arena = g.bind[dev]->arena;
@@ -2068,7 +2133,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
                               cudaMemcpyDefault, S.s_train);
       }
       if (e == cudaSuccess) e = cudaGraphLaunch(ver, S.s_train);
-      if (e == cudaSuccess) e = cudaEventRecord(J.ev_ring[dev * kMaxInflight + ev], S.s_train);
+      if (e == cudaSuccess) e = cudaEventRecord(J.ev_ring[dev * kEvRing + ev], S.s_train);
       lk.lock();
       J.launching = false;
       if (e != cudaSuccess) {
@@ -2080,8 +2145,8 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       }
       if (q.empty()) front_start = t0;
       q.push_back({it, k, dev, ev, t0, stamp});
-      J.infl.push_back({ticket, gated, J.ev_ring[dev * kMaxInflight + ev]});
-      J.last_ev = J.ev_ring[dev * kMaxInflight + ev];
+      J.infl.push_back({ticket, gated, J.ev_ring[dev * kEvRing + ev]});
+      J.last_ev = J.ev_ring[dev * kEvRing + ev];
       J.n_inflight = static_cast<int>(q.size());
       if (S.qn.load(std::memory_order_acquire) > 0) rt->cv.notify_all();  // a waiting dispatcher
       if (++J.k == n) {
@@ -2095,6 +2160,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       continue;
     }
     if (q.empty()) {  // nothing launched and nothing in flight: wait for a state change
+      flush_pend_locked();
       rt->cv.wait(lk);
       continue;
     }
@@ -2108,12 +2174,13 @@ void driver_main(sf_runtime* rt, Job* Jp) {
                            broke_for != (f.it * n + f.k);
     lk.unlock();
     cudaSetDevice(S.cuda);
+    map_pend();  // the previous retire's device interval, while this front runs
     uint64_t t_res = 0;
     cudaError_t e = cudaSuccess;
     bool broke = false;
     for (;;) {
       if (f.stamp && !t_res && cudaEventQuery(J.ev_r[f.dev]) == cudaSuccess) t_res = now_ns();
-      const cudaError_t qq = cudaEventQuery(J.ev_ring[f.dev * kMaxInflight + f.ev]);
+      const cudaError_t qq = cudaEventQuery(J.ev_ring[f.dev * kEvRing + f.ev]);
       if (qq == cudaErrorNotReady) {
         const bool req_waiting = S.qn.load(std::memory_order_relaxed) > 0;
         if (may_break && !req_waiting && queued_us() + est_us[J.k] <= budget_us) {
@@ -2131,6 +2198,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     if (broke) {
       broke_for = f.it * n + f.k;
       lk.lock();
+      push_pend();
       continue;
     }
     const uint64_t t1 = now_ns();
@@ -2138,11 +2206,11 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     // device execution interval on the host clock (0 when no anchor covers it)
     uint64_t d0 = 0, d1 = 0;
     double D0 = std::nan(""), D1 = std::nan("");
-    if (e == cudaSuccess) {
-      d0 = event_host_ns(S, J.ev_start[f.dev * kMaxInflight + f.ev], f.t0);
-      d1 = event_host_ns(S, J.ev_ring[f.dev * kMaxInflight + f.ev], f.t0);
-      D0 = event_dev_D(S, J.ev_start[f.dev * kMaxInflight + f.ev], f.t0);
-      D1 = event_dev_D(S, J.ev_ring[f.dev * kMaxInflight + f.ev], f.t0);
+    if (e == cudaSuccess && f.stamp) {  // others: deferred (pend)
+      d0 = event_host_ns(S, J.ev_start[f.dev * kEvRing + f.ev], f.t0);
+      d1 = event_host_ns(S, J.ev_ring[f.dev * kEvRing + f.ev], f.t0);
+      D0 = event_dev_D(S, J.ev_start[f.dev * kEvRing + f.ev], f.t0);
+      D1 = event_dev_D(S, J.ev_ring[f.dev * kEvRing + f.ev], f.t0);
       if (f.stamp) {  // the resume point as the GPU saw it
         const uint64_t r = event_host_ns(S, J.ev_r[f.dev], f.t0);
         if (r) t_res = r;
@@ -2163,6 +2231,7 @@ void driver_main(sf_runtime* rt, Job* Jp) {
       }
     }
     lk.lock();
+    push_pend();
     q.pop_front();
     if (!J.infl.empty()) J.infl.pop_front();
     J.n_inflight = static_cast<int>(q.size());
@@ -2193,7 +2262,8 @@ void driver_main(sf_runtime* rt, Job* Jp) {
     tev.arrival_ns = f.t0;  // train events: host dispatch (launch) time
     last_t1 = t1;
     front_start = q.empty() ? 0 : std::max(q.front().t0, t1);
-    push_trace(rt, tev, D0, D1);
+    if (f.stamp) push_trace(rt, tev, D0, D1);
+    else pend.push_back({f.dev, f.ev, f.t0, tev, D0, D1});
     // iteration-granularity (session time slicing baseline) keeps the device for the whole
     // iteration; otherwise an empty window is a scheduling point
     if (q.empty() && (!rt->cfg.iteration_granularity || J.k == 0)) release();
@@ -2358,7 +2428,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
     const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
     // blocked copies of the constant GEMV weights (allocated at bind; laid out here at the first
     // request unless sf_refresh_constants already did it; reading Q39)
-    if (direct && !B->blocked_ready) {
+    if (!B->blocked_ready) {
       layout_blocked(g, *B, S->s_infer);
       B->blocked_ready = true;
     }
@@ -2617,9 +2687,9 @@ void sf_destroy(sf_runtime* rt) {
       cudaSetDevice(rt->slots[s]->cuda);
       cudaEventDestroy(J->ev_sub[s]);
       cudaEventDestroy(J->ev_r[s]);
-      for (int i = 0; i < kMaxInflight; ++i) {
-        cudaEventDestroy(J->ev_ring[s * kMaxInflight + i]);
-        cudaEventDestroy(J->ev_start[s * kMaxInflight + i]);
+      for (int i = 0; i < kEvRing; ++i) {
+        cudaEventDestroy(J->ev_ring[s * kEvRing + i]);
+        cudaEventDestroy(J->ev_start[s * kEvRing + i]);
       }
       for (int i = 0; i < kCkEvents; ++i) cudaEventDestroy(J->ev_ck[s * kCkEvents + i]);
       cudaEventDestroy(J->ev_a[s]);
@@ -3608,15 +3678,19 @@ sf_status sf_op_mlp_chain(const float* x, int32_t M, int32_t n_layers, const int
   if (!sfk::chain_eligible(a)) return fail(SF_EUNSUPPORTED, "mlp_chain: shape outside the fused kernel");
   cudaStream_t st = as_stream(stream);
   const uint64_t wf = sfk::chain_ws_floats(a), cs = sfk::chain_counter_slots(a);
-  void *ws = nullptr, *cnt = nullptr;
+  void *ws = nullptr, *cnt = nullptr, *w0t = nullptr;
   SF_CK(cudaMallocAsync(&ws, std::max<uint64_t>(wf, 4) * 4, st));
   SF_CK(cudaMallocAsync(&cnt, cs * 4, st));
+  SF_CK(cudaMallocAsync(&w0t, sfk::chain_w0t_floats(widths[0], widths[1]) * 4, st));
   SF_CK(cudaMemsetAsync(cnt, 0, cs * 4, st));
+  SF_CK(sfk::launch_chain_w0t_layout(W[0], widths[1], widths[0], widths[1], static_cast<float*>(w0t), st));
   a.ws = static_cast<float*>(ws);
   a.counters = static_cast<unsigned*>(cnt);
+  a.w0t = static_cast<float*>(w0t);
   SF_CK(sfk::launch_chain(a, st));
   SF_CK(cudaFreeAsync(ws, st));
   SF_CK(cudaFreeAsync(cnt, st));
+  SF_CK(cudaFreeAsync(w0t, st));
   return SF_OK;
 }
 

@@ -99,7 +99,9 @@ bool make_map2d(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, 
                 uint32_t box_cols, uint32_t box_rows, bool swizzle128);
 
 // Fused batch-M (M <= 8) MLP chain: h_{l+1} = act(h_l W_l + b_l) for every layer (+ softmax)
-// in one persistent kernel (kernels_chain.cu).  layer[l].x must be layer[l-1].y.
+// in one persistent kernel (kernels_chain.cu).  layer[l].x must be layer[l-1].y.  Layer 0 is
+// read from w0t, a transposed copy W_0^T [N_0][K_0 rounded up to 4] (zero-padded) laid out by
+// launch_chain_w0t_layout (chain_w0t_floats floats).
 constexpr int kChainMaxLayers = 6;
 struct ChainLayerArgs {
   const float* W; int ldw;
@@ -117,10 +119,13 @@ struct ChainArgs {
   int sm_n = 0, sm_ldi = 0, sm_ldo = 0;
   float* ws = nullptr;
   unsigned* counters = nullptr;  // zero before the first launch; the kernel re-zeroes them
+  const float* w0t = nullptr;    // W_0^T (16-B aligned)
 };
 bool chain_eligible(const ChainArgs& a);
 uint64_t chain_ws_floats(const ChainArgs& a);
 uint64_t chain_counter_slots(const ChainArgs& a);
+uint64_t chain_w0t_floats(int K, int N);
+cudaError_t launch_chain_w0t_layout(const float* W, int ldw, int K, int N, float* Wt, cudaStream_t st);
 cudaError_t launch_chain(const ChainArgs& a, cudaStream_t st);
 // diagnostics: when set, every chain launch records per-CTA phase timestamps (u64 [SMs][64])
 void set_chain_trace(void* dev_buf);

@@ -4,6 +4,7 @@ layer {first/last CTA start, first/last return from griddepcontrol.wait, first/l
 streaming, last CTA end} relative to the first CTA start of layer 0 (sf_debug_chain_trace)."""
 import ctypes as C, json, os, sys
 import numpy as np, torch
+os.environ.setdefault("SF_CHAIN", "0")  # the per-layer GEMV chain (the fused kernel has its own trace)
 sys.path.insert(0, ".")
 import bench
 from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime

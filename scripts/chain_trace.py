@@ -28,14 +28,15 @@ lib().sf_debug_chain_trace(None)
 t = tr.view(160, 8, 8)[:, :n + 1, :].cpu().numpy().astype(np.float64)
 t0 = t[t > 0].min()
 print("event-timed us (cold L2):", np.round(res[2:], 1))
-# mlp_stream_kernel events: 0 layer start, 1 my rows streamed, 2 partials of all CTAs published
-# (grid barrier), 3 reduced (next layer's x slice / the output slice); done at [n][7]
-names = ["start", "streamed", "barrier", "reduced", "-", "-", "-", "done"]
+# mlp_fold_kernel events: layer 0: 0 start, 1 x staged, 4 columns streamed + combined;
+# layer l > 0: 0 start, 1 my rows streamed, 2 grid barrier passed, 3 reduced; done at [n][7]
+names = ["start", "streamed" , "barrier", "reduced", "l0_done", "published", "tail_landed", "done"]
+names0 = ["start", "x_staged", "x_synced", "-", "l0_combined", "l0_items_done", "-", "-"]
 for l in range(n + 1):
     row = []
     for e in range(8):
         v = t[:, l, e]
         v = v[v > 0]
         if len(v):
-            row.append(f"{names[e]} {np.median(v - t0) / 1e3:6.2f}/{np.max(v - t0) / 1e3:6.2f}")
+            row.append(f"{(names0 if l == 0 else names)[e]} {np.median(v - t0) / 1e3:6.2f}/{np.max(v - t0) / 1e3:6.2f}")
     print(f"layer {l}: " + " | ".join(row))

@@ -313,13 +313,14 @@ def test_mlp_chain_vs_oracle(ops, widths, M, biases, softmax):
 
 
 def test_mlp_chain_rejects_unsupported_shapes(ops):
-    """N % 4 != 0 (TMA row pitch) and more than 6 layers are refused, not silently wrong."""
+    """N % 4 != 0 on a row-split layer (layers >= 1 stream whole float4 rows) and more than 6
+    layers are refused, not silently wrong."""
     from paper_conf_middleware_wur0hdh21_b200._abi import SFError
     x = torch.zeros(1, 64, device="cuda")
     with pytest.raises(SFError):
-        ops.mlp_chain(x, [torch.zeros(64, 10, device="cuda"), torch.zeros(10, 8, device="cuda")],
+        ops.mlp_chain(x, [torch.zeros(64, 8, device="cuda"), torch.zeros(8, 10, device="cuda")],
                       [None, None], [True, False],
-                      [torch.zeros(1, 10, device="cuda"), torch.zeros(1, 8, device="cuda")])
+                      [torch.zeros(1, 8, device="cuda"), torch.zeros(1, 10, device="cuda")])
     Ws = [torch.zeros(64, 64, device="cuda") for _ in range(7)]
     with pytest.raises(SFError):
         ops.mlp_chain(x, Ws, [None] * 7, [True] * 7, [torch.zeros(1, 64, device="cuda") for _ in range(7)])
