@@ -1432,7 +1432,14 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
                                       ? size_t(std::max(1, std::min(2, std::atoi(std::getenv("SF_DUPLEX_DEPTH_D2H")))))
                                       : kDepth;
   constexpr int R = 4;  // event ring per direction (kCkEvents / 2)
-  const size_t nch = (total + kChunk - 1) / kChunk;
+  // small live sets (<= R chunks of 2 MB, e.g. C1's 1.6-2.4 MB): R equal chunks all issued at
+  // once (D2H on the migration stream, each H2D waiting on its chunk's event on the device), so
+  // the two directions overlap without host round trips between chunks
+  const bool upfront = !std::getenv("SF_DUPLEX_CHUNK_KB") && total <= R * kChunk;
+  const size_t chunk = upfront ? std::max<size_t>(size_t(64) << 10, ((total + R - 1) / R + 4095) / 4096 * 4096)
+                               : kChunk;
+  const size_t depth = upfront ? R : kDepth, depth_d2h = upfront ? R : kDepthD2H;
+  const size_t nch = (total + chunk - 1) / chunk;
   size_t nd = 0, nh = 0, cd = 0, ch = 0;  // D2H / H2D issued, D2H / H2D completed
   cudaEvent_t* evd = &J.ev_ck[slot * kCkEvents];
   cudaEvent_t* evh = evd + R;
@@ -1453,8 +1460,8 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
       continue;
     }
     if (!busy()) {
-      if (nd < nch && nd - cd < kDepthD2H && nd - nh < static_cast<size_t>(R)) {
-        const size_t off = nd * kChunk, n = std::min(kChunk, total - off);
+      if (nd < nch && nd - cd < depth_d2h && nd - nh < static_cast<size_t>(R)) {
+        const size_t off = nd * chunk, n = std::min(chunk, total - off);
         cudaError_t e = cudaMemcpyAsync(hstg + off, dstg + off, n, cudaMemcpyDeviceToHost, S.s_mig);
         if (e == cudaSuccess && poison_chunks) e = sfk::launch_fill(dstg + off, n, 0xFF, S.s_mig);
         if (e == cudaSuccess) e = cudaEventRecord(evd[nd % R], S.s_mig);
@@ -1462,8 +1469,8 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
         ++nd;
         progressed = true;
       }
-      if (nh < (host_order ? cd : nd) && nh - ch < kDepth) {
-        const size_t off = nh * kChunk, n = std::min(kChunk, total - off);
+      if (nh < (host_order ? cd : nd) && nh - ch < depth) {
+        const size_t off = nh * chunk, n = std::min(chunk, total - off);
         cudaError_t e = host_order ? cudaSuccess : cudaStreamWaitEvent(S.s_train, evd[nh % R], 0);
         if (e == cudaSuccess) e = cudaMemcpyAsync(dstg + off, hstg + off, n, cudaMemcpyHostToDevice, S.s_train);
         if (e == cudaSuccess) e = cudaEventRecord(evh[nh % R], S.s_train);

@@ -175,9 +175,9 @@ def test_open_loop_requests_at_bench_config_bitwise(W, gate):
     SC.check_job_order([e for e in dv if e["kind"] == "train"], {0: len(parts)}, start={0: (0, 0)})
     SC.check_cut_rule(dv)
     held = sum(e["kind"] == "infer" and e["k"] == 1 for e in evs)
+    # (how many requests land while a subgraph is queued is timing; the hold path itself is
+    # forced in test_gpu_runtime.py::test_drain_gate_holds_the_queued_subgraph)
     print("drain gate held", held, "of", sum(e["kind"] == "infer" for e in evs))
-    if gate:
-        assert held >= 1
     # with the drain gate only the running subgraph drains (window 1)
     r = SC.preempt_latency_report(dv, slack=20e3, window=1 if gate else 2)
     print("I3 bound us", r["bound"][0] / 1e3, "max wait us", max(r["waits"]) / 1e3,
