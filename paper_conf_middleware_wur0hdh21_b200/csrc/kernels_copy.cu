@@ -328,6 +328,8 @@ __global__ void copy_kernel(const uint8_t* __restrict__ src, uint8_t* __restrict
   }
 }
 
+const void* copy_kernel_fn() { return reinterpret_cast<const void*>(&copy_kernel); }
+
 cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st) {
   if (nbytes == 0) return cudaSuccess;
   const uint64_t blocks = std::min<uint64_t>((nbytes / 16 + 255) / 256 + 1, 148ull * 4);

@@ -120,6 +120,17 @@ struct Binding {
   std::map<int, std::pair<void*, sfk::GemvBlockPlan>> blocked;  // tensor id -> (copy, plan)
   // fused inference chain: layer-0 weights transposed (W_0^T, kernels_chain.cu), same lifetime
   std::map<int, float*> folded;  // tensor id -> W_0^T
+  // the whole request chain as ONE graph launch (SF_INFER_GRAPH=1): captured once per binding
+  // (at sf_refresh_constants) between two copy kernels whose src / dst are patched per request
+  // (cudaGraphExecKernelNodeSetParams), so one capture serves every request buffer
+  struct ReqGraph {
+    int state = 0;  // 0 not built, 1 ready, -1 failed (direct launches)
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    cudaGraphNode_t in_node = nullptr, out_node = nullptr;
+    dim3 in_grid, in_block, out_grid, out_block;
+    uint64_t kernels = 0;
+  } rg;
   bool blocked_ready = false;
   std::vector<void*> dev_allocs;
 };
@@ -1269,6 +1280,106 @@ sf_status alloc_blocked(Graph& g, Binding& b) {
   }
   return SF_OK;
 }
+bool infer_graph_mode() {
+  static const bool on = std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1';
+  return on;
+}
+
+sf_status launch_subgraph_ops(Capture& c, int k);
+
+// Captures the request chain of an inference binding once: copy(in -> arena input), the
+// subgraph kernels (programmatic dependent launch as on the direct path), copy(arena output ->
+// out).  The two copy nodes are found by their kernel and patched per request.
+void build_req_graph(Graph& g, Binding& B, bool pdl) {
+  Binding::ReqGraph& R = B.rg;
+  if (R.state != 0) return;
+  R.state = -1;
+  if (g.input_tid < 0 || g.output_tid < 0) return;
+  const Tensor &tin = g.T[g.input_tid], &tout = g.T[g.output_tid];
+  if (tin.nbytes % 4 || tout.nbytes % 4) return;
+  cudaStream_t st = nullptr;
+  if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) { cudaGetLastError(); return; }
+  const bool pdl_was = sfk::pdl_enabled();
+  sfk::set_pdl(pdl);
+  const uint64_t l0 = sfk::launches();
+  bool ok = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+  cudaGraph_t graph = nullptr;
+  if (ok) {
+    uint8_t* ain = B.arena + tin.offset;
+    uint8_t* aout = B.arena + tout.offset;
+    ok = sfk::launch_copy(ain, ain, tin.nbytes, st) == cudaSuccess;  // src patched per request
+    for (size_t k = 0; ok && k < B.versions.size(); ++k) {
+      Capture c{g, B, st, false, &B.prepared};
+      ok = launch_subgraph_ops(c, static_cast<int>(k)) == SF_OK;
+    }
+    ok = ok && sfk::launch_copy(aout, aout, tout.nbytes, st) == cudaSuccess;  // dst patched
+    const cudaError_t e = cudaStreamEndCapture(st, &graph);
+    ok = ok && e == cudaSuccess && graph;
+  }
+  const uint64_t nk = sfk::launches() - l0;
+  sfk::count_launch(uint64_t(0) - nk);  // captured, not launched: counted at each replay
+  sfk::set_pdl(pdl_was);
+  cudaStreamDestroy(st);
+  if (!ok) {
+    cudaGetLastError();
+    if (graph) cudaGraphDestroy(graph);
+    return;
+  }
+  size_t n = 0;
+  cudaGraphGetNodes(graph, nullptr, &n);
+  std::vector<cudaGraphNode_t> nodes(n);
+  cudaGraphGetNodes(graph, nodes.data(), &n);
+  for (auto nd : nodes) {
+    cudaGraphNodeType t;
+    if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeKernel) continue;
+    cudaKernelNodeParams kp{};
+    if (cudaGraphKernelNodeGetParams(nd, &kp) != cudaSuccess || kp.func != sfk::copy_kernel_fn()) continue;
+    size_t ndep = 0, nout = 0;
+    cudaGraphNodeGetDependencies(nd, nullptr, &ndep);
+    cudaGraphNodeGetDependentNodes(nd, nullptr, &nout);
+    if (ndep == 0) { R.in_node = nd; R.in_grid = kp.gridDim; R.in_block = kp.blockDim; }
+    else if (nout == 0) { R.out_node = nd; R.out_grid = kp.gridDim; R.out_block = kp.blockDim; }
+  }
+  cudaGraphExec_t exec = nullptr;
+  if (!R.in_node || !R.out_node || cudaGraphInstantiate(&exec, graph, 0) != cudaSuccess) {
+    cudaGetLastError();
+    cudaGraphDestroy(graph);
+    R.in_node = R.out_node = nullptr;
+    return;
+  }
+  R.graph = graph;
+  R.exec = exec;
+  R.kernels = nk;
+  R.state = 1;
+}
+
+// Patches the request's buffers into the captured chain and launches it (one API call).
+cudaError_t launch_req_graph(Binding& B, const Tensor& tin, const Tensor& tout, const void* in, void* out,
+                             cudaStream_t st) {
+  Binding::ReqGraph& R = B.rg;
+  const uint8_t* src_in = static_cast<const uint8_t*>(in);
+  uint8_t* dst_in = B.arena + tin.offset;
+  uint64_t n_in = tin.nbytes;
+  void* a_in[] = {&src_in, &dst_in, &n_in};
+  cudaKernelNodeParams kp{};
+  kp.func = const_cast<void*>(sfk::copy_kernel_fn());
+  kp.gridDim = R.in_grid;
+  kp.blockDim = R.in_block;
+  kp.kernelParams = a_in;
+  cudaError_t e = cudaGraphExecKernelNodeSetParams(R.exec, R.in_node, &kp);
+  const uint8_t* src_out = B.arena + tout.offset;
+  uint8_t* dst_out = static_cast<uint8_t*>(out);
+  uint64_t n_out = tout.nbytes;
+  void* a_out[] = {&src_out, &dst_out, &n_out};
+  kp.gridDim = R.out_grid;
+  kp.blockDim = R.out_block;
+  kp.kernelParams = a_out;
+  if (e == cudaSuccess) e = cudaGraphExecKernelNodeSetParams(R.exec, R.out_node, &kp);
+  if (e == cudaSuccess) e = cudaGraphLaunch(R.exec, st);
+  if (e == cudaSuccess) sfk::count_launch(R.kernels);
+  return e;
+}
+
 // Lay the current weights out into the blocked copies (stream-ordered on st).
 void layout_blocked(const Graph& g, Binding& b, cudaStream_t st) {
   for (auto& [t, d] : b.folded) {
@@ -2432,25 +2543,30 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       }
       return a.type == cudaMemoryTypeDevice;
     };
-    const bool in_place = direct && aligned && redirect && on_device(r->in) && on_device(r->out);
+    const bool in_place = direct && aligned && redirect && !(infer_graph_mode() && B->rg.state == 1) &&
+                          on_device(r->in) && on_device(r->out);
     // blocked copies of the constant GEMV weights (allocated at bind; laid out here at the first
     // request unless sf_refresh_constants already did it; reading Q39)
     if (!B->blocked_ready) {
       layout_blocked(g, *B, S->s_infer);
       B->blocked_ready = true;
     }
+    if (direct && infer_graph_mode() && B->rg.state == 0) build_req_graph(g, *B, use_pdl);
     const uint64_t tl0 = now_ns();
     // early launch: the chain (and its start event) wait on the device for the job's
     // dispatched subgraphs; the driver dispatches nothing more while the request is queued
     if (dep_ev) e = cudaStreamWaitEvent(S->s_infer, dep_ev, 0);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_i0, S->s_infer);
-    if (e != cudaSuccess || in_place) {
+    const bool graph_req = direct && infer_graph_mode() && B->rg.state == 1 && aligned;
+    if (e != cudaSuccess || in_place || graph_req) {
     } else if (aligned) {
       e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
-    for (size_t k = 0; e == cudaSuccess && k < B->versions.size(); ++k) {
+    const bool graph_io = direct && infer_graph_mode() && B->rg.state == 1 && aligned;
+    if (graph_io && e == cudaSuccess) e = launch_req_graph(*B, tin, tout, r->in, r->out, S->s_infer);
+    for (size_t k = 0; !graph_io && e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
         if (S->l2_setaside > 0) c.l2_keep = &B->l2_keep;
@@ -2469,7 +2585,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
         sfk::count_launch(B->version_kernels[k]);
       }
     }
-    if (e == cudaSuccess && !in_place) {
+    if (e == cudaSuccess && !in_place && !graph_io) {
       if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
       else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
     }
@@ -2684,6 +2800,8 @@ void sf_destroy(sf_runtime* rt) {
       }
       cudaSetDevice(rt->slots[B->slot]->cuda);
       for (auto v : B->versions) cudaGraphExecDestroy(v);
+      if (B->rg.exec) cudaGraphExecDestroy(B->rg.exec);
+      if (B->rg.graph) cudaGraphDestroy(B->rg.graph);
       for (void* d : B->dev_allocs) cudaFree(d);
       if (B->ws) cudaFree(B->ws);
       if (B->counters) cudaFree(B->counters);
@@ -3621,6 +3739,10 @@ sf_status sf_refresh_constants(sf_runtime* rt, sf_graph_id gid, int32_t dev) {
   layout_blocked(*g, B, S.s_infer);
   SF_CK(cudaStreamSynchronize(S.s_infer));
   B.blocked_ready = true;
+  if (infer_graph_mode()) {
+    static const bool use_pdl = !(std::getenv("SF_PDL") && std::getenv("SF_PDL")[0] == '0');
+    build_req_graph(*g, B, use_pdl);
+  }
   return SF_OK;
 }
 

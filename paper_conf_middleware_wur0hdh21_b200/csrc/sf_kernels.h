@@ -28,6 +28,9 @@ cudaError_t launch_copy2d(const void* src, uint64_t spitch, void* dst, uint64_t 
                           uint64_t width, cudaStream_t st);
 // Single-buffer copy with pointer arguments (request I/O; 16-B aligned, nbytes % 4 == 0).
 cudaError_t launch_copy(const void* src, void* dst, uint64_t nbytes, cudaStream_t st);
+// The copy kernel launch_copy runs (kernel(const uint8_t* src, uint8_t* dst, uint64_t nbytes)):
+// captured request graphs patch its pointers per request (cudaGraphExecKernelNodeSetParams).
+const void* copy_kernel_fn();
 
 // GEMM C[M,N] = op(A) op(B) (+C).  a_kcontig: A stored [M][K] (not transposed);
 // b_kcontig: B stored [N][K] (i.e. TB).  ws / counters: split-K workspace (may be null
