@@ -1045,7 +1045,8 @@ def main():
                                           "layers after, one grid barrier; device time p50)")
                                if os.environ.get("SF_CHAIN", "0") == "1" else
                                "request chain (3 LDG-streamed cluster GEMVs over blocked weights "
-                               "under PDL, fused bias/ReLU, fused softmax; device time p50)",
+                               "under PDL, fused bias/ReLU, fused softmax; direct launches behind a "
+                               "drain, one captured graph launch when the device is free; device time p50)",
                                "bound": "hbm", "algorithmic_bytes": w_bytes,
                                "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
                                "peak": hbm, "unit": "GB/s",

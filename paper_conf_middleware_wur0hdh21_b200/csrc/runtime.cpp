@@ -1280,9 +1280,14 @@ sf_status alloc_blocked(Graph& g, Binding& b) {
   }
   return SF_OK;
 }
-bool infer_graph_mode() {
-  static const bool on = std::getenv("SF_INFER_GRAPH") && std::getenv("SF_INFER_GRAPH")[0] == '1';
-  return on;
+// SF_INFER_GRAPH: 0 direct launches only; 1 every request through the captured graph; 2
+// (default, reading Q36) the graph only for requests that find the device free (a
+// preempting request's kernels are enqueued behind the drain event directly, which starts them
+// sooner; a request landing during a host round trip gets one launch call and one command fetch
+// over the busy PCIe link instead of three)
+int infer_graph_mode() {
+  static const int m = std::getenv("SF_INFER_GRAPH") ? std::atoi(std::getenv("SF_INFER_GRAPH")) : 2;
+  return m;
 }
 
 sf_status launch_subgraph_ops(Capture& c, int k);
@@ -2543,30 +2548,29 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
       }
       return a.type == cudaMemoryTypeDevice;
     };
-    const bool in_place = direct && aligned && redirect && !(infer_graph_mode() && B->rg.state == 1) &&
-                          on_device(r->in) && on_device(r->out);
+    if (direct && infer_graph_mode() && B->rg.state == 0 && B->blocked_ready) build_req_graph(g, *B, use_pdl);
+    const bool use_graph = direct && infer_graph_mode() && B->rg.state == 1 && aligned &&
+                           (infer_graph_mode() == 1 || dep_ev == nullptr);
+    const bool in_place = direct && aligned && redirect && !use_graph && on_device(r->in) && on_device(r->out);
     // blocked copies of the constant GEMV weights (allocated at bind; laid out here at the first
     // request unless sf_refresh_constants already did it; reading Q39)
     if (!B->blocked_ready) {
       layout_blocked(g, *B, S->s_infer);
       B->blocked_ready = true;
     }
-    if (direct && infer_graph_mode() && B->rg.state == 0) build_req_graph(g, *B, use_pdl);
     const uint64_t tl0 = now_ns();
     // early launch: the chain (and its start event) wait on the device for the job's
     // dispatched subgraphs; the driver dispatches nothing more while the request is queued
     if (dep_ev) e = cudaStreamWaitEvent(S->s_infer, dep_ev, 0);
     if (e == cudaSuccess) e = cudaEventRecord(S->ev_i0, S->s_infer);
-    const bool graph_req = direct && infer_graph_mode() && B->rg.state == 1 && aligned;
-    if (e != cudaSuccess || in_place || graph_req) {
+    if (e != cudaSuccess || in_place || use_graph) {
     } else if (aligned) {
       e = sfk::launch_copy(r->in, B->arena + tin.offset, tin.nbytes, S->s_infer);
     } else {
       e = cudaMemcpyAsync(B->arena + tin.offset, r->in, tin.nbytes, cudaMemcpyDefault, S->s_infer);
     }
-    const bool graph_io = direct && infer_graph_mode() && B->rg.state == 1 && aligned;
-    if (graph_io && e == cudaSuccess) e = launch_req_graph(*B, tin, tout, r->in, r->out, S->s_infer);
-    for (size_t k = 0; !graph_io && e == cudaSuccess && k < B->versions.size(); ++k) {
+    if (use_graph && e == cudaSuccess) e = launch_req_graph(*B, tin, tout, r->in, r->out, S->s_infer);
+    for (size_t k = 0; !use_graph && e == cudaSuccess && k < B->versions.size(); ++k) {
       if (direct) {
         Capture c{g, *B, S->s_infer, false, &B->prepared};
         if (S->l2_setaside > 0) c.l2_keep = &B->l2_keep;
@@ -2585,7 +2589,7 @@ void dispatcher_main(sf_runtime* rt, Slot* S) {
         sfk::count_launch(B->version_kernels[k]);
       }
     }
-    if (e == cudaSuccess && !in_place && !graph_io) {
+    if (e == cudaSuccess && !in_place && !use_graph) {
       if (aligned) e = sfk::launch_copy(B->arena + tout.offset, r->out, tout.nbytes, S->s_infer);
       else e = cudaMemcpyAsync(r->out, B->arena + tout.offset, tout.nbytes, cudaMemcpyDefault, S->s_infer);
     }

@@ -591,9 +591,11 @@ np.save(sys.argv[1], out.cpu().numpy())
                                       ({"WT": "1"}, -1), ({"WT": "1", "SF_INFER_DIRECT": "0"}, 0),
                                       ({"WT": "1", "SF_FUSE_SOFTMAX": "0", "SF_INFER_REDIRECT": "0",
                                         "SF_PDL": "0"}, 0),
-                                      ({"SF_INFER_GRAPH": "1"}, -1), ({"SF_INFER_GRAPH": "1", "SF_CHAIN": "1"}, -1)],
+                                      ({"SF_INFER_GRAPH": "1"}, -1), ({"SF_INFER_GRAPH": "1", "SF_CHAIN": "1"}, -1),
+                                      ({"SF_INFER_GRAPH": "0"}, -1)],
                          ids=["default", "tma-gemv", "chain", "chain-nopdl", "graphs", "split-gemv", "cluster-gemv",
-                              "rows", "rows-graphs", "rows-unfused", "req-graph", "req-graph-chain"])
+                              "rows", "rows-graphs", "rows-unfused", "req-graph", "req-graph-chain",
+                              "direct-only"])
 def test_inference_paths_vs_oracle(env, spin, tmp_path):
     """Every inference launch path (fused chain, PDL direct launches, captured graphs, the
     GEMV variants; device and pinned-host request buffers; spinning and blocking dispatcher)
