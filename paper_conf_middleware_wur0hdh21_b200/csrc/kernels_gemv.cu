@@ -29,10 +29,10 @@
 namespace sfk {
 namespace {
 
-constexpr int kBlkCluster = 8;   // K split = cluster size
+constexpr int kBlkCluster = 8;   // K split = cluster size (wide layers)
 constexpr int kBlkThreads = 256;
 constexpr int kBlkBatch = 8;     // rows per load batch (two batches in flight)
-constexpr int kBlkMaxKper = 2048;
+constexpr int kBlkMaxKper = 4096;
 
 __device__ __forceinline__ float4 ldg_stream(const float4* p) {
   float4 v;
@@ -49,17 +49,17 @@ __device__ __forceinline__ float4 ldg_stream_hint(const float4* p, uint64_t pol)
   return v;
 }
 
-// Wb[(cb * 8 + r) * kper * QW + row * QW + q] = W[(r * kper + row)][4 (cb QW + q) .. + 3]
+// Wb[(cb * CL + r) * kper * QW + row * QW + q] = W[(r * kper + row)][4 (cb QW + q) .. + 3]
 __global__ void gemv_block_layout_kernel(const float* __restrict__ W, float4* __restrict__ Wb, int K, int N,
-                                         int ldw, int kper, int qw, int n_cb) {
-  const long long total = static_cast<long long>(n_cb) * kBlkCluster * kper * qw;
+                                         int ldw, int kper, int qw, int n_cb, int cl) {
+  const long long total = static_cast<long long>(n_cb) * cl * kper * qw;
   for (long long i = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; i < total;
        i += static_cast<long long>(gridDim.x) * blockDim.x) {
     const int q = static_cast<int>(i % qw);
     const long long rowg = i / qw;  // (cb * 8 + r) * kper + row
     const int row = static_cast<int>(rowg % kper);
     const long long blk = rowg / kper;
-    const int r = static_cast<int>(blk % kBlkCluster), cb = static_cast<int>(blk / kBlkCluster);
+    const int r = static_cast<int>(blk % cl), cb = static_cast<int>(blk / cl);
     const int k = r * kper + row, n = 4 * (cb * qw + q);
     float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
     if (k < K) {
@@ -75,8 +75,12 @@ __global__ void gemv_block_layout_kernel(const float* __restrict__ W, float4* __
   }
 }
 
-template <int MR, int QW>
-__global__ void __cluster_dims__(kBlkCluster, 1, 1) __launch_bounds__(kBlkThreads, 2)
+// CL: CTAs per column block (the K split; a thread-block cluster reducing over DSMEM when
+// CL > 1).  CL = 1 (narrow heads, e.g. 4096 x 1000): each CTA owns whole output columns over
+// all of K, so no cluster barrier or DSMEM round trip sits at its end (ncu on the C4 head with
+// CL = 8: 30% of warp stalls in the cluster barriers); its row groups reduce as a tree.
+template <int MR, int QW, int CL>
+__global__ void __launch_bounds__(kBlkThreads, 2)
 gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, float* __restrict__ Y, int M,
                 int N, int K, int ldx, int ldy, int kper, int acc, const float* __restrict__ b1,
                 const float* __restrict__ b2, const float* __restrict__ b3, int relu,
@@ -97,11 +101,10 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
   __shared__ float4 part[MR * QW];
 
   namespace cg = cooperative_groups;
-  cg::cluster_group cluster = cg::this_cluster();
-  const int rank = static_cast<int>(cluster.block_rank());
-  const int cb = blockIdx.x / kBlkCluster;
+  const int rank = CL > 1 ? static_cast<int>(cg::this_cluster().block_rank()) : 0;
+  const int cb = blockIdx.x / CL;
   const int tid = threadIdx.x, q = tid % QW, rg = tid / QW;
-  const float4* blk = Wb + (static_cast<size_t>(cb) * kBlkCluster + rank) * kper * QW + q;
+  const float4* blk = Wb + (static_cast<size_t>(cb) * CL + rank) * kper * QW + q;
   const int nrow = kper / RL;  // rows of this thread (kper is a multiple of RL)
   const int nb = (nrow + kBlkBatch - 1) / kBlkBatch;
   float4 wa[kBlkBatch], wb[kBlkBatch];
@@ -123,9 +126,20 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     atomicMax(&tl[3], t);
   }
   const int k0 = rank * kper;
-  for (int i = tid; i < MR * kper; i += kBlkThreads) {
-    const int m = i / kper, kk = i % kper;
-    xs[i] = (m < M && k0 + kk < K) ? X[static_cast<size_t>(m) * ldx + k0 + kk] : 0.f;
+  // x slice -> smem: 16 independent loads per thread in flight before any store (one L2 round
+  // trip, not one per element: the CL = 1 head stages all of K)
+  for (int i0 = 0; i0 < MR * kper; i0 += kBlkThreads * 16) {
+    float v[16];
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const int i = i0 + tid + u * kBlkThreads, m = i / kper, kk = i % kper;
+      v[u] = (i < MR * kper && m < M && k0 + kk < K) ? X[static_cast<size_t>(m) * ldx + k0 + kk] : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const int i = i0 + tid + u * kBlkThreads;
+      if (i < MR * kper) xs[i] = v[u];
+    }
   }
   __syncthreads();
   float4 a[MR];
@@ -159,12 +173,22 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     atomicMin(&tl[4], t);
     atomicMax(&tl[5], t);
   }
-  // row groups -> quad partials, fixed order
+  // row groups -> quad partials, fixed order (CL > 1: sequential; CL = 1: a tree, RL up to 128)
 #pragma unroll
   for (int m = 0; m < MR; ++m) {
     red[rg * QW + q] = a[m];
     __syncthreads();
-    if (tid < QW) {
+    if constexpr (CL == 1) {
+      for (int sstep = RL / 2; sstep > 0; sstep >>= 1) {
+        if (rg < sstep) {
+          const float4 v = red[(rg + sstep) * QW + q];
+          float4& t = red[rg * QW + q];
+          t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+        }
+        __syncthreads();
+      }
+      if (tid < QW) part[m * QW + tid] = red[tid];
+    } else if (tid < QW) {
       float4 t = red[tid];
       for (int g = 1; g < RL; ++g) {
         const float4 v = red[g * QW + tid];
@@ -174,14 +198,18 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     }
     __syncthreads();
   }
-  cluster.sync();
+  if constexpr (CL > 1) cg::this_cluster().sync();
   if (rank == 0 && tid < MR * QW) {  // ranks in order, epilogue
     const int m = tid / QW, n = 4 * (cb * QW + tid % QW);
     if (m < M && n < N) {
       float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
-      for (int r = 0; r < kBlkCluster; ++r) {
-        const float4 v = cluster.map_shared_rank(part, r)[tid];
-        t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+      if constexpr (CL > 1) {
+        for (int r = 0; r < CL; ++r) {
+          const float4 v = cg::this_cluster().map_shared_rank(part, r)[tid];
+          t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+        }
+      } else {
+        t = part[tid];
       }
       float* o = Y + static_cast<size_t>(m) * ldy + n;
       const float r4[4] = {t.x, t.y, t.z, t.w};
@@ -204,7 +232,7 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     __shared__ float sm_red[kBlkThreads / 32];
     __threadfence();
     __syncthreads();
-    if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x / kBlkCluster - 1;
+    if (tid == 0) sm_last = atomicAdd(sm_counter, 1u) == gridDim.x / CL - 1;
     __syncthreads();
     if (sm_last) {
       if (tl && tid == 0) atomicMax(&tl[6], sfdev::globaltimer());
@@ -269,13 +297,13 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
       if (tid == 0) *sm_counter = 0u;
     }
   }
-  cluster.sync();
+  if constexpr (CL > 1) cg::this_cluster().sync();  // no CTA leaves while a peer reads its smem
   if (tl && threadIdx.x == 0) atomicMax(&tl[7], sfdev::globaltimer());
 }
 
-template <int MR, int QW>
+template <int MR, int QW, int CL>
 cudaError_t launch_blk_t(const GemmArgs& a, cudaStream_t st) {
-  auto kern = gemv_blk_kernel<MR, QW>;
+  auto kern = gemv_blk_kernel<MR, QW, CL>;
   const int kper = a.blk_kper;
   const size_t smem = static_cast<size_t>(MR) * kper * 4 + static_cast<size_t>(kBlkThreads / QW) * QW * 16;
   static std::atomic<uint64_t> configured{0};
@@ -290,18 +318,39 @@ cudaError_t launch_blk_t(const GemmArgs& a, cudaStream_t st) {
   }
   const int n_cb = (a.N + 4 * QW - 1) / (4 * QW);
   count_launch();
-  return launch_k(kern, dim3(n_cb * kBlkCluster), dim3(kBlkThreads), smem, st,
-                  static_cast<const float4*>(a.Bblk), a.A, a.C, a.M, a.N, a.K, a.lda, a.ldc, kper,
-                  a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0, a.sm_out, a.sm_ldo,
-                  a.sm_counter, a.l2_hint, static_cast<unsigned long long*>(chain_trace_buffer()));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(n_cb * CL);
+  cfg.blockDim = dim3(kBlkThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  int na = 0;
+  if (CL > 1) {
+    at[na].id = cudaLaunchAttributeClusterDimension;
+    at[na].val.clusterDim.x = CL;
+    at[na].val.clusterDim.y = 1;
+    at[na].val.clusterDim.z = 1;
+    ++na;
+  }
+  if (pdl_enabled()) {
+    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  cfg.attrs = at;
+  cfg.numAttrs = na;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<const float4*>(a.Bblk), a.A, a.C, a.M, a.N, a.K, a.lda,
+                            a.ldc, kper, a.acc ? 1 : 0, a.bias[0], a.bias[1], a.bias[2], a.relu ? 1 : 0,
+                            a.sm_out, a.sm_ldo, a.sm_counter, a.l2_hint,
+                            static_cast<unsigned long long*>(chain_trace_buffer()));
 }
 
-template <int QW>
+template <int QW, int CL>
 cudaError_t dispatch_blk_mr(const GemmArgs& a, cudaStream_t st) {
-  if (a.M == 1) return launch_blk_t<1, QW>(a, st);
-  if (a.M == 2) return launch_blk_t<2, QW>(a, st);
-  if (a.M <= 4) return launch_blk_t<4, QW>(a, st);
-  return launch_blk_t<8, QW>(a, st);
+  if (a.M == 1) return launch_blk_t<1, QW, CL>(a, st);
+  if (a.M == 2) return launch_blk_t<2, QW, CL>(a, st);
+  if (a.M <= 4) return launch_blk_t<4, QW, CL>(a, st);
+  return launch_blk_t<8, QW, CL>(a, st);
 }
 
 }  // namespace
@@ -309,6 +358,24 @@ cudaError_t dispatch_blk_mr(const GemmArgs& a, cudaStream_t st) {
 GemvBlockPlan plan_gemv_block(int M, int N, int K) {
   GemvBlockPlan p{};
   if (M < 1 || M > 8 || N < 4 || N % 4 || K < 1) return p;
+  // Cluster-free blocks (CL = 1): 8- or 16-column blocks over all of K, one CTA each, when that
+  // gives one wave of 100-296 CTAs.  SF_GEMV_HEAD: 0 never, 1 (default) narrow heads only
+  // (N <= 1184, e.g. the C4 4096 x 1000 head), 2 every eligible layer.
+  static const int head = std::getenv("SF_GEMV_HEAD") ? std::atoi(std::getenv("SF_GEMV_HEAD")) : 1;
+  if (head && K <= kBlkMaxKper && K >= 1024 && (head == 2 || N <= 4 * 2 * 148)) {
+    for (int qw : {2, 4}) {
+      const int n_cb = (N + 4 * qw - 1) / (4 * qw);
+      if (n_cb < 100 || n_cb > 296) continue;
+      const int rl = kBlkThreads / qw;
+      p.qw = qw;
+      p.cl = 1;
+      p.kper = (K + rl - 1) / rl * rl;
+      p.n_cb = n_cb;
+      p.bytes = static_cast<uint64_t>(p.n_cb) * p.kper * p.qw * 16;
+      p.ok = p.kper <= kBlkMaxKper;
+      return p;
+    }
+  }
   // ONE wave: the widest block whose grid still covers every SM (two CTAs fit per SM, so
   // 148..296 CTAs run at once; a second wave would re-pay the ramp)
   int qw = 4;
@@ -317,8 +384,9 @@ GemvBlockPlan plan_gemv_block(int M, int N, int K) {
   const int rl = kBlkThreads / qw;
   int kper = (K + kBlkCluster - 1) / kBlkCluster;
   kper = (kper + rl - 1) / rl * rl;
-  if (kper > kBlkMaxKper) return p;
+  if (kper > 2048) return p;
   p.qw = qw;
+  p.cl = kBlkCluster;
   p.kper = kper;
   p.n_cb = (N + 4 * qw - 1) / (4 * qw);
   p.bytes = static_cast<uint64_t>(p.n_cb) * kBlkCluster * kper * qw * 16;
@@ -330,7 +398,8 @@ cudaError_t launch_gemv_block_layout(const float* W, void* Wb, int K, int N, int
                                      cudaStream_t st) {
   if (!p.ok) return cudaErrorInvalidValue;
   count_launch();
-  gemv_block_layout_kernel<<<148 * 8, 256, 0, st>>>(W, static_cast<float4*>(Wb), K, N, ldw, p.kper, p.qw, p.n_cb);
+  gemv_block_layout_kernel<<<148 * 8, 256, 0, st>>>(W, static_cast<float4*>(Wb), K, N, ldw, p.kper, p.qw, p.n_cb,
+                                                    p.cl);
   return cudaGetLastError();
 }
 
@@ -339,11 +408,14 @@ bool gemv_blk_eligible(const GemmArgs& a) {
 }
 
 cudaError_t launch_gemv_blk(const GemmArgs& a, cudaStream_t st) {
+  if (a.blk_cl == 1)
+    return a.blk_qw == 2 ? dispatch_blk_mr<2, 1>(a, st) : a.blk_qw == 4 ? dispatch_blk_mr<4, 1>(a, st)
+                                                        : cudaErrorInvalidValue;
   switch (a.blk_qw) {
-    case 32: return dispatch_blk_mr<32>(a, st);
-    case 16: return dispatch_blk_mr<16>(a, st);
-    case 8: return dispatch_blk_mr<8>(a, st);
-    case 4: return dispatch_blk_mr<4>(a, st);
+    case 32: return dispatch_blk_mr<32, kBlkCluster>(a, st);
+    case 16: return dispatch_blk_mr<16, kBlkCluster>(a, st);
+    case 8: return dispatch_blk_mr<8, kBlkCluster>(a, st);
+    case 4: return dispatch_blk_mr<4, kBlkCluster>(a, st);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -863,6 +863,7 @@ sf_status launch_subgraph_ops(Capture& c, int k) {
             ga.Bblk = bk->second.first;
             ga.blk_qw = bk->second.second.qw;
             ga.blk_kper = bk->second.second.kper;
+            ga.blk_cl = bk->second.second.cl;
           }
         }
         auto sa = c.b.shadow.find(o.in[0]);

@@ -61,12 +61,12 @@ struct GemmArgs {
   uint64_t pf_bytes = 0;
   // constant B re-laid out in contiguous blocks (kernels_gemv.cu): the LDG-streamed GEMV
   const void* Bblk = nullptr;
-  int blk_qw = 0, blk_kper = 0;
+  int blk_qw = 0, blk_kper = 0, blk_cl = 8;
 };
 // Blocked layout of a constant GEMV weight (kernels_gemv.cu)
 struct GemvBlockPlan {
   bool ok = false;
-  int qw = 0, kper = 0, n_cb = 0;
+  int qw = 0, kper = 0, n_cb = 0, cl = 8;  // cl: CTAs per column block (K split)
   uint64_t bytes = 0;
 };
 GemvBlockPlan plan_gemv_block(int M, int N, int K);

@@ -891,3 +891,49 @@ def test_drain_gate_holds_the_queued_subgraph(P):
         assert rel(outs[r], R.run_inference(gi, sti, xs[r])) <= TOL
     dv = SC.device_view([dict(e, job=(1 if e["kind"] == "infer" else 0)) for e in trace])
     SC.check_no_corun(dv)
+
+
+_C4_CHILD = r"""
+import os, sys, numpy as np, torch
+sys.path.insert(0, '.')
+from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
+from sf_inputs import data as D, graphs as G
+gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M")
+xs = D.infer_inputs(gi, 4)
+with Runtime([0], dispatch_spin_us=-1) as rt:
+    ghi = rt.register(gi, 1); ghi.partition(); ghi.bind(0, staging=False)
+    ghi.load(0, D.init_state(gi, seed=D.SEED_INFER))
+    out = torch.zeros(4, 1, 1000, device="cuda")
+    host_in = torch.from_numpy(xs).pin_memory()
+    host_out = torch.zeros(4, 1, 1000).pin_memory()
+    xin = torch.from_numpy(xs).cuda()
+    for r in range(4):
+        if r % 2:
+            rt.wait(rt.submit(ghi, 0, host_in[r].data_ptr(), host_out[r].data_ptr()), 60)
+            out[r] = host_out[r].cuda()
+        else:
+            rt.wait(rt.submit(ghi, 0, xin[r].data_ptr(), out[r].data_ptr()), 60)
+np.save(sys.argv[1], out.cpu().numpy())
+"""
+
+
+@pytest.mark.parametrize("env", [{}, {"SF_GEMV_HEAD": "0"}, {"SF_GEMV_HEAD": "2"}, {"SF_INFER_GRAPH": "0"},
+                                 {"SF_INFER_GRAPH": "1"}, {"SF_CHAIN": "1"}],
+                         ids=["default", "cluster-head", "no-cluster-all", "direct-only", "graph-always",
+                              "fold-chain"])
+def test_c4_inference_model_vs_oracle(env, tmp_path):
+    """The bench's preempter model (2048-4096-4096-1000 MLP + softmax) through
+    the request path the bench times (blocked GEMVs; the cluster-free head over 8-column blocks;
+    the captured request graph) against the oracle's forward pass, device and pinned-host
+    request buffers alike."""
+    import os, subprocess, sys
+    f = tmp_path / "out.npy"
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    subprocess.run([sys.executable, "-c", _C4_CHILD, str(f)], cwd=root, env=dict(os.environ, **env),
+                   check=True, timeout=240)
+    got = np.load(f)
+    gi = G.mlp_infer((2048, 4096, 4096, 1000), name="infer_mlp_29M")
+    sti = D.init_state(gi, seed=D.SEED_INFER)
+    xs = D.infer_inputs(gi, 4)
+    for r in range(4):
+        assert rel(got[r], R.run_inference(gi, sti, xs[r])) <= TOL, (env, r)
