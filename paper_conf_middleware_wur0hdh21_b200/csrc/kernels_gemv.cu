@@ -359,9 +359,9 @@ GemvBlockPlan plan_gemv_block(int M, int N, int K) {
   GemvBlockPlan p{};
   if (M < 1 || M > 8 || N < 4 || N % 4 || K < 1) return p;
   // Cluster-free blocks (CL = 1): 8- or 16-column blocks over all of K, one CTA each, when that
-  // gives one wave of 100-296 CTAs.  SF_GEMV_HEAD: 0 never, 1 (default) narrow heads only
-  // (N <= 1184, e.g. the C4 4096 x 1000 head), 2 every eligible layer.
-  static const int head = std::getenv("SF_GEMV_HEAD") ? std::atoi(std::getenv("SF_GEMV_HEAD")) : 1;
+  // gives one wave of 100-296 CTAs (reading Q44).  SF_GEMV_HEAD: 0 never, 1 narrow
+  // heads only (N <= 1184, e.g. the C4 4096 x 1000 head), 2 (default) every eligible layer.
+  static const int head = std::getenv("SF_GEMV_HEAD") ? std::atoi(std::getenv("SF_GEMV_HEAD")) : 2;
   if (head && K <= kBlkMaxKper && K >= 1024 && (head == 2 || N <= 4 * 2 * 148)) {
     for (int qw : {2, 4}) {
       const int n_cb = (N + 4 * qw - 1) / (4 * qw);

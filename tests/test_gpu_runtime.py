@@ -917,9 +917,9 @@ np.save(sys.argv[1], out.cpu().numpy())
 """
 
 
-@pytest.mark.parametrize("env", [{}, {"SF_GEMV_HEAD": "0"}, {"SF_GEMV_HEAD": "2"}, {"SF_INFER_GRAPH": "0"},
+@pytest.mark.parametrize("env", [{}, {"SF_GEMV_HEAD": "0"}, {"SF_GEMV_HEAD": "1"}, {"SF_INFER_GRAPH": "0"},
                                  {"SF_INFER_GRAPH": "1"}, {"SF_CHAIN": "1"}],
-                         ids=["default", "cluster-head", "no-cluster-all", "direct-only", "graph-always",
+                         ids=["default", "cluster-all", "cluster-wide-layers", "direct-only", "graph-always",
                               "fold-chain"])
 def test_c4_inference_model_vs_oracle(env, tmp_path):
     """The bench's preempter model (2048-4096-4096-1000 MLP + softmax) through
