@@ -969,6 +969,7 @@ def main():
     m0 = chase_s
     link = host_link_peaks()
     dev_us = pct(main_s.get("device_us", []), 50)
+    bd = main_s.get("breakdown") or {}
     w_bytes = (2048 * 4096 + 4096 * 4096 + 4096 * 1000 + 4096 + 4096 + 1000) * 4
     tr = main_s.get("training", {})
     line = {
@@ -1050,7 +1051,13 @@ def main():
                                "bound": "hbm", "algorithmic_bytes": w_bytes,
                                "achieved": (w_bytes / (dev_us * 1e-6) / 1e9) if dev_us else None,
                                "peak": hbm, "unit": "GB/s",
-                               "frac": (w_bytes / (dev_us * 1e-6) / 1e9 / hbm) if dev_us else None},
+                               "frac": (w_bytes / (dev_us * 1e-6) / 1e9 / hbm) if dev_us else None,
+                               # the same p50 per request group: preempting requests run on an idle
+                               # device; the others land during a host round trip and share PCIe
+                               "by_group": {g: {"device_us_p50": bd[g]["device_p50"],
+                                                "frac": w_bytes / (bd[g]["device_p50"] * 1e-6) / 1e9 / hbm}
+                                            for g in ("preempting", "not_preempting")
+                                            if bd.get(g) and bd[g].get("device_p50")}},
         "e2e": {"value": pct(E, 99), "unit": UNIT, "n": len(E), "h2d_bytes_per_step": 2048 * 4 * rps,
                 "d2h_bytes_per_step": 1000 * 4 * rps, "p50_ms": pct(E, 50)},
         "gpu_launches": int(sum(a["main"]["launches"] for a in allv)),

@@ -5,6 +5,7 @@ streaming, last CTA end} relative to the first CTA start of layer 0 (sf_debug_ch
 import ctypes as C, json, os, sys
 import numpy as np, torch
 os.environ.setdefault("SF_CHAIN", "0")  # the per-layer GEMV chain (the fused kernel has its own trace)
+os.environ.setdefault("SF_INFER_GRAPH", "0")  # direct launches: the captured graph has no trace pointer
 sys.path.insert(0, ".")
 import bench
 from paper_conf_middleware_wur0hdh21_b200.runtime import Runtime
