@@ -37,7 +37,6 @@ bool pdl_enabled() { return t_pdl; }
 
 
 constexpr int kCopyThreads = 256;
-constexpr int kCopyUnroll = SF_COPY_UNROLL;
 
 __device__ __forceinline__ uint4 load_chunk(const uint8_t* src, uint64_t j, uint64_t full,
                                             uint64_t nb) {
@@ -67,6 +66,7 @@ struct SDesc {
   uint64_t begin;
 };
 
+template <int kCopyUnroll>
 __global__ void __launch_bounds__(kCopyThreads)
 mtcopy_kernel(const DCopy* __restrict__ d, int n, uint64_t base, uint64_t total, uint64_t per_block,
               int64_t patch_iter, unsigned long long* tstamp) {
@@ -288,8 +288,14 @@ cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
     nb = std::max<uint64_t>(nb, 1);
     const uint64_t per_block = (cnt + nb - 1) / nb;
     nb = (cnt + per_block - 1) / per_block;
-    mtcopy_kernel<<<static_cast<unsigned>(nb), kCopyThreads, 0, st>>>(d_descs, n, w0, w1, per_block,
-                                                                      patch_iter, tstamp);
+    // loads in flight per thread (SF_COPY_UNROLL: 8 default, 16)
+    static const int unroll = std::getenv("SF_COPY_UNROLL") ? std::atoi(std::getenv("SF_COPY_UNROLL")) : SF_COPY_UNROLL;
+    if (unroll == 16)
+      mtcopy_kernel<16><<<static_cast<unsigned>(nb), kCopyThreads, 0, st>>>(d_descs, n, w0, w1, per_block,
+                                                                            patch_iter, tstamp);
+    else
+      mtcopy_kernel<8><<<static_cast<unsigned>(nb), kCopyThreads, 0, st>>>(d_descs, n, w0, w1, per_block,
+                                                                           patch_iter, tstamp);
     count_launch();
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
