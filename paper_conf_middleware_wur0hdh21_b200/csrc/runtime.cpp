@@ -1549,10 +1549,13 @@ cudaError_t duplex_round_trip(Job& J, Slot& S, int slot, uint8_t* dstg, uint8_t*
                                       ? size_t(std::max(1, std::min(2, std::atoi(std::getenv("SF_DUPLEX_DEPTH_D2H")))))
                                       : kDepth;
   constexpr int R = 4;  // event ring per direction (kCkEvents / 2)
-  // small live sets (<= R chunks of 2 MB, e.g. C1's 1.6-2.4 MB): R equal chunks all issued at
-  // once (D2H on the migration stream, each H2D waiting on its chunk's event on the device), so
-  // the two directions overlap without host round trips between chunks
-  const bool upfront = !std::getenv("SF_DUPLEX_CHUNK_KB") && total <= R * kChunk;
+  // small live sets (2-8 MB): R equal chunks all issued at once (D2H on the migration stream,
+  // each H2D waiting on its chunk's event on the device), so the two directions overlap without
+  // host round trips between chunks.  At most one chunk of 2 MB (C1's 1.6-2.4 MB): one D2H then
+  // one H2D — measured cheaper than any split at that size, where every extra copy costs more
+  // in fixed latency than the overlap saves (scripts/pcie_small.py: 1.6 MB D2H 34 us, H2D 35,
+  // both 71 us back to back, 95-272 us as 2-8 overlapped chunks)
+  const bool upfront = !std::getenv("SF_DUPLEX_CHUNK_KB") && total > kChunk && total <= R * kChunk;
   const size_t chunk = upfront ? std::max<size_t>(size_t(64) << 10, ((total + R - 1) / R + 4095) / 4096 * 4096)
                                : kChunk;
   const size_t depth = upfront ? R : kDepth, depth_d2h = upfront ? R : kDepthD2H;
