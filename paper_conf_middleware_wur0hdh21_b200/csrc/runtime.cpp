@@ -1792,6 +1792,10 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
     Binding& BD = *g.bind[dst];
     lk.unlock();
     if ((e = cudaSetDevice(D.cuda)) != cudaSuccess) return cuda_fail(e, "set device");
+    if (dst != src) {  // as for the peer store: dst's arena may still be being released (poison)
+      cudaEventRecord(J.ev_sub[dst], D.s_mig);
+      cudaStreamWaitEvent(D.s_train, J.ev_sub[dst], 0);
+    }
     cudaEventRecord(J.ev_a[dst], D.s_train);
     // the parked bytes live in the source binding's pinned staging; a ZC swap-in reads
     // them in place when resuming on the same slot, otherwise H2D + unpack
@@ -1837,6 +1841,19 @@ sf_status do_preempt(sf_runtime* rt, Job& J, std::unique_lock<std::mutex>& lk) {
       return fail(SF_EINVAL, J.error);
     }
     const CopyList& L = it->second[k];
+    {
+      // the target arena was released by an earlier move out of that slot, whose clean-up
+      // (the poison fill in test mode) runs on the TARGET slot's migration stream: the store
+      // into it waits for that stream (a remote slot synchronised its own before the handoff)
+      Slot& T0 = slot_of(rt, target);
+      if (!T0.remote) {
+        if ((e = cudaSetDevice(T0.cuda)) != cudaSuccess ||
+            (e = cudaEventRecord(J.ev_sub[target], T0.s_mig)) != cudaSuccess ||
+            (e = cudaSetDevice(S.cuda)) != cudaSuccess ||
+            (e = cudaStreamWaitEvent(S.s_mig, J.ev_sub[target], 0)) != cudaSuccess)
+          return cuda_fail(e, "order peer store after the target's migration stream");
+      }
+    }
     tstamp_reset(S.tstamp, S.s_mig);
     cudaEventRecord(J.ev_a[src], S.s_mig);
     if (rt->cfg.migration_engine == SF_MIG_CE)  // copy engines over NVLink, no SM work
