@@ -19,7 +19,9 @@ BUILD = os.path.join(PKG, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", CSRC,
-         "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
+         "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"] + os.environ.get("SF_NVCC_EXTRA", "").split()
+# (SF_NVCC_EXTRA: extra -D switches for A/B builds of compile-time kernel parameters; delete the
+# affected _build/*.o first, the mtime check does not see flags)
 SOURCES = ["kernels_copy.cu", "kernels_gemm.cu", "kernels_gemm_tma.cu", "kernels_gemv.cu", "kernels_elem.cu",
            "kernels_chain.cu", "runtime.cpp"]
 

@@ -33,6 +33,11 @@ constexpr int kBlkCluster = 8;   // K split = cluster size (wide layers)
 constexpr int kBlkThreads = 256;
 constexpr int kBlkBatch = 8;     // rows per load batch (two batches in flight)
 constexpr int kBlkMaxKper = 4096;
+#ifndef SF_GEMV_MINB
+#define SF_GEMV_MINB 2  // CTAs per SM the cluster-free batch-1 layers are compiled for: 3 (80
+                        // registers, more of the next layer pre-launched under PDL) measured
+                        // 45.0 vs 38.8 us request device time (scripts/r2_minb.sh)
+#endif
 
 __device__ __forceinline__ float4 ldg_stream(const float4* p) {
   float4 v;
@@ -80,7 +85,7 @@ __global__ void gemv_block_layout_kernel(const float* __restrict__ W, float4* __
 // all of K, so no cluster barrier or DSMEM round trip sits at its end (ncu on the C4 head with
 // CL = 8: 30% of warp stalls in the cluster barriers); its row groups reduce as a tree.
 template <int MR, int QW, int CL>
-__global__ void __launch_bounds__(kBlkThreads, 2)
+__global__ void __launch_bounds__(kBlkThreads, CL == 1 && MR == 1 ? SF_GEMV_MINB : 2)
 gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, float* __restrict__ Y, int M,
                 int N, int K, int ldx, int ldy, int kper, int acc, const float* __restrict__ b1,
                 const float* __restrict__ b2, const float* __restrict__ b3, int relu,
