@@ -123,8 +123,13 @@ gemv_blk_kernel(const float4* __restrict__ Wb, const float* __restrict__ X, floa
     }
   };
   sfdev::griddep_launch();  // the next layer may start streaming its (constant) weights
+#ifndef SF_GEMV_NOPRE
   if (nb > 0) load(wa, 0);  // weights never depend on the predecessor: issue before the wait
   sfdev::griddep_wait();    // x is the predecessor's output
+#else  // A/B build: no weight load before the predecessor completes
+  sfdev::griddep_wait();
+  if (nb > 0) load(wa, 0);
+#endif
   if (tl && threadIdx.x == 0) {
     const unsigned long long t = sfdev::globaltimer();
     atomicMin(&tl[2], t);
