@@ -69,7 +69,7 @@ def pct(x, q):
 def block_size(args) -> int:
     """Requests per timed step: --requests-per-step, raised so that the headline percentiles rest
     on at least 1,000 requests whatever --steps is (round-1 verdict: a p99 of 20 samples)."""
-    return max(args.requests_per_step, -(-1000 // max(1, args.steps)))
+    return max(args.requests_per_step, -(-getattr(args, "min_requests", 1000) // max(1, args.steps)))
 
 
 def load_peaks():
@@ -815,6 +815,8 @@ def main():
                     help="timed steps; a step is one block of --requests-per-step Poisson arrivals")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--requests-per-step", type=int, default=50)
+    ap.add_argument("--min-requests", type=int, default=1000,
+                    help="timed requests at least (the block per step grows); 0 for short profiling runs")
     ap.add_argument("--baseline-requests", type=int, default=500,
                     help="requests per same-run baseline arm")
     ap.add_argument("--chase-cycles", type=int, default=300,

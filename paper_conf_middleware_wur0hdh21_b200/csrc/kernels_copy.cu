@@ -267,7 +267,10 @@ cudaError_t launch_mtcopy(const DCopy* d_descs, int n, uint64_t total_chunks,
   // SM (one wave: only three of this kernel's CTAs fit an SM's registers anyway): measured
   // 5.58-5.63 TB/s pack on the C2 cut 0 vs 5.50-5.54 with 8 per SM (2.7 waves), 5.0-5.1 with
   // 3-4, 4.1 with 1 (scripts/r2_bps.sh); bench p99 0.118-0.120 vs 0.122-0.123 ms.
-  static const int bps = std::getenv("SF_COPY_BPS") ? std::atoi(std::getenv("SF_COPY_BPS")) : 2;
+  // Walks above 1 GB (C3's 4.25 GB peer store, C5) keep 8 per SM: measured 5.8 TB/s there
+  // against 4.9 TB/s with 2 (scripts/bench_configs.py c3).
+  static const int bps_env = std::getenv("SF_COPY_BPS") ? std::atoi(std::getenv("SF_COPY_BPS")) : 0;
+  const int bps = bps_env > 0 ? bps_env : total_chunks * 16 <= (1ull << 30) ? 2 : 8;
   static const uint64_t min_chunks =
       std::getenv("SF_COPY_MINCHUNKS") ? std::atoll(std::getenv("SF_COPY_MINCHUNKS")) : 2048;
   uint64_t blocks = (total_chunks + min_chunks - 1) / min_chunks;

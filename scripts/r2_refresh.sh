@@ -13,12 +13,12 @@ timeout 300 python scripts/gemm_bench.py > gpurun_out/r02_gemm_bench.log 2>&1
 timeout 300 python scripts/blk_trace.py 60 > gpurun_out/r02_blk_trace.log 2>&1
 timeout 300 python scripts/subgraph_durations.py > gpurun_out/r02_subgraph_durations.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 6000 --csv \
-  --log-file gpurun_out/r02_launches.csv python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline > gpurun_out/r02_ncu_bench.log 2>&1; echo "ncu list exit $?"
+  --log-file gpurun_out/r02_launches.csv python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline --min-requests 0 > gpurun_out/r02_ncu_bench.log 2>&1; echo "ncu list exit $?"
 python scripts/launch_shares.py gpurun_out/r02_launches.csv > gpurun_out/r02_launch_shares.md
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:mtcopy -s 2 -c 2 \
-  -o gpurun_out/r02_prof_pack -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline > gpurun_out/r02_ncu_pack.log 2>&1; echo "ncu pack exit $?"
+  -o gpurun_out/r02_prof_pack -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline --min-requests 0 > gpurun_out/r02_ncu_pack.log 2>&1; echo "ncu pack exit $?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:gemv_blk -s 6 -c 3 \
-  -o gpurun_out/r02_prof_gemv -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline > gpurun_out/r02_ncu_gemv.log 2>&1; echo "ncu gemv exit $?"
+  -o gpurun_out/r02_prof_gemv -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline --min-requests 0 > gpurun_out/r02_ncu_gemv.log 2>&1; echo "ncu gemv exit $?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:gemm_tma -s 20 -c 4 \
-  -o gpurun_out/r02_prof_gemm -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline > gpurun_out/r02_ncu_gemm.log 2>&1; echo "ncu gemm exit $?"
+  -o gpurun_out/r02_prof_gemm -f python bench.py --steps 3 --warmup 3 --no-baselines --no-cpu-baseline --min-requests 0 > gpurun_out/r02_ncu_gemm.log 2>&1; echo "ncu gemm exit $?"
 ls gpurun_out | grep r02
