@@ -858,10 +858,13 @@ def main():
                     help="1: a preempting request is enqueued behind a device-side wait on the "
                          "job's in-flight subgraphs (default); 0: launched after the drain")
     args = ap.parse_args()
-    if os.environ.get("SF_BENCH_WATCHDOG_S"):  # debugging aid: dump every thread's stack, then exit
+    # watchdog: dump every thread's stack, then exit (default on for N > 1: a rank stuck on a
+    # never-completing peer handoff ends the run instead of holding every GPU of the node)
+    wd = os.environ.get("SF_BENCH_WATCHDOG_S") or ("1500" if int(os.environ.get("WORLD_SIZE", "1")) > 1 else "")
+    if wd:
         import faulthandler
         faulthandler.enable()  # a fatal signal also dumps every thread's Python stack
-        faulthandler.dump_traceback_later(float(os.environ["SF_BENCH_WATCHDOG_S"]), exit=True)
+        faulthandler.dump_traceback_later(float(wd), exit=True)
     args.world = int(os.environ.get("WORLD_SIZE", "1"))
     args.rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
